@@ -1,0 +1,373 @@
+#!/usr/bin/env python3
+"""bench.py -- payload GB/s deduplicated on B200, with roofline and CPU-oracle baselines.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload 5] [--impl ours|reference]
+
+A step = one ffm_dedup_run over the whole log (H1 hash .. H7 labels/benefit, all
+of SURVEY.md 8(a)) with the payloads already resident in HBM.  Default workload
+= BASELINE config 5 (the ~64 GB mixed application-shaped log, 2 M transfers,
+10k call sites) on one GPU; inputs (63 GB) are far larger than L2 (126 MB).
+
+  value    = sum of payload bytes / device time per step (CUDA events on the
+             library's stream), GB/s (1e9).
+  e2e      = the same metric through the public C ABI from pinned HOST buffers:
+             ffm_log_create + ffm_log_append_batch (H2D of every payload) +
+             ffm_dedup_run + D2H of duplicate_of / benefit_ns, per step.
+  roofline = the dominant kernel's algorithmic bytes / its CUDA-event time vs
+             the measured HBM copy bandwidth (MEASURED_PEAKS.json).
+  cpu_baseline = the CPU oracle (oracle/) on a bounded gid-prefix sample, 1 core.
+
+--impl reference times the oracle (the only "reference" this tier has) on the
+host cores, on this arm's config / metric / unit.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "payload GB/s deduplicated (1/2/4/8 B200) and % of HBM roofline"
+UNIT = "GB/s"
+WORKLOADS = {
+    1: "config1: 1,000 transfers 4 KB-1 MB, 30% planted dups, 50 sites",
+    2: "config2: 1M small transfers 256 B-4 KB, 60% re-uploads, 256 sites",
+    3: "config3: 10,000 x 1 MiB near-duplicates, single-byte differences",
+    4: "config4: 1,000 large transfers 16-64 MiB, 20 solver arrays x 50 iterations",
+    5: "config5: mixed application-shaped log, 2M transfers, ~64 GB, 10k call sites",
+}
+
+
+def log_msg(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def dist_env():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), \
+        int(os.environ.get("LOCAL_RANK", 0))
+
+
+def load_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.proc = None
+        self.path = f"/tmp/ffm_clocks_{os.getpid()}.csv"
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], 0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = max(mx, float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def make_log(workload, n_scale, size_scale):
+    import loggen
+    t = time.time()
+    lg = loggen.gen_config(workload, n_scale=n_scale, size_scale=size_scale)
+    lg.materialize(nthreads=0)
+    log_msg(f"[bench] generated {lg.name}: {lg.n} records, {lg.total_bytes / 1e9:.2f} GB payload, "
+            f"{lg.distinct_bytes / 1e9:.2f} GB distinct, {time.time() - t:.1f}s")
+    return lg
+
+
+def alg_bytes(lg, dup, small_bytes):
+    """Algorithmic bytes per kernel."""
+    size = lg.size.astype(np.int64)
+    n = len(size)
+    small = size <= small_bytes
+    member = dup >= 0
+    # leaders with >=1 member, counted once (their bytes are re-read from L2 by the others)
+    leaders = np.zeros(n, bool)
+    if member.any():
+        gid_to_idx = np.arange(n)           # single-GPU: gid == local index
+        leaders[gid_to_idx[dup[member]]] = True
+    out = {
+        "hash_small": int(size[small].sum()) + 8 * n + 24 * int(small.sum()),
+        "hash_large": int(size[~small].sum()) + 40 * int(((size[~small] + 32767) // 32768).sum()),
+        "verify_small": int(size[small & member].sum()) + int(size[small & leaders].sum()) + 4 * n,
+        "verify_large": int(size[~small & member].sum()) + int(size[~small & leaders].sum()),
+    }
+    out["path"] = sum(out.values()) + 64 * n    # + group-by / label metadata
+    return out
+
+
+def ncu_traffic(kernel):
+    """dram bytes per launch of `kernel` from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        k = d["kernels"].get(kernel)
+        return None if k is None else float(k["dram_bytes_per_launch"])
+    except Exception:
+        return None
+
+
+def run_ours(args):
+    import torch
+    import paper_conf_sc_weltonm19_b200 as ffm
+
+    rank, world, local = dist_env()
+    if world > 1:
+        raise SystemExit("multi-GPU sharded runs: see DESIGN.md 'Multi-GPU' (not enabled in this build)")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    lg = make_log(args.workload, args.n_scale, args.size_scale)
+    total = lg.total_bytes
+
+    # ---- device-resident log: distinct contents uploaded once, records snapshotted by the library
+    t = time.time()
+    content = torch.from_numpy(lg.buf).to(dev)
+    ptrs = (lg.c_off[lg.content] + np.uint64(content.data_ptr())).astype(np.uint64)
+    log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=total + 128 * lg.n + (1 << 20),
+                     max_records=lg.n, timing=True)
+    log.append_batch(lg.site, lg.size, ptrs, lg.dur, payload_kind=ffm.FFM_PAYLOAD_DEVICE)
+    del content
+    torch.cuda.synchronize()
+    torch.cuda.empty_cache()
+    log_msg(f"[bench] staged {total / 1e9:.2f} GB into the HBM arena in {time.time() - t:.1f}s")
+
+    dup = torch.empty(lg.n, dtype=torch.int64, device=dev)
+    ben = torch.empty(lg.n_sites, dtype=torch.int64, device=dev)
+    stream = torch.cuda.ExternalStream(log.stream, device=dev)
+    for _ in range(args.warmup):
+        log.run(dup, ben)
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    acc = {}
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(args.steps):
+        log.run(dup, ben)
+        for k, v in log.stats().items():
+            acc[k] = acc.get(k, 0) + v
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / args.steps
+    clk = clocks.stop()
+    st = {k: v / args.steps for k, v in acc.items()}
+    value = total / (ms * 1e-3) / 1e9
+
+    dup_h = dup.cpu().numpy()
+    ab = alg_bytes(lg, dup_h, 4096)
+    peak, peak_src = load_peak()
+    kern_ms = {"hash_small": st["ms_hash_small"], "hash_large": st["ms_hash_large"],
+               "verify": st["ms_verify"]}
+    dom = max(("hash_large", "hash_small"), key=lambda k: kern_ms[k])
+    dom_bytes = ab[dom]
+    dom_ms = kern_ms[dom]
+    achieved = dom_bytes / (dom_ms * 1e-3) / 1e9 if dom_ms > 0 else 0.0
+    kname = {"hash_large": "k_hash_large", "hash_small": "k_hash_small"}[dom]
+    traffic = ncu_traffic(kname)
+    roofline = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic, "alg_bytes": dom_bytes,
+                "ms": round(dom_ms, 4), "peak_source": peak_src}
+    path_gbs = ab["path"] / (ms * 1e-3) / 1e9
+    launches = int(round(st["kernel_launches"])) * args.steps
+
+    # ---- end to end through the public ABI from pinned host buffers
+    e2e = None
+    if args.e2e_steps > 0:
+        del log
+        torch.cuda.empty_cache()
+        e2e = run_e2e(args, lg, local)
+
+    # ---- CPU oracle baseline (bounded gid-prefix sample, 1 core)
+    cpu = cpu_baseline(lg, args.cpu_seconds) if args.cpu_seconds > 0 else None
+
+    out = {
+        "metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": WORKLOADS[args.workload], "records": lg.n, "payload_bytes": total,
+                   "n_sites": lg.n_sites, "seed": "0x5C19D1000%d" % args.workload,
+                   "n_scale": args.n_scale, "size_scale": args.size_scale,
+                   "l2": "inputs larger than L2 (payload %.1f GB >> 126 MB L2)" % (total / 1e9),
+                   "parallelism": "single GPU" if world == 1 else f"sharded x{world}",
+                   "chunk_bytes": 32768, "small_bytes": 4096},
+        "pct_hbm_roofline_path": round(path_gbs / peak, 4),
+        "path_alg_gbs": round(path_gbs, 1),
+        "stage_ms": {k: round(st[k], 4) for k in ("ms_hash_small", "ms_hash_large", "ms_group", "ms_verify",
+                                                  "ms_resolve", "ms_label", "ms_output", "ms_total")},
+        "clocks": clk, "gpu_launches": launches, "roofline": roofline, "e2e": e2e, "cpu_baseline": cpu,
+        "duplicates": int((dup_h >= 0).sum()),
+    }
+    print(json.dumps(out), flush=True)
+
+
+def run_e2e(args, lg, local):
+    import torch
+    import paper_conf_sc_weltonm19_b200 as ffm
+    buf = lg.buf
+    cudart = torch.cuda.cudart()
+    reg = cudart.cudaHostRegister(buf.ctypes.data, buf.nbytes, 0)
+    ptrs = lg.payload_ptrs()
+    n = lg.n
+    dup = np.empty(n, np.int64)
+    ben = np.empty(lg.n_sites, np.uint64)
+    dup_pin = torch.empty(n, dtype=torch.int64).pin_memory().numpy()
+    ben_pin = torch.empty(lg.n_sites, dtype=torch.int64).pin_memory().numpy().view(np.uint64)
+    times = []
+    for step in range(args.e2e_steps + 1):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        with ffm.FfmLog(lg.n_sites, device=local, arena_bytes=lg.total_bytes + 128 * n + (1 << 20),
+                        max_records=n) as log:
+            log.append_batch(lg.site, lg.size, ptrs, lg.dur, payload_kind=ffm.FFM_PAYLOAD_HOST)
+            log.run(dup_pin, ben_pin)
+        t1 = time.perf_counter()
+        if step > 0:                     # first step warms up
+            times.append(t1 - t0)
+    if int(reg) == 0:
+        cudart.cudaHostUnregister(buf.ctypes.data)
+    sec = statistics.median(times)
+    meta = n * (4 + 8 + 8)
+    return {"value": round(lg.total_bytes / sec / 1e9, 3), "unit": UNIT,
+            "h2d_bytes_per_step": int(lg.total_bytes + meta), "d2h_bytes_per_step": int(8 * n + 8 * lg.n_sites),
+            "steps": len(times), "s_per_step": round(sec, 4),
+            "note": "wall clock per step: create + append (pinned host -> HBM) + run + D2H, median"}
+
+
+def oracle_sample(lg, seconds_budget):
+    """gid-prefix of the log whose oracle time is ~seconds_budget (calibrated)."""
+    import oracle
+    n = lg.n
+    csum = np.cumsum(lg.size.astype(np.int64))
+    # calibrate on a small prefix
+    k = int(np.searchsorted(csum, min(csum[-1], 200_000_000))) + 1
+    k = max(1, min(k, n))
+    t = time.perf_counter()
+    oracle.dedup(lg.subset(np.arange(k)))
+    dt = max(time.perf_counter() - t, 1e-6)
+    rate = csum[k - 1] / dt
+    want = rate * seconds_budget
+    k2 = int(np.searchsorted(csum, want)) + 1
+    return max(1, min(k2, n)), rate
+
+
+def cpu_baseline(lg, seconds):
+    import oracle
+    try:
+        os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+        cores = 1
+    except Exception:
+        cores = 1
+    k, _ = oracle_sample(lg, seconds)
+    sub = lg.subset(np.arange(k))
+    t = time.perf_counter()
+    oracle.dedup(sub)
+    dt = time.perf_counter() - t
+    b = int(lg.size[:k].sum())
+    return {"value": round(b / dt / 1e9, 3), "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"gid prefix of {k} of {lg.n} records ({b / 1e9:.2f} GB of {lg.total_bytes / 1e9:.2f} GB), "
+                      f"{dt:.1f}s on 1 of {os.cpu_count()} host cores"}
+
+
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import oracle
+    lg = make_log(args.workload, args.n_scale, args.size_scale)
+    os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+    k, _ = oracle_sample(lg, args.ref_step_seconds)
+    sub = lg.subset(np.arange(k))
+    b = int(lg.size[:k].sum())
+    for _ in range(args.warmup):
+        oracle.dedup(sub)
+    ts = []
+    for _ in range(args.steps):
+        t = time.perf_counter()
+        oracle.dedup(sub)
+        ts.append(time.perf_counter() - t)
+    sec = sum(ts) / len(ts)
+    v = round(b / sec / 1e9, 3)
+    sample = f"gid prefix of {k} of {lg.n} records ({b / 1e9:.2f} GB) per step"
+    out = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(sec * 1e3, 3),
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+           "data": "synthetic",
+           "config": {"workload": WORKLOADS[args.workload], "records": lg.n, "payload_bytes": lg.total_bytes,
+                      "n_sites": lg.n_sites, "n_scale": args.n_scale, "size_scale": args.size_scale},
+           "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", type=int, default=5, choices=[1, 2, 3, 4, 5])
+    ap.add_argument("--n-scale", type=float, default=1.0)
+    ap.add_argument("--size-scale", type=float, default=1.0)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--ref-step-seconds", type=float, default=6.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        log_msg("[bench] warmup raised to 3 (timing rules)")
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,168 @@
+/*
+ * ffm.h -- C ABI of the B200-native duplicate memory-transfer detector
+ * (the transfer hot path of Diogenes' feed-forward measurement model,
+ * Welton & Miller, SC'19; /root/reference/PAPER.md, cited as P:<line>).
+ *
+ * The operation (Sec. 3.3.2 "Identifying Problematic Memory
+ * Transfers"): every recorded CPU<->GPU transfer payload is content-hashed and
+ * compared with the stored hashes of prior transfers; a match -- confirmed
+ * byte-by-byte here (reading R2) -- marks the transfer a duplicate of
+ * "the first transfer of the duplicated data".  The expected benefit of
+ * removing a duplicate is its transfer call's duration (Fig. 5
+ * RemoveMemoryTransfer), summed per call site
+ * ("single point" grouping).
+ *
+ *   duplicate_of[i] = gid of min{ j < i : size_j == size_i && bytes_j == bytes_i }, or -1
+ *   benefit_ns[s]   = sum_{i : site_i == s, duplicate_of[i] >= 0} duration_ns_i   (mod 2^64)
+ *
+ * Every function returns FFM_OK (0) or a negative ffm_status unless stated.
+ * No C++ exception crosses this boundary.  A handle is externally synchronised
+ * (one thread at a time).  After a CUDA error the handle is poisoned: every
+ * call except ffm_log_destroy / ffm_last_error returns FFM_E_STATE.
+ */
+#ifndef FFM_H
+#define FFM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum ffm_status {
+    FFM_OK = 0,
+    FFM_E_INVAL = -1,   /* NULL handle/argument, bad config, NULL payload with size > 0 */
+    FFM_E_RANGE = -2,   /* call_site >= n_sites; gids not strictly increasing */
+    FFM_E_NOMEM = -3,   /* host or device allocation failed */
+    FFM_E_CUDA  = -4,   /* a CUDA runtime call failed (handle is now poisoned) */
+    FFM_E_COMM  = -5,   /* shard exchange inconsistent (multi-rank) */
+    FFM_E_STATE = -6,   /* poisoned handle, or call out of order */
+    FFM_E_NODEV = -7    /* no CUDA device / driver (there is no CPU fallback) */
+} ffm_status;
+
+/* Opaque, library-owned log handle. */
+typedef struct ffm_log ffm_log;
+
+/* payload_kind for ffm_log_append_batch */
+enum { FFM_PAYLOAD_AUTO = 0, FFM_PAYLOAD_HOST = 1, FFM_PAYLOAD_DEVICE = 2 };
+
+/* ffm_config.flags */
+enum { FFM_FLAG_TIMING = 1u /* record per-stage CUDA events (ffm_last_run_stats) */ };
+
+typedef struct ffm_config {
+    uint32_t n_sites;      /* call_site must be < n_sites.  Sites are caller-interned stack
+                              traces, matched by instruction address. */
+    int32_t  device;       /* CUDA ordinal this log lives on */
+    int32_t  rank, world;  /* shard id / count (P > 1: see ffm_shard_* below); 0, 1 for one GPU */
+    uint64_t arena_bytes;  /* initial HBM payload arena capacity (bytes); grows x2 on demand */
+    uint64_t max_records;  /* initial record capacity hint; grows on demand */
+    uint32_t digest_bits;  /* 64 normally.  < 64 truncates the group-by digest to FORCE
+                              collisions (test / verify-stress knob, BASELINE config 3);
+                              results never change.  0 => group by size alone. */
+    uint32_t refine_bits;  /* 64 normally; < 64 weakens the first collision-resolution
+                              re-key (test knob for the worst-case resolve path). */
+    uint32_t chunk_bytes;  /* large-payload work unit, multiple of 512; 0 => 32768.
+                              Results never change. */
+    uint32_t small_bytes;  /* payloads <= this are hashed/verified one per 8-lane group;
+                              multiple of 128; 0 => 4096.  Results never change. */
+    uint32_t flags;        /* FFM_FLAG_* */
+    uint32_t reserved0;
+    void*    stream;       /* cudaStream_t to run on, or NULL: the log creates its own */
+} ffm_config;
+
+/* Fill *cfg with defaults: n_sites 1, device 0, rank 0, world 1, digest_bits 64,
+   refine_bits 64, everything else 0 / NULL. */
+void ffm_config_init(ffm_config* cfg);
+
+/* Create a log on cfg->device.  *out is owned by the library until ffm_log_destroy.
+   Errors: FFM_E_INVAL (NULL, n_sites == 0, bad chunk/small bytes, digest_bits > 64),
+   FFM_E_NODEV, FFM_E_NOMEM, FFM_E_CUDA. */
+int ffm_log_create(const ffm_config* cfg, ffm_log** out);
+
+/* Append one transfer record (the intercepted call's payload location
+   and size; its call site and time in the driver call).
+   gid = the record's local append index (program order).
+   payload_ptr is BORROWED for the call: the bytes as of this call are snapshotted
+   into HBM before return (reading R11; PAPER.md P:1459-1463 shows bytes may change
+   later), so the caller may reuse the buffer afterwards.  Host (pageable or pinned)
+   or device pointers are accepted (detected with cudaPointerGetAttributes).
+   payload_ptr may be NULL only if size == 0.  A failed append leaves the log
+   unchanged.  Errors: FFM_E_INVAL, FFM_E_RANGE (call_site >= n_sites), FFM_E_NOMEM,
+   FFM_E_CUDA, FFM_E_STATE. */
+int ffm_log_append(ffm_log* log, uint32_t call_site, uint64_t size,
+                   const void* payload_ptr, uint64_t duration_ns);
+
+/* Append n records at once (host arrays of length n).  payloads[i] follows the
+   rules of ffm_log_append; payload_kind says whether they are all HOST, all DEVICE,
+   or AUTO (detected per pointer).  gids may be NULL (local append order) or give
+   each record's GLOBAL gid, strictly increasing across all appends to this log
+   (sharded logs: records of one global program order split over ranks).
+   All-or-nothing: on error the log is unchanged. */
+int ffm_log_append_batch(ffm_log* log, uint64_t n, const uint32_t* call_sites,
+                         const uint64_t* sizes, const void* const* payloads,
+                         const uint64_t* durations_ns, const uint64_t* gids,
+                         int payload_kind);
+
+/* Run the hot path over the whole log (H1 hash, H2 group-by, H3 verify,
+   H4 collision resolve, H5 label, H6 per-site benefit, H7 return):
+     duplicate_of[n_local]  int64  gid of the earliest byte-identical record, or -1
+     benefit_ns[n_sites]    uint64 per-site sum of duplicate durations
+   Either array may be host or device memory (caller-owned; device arrays must be
+   on cfg->device).  benefit_ns may be NULL.  Idempotent: re-running over an
+   unchanged log gives identical outputs; appends after a run are allowed.
+   Synchronous: returns when the outputs are written. */
+int ffm_dedup_run(ffm_log* log, int64_t* duplicate_of, uint64_t* benefit_ns);
+
+/* Number of records appended (local) / payload bytes appended. */
+uint64_t ffm_log_count(const ffm_log* log);
+uint64_t ffm_log_payload_bytes(const ffm_log* log);
+
+/* The cudaStream_t the log runs its kernels on (for CUDA-event timing). */
+void* ffm_log_stream(const ffm_log* log);
+
+typedef struct ffm_run_stats {
+    double   ms_total;          /* CUDA-event time of the last run (FFM_FLAG_TIMING) */
+    double   ms_hash;           /* H1: hash kernels */
+    double   ms_group;          /* H2: table insert + leader lookup */
+    double   ms_verify;         /* H3: verify planning + verify kernels */
+    double   ms_resolve;        /* H4: collision-resolution rounds */
+    double   ms_label;          /* H5+H6: label + benefit */
+    double   ms_output;         /* H7: output copies */
+    double   ms_hash_large;     /* the large-payload hash kernel alone */
+    double   ms_hash_small;     /* the small-payload hash kernel alone */
+    uint64_t n_records;
+    uint64_t payload_bytes;     /* sum of sizes */
+    uint64_t n_members;         /* records whose group candidate is an earlier record */
+    uint64_t n_residual;        /* members that failed byte verification (collisions) */
+    uint64_t resolve_rounds;
+    uint64_t kernel_launches;   /* kernels this library launched in the last run */
+    uint64_t hash_items;        /* large-payload hash work units */
+    uint64_t verify_items;      /* large-payload verify work units */
+} ffm_run_stats;
+
+/* Statistics of the last ffm_dedup_run. */
+int ffm_last_run_stats(const ffm_log* log, ffm_run_stats* out);
+
+/* Debug / conformance: copy the last run's 64-bit payload digests (host array [n]).
+   The digest is specified in DESIGN.md "Digest"; it is an implementation detail
+   and never part of the result. */
+int ffm_debug_digests(ffm_log* log, uint64_t* digests_out);
+
+/* Destroy the log and release its memory.  NULL is a no-op (returns FFM_OK). */
+int ffm_log_destroy(ffm_log* log);
+
+/* Static text for a status code. */
+const char* ffm_strerror(int status);
+
+/* Detail of the last error on this handle (including CUDA error text); "" if none.
+   Valid until the next call on the handle. */
+const char* ffm_last_error(const ffm_log* log);
+
+/* Library build identification, e.g. "ffm 0.1 sm_100a". */
+const char* ffm_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* FFM_H */

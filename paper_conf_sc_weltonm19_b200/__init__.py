@@ -1,0 +1,273 @@
+"""paper_conf_sc_weltonm19_b200 -- B200-native duplicate memory-transfer detection.
+
+Thin ctypes binding over ``libffm.so`` (include/ffm.h).  Argument marshalling
+only: every step of the hot path runs in the library's sm_100a kernels.  There
+is no CPU fallback -- if the CUDA library is missing or no device is present,
+the calls raise.
+
+Raw functions keep the C names (``ffm_log_create``, ``ffm_log_append``,
+``ffm_log_append_batch``, ``ffm_dedup_run``, ...); ``FfmLog`` is a small
+convenience wrapper used by the tests and bench.py.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from ._build import LIB as _LIB_PATH
+
+FFM_OK, FFM_E_INVAL, FFM_E_RANGE, FFM_E_NOMEM, FFM_E_CUDA, FFM_E_COMM, FFM_E_STATE, FFM_E_NODEV = \
+    0, -1, -2, -3, -4, -5, -6, -7
+FFM_PAYLOAD_AUTO, FFM_PAYLOAD_HOST, FFM_PAYLOAD_DEVICE = 0, 1, 2
+FFM_FLAG_TIMING = 1
+
+# every symbol include/ffm.h declares (checked by tests/test_abi.py)
+EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_append_batch",
+           "ffm_dedup_run", "ffm_log_count", "ffm_log_payload_bytes", "ffm_log_stream",
+           "ffm_last_run_stats", "ffm_debug_digests", "ffm_log_destroy", "ffm_strerror",
+           "ffm_last_error", "ffm_version"]
+
+
+class FfmConfig(ctypes.Structure):
+    _fields_ = [("n_sites", ctypes.c_uint32), ("device", ctypes.c_int32), ("rank", ctypes.c_int32),
+                ("world", ctypes.c_int32), ("arena_bytes", ctypes.c_uint64),
+                ("max_records", ctypes.c_uint64), ("digest_bits", ctypes.c_uint32),
+                ("refine_bits", ctypes.c_uint32), ("chunk_bytes", ctypes.c_uint32),
+                ("small_bytes", ctypes.c_uint32), ("flags", ctypes.c_uint32),
+                ("reserved0", ctypes.c_uint32), ("stream", ctypes.c_void_p)]
+
+
+class FfmRunStats(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_double) for k in ("ms_total", "ms_hash", "ms_group", "ms_verify", "ms_resolve",
+                                                 "ms_label", "ms_output", "ms_hash_large", "ms_hash_small")] + \
+               [(k, ctypes.c_uint64) for k in ("n_records", "payload_bytes", "n_members", "n_residual",
+                                                "resolve_rounds", "kernel_launches", "hash_items",
+                                                "verify_items")]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class FfmError(RuntimeError):
+    def __init__(self, code, msg=""):
+        super().__init__(f"{ffm_strerror(code)} ({code}){': ' + msg if msg else ''}")
+        self.code = code
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libffm.so (in-tree).  Raises if it is missing: there is no fallback."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_LIB_PATH):
+            raise ImportError(f"{_LIB_PATH} is missing: run __graft_entry__.build() "
+                              "(the CUDA library is the only implementation)")
+        L = ctypes.CDLL(_LIB_PATH)
+        vp, u64, u32, i32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
+        L.ffm_config_init.argtypes = [ctypes.POINTER(FfmConfig)]
+        L.ffm_config_init.restype = None
+        L.ffm_log_create.argtypes = [ctypes.POINTER(FfmConfig), ctypes.POINTER(vp)]
+        L.ffm_log_create.restype = i32
+        L.ffm_log_append.argtypes = [vp, u32, u64, vp, u64]
+        L.ffm_log_append.restype = i32
+        L.ffm_log_append_batch.argtypes = [vp, u64, vp, vp, vp, vp, vp, i32]
+        L.ffm_log_append_batch.restype = i32
+        L.ffm_dedup_run.argtypes = [vp, vp, vp]
+        L.ffm_dedup_run.restype = i32
+        L.ffm_log_count.argtypes = [vp]
+        L.ffm_log_count.restype = u64
+        L.ffm_log_payload_bytes.argtypes = [vp]
+        L.ffm_log_payload_bytes.restype = u64
+        L.ffm_log_stream.argtypes = [vp]
+        L.ffm_log_stream.restype = vp
+        L.ffm_last_run_stats.argtypes = [vp, ctypes.POINTER(FfmRunStats)]
+        L.ffm_last_run_stats.restype = i32
+        L.ffm_debug_digests.argtypes = [vp, vp]
+        L.ffm_debug_digests.restype = i32
+        L.ffm_log_destroy.argtypes = [vp]
+        L.ffm_log_destroy.restype = i32
+        L.ffm_strerror.argtypes = [i32]
+        L.ffm_strerror.restype = ctypes.c_char_p
+        L.ffm_last_error.argtypes = [vp]
+        L.ffm_last_error.restype = ctypes.c_char_p
+        L.ffm_version.argtypes = []
+        L.ffm_version.restype = ctypes.c_char_p
+        _lib = L
+    return _lib
+
+
+# ---- raw C-named wrappers (argument marshalling only) -----------------------
+def ffm_config_init() -> FfmConfig:
+    c = FfmConfig()
+    lib().ffm_config_init(ctypes.byref(c))
+    return c
+
+
+def ffm_strerror(code: int) -> str:
+    return lib().ffm_strerror(code).decode()
+
+
+def ffm_version() -> str:
+    return lib().ffm_version().decode()
+
+
+def ffm_log_create(cfg: FfmConfig) -> int:
+    h = ctypes.c_void_p()
+    rc = lib().ffm_log_create(ctypes.byref(cfg), ctypes.byref(h))
+    if rc != FFM_OK:
+        raise FfmError(rc)
+    return h.value
+
+
+def ffm_last_error(h) -> str:
+    return lib().ffm_last_error(h).decode()
+
+
+def _check(h, rc):
+    if rc != FFM_OK:
+        raise FfmError(rc, ffm_last_error(h) if h else "")
+
+
+def ffm_log_append(h, call_site: int, size: int, payload_ptr: int, duration_ns: int):
+    _check(h, lib().ffm_log_append(h, call_site, size, payload_ptr, duration_ns))
+
+
+def _addr(a):
+    """Address of a numpy array or torch tensor (host or device)."""
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data
+    if hasattr(a, "data_ptr"):
+        return a.data_ptr()
+    return int(a)
+
+
+def ffm_log_append_batch(h, call_sites, sizes, payload_ptrs, durations_ns, gids=None,
+                         payload_kind: int = FFM_PAYLOAD_AUTO):
+    sites = np.ascontiguousarray(call_sites, dtype=np.uint32)
+    sz = np.ascontiguousarray(sizes, dtype=np.uint64)
+    pp = np.ascontiguousarray(payload_ptrs, dtype=np.uint64)
+    du = np.ascontiguousarray(durations_ns, dtype=np.uint64)
+    g = None if gids is None else np.ascontiguousarray(gids, dtype=np.uint64)
+    n = len(sites)
+    if not (len(sz) == len(pp) == len(du) == n) or (g is not None and len(g) != n):
+        raise ValueError("array lengths differ")
+    _check(h, lib().ffm_log_append_batch(h, n, _addr(sites), _addr(sz), _addr(pp), _addr(du),
+                                         _addr(g), payload_kind))
+
+
+def ffm_dedup_run(h, duplicate_of, benefit_ns):
+    """duplicate_of / benefit_ns: numpy arrays (host) or torch CUDA tensors (device)."""
+    _check(h, lib().ffm_dedup_run(h, _addr(duplicate_of), _addr(benefit_ns)))
+
+
+def ffm_log_count(h) -> int:
+    return int(lib().ffm_log_count(h))
+
+
+def ffm_log_payload_bytes(h) -> int:
+    return int(lib().ffm_log_payload_bytes(h))
+
+
+def ffm_log_stream(h) -> int:
+    return lib().ffm_log_stream(h) or 0
+
+
+def ffm_last_run_stats(h) -> dict:
+    s = FfmRunStats()
+    _check(h, lib().ffm_last_run_stats(h, ctypes.byref(s)))
+    return s.as_dict()
+
+
+def ffm_debug_digests(h) -> np.ndarray:
+    out = np.empty(max(1, ffm_log_count(h)), np.uint64)
+    _check(h, lib().ffm_debug_digests(h, _addr(out)))
+    return out[:ffm_log_count(h)]
+
+
+def ffm_log_destroy(h):
+    _check(None, lib().ffm_log_destroy(h))
+
+
+# ---- convenience wrapper ----------------------------------------------------
+class FfmLog:
+    """Owns one ffm_log handle."""
+
+    def __init__(self, n_sites: int, device: int = 0, *, arena_bytes: int = 0, max_records: int = 0,
+                 digest_bits: int = 64, refine_bits: int = 64, chunk_bytes: int = 0, small_bytes: int = 0,
+                 timing: bool = False, stream: int = 0, rank: int = 0, world: int = 1):
+        cfg = ffm_config_init()
+        cfg.n_sites, cfg.device, cfg.rank, cfg.world = n_sites, device, rank, world
+        cfg.arena_bytes, cfg.max_records = arena_bytes, max_records
+        cfg.digest_bits, cfg.refine_bits = digest_bits, refine_bits
+        cfg.chunk_bytes, cfg.small_bytes = chunk_bytes, small_bytes
+        cfg.flags = FFM_FLAG_TIMING if timing else 0
+        cfg.stream = stream or None
+        self.n_sites = n_sites
+        self.h = ffm_log_create(cfg)
+
+    def append(self, call_site, size, payload_ptr, duration_ns):
+        ffm_log_append(self.h, call_site, size, payload_ptr, duration_ns)
+
+    def append_batch(self, call_sites, sizes, payload_ptrs, durations_ns, gids=None,
+                     payload_kind=FFM_PAYLOAD_AUTO):
+        ffm_log_append_batch(self.h, call_sites, sizes, payload_ptrs, durations_ns, gids, payload_kind)
+
+    def append_log(self, log, ptrs=None, payload_kind=FFM_PAYLOAD_HOST, gids=None, idx=None):
+        """Append a log object with site/size/dur arrays and payload_ptrs() (host payloads by
+        default, or the device addresses `ptrs`)."""
+        p = log.payload_ptrs() if ptrs is None else ptrs
+        if idx is None:
+            self.append_batch(log.site, log.size, p, log.dur, gids, payload_kind)
+        else:
+            self.append_batch(log.site[idx], log.size[idx], np.asarray(p)[idx], log.dur[idx],
+                              gids, payload_kind)
+
+    def run(self, duplicate_of=None, benefit_ns=None):
+        n = self.count
+        if duplicate_of is None:
+            duplicate_of = np.empty(max(n, 1), np.int64)
+        if benefit_ns is None:
+            benefit_ns = np.empty(self.n_sites, np.uint64)
+        ffm_dedup_run(self.h, duplicate_of, benefit_ns)
+        return duplicate_of[:n] if isinstance(duplicate_of, np.ndarray) else duplicate_of, benefit_ns
+
+    @property
+    def count(self):
+        return ffm_log_count(self.h)
+
+    @property
+    def payload_bytes(self):
+        return ffm_log_payload_bytes(self.h)
+
+    @property
+    def stream(self):
+        return ffm_log_stream(self.h)
+
+    def stats(self):
+        return ffm_last_run_stats(self.h)
+
+    def digests(self):
+        return ffm_debug_digests(self.h)
+
+    def close(self):
+        if self.h:
+            ffm_log_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

@@ -1,0 +1,616 @@
+// ffm_api.cu -- the C ABI (include/ffm.h): log management, HBM staging (H0) and the
+// run pipeline (H1..H7).  No C++ exception crosses the boundary; every CUDA error
+// poisons the handle.  There is no CPU fallback: without a device, create fails.
+#include <cuda_runtime.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "ffm_internal.h"
+
+using namespace ffm;
+
+namespace {
+
+constexpr uint64_t kRingBytes = 16ull << 20;      // per half of the pinned staging ring
+constexpr uint64_t kDirectCopy = 4ull << 20;      // host payloads above this bypass the ring
+constexpr uint64_t kGatherMax = 1ull << 20;       // device payloads up to this use k_gather
+
+struct CudaFail {
+    cudaError_t e;
+    const char* what;
+};
+
+inline void ck(cudaError_t e, const char* what) {
+    if (e != cudaSuccess) throw CudaFail{e, what};
+}
+
+inline uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+inline uint64_t pow2_at_least(uint64_t x) {
+    uint64_t p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+
+int fail_cuda(ffm_log* log, const CudaFail& f) {
+    log->poisoned = true;
+    log->last_error = std::string(f.what) + ": " + cudaGetErrorString(f.e);
+    cudaGetLastError();
+    return FFM_E_CUDA;
+}
+
+int set_err(ffm_log* log, int code, const std::string& msg) {
+    if (log) log->last_error = msg;
+    return code;
+}
+
+template <class T>
+void dev_grow(T*& p, uint64_t& cap, uint64_t need, uint64_t keep, cudaStream_t st) {
+    if (need <= cap) return;
+    uint64_t nc = std::max<uint64_t>(need, cap * 2);
+    T* np = nullptr;
+    ck(cudaMalloc(&np, nc * sizeof(T)), "cudaMalloc(metadata)");
+    if (p && keep) ck(cudaMemcpyAsync(np, p, keep * sizeof(T), cudaMemcpyDeviceToDevice, st), "grow copy");
+    ck(cudaStreamSynchronize(st), "grow sync");
+    if (p) ck(cudaFree(p), "cudaFree");
+    p = np;
+    cap = nc;
+}
+
+template <class T>
+void dev_alloc(T*& p, uint64_t count) {
+    if (p) cudaFree(p);
+    p = nullptr;
+    ck(cudaMalloc(&p, std::max<uint64_t>(count, 1) * sizeof(T)), "cudaMalloc(work)");
+}
+
+// ---------------------------------------------------------------- staging (H0)
+void ring_flush(ffm_log* L) {
+    if (!L->ring_fill) return;
+    int c = L->ring_cur;
+    ck(cudaMemcpyAsync(L->arena + L->ring_arena_start, L->ring[c], L->ring_fill, cudaMemcpyHostToDevice,
+                       L->stage_stream),
+       "ring H2D");
+    ck(cudaEventRecord(L->ring_ev[c], L->stage_stream), "ring event");
+    L->ring_cur = c ^ 1;
+    ck(cudaEventSynchronize(L->ring_ev[L->ring_cur]), "ring wait");   // other half free again
+    L->ring_fill = 0;
+}
+
+void ensure_arena(ffm_log* L, uint64_t need) {
+    if (need <= L->arena_cap) return;
+    ring_flush(L);
+    ck(cudaStreamSynchronize(L->stage_stream), "arena sync");
+    ck(cudaStreamSynchronize(L->stream), "arena sync");
+    uint64_t nc = std::max<uint64_t>(need, std::max<uint64_t>(L->arena_cap * 2, 64ull << 20));
+    uint8_t* na = nullptr;
+    if (cudaMalloc(&na, nc) != cudaSuccess) {
+        cudaGetLastError();
+        nc = need;   // retry exact
+        ck(cudaMalloc(&na, nc), "cudaMalloc(arena)");
+    }
+    if (L->arena && L->arena_used)
+        ck(cudaMemcpyAsync(na, L->arena, L->arena_used, cudaMemcpyDeviceToDevice, L->stage_stream), "arena copy");
+    ck(cudaStreamSynchronize(L->stage_stream), "arena copy sync");
+    if (L->arena) ck(cudaFree(L->arena), "cudaFree(arena)");
+    L->arena = na;
+    L->arena_cap = nc;
+}
+
+void stage_host(ffm_log* L, const void* src, uint64_t size, uint64_t off) {
+    if (size > kDirectCopy) {
+        ring_flush(L);
+        ck(cudaMemcpyAsync(L->arena + off, src, size, cudaMemcpyHostToDevice, L->stage_stream), "H2D");
+        ck(cudaStreamSynchronize(L->stage_stream), "H2D sync");   // snapshot before return
+        return;
+    }
+    if (L->ring_fill && (off < L->ring_arena_start || off + size - L->ring_arena_start > L->ring_bytes))
+        ring_flush(L);
+    if (!L->ring_fill) L->ring_arena_start = off;
+    memcpy(L->ring[L->ring_cur] + (off - L->ring_arena_start), src, size);
+    L->ring_fill = off + size - L->ring_arena_start;
+}
+
+bool is_device_ptr(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+void upload_meta(ffm_log* L) {
+    uint64_t n = L->h_size.size();
+    if (L->d_meta_n == n) return;
+    uint64_t c0 = L->d_meta_cap, keep = L->d_meta_n;
+    uint64_t cap = c0;
+    dev_grow(L->d_off, cap, n, keep, L->stage_stream);
+    cap = c0;
+    dev_grow(L->d_size, cap, n, keep, L->stage_stream);
+    cap = c0;
+    dev_grow(L->d_site, cap, n, keep, L->stage_stream);
+    cap = c0;
+    dev_grow(L->d_dur, cap, n, keep, L->stage_stream);
+    cap = c0;
+    dev_grow(L->d_gid, cap, n, keep, L->stage_stream);
+    L->d_meta_cap = cap;
+    uint64_t a = L->d_meta_n, k = n - a;
+    cudaStream_t s = L->stage_stream;
+    ck(cudaMemcpyAsync(L->d_off + a, L->h_off.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
+    ck(cudaMemcpyAsync(L->d_size + a, L->h_size.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
+    ck(cudaMemcpyAsync(L->d_site + a, L->h_site.data() + a, k * 4, cudaMemcpyHostToDevice, s), "meta H2D");
+    ck(cudaMemcpyAsync(L->d_dur + a, L->h_dur.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
+    ck(cudaMemcpyAsync(L->d_gid + a, L->h_gid.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
+    ck(cudaStreamSynchronize(s), "meta sync");
+    L->d_meta_n = n;
+}
+
+uint64_t large_chunks(const ffm_log* L, uint64_t size) {
+    uint64_t cb = L->params.chunk_bytes;
+    return size > L->params.small_bytes ? (size + cb - 1) / cb : 0;
+}
+
+int check_state(ffm_log* L) {
+    if (!L) return FFM_E_INVAL;
+    if (L->poisoned) return FFM_E_STATE;
+    return FFM_OK;
+}
+
+// Validate + assign arena offsets for a batch; returns FFM_OK or an error without
+// touching the log.
+int plan_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes, const void* const* payloads,
+               const uint64_t* gids, std::vector<uint64_t>& offs, uint64_t& arena_end) {
+    uint64_t cur = L->arena_used;
+    uint64_t last = L->last_gid;
+    bool any = L->any_gid || !L->h_gid.empty();
+    uint64_t base_n = L->h_size.size();
+    if (base_n + n >= 0xFFFFFFFFull) return set_err(L, FFM_E_RANGE, "too many records for one log (2^32-1)");
+    offs.resize(n);
+    for (uint64_t i = 0; i < n; ++i) {
+        if (sites[i] >= L->cfg.n_sites) return set_err(L, FFM_E_RANGE, "call_site >= n_sites");
+        if (sizes[i] > 0 && payloads[i] == nullptr) return set_err(L, FFM_E_INVAL, "NULL payload with size > 0");
+        uint64_t g = gids ? gids[i] : (any ? last + 1 : 0);
+        if (gids && any && g <= last) return set_err(L, FFM_E_RANGE, "gids must be strictly increasing");
+        last = g;
+        any = true;
+        cur = align_up(cur, kArenaAlign);
+        offs[i] = cur;
+        cur += sizes[i];
+    }
+    arena_end = cur;
+    return FFM_OK;
+}
+
+void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes, const uint64_t* durs,
+               const uint64_t* gids, const std::vector<uint64_t>& offs, uint64_t arena_end) {
+    bool any = !L->h_gid.empty();
+    for (uint64_t i = 0; i < n; ++i) {
+        L->h_site.push_back(sites[i]);
+        L->h_size.push_back(sizes[i]);
+        L->h_off.push_back(offs[i]);
+        L->h_dur.push_back(durs[i]);
+        uint64_t g = gids ? gids[i] : (any ? L->last_gid + 1 : 0);
+        L->h_gid.push_back(g);
+        L->last_gid = g;
+        any = true;
+        L->payload_bytes += sizes[i];
+        L->n_large_chunks += large_chunks(L, sizes[i]);
+    }
+    if (gids) L->any_gid = true;
+    L->arena_used = arena_end;
+}
+
+// ---------------------------------------------------------------- work buffers
+void ensure_work(ffm_log* L, uint64_t n) {
+    Work& W = L->work;
+    uint64_t tcap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
+    if (n > W.n_cap || W.accA == nullptr) {
+        uint64_t c = std::max<uint64_t>(n, 1024);
+        dev_alloc(W.accA, c);
+        dev_alloc(W.accB, c);
+        dev_alloc(W.key, c);
+        dev_alloc(W.digest, c);
+        dev_alloc(W.slot, c);
+        dev_alloc(W.leader, c);
+        dev_alloc(W.eq, c);
+        dev_alloc(W.mis, c);
+        dev_alloc(W.res[0], c);
+        dev_alloc(W.res[1], c);
+        dev_alloc(W.lcount, c + 1);
+        dev_alloc(W.lstart, c + 1);
+        dev_alloc(W.hcount, c + 1);
+        dev_alloc(W.hstart, c + 1);
+        dev_alloc(W.dup, c);
+        if (!W.counters) dev_alloc(W.counters, 16);
+        size_t cb = cub_scan_bytes(c + 1);
+        if (W.cub_tmp) cudaFree(W.cub_tmp);
+        W.cub_tmp = nullptr;
+        ck(cudaMalloc(&W.cub_tmp, std::max<size_t>(cb, 256)), "cudaMalloc(cub)");
+        W.cub_tmp_bytes = std::max<size_t>(cb, 256);
+        W.n_cap = c;
+    }
+    if (tcap > W.t_cap) {
+        dev_alloc(W.tkey, tcap);
+        dev_alloc(W.tval, tcap);
+        W.t_cap = tcap;
+    }
+    if (L->n_large_chunks > W.hitem_cap) {
+        uint64_t c = L->n_large_chunks + L->n_large_chunks / 4 + 64;
+        dev_alloc(W.hitems, c);
+        dev_alloc(W.vitems, c);
+        dev_alloc(W.hpart, 2 * c);
+        W.hitem_cap = W.vitem_cap = c;
+    }
+    if (L->cfg.n_sites > W.site_cap) {
+        dev_alloc(W.ben, L->cfg.n_sites);
+        W.site_cap = L->cfg.n_sites;
+    }
+}
+
+DevLog dev_view(const ffm_log* L) {
+    DevLog d;
+    d.arena = L->arena;
+    d.off = L->d_off;
+    d.size = L->d_size;
+    d.site = L->d_site;
+    d.dur = L->d_dur;
+    d.gid = L->d_gid;
+    d.n = (uint32_t)L->h_size.size();
+    return d;
+}
+
+float ev_ms(cudaEvent_t a, cudaEvent_t b) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) {
+        cudaGetLastError();
+        return 0.f;
+    }
+    return ms;
+}
+
+#define LCHK(x)                                                                \
+    do {                                                                       \
+        int _k = (x);                                                          \
+        if (_k < 0) throw CudaFail{cudaGetLastError(), "kernel launch " #x};   \
+        launches += (uint64_t)_k;                                              \
+    } while (0)
+
+}  // namespace
+
+// ======================================================================== ABI
+extern "C" {
+
+void ffm_config_init(ffm_config* cfg) {
+    if (!cfg) return;
+    memset(cfg, 0, sizeof(*cfg));
+    cfg->n_sites = 1;
+    cfg->world = 1;
+    cfg->digest_bits = 64;
+    cfg->refine_bits = 64;
+}
+
+const char* ffm_version(void) { return "ffm 0.1 sm_100a"; }
+
+const char* ffm_strerror(int s) {
+    switch (s) {
+        case FFM_OK: return "ok";
+        case FFM_E_INVAL: return "invalid argument";
+        case FFM_E_RANGE: return "argument out of range";
+        case FFM_E_NOMEM: return "out of memory";
+        case FFM_E_CUDA: return "CUDA error";
+        case FFM_E_COMM: return "shard exchange error";
+        case FFM_E_STATE: return "invalid state (poisoned handle)";
+        case FFM_E_NODEV: return "no CUDA device";
+        default: return "unknown status";
+    }
+}
+
+const char* ffm_last_error(const ffm_log* log) { return log ? log->last_error.c_str() : ""; }
+
+int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
+    if (!cfg || !out) return FFM_E_INVAL;
+    *out = nullptr;
+    if (cfg->n_sites == 0 || cfg->digest_bits > 64 || cfg->refine_bits > 64 || cfg->world < 1 ||
+        cfg->rank < 0 || cfg->rank >= cfg->world)
+        return FFM_E_INVAL;
+    uint32_t chunk = cfg->chunk_bytes ? cfg->chunk_bytes : 32768;
+    uint32_t small = cfg->small_bytes ? cfg->small_bytes : 4096;
+    if (chunk % 1024 || small % 128 || chunk == 0) return FFM_E_INVAL;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return FFM_E_NODEV;
+    }
+    if (cfg->device < 0 || cfg->device >= ndev) return FFM_E_INVAL;
+    ffm_log* L = new (std::nothrow) ffm_log();
+    if (!L) return FFM_E_NOMEM;
+    L->cfg = *cfg;
+    L->device = cfg->device;
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        int prop_major = 0;
+        ck(cudaDeviceGetAttribute(&prop_major, cudaDevAttrComputeCapabilityMajor, L->device), "attr");
+        if (prop_major < 10) {
+            delete L;
+            return FFM_E_NODEV;   // built for sm_100a only
+        }
+        ck(cudaDeviceGetAttribute(&L->params.num_sms, cudaDevAttrMultiProcessorCount, L->device), "attr");
+        L->params.chunk_bytes = chunk;
+        L->params.small_bytes = small;
+        L->params.digest_mask = cfg->digest_bits >= 64 ? ~0ull : ((1ull << cfg->digest_bits) - 1);
+        L->params.refine_mask = cfg->refine_bits >= 64 ? ~0ull : ((1ull << cfg->refine_bits) - 1);
+        if (cfg->stream) {
+            L->stream = (cudaStream_t)cfg->stream;
+        } else {
+            ck(cudaStreamCreateWithFlags(&L->stream, cudaStreamNonBlocking), "stream");
+            L->own_stream = true;
+        }
+        ck(cudaStreamCreateWithFlags(&L->stage_stream, cudaStreamNonBlocking), "stream");
+        L->ring_bytes = kRingBytes;
+        for (int i = 0; i < 2; ++i) {
+            ck(cudaHostAlloc((void**)&L->ring[i], kRingBytes, cudaHostAllocDefault), "cudaHostAlloc(ring)");
+            ck(cudaEventCreateWithFlags(&L->ring_ev[i], cudaEventDisableTiming), "event");
+            ck(cudaEventRecord(L->ring_ev[i], L->stage_stream), "event");
+        }
+        for (auto& e : L->ev) ck(cudaEventCreate(&e), "event");
+        ck(cudaHostAlloc((void**)&L->h_counters, 16 * sizeof(uint32_t), cudaHostAllocDefault), "cudaHostAlloc");
+        if (cfg->arena_bytes) ensure_arena(L, cfg->arena_bytes);
+        if (cfg->max_records) {
+            L->h_site.reserve(cfg->max_records);
+            L->h_size.reserve(cfg->max_records);
+            L->h_off.reserve(cfg->max_records);
+            L->h_dur.reserve(cfg->max_records);
+            L->h_gid.reserve(cfg->max_records);
+        }
+    } catch (const CudaFail& f) {
+        int code = (f.e == cudaErrorMemoryAllocation) ? FFM_E_NOMEM : FFM_E_CUDA;
+        cudaGetLastError();
+        ffm_log_destroy(L);
+        return code;
+    } catch (const std::bad_alloc&) {
+        ffm_log_destroy(L);
+        return FFM_E_NOMEM;
+    }
+    *out = L;
+    return FFM_OK;
+}
+
+int ffm_log_append_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes,
+                         const void* const* payloads, const uint64_t* durs, const uint64_t* gids, int kind) {
+    int st = check_state(L);
+    if (st) return st;
+    if (n == 0) return FFM_OK;
+    if (!sites || !sizes || !payloads || !durs) return set_err(L, FFM_E_INVAL, "NULL array");
+    if (kind < FFM_PAYLOAD_AUTO || kind > FFM_PAYLOAD_DEVICE) return set_err(L, FFM_E_INVAL, "bad payload_kind");
+    std::vector<uint64_t> offs;
+    uint64_t end = 0;
+    int rc = plan_batch(L, n, sites, sizes, payloads, gids, offs, end);
+    if (rc) return rc;
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        ensure_arena(L, end);
+        std::vector<uint64_t> desc;
+        bool any_device = false;
+        for (uint64_t i = 0; i < n; ++i) {
+            if (sizes[i] == 0) continue;
+            bool dev = kind == FFM_PAYLOAD_DEVICE || (kind == FFM_PAYLOAD_AUTO && is_device_ptr(payloads[i]));
+            // the ring uploads one contiguous arena range: close it before a record that
+            // is written into the arena by another path
+            if (dev && L->ring_fill) ring_flush(L);
+            if (!dev) {
+                stage_host(L, payloads[i], sizes[i], offs[i]);
+            } else if (sizes[i] > kGatherMax) {
+                any_device = true;
+                ck(cudaMemcpyAsync(L->arena + offs[i], payloads[i], sizes[i], cudaMemcpyDeviceToDevice,
+                                   L->stage_stream),
+                   "D2D");
+            } else {
+                any_device = true;
+                desc.push_back((uint64_t)(uintptr_t)payloads[i]);
+                desc.push_back(offs[i]);
+                desc.push_back(sizes[i]);
+            }
+        }
+        if (!desc.empty()) {
+            uint64_t nd = desc.size() / 3;
+            uint64_t cap = L->desc_cap;
+            if (desc.size() > cap) {
+                if (L->d_desc) ck(cudaFree(L->d_desc), "cudaFree");
+                L->d_desc = nullptr;
+                cap = std::max<uint64_t>(desc.size(), 2 * cap);
+                ck(cudaMalloc(&L->d_desc, cap * sizeof(uint64_t)), "cudaMalloc(desc)");
+                L->desc_cap = cap;
+            }
+            ck(cudaMemcpyAsync(L->d_desc, desc.data(), desc.size() * 8, cudaMemcpyHostToDevice, L->stage_stream),
+               "desc H2D");
+            if (launch_gather(L->d_desc, (uint32_t)nd, L->arena, L->stage_stream) < 0)
+                throw CudaFail{cudaGetLastError(), "k_gather"};
+        }
+        if (any_device) ck(cudaStreamSynchronize(L->stage_stream), "D2D sync");   // snapshot before return
+        push_meta(L, n, sites, sizes, durs, gids, offs, end);
+        L->digests_valid = false;
+        if (n > 1) upload_meta(L);
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    } catch (const std::bad_alloc&) {
+        return set_err(L, FFM_E_NOMEM, "host allocation failed");
+    }
+    return FFM_OK;
+}
+
+int ffm_log_append(ffm_log* L, uint32_t site, uint64_t size, const void* payload, uint64_t dur) {
+    const void* p[1] = {payload};
+    return ffm_log_append_batch(L, 1, &site, &size, p, &dur, nullptr, FFM_PAYLOAD_AUTO);
+}
+
+uint64_t ffm_log_count(const ffm_log* L) { return L ? (uint64_t)L->h_size.size() : 0; }
+uint64_t ffm_log_payload_bytes(const ffm_log* L) { return L ? L->payload_bytes : 0; }
+void* ffm_log_stream(const ffm_log* L) { return L ? (void*)L->stream : nullptr; }
+
+int ffm_last_run_stats(const ffm_log* L, ffm_run_stats* out) {
+    if (!L || !out) return FFM_E_INVAL;
+    *out = L->stats;
+    return FFM_OK;
+}
+
+int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
+    int st = check_state(L);
+    if (st) return st;
+    uint64_t n = L->h_size.size();
+    if (n > 0 && !dup_out) return set_err(L, FFM_E_INVAL, "duplicate_of is NULL");
+    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
+    uint64_t launches = 0;
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        // H0 tail: flush staged payloads and metadata, order the run after them
+        ring_flush(L);
+        upload_meta(L);
+        ck(cudaEventRecord(L->ring_ev[L->ring_cur], L->stage_stream), "event");
+        ck(cudaStreamWaitEvent(L->stream, L->ring_ev[L->ring_cur], 0), "wait staging");
+        ensure_work(L, n);
+        Work& W = L->work;
+        cudaStream_t s = L->stream;
+        DevLog D = dev_view(L);
+        const uint32_t ns = L->cfg.n_sites;
+        bool dup_dev = dup_out && is_device_ptr(dup_out);
+        bool ben_dev = ben_out && is_device_ptr(ben_out);
+        int64_t* d_dup = dup_dev ? dup_out : W.dup;
+        uint64_t* d_ben = ben_dev ? ben_out : W.ben;
+
+        if (timing) ck(cudaEventRecord(L->ev[0], s), "event");
+        if (launch_zero_counters(W, s) < 0) throw CudaFail{cudaGetLastError(), "zero counters"};
+        // H1 hash
+        LCHK(launch_hash_small(D, W, L->params, s));
+        if (timing) ck(cudaEventRecord(L->ev[8], s), "event");
+        if (L->n_large_chunks) {
+            LCHK(launch_hash_plan(D, W, L->params, s));
+            if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
+            LCHK(launch_hash_large(D, W, L->params, L->n_large_chunks, s));
+            if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
+            LCHK(launch_hash_combine(D, W, L->params, s));
+        }
+        if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
+        // H2 group-by (round 0, all records)
+        uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
+        LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, s));
+        if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
+        // H3 verify
+        LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], L->n_large_chunks ? W.vitem_cap : 0, s));
+        if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
+        // H5 + H6 label and benefit
+        LCHK(launch_label(D, W, ns, d_dup, d_ben, s));
+        if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
+        ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+        ck(cudaStreamSynchronize(s), "run sync");
+        uint64_t n_members = L->h_counters[1];
+        uint64_t nres = L->h_counters[0];
+        uint64_t n_res_total = nres;
+        uint64_t rounds = 0;
+        if (nres) {
+            // H4 collision resolution: exact classes among the residual members
+            if (timing) ck(cudaEventRecord(L->ev[6], s), "event");
+            int cur = 0;
+            while (nres) {
+                ++rounds;
+                if (rounds > n + 2) throw CudaFail{cudaErrorUnknown, "collision resolution did not converge"};
+                ck(cudaMemsetAsync(W.counters, 0, sizeof(uint32_t), s), "memset");
+                uint64_t capr = std::max<uint64_t>(1024, pow2_at_least(2 * nres));
+                LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)rounds, s));
+                LCHK(launch_verify(D, W, L->params, W.res[cur], (uint32_t)nres, W.res[cur ^ 1],
+                                   L->n_large_chunks ? W.vitem_cap : 0, s));
+                ck(cudaMemcpyAsync(L->h_counters, W.counters, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+                ck(cudaStreamSynchronize(s), "round sync");
+                nres = L->h_counters[0];
+                n_res_total += nres;
+                cur ^= 1;
+            }
+            LCHK(launch_label(D, W, ns, d_dup, d_ben, s));
+            if (timing) ck(cudaEventRecord(L->ev[7], s), "event");
+        }
+        // H7 return
+        if (timing) ck(cudaEventRecord(L->ev[9], s), "event");
+        if (!dup_dev && n)
+            ck(cudaMemcpyAsync(dup_out, d_dup, n * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
+        if (ben_out && !ben_dev)
+            ck(cudaMemcpyAsync(ben_out, d_ben, ns * sizeof(uint64_t), cudaMemcpyDeviceToHost, s), "D2H ben");
+        if (timing) ck(cudaEventRecord(L->ev[5], s), "event");
+        ck(cudaStreamSynchronize(s), "output sync");
+        ck(cudaGetLastError(), "run");
+
+        ffm_run_stats& S = L->stats;
+        memset(&S, 0, sizeof(S));
+        S.n_records = n;
+        S.payload_bytes = L->payload_bytes;
+        S.n_members = n_members;
+        S.n_residual = n_res_total;
+        S.resolve_rounds = rounds;
+        S.kernel_launches = launches;
+        S.hash_items = L->n_large_chunks;
+        if (timing) {
+            S.ms_hash_small = ev_ms(L->ev[0], L->ev[8]);
+            S.ms_hash_large = L->n_large_chunks ? ev_ms(L->ev[10], L->ev[11]) : 0.0;
+            S.ms_hash = ev_ms(L->ev[0], L->ev[1]);
+            S.ms_group = ev_ms(L->ev[1], L->ev[2]);
+            S.ms_verify = ev_ms(L->ev[2], L->ev[3]);
+            S.ms_label = ev_ms(L->ev[3], L->ev[4]);
+            S.ms_resolve = rounds ? ev_ms(L->ev[6], L->ev[7]) : 0.0;
+            S.ms_output = ev_ms(L->ev[9], L->ev[5]);
+            S.ms_total = ev_ms(L->ev[0], L->ev[5]);
+        }
+        L->digests_valid = true;
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    } catch (const std::bad_alloc&) {
+        return set_err(L, FFM_E_NOMEM, "host allocation failed");
+    }
+    return FFM_OK;
+}
+
+int ffm_debug_digests(ffm_log* L, uint64_t* out) {
+    int st = check_state(L);
+    if (st) return st;
+    if (!out) return FFM_E_INVAL;
+    if (!L->digests_valid) return set_err(L, FFM_E_STATE, "no run since the last append");
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        uint64_t n = L->h_size.size();
+        if (n) ck(cudaMemcpy(out, L->work.digest, n * 8, cudaMemcpyDeviceToHost), "D2H digests");
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    }
+    return FFM_OK;
+}
+
+int ffm_log_destroy(ffm_log* L) {
+    if (!L) return FFM_OK;
+    cudaSetDevice(L->device);
+    if (L->stream) cudaStreamSynchronize(L->stream);
+    if (L->stage_stream) cudaStreamSynchronize(L->stage_stream);
+    Work& W = L->work;
+    void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
+                    W.lcount, W.lstart, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
+                    W.dup, W.ben, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid,
+                    L->arena, L->d_desc};
+    for (void* p : ptrs)
+        if (p) cudaFree(p);
+    for (int i = 0; i < 2; ++i) {
+        if (L->ring[i]) cudaFreeHost(L->ring[i]);
+        if (L->ring_ev[i]) cudaEventDestroy(L->ring_ev[i]);
+    }
+    for (auto e : L->ev)
+        if (e) cudaEventDestroy(e);
+    if (L->h_counters) cudaFreeHost(L->h_counters);
+    if (L->stage_stream) cudaStreamDestroy(L->stage_stream);
+    if (L->own_stream && L->stream) cudaStreamDestroy(L->stream);
+    cudaGetLastError();
+    delete L;
+    return FFM_OK;
+}
+
+}  // extern "C"

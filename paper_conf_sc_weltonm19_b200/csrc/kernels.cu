@@ -1,0 +1,733 @@
+// kernels.cu -- sm_100a kernels of the duplicate-transfer hot path.
+//
+// Steps:
+//   H1 hash    k_hash_small / k_hash_large   ("the data being transferred is hashed")
+//   H2 group   k_group_insert / k_leader     ("compared to the stored hashes from prior transfers")
+//   H3 verify  k_verify_small / k_verify_large (reading R2: every hash match is byte-verified)
+//   H4 resolve k_refine + H2/H3 over the residuals (exact classes under digest collisions)
+//   H5/H6      k_label  ("marks the transfer as being a duplicate ... the location of the
+//              first transfer"; Fig. 5 P:956-960 benefit = duration; P:1021-1026 per call site)
+//
+// All of it is integer, HBM-bound streaming: 256-bit non-coalescing-free loads
+// (LDG.256, sm_100), per-lane NH multiply-accumulate, warp / 8-lane shuffles.
+// No tensor cores: there is no dense contraction on this path.
+#include <cub/cub.cuh>
+
+#include "ffm_internal.h"
+
+namespace ffm {
+
+// ----------------------------------------------------------------------------
+// Digest.  16-byte words W[q], q < ceil(n/16), zero-padded;
+// four little-endian u32 lanes w0..w3.  Position g = q mod 16, stripe s = q div 16.
+// k_j = KA[g][j] + s * DA[j]  (mod 2^32), j = 0..5
+// A = sum (w0+k0)(w1+k1) + (w2+k2)(w3+k3)   B = sum (w0+k2)(w1+k3) + (w2+k4)(w3+k5)   (mod 2^64)
+// digest = fmix64(A ^ fmix64(B ^ n * 0x9E3779B97F4A7C15))
+// The per-stripe key steps DA are compile-time constants (immediate operands), so a
+// lane keeps only its 12 current keys in registers.
+// ----------------------------------------------------------------------------
+struct NHKeys {
+    uint32_t ka[16][6];
+};
+
+constexpr uint64_t sm64(uint64_t x) {
+    x += 0x9E3779B97F4A7C15ull;
+    x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+    x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+    return x ^ (x >> 31);
+}
+
+constexpr NHKeys make_nh_keys() {
+    NHKeys k{};
+    uint64_t s = 0xD10E5E5FF1ull;
+    for (int g = 0; g < 16; ++g)
+        for (int j = 0; j < 6; ++j) k.ka[g][j] = (uint32_t)(sm64(s++) >> 16);
+    return k;
+}
+
+// per-stripe key increments (odd => full period mod 2^32)
+__host__ __device__ constexpr uint32_t kDA(int j) {
+    return j == 0 ? 0x9E3779B9u : j == 1 ? 0x7F4A7C15u : j == 2 ? 0xF39CC061u
+         : j == 3 ? 0x5CEDC835u : j == 4 ? 0x1B873593u : 0xCC9E2D51u;
+}
+
+__constant__ NHKeys c_nh = make_nh_keys();
+
+__host__ __device__ __forceinline__ uint64_t fmix64(uint64_t k) {
+    k ^= k >> 33;
+    k *= 0xff51afd7ed558ccdull;
+    k ^= k >> 33;
+    k *= 0xc4ceb9fe1a85ec53ull;
+    k ^= k >> 33;
+    return k;
+}
+
+__device__ __forceinline__ uint64_t finalize_digest(uint64_t A, uint64_t B, uint64_t n) {
+    return fmix64(A ^ fmix64(B ^ (n * 0x9E3779B97F4A7C15ull)));
+}
+
+__device__ __forceinline__ uint64_t not_empty(uint64_t k) { return k == kEmptyKey ? k - 1 : k; }
+
+__device__ __forceinline__ uint64_t group_key(uint64_t digest, uint64_t n, uint64_t mask) {
+    return not_empty(fmix64((digest & mask) ^ fmix64(n + 0x632BE59BD9B4E019ull)));
+}
+
+// 32-byte block = two 16-byte words.
+struct Blk {
+    uint32_t v[8];
+};
+
+// Streamed payload bytes: read once, do not pollute L1, evict first from L2.
+__device__ __forceinline__ Blk ld_stream(const uint8_t* p) {
+    Blk r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::evict_first.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.v[0]), "=r"(r.v[1]), "=r"(r.v[2]), "=r"(r.v[3]), "=r"(r.v[4]), "=r"(r.v[5]),
+                   "=r"(r.v[6]), "=r"(r.v[7])
+                 : "l"(p));
+    return r;
+}
+
+// Leader bytes during verify: re-read by every member of the class -> keep in L2.
+__device__ __forceinline__ Blk ld_keep(const uint8_t* p) {
+    Blk r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::evict_last.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.v[0]), "=r"(r.v[1]), "=r"(r.v[2]), "=r"(r.v[3]), "=r"(r.v[4]), "=r"(r.v[5]),
+                   "=r"(r.v[6]), "=r"(r.v[7])
+                 : "l"(p));
+    return r;
+}
+
+__device__ __forceinline__ Blk zero_blk() {
+    Blk r;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) r.v[i] = 0;
+    return r;
+}
+
+// Zero the bytes of block b at or beyond n (only the record's last block is partial).
+__device__ __forceinline__ void mask_tail(Blk& x, uint64_t n, uint64_t b) {
+    int64_t valid = (int64_t)n - (int64_t)(32 * b);
+    if (valid >= 32) return;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+        int64_t vb = valid - 4 * i;
+        uint32_t m = vb >= 4 ? 0xFFFFFFFFu : (vb <= 0 ? 0u : ((1u << (8 * vb)) - 1u));
+        x.v[i] &= m;
+    }
+}
+
+struct LaneKeys {
+    uint32_t k[2][6];
+};
+
+// Keys of positions p0, p0+1 at stripe s.
+__device__ __forceinline__ void load_keys(LaneKeys& K, int p0, uint32_t s) {
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int j = 0; j < 6; ++j) K.k[h][j] = c_nh.ka[p0 + h][j] + s * kDA(j);
+}
+
+// Advance MULT stripes (immediate-operand adds).
+template <uint32_t MULT>
+__device__ __forceinline__ void advance(LaneKeys& K) {
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int j = 0; j < 6; ++j) K.k[h][j] += kDA(j) * MULT;
+}
+
+__device__ __forceinline__ void nh_word(uint32_t w0, uint32_t w1, uint32_t w2, uint32_t w3, const uint32_t* k,
+                                        uint64_t& A, uint64_t& B) {
+    A += (uint64_t)(w0 + k[0]) * (uint64_t)(w1 + k[1]);
+    A += (uint64_t)(w2 + k[2]) * (uint64_t)(w3 + k[3]);
+    B += (uint64_t)(w0 + k[2]) * (uint64_t)(w1 + k[3]);
+    B += (uint64_t)(w2 + k[4]) * (uint64_t)(w3 + k[5]);
+}
+
+// NH of block b (words 2b, 2b+1) of a record of n bytes; the second word only if it
+// exists (16*(2b+1) < n).
+__device__ __forceinline__ void nh_blk(const Blk& x, const LaneKeys& K, uint64_t n, uint64_t b, uint64_t& A,
+                                       uint64_t& B) {
+    nh_word(x.v[0], x.v[1], x.v[2], x.v[3], K.k[0], A, B);
+    if (32 * b + 16 < n) nh_word(x.v[4], x.v[5], x.v[6], x.v[7], K.k[1], A, B);
+}
+
+// ----------------------------------------------------------------------------
+// H1a: payloads <= small_bytes, one 8-lane group ("octet") per record.  Lane g
+// reads 32-B block g of each 256-B stripe: positions 2g, 2g+1.
+// ----------------------------------------------------------------------------
+constexpr int kSmallU = 4;
+
+__global__ void __launch_bounds__(256, 3) k_hash_small(DevLog L, uint32_t small_bytes, uint64_t* __restrict__ accA,
+                                                    uint64_t* __restrict__ accB) {
+    const int g = threadIdx.x & 7;
+    const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
+    const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
+    const unsigned omask = 0xFFu << (threadIdx.x & 24);
+    LaneKeys K0;
+    load_keys(K0, 2 * g, 0);
+    for (uint32_t r = oct; r < L.n; r += noct) {
+        const uint64_t n = L.size[r];
+        if (n > small_bytes) continue;
+        const uint8_t* base = L.arena + L.off[r];
+        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
+        LaneKeys K = K0;
+        uint64_t A = 0, B = 0;
+        for (uint32_t b0 = 0; b0 < nblk; b0 += 8 * kSmallU) {
+            Blk x[kSmallU];
+#pragma unroll
+            for (int u = 0; u < kSmallU; ++u) {
+                uint32_t b = b0 + 8 * u + g;
+                x[u] = b < nblk ? ld_stream(base + 32ull * b) : zero_blk();
+            }
+#pragma unroll
+            for (int u = 0; u < kSmallU; ++u) {
+                uint32_t b = b0 + 8 * u + g;
+                if (b < nblk) {
+                    mask_tail(x[u], n, b);
+                    nh_blk(x[u], K, n, b, A, B);
+                }
+                advance<1>(K);
+            }
+        }
+#pragma unroll
+        for (int o = 4; o; o >>= 1) {
+            A += __shfl_xor_sync(omask, A, o);
+            B += __shfl_xor_sync(omask, B, o);
+        }
+        if (g == 0) {
+            accA[r] = A;
+            accB[r] = B;
+        }
+    }
+}
+
+// ----------------------------------------------------------------------------
+// H1b: payloads > small_bytes, one warp per (record, chunk) work unit.  Lane l
+// reads block b0 + l + 32t: positions 2(l mod 8), stripe (b0 + l)/8 + 4t.
+// Each unit writes its partial (A, B); k_hash_combine sums them per record.
+// ----------------------------------------------------------------------------
+constexpr int kLargeU = 4;
+
+__global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __restrict__ items,
+                                                    const uint32_t* __restrict__ n_items_ptr, uint32_t chunk_bytes,
+                                                    uint64_t* __restrict__ part) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    const uint32_t n_items = *n_items_ptr;
+    const uint32_t cblk = chunk_bytes >> 5;
+    for (uint32_t it = warp; it < n_items; it += nwarps) {
+        const uint2 w = items[it];
+        const uint32_t r = w.x;
+        const uint64_t n = L.size[r];
+        const uint8_t* base = L.arena + L.off[r];
+        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
+        const uint32_t bb = w.y * cblk;
+        const uint32_t be = min(bb + cblk, nblk);
+        LaneKeys K;
+        load_keys(K, 2 * (lane & 7), (uint32_t)((bb + lane) >> 3));
+        uint64_t A = 0, B = 0;
+        for (uint32_t b0 = bb; b0 < be; b0 += 32 * kLargeU) {
+            Blk x[kLargeU];
+#pragma unroll
+            for (int u = 0; u < kLargeU; ++u) {
+                uint32_t b = b0 + 32 * u + lane;
+                x[u] = b < be ? ld_stream(base + 32ull * b) : zero_blk();
+            }
+#pragma unroll
+            for (int u = 0; u < kLargeU; ++u) {
+                uint32_t b = b0 + 32 * u + lane;
+                if (b < be) {
+                    mask_tail(x[u], n, b);
+                    nh_blk(x[u], K, n, b, A, B);
+                }
+                advance<4>(K);
+            }
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
+            B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
+        }
+        if (lane == 0) {
+            part[2ull * it] = A;
+            part[2ull * it + 1] = B;
+        }
+    }
+}
+
+// Combine the chunk partial sums of multi-chunk records (NH is a plain sum, so the
+// record's accumulators are the sums of its chunks' -- no atomics, deterministic).
+__global__ void k_hash_combine(DevLog L, uint32_t small_bytes, const uint32_t* __restrict__ start,
+                               const uint64_t* __restrict__ part, uint64_t* __restrict__ accA,
+                               uint64_t* __restrict__ accB) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (r >= L.n) return;
+    if (L.size[r] <= small_bytes) return;
+    const uint32_t s = start[r], e = start[r + 1];
+    uint64_t A = 0, B = 0;
+    for (uint32_t it = s + lane; it < e; it += 32) {
+        A += part[2ull * it];
+        B += part[2ull * it + 1];
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
+        B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
+    }
+    if (lane == 0) {
+        accA[r] = A;
+        accB[r] = B;
+    }
+}
+
+// Work-unit planning for H1b / H3b: counts -> exclusive scan -> scatter.
+__global__ void k_hash_count(DevLog L, uint32_t small_bytes, uint32_t chunk_bytes, uint32_t* __restrict__ cnt) {
+    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r > L.n) return;
+    uint32_t c = 0;
+    if (r < L.n) {
+        uint64_t n = L.size[r];
+        if (n > small_bytes) c = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
+    }
+    cnt[r] = c;
+}
+
+__global__ void k_hash_fill(DevLog L, uint32_t small_bytes, uint32_t chunk_bytes, const uint32_t* __restrict__ start,
+                            uint2* __restrict__ items) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (r >= L.n) return;
+    uint64_t n = L.size[r];
+    if (n <= small_bytes) return;
+    uint32_t c_n = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
+    uint32_t s = start[r];
+    for (uint32_t c = lane; c < c_n; c += 32) items[s + c] = make_uint2(r, c);
+}
+
+// ----------------------------------------------------------------------------
+// H2: group-by (size, digest) in an open-addressing table; value = min local index
+// ("the first transfer").  Round 0 keys all records from their digest;
+// resolve rounds re-key residual lists (k_refine) and reuse this kernel.
+// ----------------------------------------------------------------------------
+__global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
+                               uint64_t cap_mask, uint64_t digest_mask, int round) {
+    uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n_list) return;
+    uint32_t r = list ? list[i] : i;
+    uint64_t key;
+    if (round == 0) {
+        uint64_t n = L.size[r];
+        uint64_t d = finalize_digest(W.accA[r], W.accB[r], n);
+        W.digest[r] = d;
+        key = group_key(d, n, digest_mask);
+        W.key[r] = key;
+    } else {
+        key = W.key[r];
+    }
+    uint64_t h = key & cap_mask;
+    while (true) {
+        unsigned long long prev =
+            atomicCAS((unsigned long long*)&W.tkey[h], (unsigned long long)kEmptyKey, (unsigned long long)key);
+        if (prev == kEmptyKey || prev == key) break;
+        h = (h + 1) & cap_mask;
+    }
+    atomicMin(&W.tval[h], r);
+    W.slot[r] = (uint32_t)h;
+}
+
+// Leader lookup; members (leader != self) are reset for verification and, when large,
+// counted into their leader's verify work range (grouped by leader for L2 reuse).
+__global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list, uint32_t small_bytes,
+                         uint32_t chunk_bytes) {
+    uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    bool member = false;
+    if (i < n_list) {
+        uint32_t r = list ? list[i] : i;
+        uint32_t ld = W.tval[W.slot[r]];
+        W.leader[r] = ld;
+        if (ld != r) {
+            member = true;
+            W.eq[r] = 1;
+            W.mis[r] = ~0ull;
+            uint64_t n = L.size[r];
+            if (n > small_bytes) atomicAdd(&W.lcount[ld], (uint32_t)((n + chunk_bytes - 1) / chunk_bytes));
+        }
+    }
+    unsigned b = __ballot_sync(0xFFFFFFFFu, member);
+    if ((threadIdx.x & 31) == 0 && b) atomicAdd(&W.counters[1], (uint32_t)__popc(b));
+}
+
+__global__ void k_verify_fill(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
+                              uint32_t small_bytes, uint32_t chunk_bytes) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (i >= n_list) return;
+    const uint32_t m = list ? list[i] : i;
+    const uint32_t ld = W.leader[m];
+    if (ld == m) return;
+    const uint64_t n = L.size[m];
+    if (n <= small_bytes) return;
+    const uint32_t c_n = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
+    uint32_t p = 0;
+    if (lane == 0) p = atomicAdd(&W.lstart[ld], c_n);
+    p = __shfl_sync(0xFFFFFFFFu, p, 0);
+    for (uint32_t c = lane; c < c_n; c += 32) W.vitems[p + c] = make_uint2(m, c);
+}
+
+// ----------------------------------------------------------------------------
+// H3: byte verification of every member against its candidate leader.  Records the
+// first mismatching 16-B word (exact minimum: a chunk is skipped only when a
+// mismatch at a lower word is already known), and appends failures to a residual list.
+// ----------------------------------------------------------------------------
+__device__ __forceinline__ int blk_diff(const Blk& x, const Blk& y) {
+    // -1: equal; 0: first word differs; 1: only second word differs
+    uint32_t d0 = (x.v[0] ^ y.v[0]) | (x.v[1] ^ y.v[1]) | (x.v[2] ^ y.v[2]) | (x.v[3] ^ y.v[3]);
+    uint32_t d1 = (x.v[4] ^ y.v[4]) | (x.v[5] ^ y.v[5]) | (x.v[6] ^ y.v[6]) | (x.v[7] ^ y.v[7]);
+    return d0 ? 0 : (d1 ? 1 : -1);
+}
+
+__device__ __forceinline__ void report_mismatch(Work& W, uint32_t m, uint64_t word, uint32_t* res_out, bool atomic) {
+    if (atomic) {
+        atomicMin((unsigned long long*)&W.mis[m], (unsigned long long)word);
+        if (atomicExch(&W.eq[m], 0u) == 1u) res_out[atomicAdd(&W.counters[0], 1u)] = m;
+    } else {
+        W.mis[m] = word;
+        W.eq[m] = 0;
+        res_out[atomicAdd(&W.counters[0], 1u)] = m;
+    }
+}
+
+constexpr int kVerifyU = 2;
+
+__global__ void __launch_bounds__(256, 3) k_verify_small(DevLog L, Work W, const uint32_t* __restrict__ list,
+                                                      uint32_t n_list, uint32_t small_bytes, uint32_t* res_out) {
+    const int g = threadIdx.x & 7;
+    const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
+    const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
+    const unsigned omask = 0xFFu << (threadIdx.x & 24);
+    for (uint32_t i = oct; i < n_list; i += noct) {
+        const uint32_t m = list ? list[i] : i;
+        const uint32_t ld = W.leader[m];
+        if (ld == m) continue;
+        const uint64_t n = L.size[m];
+        if (n > small_bytes) continue;
+        uint64_t word = ~0ull;
+        if (L.size[ld] != n) {
+            word = 0;
+        } else {
+            const uint8_t* pm = L.arena + L.off[m];
+            const uint8_t* pl = L.arena + L.off[ld];
+            const uint32_t nblk = (uint32_t)((n + 31) >> 5);
+            for (uint32_t b0 = 0; b0 < nblk; b0 += 8 * kVerifyU) {
+                Blk x[kVerifyU], y[kVerifyU];
+#pragma unroll
+                for (int u = 0; u < kVerifyU; ++u) {
+                    uint32_t b = b0 + 8 * u + g;
+                    x[u] = b < nblk ? ld_stream(pm + 32ull * b) : zero_blk();
+                    y[u] = b < nblk ? ld_keep(pl + 32ull * b) : zero_blk();
+                }
+                uint64_t found = ~0ull;
+#pragma unroll
+                for (int u = 0; u < kVerifyU; ++u) {
+                    uint32_t b = b0 + 8 * u + g;
+                    if (b < nblk) {
+                        mask_tail(x[u], n, b);
+                        mask_tail(y[u], n, b);
+                        int d = blk_diff(x[u], y[u]);
+                        if (d >= 0 && found == ~0ull) found = 2ull * b + d;
+                    }
+                }
+                // octet min over lanes
+#pragma unroll
+                for (int o = 4; o; o >>= 1) {
+                    uint64_t other = __shfl_xor_sync(omask, found, o);
+                    found = other < found ? other : found;
+                }
+                if (found != ~0ull) {
+                    word = found;
+                    break;
+                }
+            }
+        }
+        if (word != ~0ull && g == 0) report_mismatch(W, m, word, res_out, false);
+    }
+}
+
+__global__ void __launch_bounds__(256, 3) k_verify_large(DevLog L, Work W, const uint2* __restrict__ items,
+                                                      const uint32_t* __restrict__ n_items_ptr, uint32_t chunk_bytes,
+                                                      uint32_t* res_out) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    const uint32_t n_items = *n_items_ptr;
+    const uint32_t cblk = chunk_bytes >> 5;
+    for (uint32_t it = warp; it < n_items; it += nwarps) {
+        const uint2 w = items[it];
+        const uint32_t m = w.x;
+        const uint32_t ld = W.leader[m];
+        const uint64_t n = L.size[m];
+        if (L.size[ld] != n) {
+            if (lane == 0) report_mismatch(W, m, 0, res_out, true);
+            continue;
+        }
+        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
+        const uint32_t bb = w.y * cblk;
+        const uint32_t be = min(bb + cblk, nblk);
+        uint64_t known = lane == 0 ? *((volatile uint64_t*)&W.mis[m]) : 0;
+        known = __shfl_sync(0xFFFFFFFFu, known, 0);
+        if (2 * bb >= known) continue;   // a mismatch at a lower word is already known
+        const uint8_t* pm = L.arena + L.off[m];
+        const uint8_t* pl = L.arena + L.off[ld];
+        uint64_t word = ~0ull;
+        for (uint32_t b0 = bb; b0 < be; b0 += 32 * kVerifyU) {
+            Blk x[kVerifyU], y[kVerifyU];
+#pragma unroll
+            for (int u = 0; u < kVerifyU; ++u) {
+                uint32_t b = b0 + 32 * u + lane;
+                x[u] = b < be ? ld_stream(pm + 32ull * b) : zero_blk();
+                y[u] = b < be ? ld_keep(pl + 32ull * b) : zero_blk();
+            }
+            uint64_t found = ~0ull;
+#pragma unroll
+            for (int u = 0; u < kVerifyU; ++u) {
+                uint32_t b = b0 + 32 * u + lane;
+                if (b < be) {
+                    mask_tail(x[u], n, b);
+                    mask_tail(y[u], n, b);
+                    int d = blk_diff(x[u], y[u]);
+                    if (d >= 0 && found == ~0ull) found = 2ull * b + d;
+                }
+            }
+            if (__any_sync(0xFFFFFFFFu, found != ~0ull)) {
+#pragma unroll
+                for (int o = 16; o; o >>= 1) {
+                    uint64_t other = __shfl_xor_sync(0xFFFFFFFFu, found, o);
+                    found = other < found ? other : found;
+                }
+                word = found;
+                break;
+            }
+        }
+        if (word != ~0ull && lane == 0) report_mismatch(W, m, word, res_out, true);
+    }
+}
+
+// ----------------------------------------------------------------------------
+// H4: re-key residual members.  Round 1 refines by the full, untruncated NH sums;
+// later rounds by (first mismatching word index vs the previous leader, that word).
+// Byte-equal records always receive equal keys, so exactness never depends on the key.
+// ----------------------------------------------------------------------------
+__global__ void k_refine(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list, int round,
+                         uint64_t refine_mask) {
+    uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n_list) return;
+    uint32_t m = list[i];
+    uint64_t ref;
+    if (round == 1) {
+        ref = (fmix64(W.accA[m]) ^ W.accB[m]) & refine_mask;
+    } else {
+        uint64_t q = W.mis[m];
+        uint64_t n = L.size[m];
+        uint32_t w[4] = {0, 0, 0, 0};
+        if (16 * q < n) {
+            const uint8_t* p = L.arena + L.off[m] + 16 * q;
+            for (int j = 0; j < 16 && 16 * q + j < n; ++j) w[j >> 2] |= (uint32_t)p[j] << (8 * (j & 3));
+        }
+        ref = fmix64(q * 0x9E3779B97F4A7C15ull ^ ((uint64_t)w[1] << 32 | w[0])) ^ fmix64((uint64_t)w[3] << 32 | w[2]);
+    }
+    W.key[m] = not_empty(fmix64(W.key[m] ^ fmix64(ref + (uint64_t)round)));
+}
+
+// ----------------------------------------------------------------------------
+// H5 + H6: labels and per-site benefit (u64 atomics: exact and order independent).
+// ----------------------------------------------------------------------------
+template <bool kSmem>
+__global__ void __launch_bounds__(256) k_label(DevLog L, const uint32_t* __restrict__ leader, uint32_t n_sites,
+                                               int64_t* __restrict__ dup_out, uint64_t* __restrict__ ben) {
+    extern __shared__ unsigned long long sben[];
+    if (kSmem) {
+        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) sben[s] = 0;
+        __syncthreads();
+    }
+    for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < L.n; r += gridDim.x * blockDim.x) {
+        uint32_t ld = leader[r];
+        int64_t d = ld == r ? -1 : (int64_t)L.gid[ld];
+        dup_out[r] = d;
+        if (d >= 0) {
+            if (kSmem)
+                atomicAdd(&sben[L.site[r]], (unsigned long long)L.dur[r]);
+            else
+                atomicAdd((unsigned long long*)&ben[L.site[r]], (unsigned long long)L.dur[r]);
+        }
+    }
+    if (kSmem) {
+        __syncthreads();
+        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x)
+            if (sben[s]) atomicAdd((unsigned long long*)&ben[s], sben[s]);
+    }
+}
+
+// ----------------------------------------------------------------------------
+// H0 helper: snapshot device-resident payloads into the arena (one warp per record).
+// desc[3i] = src address, desc[3i+1] = arena offset, desc[3i+2] = size.
+// ----------------------------------------------------------------------------
+__global__ void k_gather(const uint64_t* __restrict__ desc, uint32_t n, uint8_t* __restrict__ arena) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t i = warp; i < n; i += nwarps) {
+        const uint8_t* src = (const uint8_t*)desc[3 * i];
+        uint8_t* dst = arena + desc[3 * i + 1];
+        const uint64_t sz = desc[3 * i + 2];
+        if (((uintptr_t)src & 15) == 0) {
+            const uint64_t nv = sz >> 4;
+            for (uint64_t k = lane; k < nv; k += 32) ((uint4*)dst)[k] = ((const uint4*)src)[k];
+            for (uint64_t k = (nv << 4) + lane; k < sz; k += 32) dst[k] = src[k];
+        } else {
+            for (uint64_t k = lane; k < sz; k += 32) dst[k] = src[k];
+        }
+    }
+}
+
+// ----------------------------------------------------------------------------
+// Launchers
+// ----------------------------------------------------------------------------
+static inline uint32_t blocks_for(uint64_t threads, uint32_t bs = 256) {
+    return (uint32_t)((threads + bs - 1) / bs);
+}
+
+#define FFM_LAUNCH_CHECK() \
+    do {                                      \
+        if (cudaGetLastError() != cudaSuccess) return -1; \
+    } while (0)
+
+size_t cub_scan_bytes(uint64_t n) {
+    size_t bytes = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, bytes, (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n);
+    return bytes;
+}
+
+int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
+    if (L.n == 0) return 0;
+    uint32_t grid = (uint32_t)P.num_sms * 8;
+    uint32_t need = blocks_for((uint64_t)L.n * 8);
+    k_hash_small<<<need < grid ? need : grid, 256, 0, st>>>(L, P.small_bytes, W.accA, W.accB);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
+int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
+    k_hash_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hcount);
+    FFM_LAUNCH_CHECK();
+    size_t bytes = W.cub_tmp_bytes;
+    if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.hcount, W.hstart, (int)(L.n + 1), st) != cudaSuccess)
+        return -1;
+    if (L.n) {
+        k_hash_fill<<<blocks_for((uint64_t)L.n * 32), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hstart,
+                                                                    W.hitems);
+        FFM_LAUNCH_CHECK();
+    }
+    return 3;
+}
+
+int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st) {
+    if (n_items == 0) return 0;
+    uint32_t grid = (uint32_t)P.num_sms * 8;
+    uint32_t need = blocks_for(n_items * 32);
+    k_hash_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W.hitems, W.hstart + L.n, P.chunk_bytes, W.hpart);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
+int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
+    if (L.n == 0) return 0;
+    k_hash_combine<<<blocks_for((uint64_t)L.n * 32), 256, 0, st>>>(L, P.small_bytes, W.hstart, W.hpart, W.accA,
+                                                                     W.accB);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
+int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list, uint64_t cap,
+                 int round, cudaStream_t st) {
+    if (n_list == 0) return 0;
+    int k = 0;
+    if (round > 0) {
+        k_refine<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, round, P.refine_mask);
+        FFM_LAUNCH_CHECK();
+        ++k;
+    }
+    if (cudaMemsetAsync(W.tkey, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(W.tval, 0xFF, cap * sizeof(uint32_t), st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(W.lcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
+    k_group_insert<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, cap - 1, P.digest_mask, round);
+    FFM_LAUNCH_CHECK();
+    k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes);
+    FFM_LAUNCH_CHECK();
+    return k + 2;
+}
+
+int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
+                  uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st) {
+    if (n_list == 0) return 0;
+    int k = 0;
+    // large members: per-leader ranges (scan of lcount) then scatter work units
+    size_t bytes = W.cub_tmp_bytes;
+    if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.lcount, W.lstart, (int)(L.n + 1), st) != cudaSuccess)
+        return -1;
+    ++k;
+    // lstart[n] holds the total; keep it aside, the scatter advances lstart as cursors
+    uint32_t* n_vitems = W.counters + 2;
+    if (cudaMemcpyAsync(n_vitems, W.lstart + L.n, sizeof(uint32_t), cudaMemcpyDeviceToDevice, st) != cudaSuccess)
+        return -1;
+    if (vitem_cap) {
+        k_verify_fill<<<blocks_for((uint64_t)n_list * 32), 256, 0, st>>>(L, W, list, n_list, P.small_bytes,
+                                                                          P.chunk_bytes);
+        FFM_LAUNCH_CHECK();
+        ++k;
+    }
+    uint32_t grid = (uint32_t)P.num_sms * 8;
+    uint32_t need = blocks_for((uint64_t)n_list * 8);
+    k_verify_small<<<need < grid ? need : grid, 256, 0, st>>>(L, W, list, n_list, P.small_bytes, res_out);
+    FFM_LAUNCH_CHECK();
+    ++k;
+    if (vitem_cap) {
+        need = blocks_for(vitem_cap * 32);
+        k_verify_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.vitems, n_vitems, P.chunk_bytes, res_out);
+        FFM_LAUNCH_CHECK();
+        ++k;
+    }
+    return k;
+}
+
+int launch_label(const DevLog& L, Work& W, uint32_t n_sites, int64_t* dup_out, uint64_t* ben_out, cudaStream_t st) {
+    if (cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    if (L.n == 0) return 0;
+    uint32_t grid = blocks_for(L.n);
+    if (grid > 148u * 8) grid = 148u * 8;
+    if (n_sites <= 4096) {
+        k_label<true><<<grid, 256, n_sites * sizeof(uint64_t), st>>>(L, W.leader, n_sites, dup_out, ben_out);
+    } else {
+        k_label<false><<<grid, 256, 0, st>>>(L, W.leader, n_sites, dup_out, ben_out);
+    }
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
+int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st) {
+    if (n == 0) return 0;
+    uint32_t grid = blocks_for((uint64_t)n * 32);
+    if (grid > 148u * 16) grid = 148u * 16;
+    k_gather<<<grid, 256, 0, st>>>(d_desc, n, arena);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
+int launch_zero_counters(Work& W, cudaStream_t st) {
+    return cudaMemsetAsync(W.counters, 0, 16 * sizeof(uint32_t), st) == cudaSuccess ? 0 : -1;
+}
+
+}  // namespace ffm

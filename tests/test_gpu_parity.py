@@ -1,0 +1,230 @@
+"""Parity of the CUDA path (through the C ABI) against the CPU oracle -- bit-exact.
+
+All outputs are integers (gids and nanoseconds), so the bar is bit-exact equality
+of duplicate_of and benefit_ns with oracle/ffm_oracle.c on the same seeded logs.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import loggen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+@pytest.fixture(scope="module")
+def ffm():
+    import torch
+    assert torch.cuda.is_available(), "the -m gpu tests need a CUDA device"
+    import paper_conf_sc_weltonm19_b200 as m
+    return m
+
+
+def gpu_dedup(ffm, lg, device_payloads=False, **kw):
+    with ffm.FfmLog(lg.n_sites, device=0, timing=True, **kw) as log:
+        if device_payloads:
+            import torch
+            buf = torch.from_numpy(lg.materialize()).cuda()
+            ptrs = (lg.c_off[lg.content] + np.uint64(buf.data_ptr())).astype(np.uint64)
+            log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE)
+            del buf
+        else:
+            log.append_log(lg)
+        dup, ben = log.run()
+        return dup.copy(), ben.copy(), log.stats()
+
+
+def assert_same(lg, dup, ben, hash_bits=64):
+    want_dup, want_ben = oracle.dedup(lg, hash_bits=hash_bits)
+    np.testing.assert_array_equal(dup, want_dup)
+    np.testing.assert_array_equal(ben, want_ben)
+
+
+@pytest.mark.parametrize("name", sorted(f for f in os.listdir(GOLDEN) if f.endswith(".json")))
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_golden(ffm, name, digest_bits):
+    fx = json.load(open(os.path.join(GOLDEN, name)))
+    lg = loggen.from_payloads([bytes.fromhex(r["hex"]) for r in fx["records"]],
+                              [r["site"] for r in fx["records"]], [r["dur"] for r in fx["records"]],
+                              fx["n_sites"])
+    dup, ben, _ = gpu_dedup(ffm, lg, digest_bits=digest_bits)
+    assert dup.tolist() == fx["expect_duplicate_of"]
+    assert ben.tolist() == fx["expect_benefit_ns"]
+
+
+def _rand_log(seed, n, alphabet, max_len):
+    rng = np.random.default_rng(seed)
+    base = [rng.integers(0, 256, int(rng.integers(0, max_len + 1)), dtype=np.uint8).tobytes()
+            for _ in range(alphabet)]
+    pay = []
+    for _ in range(n):
+        b = base[int(rng.integers(0, alphabet))]
+        u = rng.random()
+        if u < 0.25 and b:
+            a = bytearray(b)
+            a[int(rng.integers(0, len(a)))] ^= 1 + int(rng.integers(0, 255))
+            b = bytes(a)
+        elif u < 0.3:
+            b = b[:-1]
+        pay.append(b)
+    ns = int(rng.integers(1, 7))
+    return loggen.from_payloads(pay, rng.integers(0, ns, n), rng.integers(0, 1 << 40, n), ns)
+
+
+@pytest.mark.parametrize("seed", range(12))
+@pytest.mark.parametrize("digest_bits,refine_bits", [(64, 64), (8, 64), (0, 64), (0, 0)])
+def test_random_tiny_logs(ffm, seed, digest_bits, refine_bits):
+    lg = _rand_log(seed, int(np.random.default_rng(seed).integers(1, 400)), 12, 700)
+    dup, ben, st = gpu_dedup(ffm, lg, digest_bits=digest_bits, refine_bits=refine_bits,
+                             chunk_bytes=1024, small_bytes=128)
+    assert_same(lg, dup, ben)
+
+
+@pytest.mark.parametrize("chunk,small", [(1024, 128), (4096, 4096), (32768, 4096), (65536, 16384)])
+@pytest.mark.parametrize("device_payloads", [False, True])
+def test_configs_reduced(ffm, chunk, small, device_payloads):
+    for k, ns, ss in [(1, 0.3, 0.25), (2, 0.01, 1.0), (3, 0.03, 1 / 16), (4, 0.1, 1 / 64), (5, 0.003, 1 / 32)]:
+        lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
+        dup, ben, st = gpu_dedup(ffm, lg, device_payloads, chunk_bytes=chunk, small_bytes=small)
+        assert_same(lg, dup, ben)
+        np.testing.assert_array_equal(dup, lg.planted_duplicate_of())
+
+
+@pytest.mark.parametrize("digest_bits,refine_bits", [(64, 64), (16, 64), (0, 64), (0, 0)])
+def test_forced_collisions_config3(ffm, digest_bits, refine_bits):
+    lg = loggen.gen_config(3, n_scale=0.02 if refine_bits else 0.006, size_scale=1 / 32)
+    dup, ben, st = gpu_dedup(ffm, lg, digest_bits=digest_bits, refine_bits=refine_bits, chunk_bytes=4096)
+    assert_same(lg, dup, ben)
+    if digest_bits == 0:
+        assert st["n_residual"] > 0 and st["resolve_rounds"] >= 1
+
+
+def test_digest_spec_and_chunk_invariance(ffm):
+    from digest_spec import digest
+    rng = np.random.default_rng(9)
+    sizes = [0, 1, 15, 16, 17, 31, 32, 33, 255, 256, 257, 4095, 4096, 4097, 32767, 32768, 32769,
+             100000, (1 << 20) + 3]
+    pay = [rng.integers(0, 256, s, dtype=np.uint8).tobytes() for s in sizes]
+    lg = loggen.from_payloads(pay)
+    want = [digest(p) for p in pay]
+    for chunk, small in [(1024, 128), (32768, 4096), (65536, 0)]:
+        with ffm.FfmLog(1, chunk_bytes=chunk, small_bytes=small) as log:
+            log.append_log(lg)
+            log.run()
+            got = log.digests()
+        assert [int(x) for x in got] == want, (chunk, small)
+
+
+def test_flip_at_boundaries(ffm):
+    rng = np.random.default_rng(4)
+    size = 3 * 4096 + 77
+    base = rng.integers(0, 256, size, dtype=np.uint8).tobytes()
+    pay = [base]
+    for p in [0, 15, 16, 31, 32, 1023, 1024, 4095, 4096, 8191, 8192, size - 1]:
+        a = bytearray(base)
+        a[p] ^= 0x80
+        pay += [bytes(a), base]
+    lg = loggen.from_payloads(pay)
+    for chunk, small in [(1024, 128), (4096, 16384)]:
+        for db in (64, 0):
+            dup, ben, _ = gpu_dedup(ffm, lg, chunk_bytes=chunk, small_bytes=small, digest_bits=db)
+            assert dup.tolist() == [-1] + [-1, 0] * 12
+
+
+def test_repeat_runs_and_appends_after_run(ffm):
+    lg = loggen.gen_config(2, n_scale=0.005)
+    half = lg.n // 2
+    with ffm.FfmLog(lg.n_sites) as log:
+        ptrs = lg.payload_ptrs()
+        log.append_batch(lg.site[:half], lg.size[:half], ptrs[:half], lg.dur[:half])
+        d1, b1 = [x.copy() for x in log.run()]
+        sub = lg.subset(np.arange(half))
+        assert_same(sub, d1, b1)
+        log.append_batch(lg.site[half:], lg.size[half:], ptrs[half:], lg.dur[half:])
+        outs = [tuple(x.copy() for x in log.run()) for _ in range(3)]
+    for d, b in outs:
+        np.testing.assert_array_equal(d, outs[0][0])
+        np.testing.assert_array_equal(b, outs[0][1])
+    assert_same(lg, *outs[0])
+
+
+def test_single_appends_mixed_host_device(ffm):
+    import torch
+    lg = loggen.gen_config(1, n_scale=0.1, size_scale=0.1)
+    buf = torch.from_numpy(lg.materialize()).cuda()
+    with ffm.FfmLog(lg.n_sites) as log:
+        hp = lg.payload_ptrs()
+        for i in range(lg.n):
+            c = int(lg.content[i])
+            p = int(hp[i]) if i % 2 else buf.data_ptr() + int(lg.c_off[c])
+            log.append(int(lg.site[i]), int(lg.size[i]), p, int(lg.dur[i]))
+        dup, ben = log.run()
+    assert_same(lg, dup, ben)
+
+
+def test_device_outputs(ffm):
+    import torch
+    lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 64)
+    with ffm.FfmLog(lg.n_sites) as log:
+        log.append_log(lg)
+        d = torch.empty(lg.n, dtype=torch.int64, device="cuda")
+        b = torch.empty(lg.n_sites, dtype=torch.int64, device="cuda")
+        log.run(d, b)
+        assert_same(lg, d.cpu().numpy(), b.cpu().numpy().view(np.uint64))
+
+
+def test_snapshot_semantics(ffm):
+    a = np.frombuffer(b"0123456789abcdef" * 4, np.uint8).copy()
+    with ffm.FfmLog(1) as log:
+        log.append(0, a.nbytes, a.ctypes.data, 5)
+        a[3] ^= 1                                   # caller mutates after append
+        log.append(0, a.nbytes, a.ctypes.data, 7)
+        a[3] ^= 1
+        log.append(0, a.nbytes, a.ctypes.data, 11)
+        dup, ben = log.run()
+    assert dup.tolist() == [-1, -1, 0] and ben.tolist() == [11]
+
+
+def test_errors_leave_log_unchanged(ffm):
+    x = np.zeros(64, np.uint8)
+    with ffm.FfmLog(2) as log:
+        log.append(1, 64, x.ctypes.data, 1)
+        with pytest.raises(ffm.FfmError) as e:
+            log.append(2, 64, x.ctypes.data, 1)
+        assert e.value.code == ffm.FFM_E_RANGE
+        with pytest.raises(ffm.FfmError) as e:
+            log.append(0, 8, 0, 1)
+        assert e.value.code == ffm.FFM_E_INVAL
+        with pytest.raises(ffm.FfmError) as e:
+            log.append_batch([0, 1], [64, 64], [x.ctypes.data] * 2, [1, 1], gids=[5, 5])
+        assert e.value.code == ffm.FFM_E_RANGE
+        log.append(0, 0, 0, 3)                      # size 0 with NULL is fine
+        assert log.count == 2
+        dup, ben = log.run()
+        assert dup.tolist() == [-1, -1]
+
+
+def test_gids_are_reported(ffm):
+    x = np.frombuffer(b"abcdefgh" * 8, np.uint8).copy()
+    with ffm.FfmLog(1) as log:
+        log.append_batch([0, 0, 0], [64, 32, 64], [x.ctypes.data] * 3, [1, 2, 3], gids=[10, 20, 35])
+        dup, ben = log.run()
+    assert dup.tolist() == [-1, -1, 10] and ben.tolist() == [3]
+
+
+@pytest.mark.parametrize("k", [1, 2, 3])
+def test_full_size_configs_1_to_3(ffm, k):
+    lg = loggen.gen_config(k)
+    lg.materialize(nthreads=0)
+    dup, ben, st = gpu_dedup(ffm, lg)
+    assert_same(lg, dup, ben)
+    if k == 3:
+        dup0, ben0, st0 = gpu_dedup(ffm, lg, digest_bits=0)
+        np.testing.assert_array_equal(dup0, dup)
+        np.testing.assert_array_equal(ben0, ben)
+        assert st0["n_residual"] > 0
