@@ -224,6 +224,8 @@ void ensure_work(ffm_log* L, uint64_t n) {
         dev_alloc(W.res[1], c);
         dev_alloc(W.lcount, c + 1);
         dev_alloc(W.lstart, c + 1);
+        dev_alloc(W.gcount, c + 1);
+        dev_alloc(W.pos, c);
         dev_alloc(W.hcount, c + 1);
         dev_alloc(W.hstart, c + 1);
         dev_alloc(W.dup, c);
@@ -249,6 +251,8 @@ void ensure_work(ffm_log* L, uint64_t n) {
     }
     if (L->cfg.n_sites > W.site_cap) {
         dev_alloc(W.ben, L->cfg.n_sites);
+        if ((uint64_t)L->cfg.n_sites * 8 <= (uint64_t)L->params.max_smem)
+            dev_alloc(W.label_part, (uint64_t)label_hist_rows(L->params.num_sms) * L->cfg.n_sites);
         W.site_cap = L->cfg.n_sites;
     }
 }
@@ -341,6 +345,7 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
             return FFM_E_NODEV;   // built for sm_100a only
         }
         ck(cudaDeviceGetAttribute(&L->params.num_sms, cudaDevAttrMultiProcessorCount, L->device), "attr");
+        ck(cudaDeviceGetAttribute(&L->params.max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, L->device), "attr");
         L->params.chunk_bytes = chunk;
         L->params.small_bytes = small;
         L->params.digest_mask = cfg->digest_bits >= 64 ? ~0ull : ((1ull << cfg->digest_bits) - 1);
@@ -352,6 +357,8 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
             L->own_stream = true;
         }
         ck(cudaStreamCreateWithFlags(&L->stage_stream, cudaStreamNonBlocking), "stream");
+        ck(cudaStreamCreateWithFlags(&L->side_stream, cudaStreamNonBlocking), "stream");
+        for (auto& e : L->fork_ev) ck(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
         L->ring_bytes = kRingBytes;
         for (int i = 0; i < 2; ++i) {
             ck(cudaHostAlloc((void**)&L->ring[i], kRingBytes, cudaHostAllocDefault), "cudaHostAlloc(ring)");
@@ -485,9 +492,14 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
 
         if (timing) ck(cudaEventRecord(L->ev[0], s), "event");
         if (launch_zero_counters(W, s) < 0) throw CudaFail{cudaGetLastError(), "zero counters"};
-        // H1 hash
-        LCHK(launch_hash_small(D, W, L->params, s));
-        if (timing) ck(cudaEventRecord(L->ev[8], s), "event");
+        // H1 hash: small payloads on the side stream, concurrently with the large path
+        cudaStream_t side = L->side_stream;
+        ck(cudaEventRecord(L->fork_ev[0], s), "event");
+        ck(cudaStreamWaitEvent(side, L->fork_ev[0], 0), "fork");
+        if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
+        LCHK(launch_hash_small(D, W, L->params, side));
+        if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
+        ck(cudaEventRecord(L->fork_ev[1], side), "event");
         if (L->n_large_chunks) {
             LCHK(launch_hash_plan(D, W, L->params, s));
             if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
@@ -495,16 +507,18 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
             if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
             LCHK(launch_hash_combine(D, W, L->params, s));
         }
+        ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
         if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
         // H2 group-by (round 0, all records)
         uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
         LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, s));
         if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
         // H3 verify
-        LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], L->n_large_chunks ? W.vitem_cap : 0, s));
+        LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], L->n_large_chunks ? W.vitem_cap : 0, s, side,
+                           L->fork_ev[2], L->fork_ev[3]));
         if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
         // H5 + H6 label and benefit
-        LCHK(launch_label(D, W, ns, d_dup, d_ben, s));
+        LCHK(launch_label(D, W, L->params, ns, d_dup, d_ben, s));
         if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
         ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
         ck(cudaStreamSynchronize(s), "run sync");
@@ -523,14 +537,14 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
                 uint64_t capr = std::max<uint64_t>(1024, pow2_at_least(2 * nres));
                 LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)rounds, s));
                 LCHK(launch_verify(D, W, L->params, W.res[cur], (uint32_t)nres, W.res[cur ^ 1],
-                                   L->n_large_chunks ? W.vitem_cap : 0, s));
+                                   L->n_large_chunks ? W.vitem_cap : 0, s, nullptr, nullptr, nullptr));
                 ck(cudaMemcpyAsync(L->h_counters, W.counters, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
                 ck(cudaStreamSynchronize(s), "round sync");
                 nres = L->h_counters[0];
                 n_res_total += nres;
                 cur ^= 1;
             }
-            LCHK(launch_label(D, W, ns, d_dup, d_ben, s));
+            LCHK(launch_label(D, W, L->params, ns, d_dup, d_ben, s));
             if (timing) ck(cudaEventRecord(L->ev[7], s), "event");
         }
         // H7 return
@@ -553,7 +567,7 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         S.kernel_launches = launches;
         S.hash_items = L->n_large_chunks;
         if (timing) {
-            S.ms_hash_small = ev_ms(L->ev[0], L->ev[8]);
+            S.ms_hash_small = ev_ms(L->ev[12], L->ev[8]);
             S.ms_hash_large = L->n_large_chunks ? ev_ms(L->ev[10], L->ev[11]) : 0.0;
             S.ms_hash = ev_ms(L->ev[0], L->ev[1]);
             S.ms_group = ev_ms(L->ev[1], L->ev[2]);
@@ -594,8 +608,8 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->stage_stream) cudaStreamSynchronize(L->stage_stream);
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
-                    W.lcount, W.lstart, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
-                    W.dup, W.ben, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid,
+                    W.lcount, W.lstart, W.gcount, W.pos, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
+                    W.dup, W.ben, W.label_part, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid,
                     L->arena, L->d_desc};
     for (void* p : ptrs)
         if (p) cudaFree(p);
@@ -607,6 +621,9 @@ int ffm_log_destroy(ffm_log* L) {
         if (e) cudaEventDestroy(e);
     if (L->h_counters) cudaFreeHost(L->h_counters);
     if (L->stage_stream) cudaStreamDestroy(L->stage_stream);
+    if (L->side_stream) cudaStreamDestroy(L->side_stream);
+    for (auto e : L->fork_ev)
+        if (e) cudaEventDestroy(e);
     if (L->own_stream && L->stream) cudaStreamDestroy(L->stream);
     cudaGetLastError();
     delete L;

@@ -38,7 +38,9 @@ struct Work {
     uint64_t* mis = nullptr;       // [n] first mismatching 16-B word vs leader
     uint32_t* res[2] = {nullptr, nullptr};  // residual lists (double buffer)
     uint32_t* lcount = nullptr;    // [n+1] per-leader verify chunk counts
-    uint32_t* lstart = nullptr;    // [n+1] exclusive scan of lcount (then cursors)
+    uint32_t* lstart = nullptr;    // [n+1] exclusive scan of lcount: group base of each leader
+    uint32_t* gcount = nullptr;    // [n+1] large members per leader (chunk-major stride)
+    uint32_t* pos = nullptr;       // [n] position of a large member within its leader's group
     uint2* hitems = nullptr;       // large-payload hash work units (record, chunk)
     uint2* vitems = nullptr;       // large-payload verify work units (member, chunk)
     uint32_t* hcount = nullptr;    // [n+1] per-record hash chunk counts
@@ -48,6 +50,7 @@ struct Work {
     uint32_t* tval = nullptr;      // [cap] table min local index
     int64_t* dup = nullptr;        // [n] output staging
     uint64_t* ben = nullptr;       // [n_sites]
+    uint64_t* label_part = nullptr; // [label_hist_rows * n_sites] per-block benefit partials
     uint32_t* counters = nullptr;  // device counters: [0] nres, [1] n_members, [2..] misc
     void* cub_tmp = nullptr;
     size_t cub_tmp_bytes = 0;
@@ -60,6 +63,7 @@ struct Params {
     uint32_t chunk_bytes;
     uint32_t small_bytes;
     int num_sms;
+    int max_smem;      // opt-in dynamic shared memory per block (bytes)
 };
 
 // ---- kernel launchers (kernels.cu).  All asynchronous on `st`; each returns the
@@ -71,9 +75,11 @@ int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t 
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
                  uint64_t cap, int round, cudaStream_t st);
 int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
-                  uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st);
-int launch_label(const DevLog& L, Work& W, uint32_t n_sites, int64_t* dup_out, uint64_t* ben_out,
-                 cudaStream_t st);
+                  uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st, cudaStream_t side, cudaEvent_t ev_fork,
+                  cudaEvent_t ev_join);
+int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out,
+                 uint64_t* ben_out, cudaStream_t st);
+uint32_t label_hist_rows(int num_sms);
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 size_t cub_scan_bytes(uint64_t n);
@@ -86,6 +92,8 @@ struct ffm_log {
     int device = 0;
     cudaStream_t stream = nullptr;
     cudaStream_t stage_stream = nullptr;
+    cudaStream_t side_stream = nullptr;   // small-payload kernels run concurrently here
+    cudaEvent_t fork_ev[4] = {};
     bool own_stream = false;
     bool poisoned = false;
     std::string last_error;

@@ -13,6 +13,9 @@
 // No tensor cores: there is no dense contraction on this path.
 #include <cub/cub.cuh>
 
+#include <mutex>
+#include <unordered_map>
+
 #include "ffm_internal.h"
 
 namespace ffm {
@@ -153,13 +156,35 @@ __device__ __forceinline__ void nh_blk(const Blk& x, const LaneKeys& K, uint64_t
     if (32 * b + 16 < n) nh_word(x.v[4], x.v[5], x.v[6], x.v[7], K.k[1], A, B);
 }
 
+// Each warp scans 32 consecutive list entries, ballots the ones that need work and
+// then serves them one at a time with all 32 lanes (cheap skipping of small records).
+#define FFM_WARP_COMPACT(n_list, list, PRED, ...)                                         \
+    {                                                                                      \
+        const int lane_ = threadIdx.x & 31;                                                \
+        const uint32_t i_ = blockIdx.x * blockDim.x + threadIdx.x;                         \
+        uint32_t r_ = 0;                                                                   \
+        bool act_ = false;                                                                 \
+        if (i_ < (n_list)) {                                                               \
+            r_ = (list) ? (list)[i_] : i_;                                                 \
+            act_ = (PRED);                                                                 \
+        }                                                                                  \
+        unsigned bal_ = __ballot_sync(0xFFFFFFFFu, act_);                                  \
+        while (bal_) {                                                                     \
+            const int src_ = __ffs(bal_) - 1;                                              \
+            bal_ &= bal_ - 1;                                                              \
+            const uint32_t rec = __shfl_sync(0xFFFFFFFFu, r_, src_);                       \
+            const int lane = lane_;                                                        \
+            __VA_ARGS__                                                                    \
+        }                                                                                  \
+    }
+
 // ----------------------------------------------------------------------------
 // H1a: payloads <= small_bytes, one 8-lane group ("octet") per record.  Lane g
 // reads 32-B block g of each 256-B stripe: positions 2g, 2g+1.
 // ----------------------------------------------------------------------------
-constexpr int kSmallU = 4;
+constexpr int kSmallU = 2;
 
-__global__ void __launch_bounds__(256, 3) k_hash_small(DevLog L, uint32_t small_bytes, uint64_t* __restrict__ accA,
+__global__ void __launch_bounds__(256, 4) k_hash_small(DevLog L, uint32_t small_bytes, uint64_t* __restrict__ accA,
                                                     uint64_t* __restrict__ accB) {
     const int g = threadIdx.x & 7;
     const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
@@ -258,30 +283,28 @@ __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __
     }
 }
 
-// Combine the chunk partial sums of multi-chunk records (NH is a plain sum, so the
-// record's accumulators are the sums of its chunks' -- no atomics, deterministic).
+// Combine the chunk partial sums of large records (NH is a plain sum, so the record's
+// accumulators are the sums of its chunks' -- no atomics, deterministic).
 __global__ void k_hash_combine(DevLog L, uint32_t small_bytes, const uint32_t* __restrict__ start,
                                const uint64_t* __restrict__ part, uint64_t* __restrict__ accA,
                                uint64_t* __restrict__ accB) {
-    const int lane = threadIdx.x & 31;
-    const uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (r >= L.n) return;
-    if (L.size[r] <= small_bytes) return;
-    const uint32_t s = start[r], e = start[r + 1];
-    uint64_t A = 0, B = 0;
-    for (uint32_t it = s + lane; it < e; it += 32) {
-        A += part[2ull * it];
-        B += part[2ull * it + 1];
-    }
-#pragma unroll
-    for (int o = 16; o; o >>= 1) {
-        A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
-        B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
-    }
-    if (lane == 0) {
-        accA[r] = A;
-        accB[r] = B;
-    }
+    const uint32_t* nolist = nullptr;
+    FFM_WARP_COMPACT(L.n, nolist, (L.size[r_] > small_bytes), {
+        const uint32_t s0 = start[rec], e0 = start[rec + 1];
+        uint64_t A = 0, B = 0;
+        for (uint32_t it = s0 + lane; it < e0; it += 32) {
+            A += part[2ull * it];
+            B += part[2ull * it + 1];
+        }
+        for (int o = 16; o; o >>= 1) {
+            A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
+            B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
+        }
+        if (lane == 0) {
+            accA[rec] = A;
+            accB[rec] = B;
+        }
+    })
 }
 
 // Work-unit planning for H1b / H3b: counts -> exclusive scan -> scatter.
@@ -298,14 +321,12 @@ __global__ void k_hash_count(DevLog L, uint32_t small_bytes, uint32_t chunk_byte
 
 __global__ void k_hash_fill(DevLog L, uint32_t small_bytes, uint32_t chunk_bytes, const uint32_t* __restrict__ start,
                             uint2* __restrict__ items) {
-    const int lane = threadIdx.x & 31;
-    const uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (r >= L.n) return;
-    uint64_t n = L.size[r];
-    if (n <= small_bytes) return;
-    uint32_t c_n = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
-    uint32_t s = start[r];
-    for (uint32_t c = lane; c < c_n; c += 32) items[s + c] = make_uint2(r, c);
+    const uint32_t* nolist = nullptr;
+    FFM_WARP_COMPACT(L.n, nolist, (L.size[r_] > small_bytes), {
+        const uint32_t c_n = start[rec + 1] - start[rec];
+        const uint32_t s0 = start[rec];
+        for (uint32_t c = lane; c < c_n; c += 32) items[s0 + c] = make_uint2(rec, c);
+    })
 }
 
 // ----------------------------------------------------------------------------
@@ -339,8 +360,11 @@ __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ li
     W.slot[r] = (uint32_t)h;
 }
 
-// Leader lookup; members (leader != self) are reset for verification and, when large,
-// counted into their leader's verify work range (grouped by leader for L2 reuse).
+// Leader lookup.  Members (leader != self) are reset for verification; a large
+// member of its leader's size gets a position in its leader's group so that the
+// verify work of a class is laid out chunk-major: (chunk c, member p) at
+// lstart[leader] + c * gcount[leader] + p -- all members read leader chunk c back
+// to back, so the leader streams from HBM once and is re-read from L2.
 __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list, uint32_t small_bytes,
                          uint32_t chunk_bytes) {
     uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -354,7 +378,10 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
             W.eq[r] = 1;
             W.mis[r] = ~0ull;
             uint64_t n = L.size[r];
-            if (n > small_bytes) atomicAdd(&W.lcount[ld], (uint32_t)((n + chunk_bytes - 1) / chunk_bytes));
+            if (n > small_bytes && L.size[ld] == n) {
+                atomicAdd(&W.lcount[ld], (uint32_t)((n + chunk_bytes - 1) / chunk_bytes));
+                W.pos[r] = atomicAdd(&W.gcount[ld], 1u);
+            }
         }
     }
     unsigned b = __ballot_sync(0xFFFFFFFFu, member);
@@ -363,19 +390,14 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
 
 __global__ void k_verify_fill(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
                               uint32_t small_bytes, uint32_t chunk_bytes) {
-    const int lane = threadIdx.x & 31;
-    const uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (i >= n_list) return;
-    const uint32_t m = list ? list[i] : i;
-    const uint32_t ld = W.leader[m];
-    if (ld == m) return;
-    const uint64_t n = L.size[m];
-    if (n <= small_bytes) return;
-    const uint32_t c_n = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
-    uint32_t p = 0;
-    if (lane == 0) p = atomicAdd(&W.lstart[ld], c_n);
-    p = __shfl_sync(0xFFFFFFFFu, p, 0);
-    for (uint32_t c = lane; c < c_n; c += 32) W.vitems[p + c] = make_uint2(m, c);
+    FFM_WARP_COMPACT(n_list, list,
+                     (W.leader[r_] != r_ && L.size[r_] > small_bytes && L.size[W.leader[r_]] == L.size[r_]), {
+        const uint32_t ld = W.leader[rec];
+        const uint64_t n = L.size[rec];
+        const uint32_t c_n = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
+        const uint32_t base = W.lstart[ld], k = W.gcount[ld], p = W.pos[rec];
+        for (uint32_t c = lane; c < c_n; c += 32) W.vitems[base + c * k + p] = make_uint2(rec, c);
+    })
 }
 
 // ----------------------------------------------------------------------------
@@ -403,7 +425,7 @@ __device__ __forceinline__ void report_mismatch(Work& W, uint32_t m, uint64_t wo
 
 constexpr int kVerifyU = 2;
 
-__global__ void __launch_bounds__(256, 3) k_verify_small(DevLog L, Work W, const uint32_t* __restrict__ list,
+__global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const uint32_t* __restrict__ list,
                                                       uint32_t n_list, uint32_t small_bytes, uint32_t* res_out) {
     const int g = threadIdx.x & 7;
     const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
@@ -414,9 +436,10 @@ __global__ void __launch_bounds__(256, 3) k_verify_small(DevLog L, Work W, const
         const uint32_t ld = W.leader[m];
         if (ld == m) continue;
         const uint64_t n = L.size[m];
-        if (n > small_bytes) continue;
+        const bool size_differs = L.size[ld] != n;     // (any size: large ones are not laid out)
+        if (n > small_bytes && !size_differs) continue;
         uint64_t word = ~0ull;
-        if (L.size[ld] != n) {
+        if (size_differs) {
             word = 0;
         } else {
             const uint8_t* pm = L.arena + L.off[m];
@@ -543,31 +566,43 @@ __global__ void k_refine(DevLog L, Work W, const uint32_t* __restrict__ list, ui
 }
 
 // ----------------------------------------------------------------------------
-// H5 + H6: labels and per-site benefit (u64 atomics: exact and order independent).
+// H5 + H6: labels and per-site benefit.  Integer sums are exact and order
+// independent.  With n_sites fitting in shared memory each block keeps a private
+// histogram (no global atomic contention on hot call sites -- Zipf-skewed logs put
+// 10% of all records on one site) and a second kernel sums the block partials.
 // ----------------------------------------------------------------------------
-template <bool kSmem>
-__global__ void __launch_bounds__(256) k_label(DevLog L, const uint32_t* __restrict__ leader, uint32_t n_sites,
-                                               int64_t* __restrict__ dup_out, uint64_t* __restrict__ ben) {
+__global__ void __launch_bounds__(512) k_label_hist(DevLog L, const uint32_t* __restrict__ leader, uint32_t n_sites,
+                                                    int64_t* __restrict__ dup_out, uint64_t* __restrict__ part) {
     extern __shared__ unsigned long long sben[];
-    if (kSmem) {
-        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) sben[s] = 0;
-        __syncthreads();
-    }
+    for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) sben[s] = 0;
+    __syncthreads();
     for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < L.n; r += gridDim.x * blockDim.x) {
         uint32_t ld = leader[r];
         int64_t d = ld == r ? -1 : (int64_t)L.gid[ld];
         dup_out[r] = d;
-        if (d >= 0) {
-            if (kSmem)
-                atomicAdd(&sben[L.site[r]], (unsigned long long)L.dur[r]);
-            else
-                atomicAdd((unsigned long long*)&ben[L.site[r]], (unsigned long long)L.dur[r]);
-        }
+        if (d >= 0) atomicAdd(&sben[L.site[r]], (unsigned long long)L.dur[r]);
     }
-    if (kSmem) {
-        __syncthreads();
-        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x)
-            if (sben[s]) atomicAdd((unsigned long long*)&ben[s], sben[s]);
+    __syncthreads();
+    uint64_t* row = part + (uint64_t)blockIdx.x * n_sites;
+    for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) row[s] = sben[s];
+}
+
+__global__ void k_site_reduce(const uint64_t* __restrict__ part, uint32_t rows, uint32_t n_sites,
+                              uint64_t* __restrict__ ben) {
+    uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n_sites) return;
+    uint64_t acc = 0;
+    for (uint32_t b = 0; b < rows; ++b) acc += part[(uint64_t)b * n_sites + s];
+    ben[s] = acc;
+}
+
+__global__ void __launch_bounds__(256) k_label_global(DevLog L, const uint32_t* __restrict__ leader,
+                                                      int64_t* __restrict__ dup_out, uint64_t* __restrict__ ben) {
+    for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < L.n; r += gridDim.x * blockDim.x) {
+        uint32_t ld = leader[r];
+        int64_t d = ld == r ? -1 : (int64_t)L.gid[ld];
+        dup_out[r] = d;
+        if (d >= 0) atomicAdd((unsigned long long*)&ben[L.site[r]], (unsigned long long)L.dur[r]);
     }
 }
 
@@ -600,6 +635,26 @@ static inline uint32_t blocks_for(uint64_t threads, uint32_t bs = 256) {
     return (uint32_t)((threads + bs - 1) / bs);
 }
 
+// Persistent launch: exactly the resident blocks (num_sms x occupancy), one wave.
+static uint32_t resident_grid(const void* kernel, int num_sms, int block = 256) {
+    static std::mutex mu;
+    static std::unordered_map<const void*, int> cache;
+    std::lock_guard<std::mutex> g(mu);
+    auto it = cache.find(kernel);
+    int occ;
+    if (it == cache.end()) {
+        occ = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, block, 0) != cudaSuccess || occ < 1) {
+            cudaGetLastError();
+            occ = 1;
+        }
+        cache[kernel] = occ;
+    } else {
+        occ = it->second;
+    }
+    return (uint32_t)(occ * num_sms);
+}
+
 #define FFM_LAUNCH_CHECK() \
     do {                                      \
         if (cudaGetLastError() != cudaSuccess) return -1; \
@@ -613,7 +668,7 @@ size_t cub_scan_bytes(uint64_t n) {
 
 int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
     if (L.n == 0) return 0;
-    uint32_t grid = (uint32_t)P.num_sms * 8;
+    uint32_t grid = resident_grid((const void*)k_hash_small, P.num_sms);
     uint32_t need = blocks_for((uint64_t)L.n * 8);
     k_hash_small<<<need < grid ? need : grid, 256, 0, st>>>(L, P.small_bytes, W.accA, W.accB);
     FFM_LAUNCH_CHECK();
@@ -627,7 +682,7 @@ int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st)
     if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.hcount, W.hstart, (int)(L.n + 1), st) != cudaSuccess)
         return -1;
     if (L.n) {
-        k_hash_fill<<<blocks_for((uint64_t)L.n * 32), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hstart,
+        k_hash_fill<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hstart,
                                                                     W.hitems);
         FFM_LAUNCH_CHECK();
     }
@@ -636,7 +691,7 @@ int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st)
 
 int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st) {
     if (n_items == 0) return 0;
-    uint32_t grid = (uint32_t)P.num_sms * 8;
+    uint32_t grid = resident_grid((const void*)k_hash_large, P.num_sms);
     uint32_t need = blocks_for(n_items * 32);
     k_hash_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W.hitems, W.hstart + L.n, P.chunk_bytes, W.hpart);
     FFM_LAUNCH_CHECK();
@@ -645,7 +700,7 @@ int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_item
 
 int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
     if (L.n == 0) return 0;
-    k_hash_combine<<<blocks_for((uint64_t)L.n * 32), 256, 0, st>>>(L, P.small_bytes, W.hstart, W.hpart, W.accA,
+    k_hash_combine<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, P.small_bytes, W.hstart, W.hpart, W.accA,
                                                                      W.accB);
     FFM_LAUNCH_CHECK();
     return 1;
@@ -663,6 +718,7 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
     if (cudaMemsetAsync(W.tkey, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
     if (cudaMemsetAsync(W.tval, 0xFF, cap * sizeof(uint32_t), st) != cudaSuccess) return -1;
     if (cudaMemsetAsync(W.lcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(W.gcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
     k_group_insert<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, cap - 1, P.digest_mask, round);
     FFM_LAUNCH_CHECK();
     k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes);
@@ -671,48 +727,71 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
 }
 
 int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
-                  uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st) {
+                  uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st, cudaStream_t side, cudaEvent_t ev_fork,
+                  cudaEvent_t ev_join) {
     if (n_list == 0) return 0;
     int k = 0;
-    // large members: per-leader ranges (scan of lcount) then scatter work units
-    size_t bytes = W.cub_tmp_bytes;
-    if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.lcount, W.lstart, (int)(L.n + 1), st) != cudaSuccess)
-        return -1;
-    ++k;
-    // lstart[n] holds the total; keep it aside, the scatter advances lstart as cursors
-    uint32_t* n_vitems = W.counters + 2;
-    if (cudaMemcpyAsync(n_vitems, W.lstart + L.n, sizeof(uint32_t), cudaMemcpyDeviceToDevice, st) != cudaSuccess)
-        return -1;
-    if (vitem_cap) {
-        k_verify_fill<<<blocks_for((uint64_t)n_list * 32), 256, 0, st>>>(L, W, list, n_list, P.small_bytes,
-                                                                          P.chunk_bytes);
-        FFM_LAUNCH_CHECK();
-        ++k;
+    // small members (and any size-mismatched member) on the side stream, concurrently
+    // with the bandwidth-bound large path: the latency-bound small kernel fills gaps.
+    cudaStream_t ss = side ? side : st;
+    if (side) {
+        if (cudaEventRecord(ev_fork, st) != cudaSuccess || cudaStreamWaitEvent(side, ev_fork, 0) != cudaSuccess)
+            return -1;
     }
-    uint32_t grid = (uint32_t)P.num_sms * 8;
+    uint32_t grid_s = resident_grid((const void*)k_verify_small, P.num_sms);
     uint32_t need = blocks_for((uint64_t)n_list * 8);
-    k_verify_small<<<need < grid ? need : grid, 256, 0, st>>>(L, W, list, n_list, P.small_bytes, res_out);
+    k_verify_small<<<need < grid_s ? need : grid_s, 256, 0, ss>>>(L, W, list, n_list, P.small_bytes, res_out);
     FFM_LAUNCH_CHECK();
     ++k;
     if (vitem_cap) {
+        // large members: chunk-major groups per leader (scan of lcount) then scatter work units
+        size_t bytes = W.cub_tmp_bytes;
+        if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.lcount, W.lstart, (int)(L.n + 1), st) != cudaSuccess)
+            return -1;
+        ++k;
+        uint32_t* n_vitems = W.lstart + L.n;   // total large verify work units
+        k_verify_fill<<<blocks_for((uint64_t)n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes,
+                                                                    P.chunk_bytes);
+        FFM_LAUNCH_CHECK();
+        ++k;
+        uint32_t grid = resident_grid((const void*)k_verify_large, P.num_sms);
         need = blocks_for(vitem_cap * 32);
         k_verify_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.vitems, n_vitems, P.chunk_bytes, res_out);
         FFM_LAUNCH_CHECK();
         ++k;
     }
+    if (side) {
+        if (cudaEventRecord(ev_join, side) != cudaSuccess || cudaStreamWaitEvent(st, ev_join, 0) != cudaSuccess)
+            return -1;
+    }
     return k;
 }
 
-int launch_label(const DevLog& L, Work& W, uint32_t n_sites, int64_t* dup_out, uint64_t* ben_out, cudaStream_t st) {
-    if (cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * sizeof(uint64_t), st) != cudaSuccess) return -1;
-    if (L.n == 0) return 0;
-    uint32_t grid = blocks_for(L.n);
-    if (grid > 148u * 8) grid = 148u * 8;
-    if (n_sites <= 4096) {
-        k_label<true><<<grid, 256, n_sites * sizeof(uint64_t), st>>>(L, W.leader, n_sites, dup_out, ben_out);
-    } else {
-        k_label<false><<<grid, 256, 0, st>>>(L, W.leader, n_sites, dup_out, ben_out);
+uint32_t label_hist_rows(int num_sms) { return (uint32_t)num_sms * 2; }
+
+int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out, uint64_t* ben_out,
+                 cudaStream_t st) {
+    if (L.n == 0) return cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * sizeof(uint64_t), st) == cudaSuccess ? 0 : -1;
+    const size_t smem = (size_t)n_sites * sizeof(uint64_t);
+    if (W.label_part && smem <= (size_t)P.max_smem) {
+        static int configured_smem = 0;
+        if ((int)smem > configured_smem) {
+            if (cudaFuncSetAttribute(k_label_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, P.max_smem) !=
+                cudaSuccess)
+                return -1;
+            configured_smem = P.max_smem;
+        }
+        const uint32_t rows = label_hist_rows(P.num_sms);
+        k_label_hist<<<rows, 512, smem, st>>>(L, W.leader, n_sites, dup_out, W.label_part);
+        FFM_LAUNCH_CHECK();
+        k_site_reduce<<<blocks_for(n_sites), 256, 0, st>>>(W.label_part, rows, n_sites, ben_out);
+        FFM_LAUNCH_CHECK();
+        return 2;
     }
+    if (cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    uint32_t grid = blocks_for(L.n);
+    if (grid > (uint32_t)P.num_sms * 8) grid = (uint32_t)P.num_sms * 8;
+    k_label_global<<<grid, 256, 0, st>>>(L, W.leader, dup_out, ben_out);
     FFM_LAUNCH_CHECK();
     return 1;
 }
