@@ -148,6 +148,58 @@ int ffm_last_run_stats(const ffm_log* log, ffm_run_stats* out);
    and never part of the result. */
 int ffm_debug_digests(ffm_log* log, uint64_t* digests_out);
 
+/* ---------------------------------------------------------------------------
+ * Sharded logs (world > 1).  One process per GPU.
+ * Exact byte equality is transitive, so the per-rank results merge through one
+ * exchange of class-representative tuples.  Per run, on every rank:
+ *   1. ffm_shard_local   -- H1..H4 on this rank's records; export one ffm_rep per
+ *                           exact local class into caller DEVICE memory.
+ *   2. caller all-gathers the reps of all ranks, in rank order, into one device array
+ *      (e.g. torch.distributed all_gather over NCCL / NVLink), with the counts.
+ *   3. ffm_shard_merge   -- global group-by over all reps; a remote candidate is
+ *                           byte-verified by loading its bytes straight from the peer
+ *                           GPU's arena (IPC-mapped, over NVLink) inside the kernel;
+ *                           writes duplicate_of for this rank's records (global gids)
+ *                           and this rank's PARTIAL benefit.
+ *   4. caller all-reduces the partial benefits (uint64 sum).
+ * Peer arenas are mapped once per arena allocation: exchange ffm_shard_ipc_handle
+ * outputs (after the last append) and call ffm_shard_open_peer for every other rank.
+ * ------------------------------------------------------------------------- */
+typedef struct ffm_rep {
+    uint64_t key;    /* group key of the payload digest (identical function on every rank) */
+    uint64_t size;   /* payload bytes */
+    uint64_t gid;    /* global gid of the class's first record on the owning rank */
+    uint64_t off;    /* arena offset on the owning rank */
+} ffm_rep;
+
+enum { FFM_SHARD_SITE_LPT = 0,     /* whole call sites, bin-packed by bytes (largest first) */
+       FFM_SHARD_CONTIGUOUS = 1 }; /* contiguous gid ranges of ~equal bytes */
+
+/* Host-only shard planner: rank_out[i] in [0, world) for each of n records.
+   SITE_LPT keeps every re-upload of a call site (the dominant duplicate pattern,
+   P:1194-1197) on one rank.  Errors: FFM_E_INVAL, FFM_E_RANGE (site >= n_sites). */
+int ffm_shard_plan(uint64_t n, const uint32_t* call_sites, const uint64_t* sizes, uint32_t n_sites,
+                   int32_t world, int policy, int32_t* rank_out);
+
+/* 64-byte CUDA IPC handle of this log's HBM arena (valid until the arena grows:
+   exchange after the last append). */
+int ffm_shard_ipc_handle(ffm_log* log, void* handle_out);
+
+/* Map peer `rank`'s arena from its ffm_shard_ipc_handle bytes (no-op for own rank;
+   re-mapping the same handle is free). */
+int ffm_shard_open_peer(ffm_log* log, int32_t rank, const void* handle);
+
+/* Step 1.  reps_out: device array of at least ffm_log_count(log) entries.
+   *n_reps_out = number written (in local gid order). */
+int ffm_shard_local(ffm_log* log, ffm_rep* reps_out, uint64_t cap, uint64_t* n_reps_out);
+
+/* Step 3.  all_reps: device array of all ranks' reps, rank-major; counts: host array
+   [world].  counts[rank] must equal this rank's last n_reps (else FFM_E_COMM).
+   duplicate_of [n_local] (host or device) receives global gids; benefit_partial
+   [n_sites] receives this rank's partial sums (all-reduce them). */
+int ffm_shard_merge(ffm_log* log, const ffm_rep* all_reps, const uint64_t* counts, int64_t* duplicate_of,
+                    uint64_t* benefit_partial);
+
 /* Destroy the log and release its memory.  NULL is a no-op (returns FFM_OK). */
 int ffm_log_destroy(ffm_log* log);
 

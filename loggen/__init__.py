@@ -101,7 +101,7 @@ class Log:
             off[1:] = np.cumsum(slot[:-1], dtype=np.uint64)
         total = int(slot.sum()) if len(sz) else 0
         if buf is None:
-            buf = np.empty(max(total, 16), dtype=np.uint8)
+            buf = np.zeros(max(total, 16), dtype=np.uint8)   # calloc: padding deterministic
         elif buf.nbytes < total:
             raise ValueError("buffer too small")
         lib = _get_lib()

@@ -27,7 +27,10 @@ FFM_FLAG_TIMING = 1
 EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_append_batch",
            "ffm_dedup_run", "ffm_log_count", "ffm_log_payload_bytes", "ffm_log_stream",
            "ffm_last_run_stats", "ffm_debug_digests", "ffm_log_destroy", "ffm_strerror",
-           "ffm_last_error", "ffm_version"]
+           "ffm_last_error", "ffm_version", "ffm_shard_plan", "ffm_shard_ipc_handle", "ffm_shard_open_peer",
+           "ffm_shard_local", "ffm_shard_merge"]
+FFM_SHARD_SITE_LPT, FFM_SHARD_CONTIGUOUS = 0, 1
+REP_WORDS = 4        # ffm_rep = {key, size, gid, off}, 4 x u64
 
 
 class FfmConfig(ctypes.Structure):
@@ -96,6 +99,16 @@ def lib() -> ctypes.CDLL:
         L.ffm_last_error.restype = ctypes.c_char_p
         L.ffm_version.argtypes = []
         L.ffm_version.restype = ctypes.c_char_p
+        L.ffm_shard_plan.argtypes = [u64, vp, vp, u32, ctypes.c_int32, i32, vp]
+        L.ffm_shard_plan.restype = i32
+        L.ffm_shard_ipc_handle.argtypes = [vp, vp]
+        L.ffm_shard_ipc_handle.restype = i32
+        L.ffm_shard_open_peer.argtypes = [vp, ctypes.c_int32, vp]
+        L.ffm_shard_open_peer.restype = i32
+        L.ffm_shard_local.argtypes = [vp, vp, u64, ctypes.POINTER(u64)]
+        L.ffm_shard_local.restype = i32
+        L.ffm_shard_merge.argtypes = [vp, vp, vp, vp, vp]
+        L.ffm_shard_merge.restype = i32
         _lib = L
     return _lib
 
@@ -192,6 +205,40 @@ def ffm_debug_digests(h) -> np.ndarray:
 
 def ffm_log_destroy(h):
     _check(None, lib().ffm_log_destroy(h))
+
+
+def ffm_shard_plan(call_sites, sizes, n_sites: int, world: int, policy: int = FFM_SHARD_SITE_LPT) -> np.ndarray:
+    """Host-only: rank of each record (site-affinity LPT or contiguous byte-balanced ranges)."""
+    sites = np.ascontiguousarray(call_sites, dtype=np.uint32)
+    sz = np.ascontiguousarray(sizes, dtype=np.uint64)
+    out = np.empty(max(len(sites), 1), np.int32)
+    rc = lib().ffm_shard_plan(len(sites), _addr(sites), _addr(sz), n_sites, world, policy, _addr(out))
+    if rc != FFM_OK:
+        raise FfmError(rc)
+    return out[:len(sites)]
+
+
+def ffm_shard_ipc_handle(h) -> bytes:
+    buf = ctypes.create_string_buffer(64)
+    _check(h, lib().ffm_shard_ipc_handle(h, buf))
+    return buf.raw
+
+
+def ffm_shard_open_peer(h, rank: int, handle: bytes):
+    buf = ctypes.create_string_buffer(bytes(handle), 64)
+    _check(h, lib().ffm_shard_open_peer(h, rank, buf))
+
+
+def ffm_shard_local(h, reps_out, cap: int) -> int:
+    """reps_out: device buffer (torch CUDA tensor) of >= ffm_log_count ffm_rep entries."""
+    n = ctypes.c_uint64()
+    _check(h, lib().ffm_shard_local(h, _addr(reps_out), cap, ctypes.byref(n)))
+    return int(n.value)
+
+
+def ffm_shard_merge(h, all_reps, counts, duplicate_of, benefit_partial):
+    c = np.ascontiguousarray(counts, dtype=np.uint64)
+    _check(h, lib().ffm_shard_merge(h, _addr(all_reps), _addr(c), _addr(duplicate_of), _addr(benefit_partial)))
 
 
 # ---- convenience wrapper ----------------------------------------------------

@@ -5,7 +5,7 @@ import subprocess
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB = os.path.join(HERE, "libffm.so")
-SOURCES = [os.path.join(HERE, "csrc", f) for f in ("kernels.cu", "ffm_api.cu")]
+SOURCES = [os.path.join(HERE, "csrc", f) for f in ("kernels.cu", "shard.cu", "ffm_api.cu", "shard_plan.cpp")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-shared", "-Xcompiler", "-fPIC", "-O3", "-lineinfo", "-std=c++17",
          "-gencode", "arch=compute_100a,code=sm_100a"]
@@ -15,7 +15,7 @@ def _stale() -> bool:
     if not os.path.exists(LIB):
         return True
     t = os.path.getmtime(LIB)
-    deps = SOURCES + glob.glob(os.path.join(HERE, "csrc", "*.h")) + \
+    deps = SOURCES + glob.glob(os.path.join(HERE, "csrc", "*.h")) + glob.glob(os.path.join(HERE, "csrc", "*.cuh")) + \
         glob.glob(os.path.join(HERE, "..", "include", "*.h"))
     return any(os.path.getmtime(d) > t for d in deps)
 

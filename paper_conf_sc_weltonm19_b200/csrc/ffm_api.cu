@@ -20,6 +20,10 @@ constexpr uint64_t kRingBytes = 16ull << 20;      // per half of the pinned stag
 constexpr uint64_t kDirectCopy = 4ull << 20;      // host payloads above this bypass the ring
 constexpr uint64_t kGatherMax = 1ull << 20;       // device payloads up to this use k_gather
 
+struct LocalRun {
+    uint64_t n_members, n_res_total, rounds;
+};
+
 struct CudaFail {
     cudaError_t e;
     const char* what;
@@ -285,6 +289,192 @@ float ev_ms(cudaEvent_t a, cudaEvent_t b) {
         launches += (uint64_t)_k;                                              \
     } while (0)
 
+
+// ---------------------------------------------------------------- run pipeline
+void run_prologue(ffm_log* L) {
+    ck(cudaSetDevice(L->device), "cudaSetDevice");
+    // H0 tail: flush staged payloads and metadata, order the run after them
+    ring_flush(L);
+    upload_meta(L);
+    ck(cudaEventRecord(L->ring_ev[L->ring_cur], L->stage_stream), "event");
+    ck(cudaStreamWaitEvent(L->stream, L->ring_ev[L->ring_cur], 0), "wait staging");
+    ensure_work(L, L->h_size.size());
+}
+
+// H1..H4 over the local log: on return W.leader holds every record's final local
+// leader (the min local index of its exact byte class).  With `label` the H5/H6
+// kernels are queued before the first sync (single-GPU fast path: one sync when
+// there are no digest collisions) and re-run after collision resolution.
+LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup, uint64_t* d_ben) {
+    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
+    const uint64_t n = L->h_size.size();
+    Work& W = L->work;
+    cudaStream_t s = L->stream;
+    DevLog D = dev_view(L);
+    const uint32_t ns = L->cfg.n_sites;
+    LocalRun R{};
+    if (timing) ck(cudaEventRecord(L->ev[0], s), "event");
+    if (launch_zero_counters(W, s) < 0) throw CudaFail{cudaGetLastError(), "zero counters"};
+    // H1 hash: small payloads on the side stream, concurrently with the large path
+    cudaStream_t side = L->side_stream;
+    ck(cudaEventRecord(L->fork_ev[0], s), "event");
+    ck(cudaStreamWaitEvent(side, L->fork_ev[0], 0), "fork");
+    if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
+    LCHK(launch_hash_small(D, W, L->params, side));
+    if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
+    ck(cudaEventRecord(L->fork_ev[1], side), "event");
+    if (L->n_large_chunks) {
+        LCHK(launch_hash_plan(D, W, L->params, s));
+        if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
+        LCHK(launch_hash_large(D, W, L->params, L->n_large_chunks, s));
+        if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
+        LCHK(launch_hash_combine(D, W, L->params, s));
+    }
+    ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
+    if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
+    // H2 group-by (round 0, all records)
+    uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
+    LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, s));
+    if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
+    // H3 verify
+    LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], L->n_large_chunks ? W.vitem_cap : 0, s, side,
+                       L->fork_ev[2], L->fork_ev[3]));
+    if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
+    // H5 + H6 (speculative: valid unless H3 found residuals)
+    if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, d_ben, s));
+    if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
+    ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+    ck(cudaStreamSynchronize(s), "run sync");
+    R.n_members = L->h_counters[1];
+    uint64_t nres = L->h_counters[0];
+    R.n_res_total = nres;
+    if (nres) {
+        // H4 collision resolution: exact classes among the residual members
+        if (timing) ck(cudaEventRecord(L->ev[6], s), "event");
+        int cur = 0;
+        while (nres) {
+            ++R.rounds;
+            if (R.rounds > n + 2) throw CudaFail{cudaErrorUnknown, "collision resolution did not converge"};
+            ck(cudaMemsetAsync(W.counters, 0, sizeof(uint32_t), s), "memset");
+            uint64_t capr = std::max<uint64_t>(1024, pow2_at_least(2 * nres));
+            LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)R.rounds, s));
+            LCHK(launch_verify(D, W, L->params, W.res[cur], (uint32_t)nres, W.res[cur ^ 1],
+                               L->n_large_chunks ? W.vitem_cap : 0, s, nullptr, nullptr, nullptr));
+            ck(cudaMemcpyAsync(L->h_counters, W.counters, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+            ck(cudaStreamSynchronize(s), "round sync");
+            nres = L->h_counters[0];
+            R.n_res_total += nres;
+            cur ^= 1;
+        }
+        if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, d_ben, s));
+        if (timing) ck(cudaEventRecord(L->ev[7], s), "event");
+    }
+    return R;
+}
+
+void fill_stats(ffm_log* L, const LocalRun& R, uint64_t launches, bool single) {
+    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
+    ffm_run_stats& S = L->stats;
+    memset(&S, 0, sizeof(S));
+    S.n_records = L->h_size.size();
+    S.payload_bytes = L->payload_bytes;
+    S.n_members = R.n_members;
+    S.n_residual = R.n_res_total;
+    S.resolve_rounds = R.rounds;
+    S.kernel_launches = launches;
+    S.hash_items = L->n_large_chunks;
+    if (timing) {
+        S.ms_hash_small = ev_ms(L->ev[12], L->ev[8]);
+        S.ms_hash_large = L->n_large_chunks ? ev_ms(L->ev[10], L->ev[11]) : 0.0;
+        S.ms_hash = ev_ms(L->ev[0], L->ev[1]);
+        S.ms_group = ev_ms(L->ev[1], L->ev[2]);
+        S.ms_verify = ev_ms(L->ev[2], L->ev[3]);
+        S.ms_label = single ? ev_ms(L->ev[3], L->ev[4]) : 0.0;
+        S.ms_resolve = R.rounds ? ev_ms(L->ev[6], L->ev[7]) : 0.0;
+        if (single) {
+            S.ms_output = ev_ms(L->ev[9], L->ev[5]);
+            S.ms_total = ev_ms(L->ev[0], L->ev[5]);
+        }
+    }
+    L->digests_valid = true;
+}
+
+
+// ---------------------------------------------------------------- sharded runs
+void ensure_shard(ffm_log* L, uint64_t n, uint64_t M, uint64_t nloc, uint64_t vcap, int world) {
+    ShardWork& S = L->shard;
+    if (n + 1 > S.n_cap || !S.flag) {
+        uint64_t c = std::max<uint64_t>(n + 1, 1024);
+        dev_alloc(S.flag, c);
+        dev_alloc(S.rep_idx, c);
+        S.n_cap = c;
+        size_t cb = cub_scan_bytes(c);
+        if (cb > L->work.cub_tmp_bytes) {
+            if (L->work.cub_tmp) cudaFree(L->work.cub_tmp);
+            L->work.cub_tmp = nullptr;
+            ck(cudaMalloc(&L->work.cub_tmp, cb), "cudaMalloc(cub)");
+            L->work.cub_tmp_bytes = cb;
+        }
+    }
+    uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(M, 1)));
+    if (cap > S.t_cap) {
+        dev_alloc(S.tkey, cap);
+        dev_alloc(S.tgid, cap);
+        dev_alloc(S.tidx, cap);
+        S.t_cap = cap;
+    }
+    if (M > S.m_cap || !S.tslot) {
+        uint64_t c = std::max<uint64_t>(M, 1024);
+        dev_alloc(S.tslot, c);
+        dev_alloc(S.sort_keys_in, c);
+        dev_alloc(S.sort_keys_out, c);
+        dev_alloc(S.sort_vals_in, c);
+        dev_alloc(S.order, c);
+        size_t sb = sort_tmp_bytes((uint32_t)c);
+        if (S.sort_tmp) cudaFree(S.sort_tmp);
+        S.sort_tmp = nullptr;
+        ck(cudaMalloc(&S.sort_tmp, std::max<size_t>(sb, 256)), "cudaMalloc(sort)");
+        S.sort_tmp_bytes = std::max<size_t>(sb, 256);
+        S.m_cap = c;
+    }
+    if (nloc + 1 > S.l_cap || !S.state) {
+        uint64_t c = std::max<uint64_t>(nloc + 1, 1024);
+        dev_alloc(S.state, c);
+        dev_alloc(S.cand, c);
+        dev_alloc(S.vcount, c);
+        dev_alloc(S.vstart, c);
+        dev_alloc(S.G, c);
+        dev_alloc(S.slow_list, c);
+        S.l_cap = c;
+        size_t cb = cub_scan_bytes(c);
+        if (cb > L->work.cub_tmp_bytes) {
+            if (L->work.cub_tmp) cudaFree(L->work.cub_tmp);
+            L->work.cub_tmp = nullptr;
+            ck(cudaMalloc(&L->work.cub_tmp, cb), "cudaMalloc(cub)");
+            L->work.cub_tmp_bytes = cb;
+        }
+    }
+    if (vcap > S.v_cap || !S.vitems) {
+        uint64_t c = std::max<uint64_t>(vcap, 1024);
+        dev_alloc(S.vitems, c);
+        S.v_cap = c;
+    }
+    if ((uint64_t)world > S.w_cap || !S.rank_lo) {
+        dev_alloc(S.rank_lo, world);
+        dev_alloc(S.bases, world);
+        if (!S.n_slow) dev_alloc(S.n_slow, 1);
+        S.w_cap = world;
+    }
+}
+
+void free_shard(ShardWork& S) {
+    void* ptrs[] = {S.flag, S.rep_idx, S.tkey, S.tgid, S.tidx, S.tslot, S.state, S.cand, S.vcount, S.vstart,
+                    S.G, S.slow_list, S.vitems, S.rank_lo, (void*)S.bases, S.n_slow, S.sort_keys_in,
+                    S.sort_keys_out, S.sort_vals_in, S.order, S.sort_tmp};
+    for (void* p : ptrs)
+        if (p) cudaFree(p);
+}
+
 }  // namespace
 
 // ======================================================================== ABI
@@ -471,83 +661,20 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
     if (st) return st;
     uint64_t n = L->h_size.size();
     if (n > 0 && !dup_out) return set_err(L, FFM_E_INVAL, "duplicate_of is NULL");
-    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
-    uint64_t launches = 0;
+    if (L->cfg.world > 1) return set_err(L, FFM_E_STATE, "sharded log: use ffm_shard_local / ffm_shard_merge");
     try {
-        ck(cudaSetDevice(L->device), "cudaSetDevice");
-        // H0 tail: flush staged payloads and metadata, order the run after them
-        ring_flush(L);
-        upload_meta(L);
-        ck(cudaEventRecord(L->ring_ev[L->ring_cur], L->stage_stream), "event");
-        ck(cudaStreamWaitEvent(L->stream, L->ring_ev[L->ring_cur], 0), "wait staging");
-        ensure_work(L, n);
+        run_prologue(L);
         Work& W = L->work;
         cudaStream_t s = L->stream;
-        DevLog D = dev_view(L);
         const uint32_t ns = L->cfg.n_sites;
         bool dup_dev = dup_out && is_device_ptr(dup_out);
         bool ben_dev = ben_out && is_device_ptr(ben_out);
         int64_t* d_dup = dup_dev ? dup_out : W.dup;
         uint64_t* d_ben = ben_dev ? ben_out : W.ben;
-
-        if (timing) ck(cudaEventRecord(L->ev[0], s), "event");
-        if (launch_zero_counters(W, s) < 0) throw CudaFail{cudaGetLastError(), "zero counters"};
-        // H1 hash: small payloads on the side stream, concurrently with the large path
-        cudaStream_t side = L->side_stream;
-        ck(cudaEventRecord(L->fork_ev[0], s), "event");
-        ck(cudaStreamWaitEvent(side, L->fork_ev[0], 0), "fork");
-        if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
-        LCHK(launch_hash_small(D, W, L->params, side));
-        if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
-        ck(cudaEventRecord(L->fork_ev[1], side), "event");
-        if (L->n_large_chunks) {
-            LCHK(launch_hash_plan(D, W, L->params, s));
-            if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
-            LCHK(launch_hash_large(D, W, L->params, L->n_large_chunks, s));
-            if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
-            LCHK(launch_hash_combine(D, W, L->params, s));
-        }
-        ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
-        if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
-        // H2 group-by (round 0, all records)
-        uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
-        LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, s));
-        if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
-        // H3 verify
-        LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], L->n_large_chunks ? W.vitem_cap : 0, s, side,
-                           L->fork_ev[2], L->fork_ev[3]));
-        if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
-        // H5 + H6 label and benefit
-        LCHK(launch_label(D, W, L->params, ns, d_dup, d_ben, s));
-        if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
-        ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
-        ck(cudaStreamSynchronize(s), "run sync");
-        uint64_t n_members = L->h_counters[1];
-        uint64_t nres = L->h_counters[0];
-        uint64_t n_res_total = nres;
-        uint64_t rounds = 0;
-        if (nres) {
-            // H4 collision resolution: exact classes among the residual members
-            if (timing) ck(cudaEventRecord(L->ev[6], s), "event");
-            int cur = 0;
-            while (nres) {
-                ++rounds;
-                if (rounds > n + 2) throw CudaFail{cudaErrorUnknown, "collision resolution did not converge"};
-                ck(cudaMemsetAsync(W.counters, 0, sizeof(uint32_t), s), "memset");
-                uint64_t capr = std::max<uint64_t>(1024, pow2_at_least(2 * nres));
-                LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)rounds, s));
-                LCHK(launch_verify(D, W, L->params, W.res[cur], (uint32_t)nres, W.res[cur ^ 1],
-                                   L->n_large_chunks ? W.vitem_cap : 0, s, nullptr, nullptr, nullptr));
-                ck(cudaMemcpyAsync(L->h_counters, W.counters, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
-                ck(cudaStreamSynchronize(s), "round sync");
-                nres = L->h_counters[0];
-                n_res_total += nres;
-                cur ^= 1;
-            }
-            LCHK(launch_label(D, W, L->params, ns, d_dup, d_ben, s));
-            if (timing) ck(cudaEventRecord(L->ev[7], s), "event");
-        }
+        uint64_t launches = 0;
+        LocalRun R = run_local(L, launches, true, d_dup, d_ben);
         // H7 return
+        const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
         if (timing) ck(cudaEventRecord(L->ev[9], s), "event");
         if (!dup_dev && n)
             ck(cudaMemcpyAsync(dup_out, d_dup, n * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
@@ -556,28 +683,159 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         if (timing) ck(cudaEventRecord(L->ev[5], s), "event");
         ck(cudaStreamSynchronize(s), "output sync");
         ck(cudaGetLastError(), "run");
+        fill_stats(L, R, launches, true);
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    } catch (const std::bad_alloc&) {
+        return set_err(L, FFM_E_NOMEM, "host allocation failed");
+    }
+    return FFM_OK;
+}
 
-        ffm_run_stats& S = L->stats;
-        memset(&S, 0, sizeof(S));
-        S.n_records = n;
-        S.payload_bytes = L->payload_bytes;
-        S.n_members = n_members;
-        S.n_residual = n_res_total;
-        S.resolve_rounds = rounds;
-        S.kernel_launches = launches;
-        S.hash_items = L->n_large_chunks;
-        if (timing) {
-            S.ms_hash_small = ev_ms(L->ev[12], L->ev[8]);
-            S.ms_hash_large = L->n_large_chunks ? ev_ms(L->ev[10], L->ev[11]) : 0.0;
-            S.ms_hash = ev_ms(L->ev[0], L->ev[1]);
-            S.ms_group = ev_ms(L->ev[1], L->ev[2]);
-            S.ms_verify = ev_ms(L->ev[2], L->ev[3]);
-            S.ms_label = ev_ms(L->ev[3], L->ev[4]);
-            S.ms_resolve = rounds ? ev_ms(L->ev[6], L->ev[7]) : 0.0;
-            S.ms_output = ev_ms(L->ev[9], L->ev[5]);
-            S.ms_total = ev_ms(L->ev[0], L->ev[5]);
+int ffm_shard_ipc_handle(ffm_log* L, void* out) {
+    int st = check_state(L);
+    if (st) return st;
+    if (!out) return FFM_E_INVAL;
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        ensure_arena(L, 1);
+        cudaIpcMemHandle_t h;
+        ck(cudaIpcGetMemHandle(&h, L->arena), "cudaIpcGetMemHandle");
+        static_assert(sizeof(h) == 64, "IPC handle size");
+        memcpy(out, &h, 64);
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    }
+    return FFM_OK;
+}
+
+int ffm_shard_open_peer(ffm_log* L, int32_t peer, const void* handle) {
+    int st = check_state(L);
+    if (st) return st;
+    if (!handle || peer < 0 || peer >= L->cfg.world) return set_err(L, FFM_E_INVAL, "bad peer rank / handle");
+    if (peer == L->cfg.rank) return FFM_OK;
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        if (L->peer_ptr.size() < (size_t)L->cfg.world) {
+            L->peer_ptr.resize(L->cfg.world, nullptr);
+            L->peer_handle.resize(L->cfg.world);
         }
-        L->digests_valid = true;
+        std::string hb((const char*)handle, 64);
+        if (L->peer_ptr[peer] && L->peer_handle[peer] == hb) return FFM_OK;
+        if (L->peer_ptr[peer]) ck(cudaIpcCloseMemHandle(L->peer_ptr[peer]), "cudaIpcCloseMemHandle");
+        L->peer_ptr[peer] = nullptr;
+        cudaIpcMemHandle_t h;
+        memcpy(&h, handle, 64);
+        void* p = nullptr;
+        ck(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+        L->peer_ptr[peer] = p;
+        L->peer_handle[peer] = hb;
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    }
+    return FFM_OK;
+}
+
+int ffm_shard_local(ffm_log* L, ffm_rep* reps_out, uint64_t cap, uint64_t* n_reps_out) {
+    int st = check_state(L);
+    if (st) return st;
+    uint64_t n = L->h_size.size();
+    if (!n_reps_out || (n && !reps_out)) return set_err(L, FFM_E_INVAL, "NULL argument");
+    if (cap < n) return set_err(L, FFM_E_RANGE, "reps_out capacity < ffm_log_count");
+    try {
+        run_prologue(L);
+        uint64_t launches = 0;
+        LocalRun R = run_local(L, launches, false, nullptr, nullptr);
+        ensure_shard(L, n, 1, 1, 1, std::max(L->cfg.world, 1));
+        DevLog D = dev_view(L);
+        cudaStream_t s = L->stream;
+        LCHK(launch_rep_export(D, L->work, L->shard, L->params, (RepTuple*)reps_out, s));
+        ck(cudaMemcpyAsync(L->h_counters, L->shard.rep_idx + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+        ck(cudaStreamSynchronize(s), "shard local sync");
+        L->n_reps = L->h_counters[0];
+        L->reps_valid = true;
+        *n_reps_out = L->n_reps;
+        fill_stats(L, R, launches, false);
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    } catch (const std::bad_alloc&) {
+        return set_err(L, FFM_E_NOMEM, "host allocation failed");
+    }
+    return FFM_OK;
+}
+
+int ffm_shard_merge(ffm_log* L, const ffm_rep* all_reps, const uint64_t* counts, int64_t* dup_out,
+                    uint64_t* ben_out) {
+    int st = check_state(L);
+    if (st) return st;
+    const int world = L->cfg.world, rank = L->cfg.rank;
+    uint64_t n = L->h_size.size();
+    if (!counts || (n && !dup_out) || !ben_out) return set_err(L, FFM_E_INVAL, "NULL argument");
+    if (!L->reps_valid) return set_err(L, FFM_E_STATE, "ffm_shard_local must run first");
+    uint64_t M = 0, lo = 0;
+    std::vector<uint32_t> rank_lo(world);
+    for (int r = 0; r < world; ++r) {
+        rank_lo[r] = (uint32_t)M;
+        if (r == rank) lo = M;
+        M += counts[r];
+    }
+    if (counts[rank] != L->n_reps) return set_err(L, FFM_E_COMM, "counts[rank] != this rank's n_reps");
+    if (M >= 0xFFFFFFFFull) return set_err(L, FFM_E_RANGE, "too many representatives");
+    if (M && !all_reps) return set_err(L, FFM_E_INVAL, "NULL all_reps");
+    std::vector<const uint8_t*> bases(world, nullptr);
+    for (int r = 0; r < world; ++r) {
+        if (r == rank) {
+            bases[r] = L->arena;
+        } else if (counts[r]) {
+            if ((size_t)r >= L->peer_ptr.size() || !L->peer_ptr[r])
+                return set_err(L, FFM_E_STATE, "peer arena not mapped (ffm_shard_open_peer)");
+            bases[r] = (const uint8_t*)L->peer_ptr[r];
+        }
+    }
+    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        const uint64_t nloc = L->n_reps;
+        uint64_t vcap = nloc + L->n_large_chunks + 64;
+        ensure_shard(L, n, M, nloc, vcap, world);
+        ShardWork& S = L->shard;
+        Work& W = L->work;
+        cudaStream_t s = L->stream;
+        DevLog D = dev_view(L);
+        uint64_t launches = 0;
+        if (timing) ck(cudaEventRecord(L->ev[13], s), "event");
+        ck(cudaMemcpyAsync(S.rank_lo, rank_lo.data(), world * sizeof(uint32_t), cudaMemcpyHostToDevice, s), "H2D");
+        ck(cudaMemcpyAsync((void*)S.bases, bases.data(), world * sizeof(void*), cudaMemcpyHostToDevice, s), "H2D");
+        uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(M, 1)));
+        LCHK(launch_merge(D, W, S, L->params, (const RepTuple*)all_reps, (uint32_t)M, (uint32_t)lo, (uint32_t)nloc,
+                          world, rank, cap, s));
+        ck(cudaMemcpyAsync(L->h_counters, S.n_slow, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+        ck(cudaStreamSynchronize(s), "merge sync");
+        uint32_t n_slow = L->h_counters[0];
+        if (n_slow) {
+            LCHK(launch_sort_prep(S, (const RepTuple*)all_reps, (uint32_t)M, s));
+            LCHK(launch_merge_slow(D, W, S, L->params, (const RepTuple*)all_reps, (uint32_t)M, (uint32_t)lo, world,
+                                   rank, n_slow, s));
+        }
+        bool dup_dev = dup_out && is_device_ptr(dup_out);
+        bool ben_dev = is_device_ptr(ben_out);
+        int64_t* d_dup = dup_dev ? dup_out : W.dup;
+        uint64_t* d_ben = ben_dev ? ben_out : W.ben;
+        LCHK(launch_merge_label(D, W, S, L->params, L->cfg.n_sites, d_dup, d_ben, s));
+        if (!dup_dev && n)
+            ck(cudaMemcpyAsync(dup_out, d_dup, n * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
+        if (!ben_dev)
+            ck(cudaMemcpyAsync(ben_out, d_ben, L->cfg.n_sites * sizeof(uint64_t), cudaMemcpyDeviceToHost, s),
+               "D2H ben");
+        if (timing) ck(cudaEventRecord(L->ev[14], s), "event");
+        ck(cudaStreamSynchronize(s), "merge output sync");
+        ck(cudaGetLastError(), "merge");
+        L->stats.kernel_launches += launches;
+        L->stats.n_residual += n_slow;
+        if (timing) {
+            L->stats.ms_output = ev_ms(L->ev[13], L->ev[14]);
+            L->stats.ms_total = ev_ms(L->ev[0], L->ev[14]);
+        }
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
     } catch (const std::bad_alloc&) {
@@ -613,6 +871,9 @@ int ffm_log_destroy(ffm_log* L) {
                     L->arena, L->d_desc};
     for (void* p : ptrs)
         if (p) cudaFree(p);
+    free_shard(L->shard);
+    for (void* p : L->peer_ptr)
+        if (p) cudaIpcCloseMemHandle(p);
     for (int i = 0; i < 2; ++i) {
         if (L->ring[i]) cudaFreeHost(L->ring[i]);
         if (L->ring_ev[i]) cudaEventDestroy(L->ring_ev[i]);

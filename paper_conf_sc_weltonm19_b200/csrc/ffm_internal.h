@@ -57,6 +57,41 @@ struct Work {
     uint64_t n_cap = 0, t_cap = 0, hitem_cap = 0, vitem_cap = 0, site_cap = 0;
 };
 
+// One representative per exact local class, exported for the cross-shard merge.
+// Layout identical to ffm_rep (include/ffm.h).
+struct RepTuple {
+    uint64_t key;    // group key of the full digest (same function on every rank)
+    uint64_t size;
+    uint64_t gid;    // global gid of the class's first local record
+    uint64_t off;    // arena offset on the owning rank
+};
+
+struct ShardWork {
+    uint32_t* flag = nullptr;        // [n+1]
+    uint32_t* rep_idx = nullptr;     // [n+1] exclusive scan of flag: tuple index of each local rep
+    uint64_t* tkey = nullptr;        // [cap]
+    uint64_t* tgid = nullptr;        // [cap]
+    uint32_t* tidx = nullptr;        // [cap]
+    uint32_t* tslot = nullptr;       // [M]
+    uint32_t* state = nullptr;       // [nloc]
+    uint32_t* cand = nullptr;        // [nloc]
+    uint32_t* vcount = nullptr;      // [nloc+1]
+    uint32_t* vstart = nullptr;      // [nloc+1]
+    uint64_t* G = nullptr;           // [nloc] global leader gid of each local representative
+    uint32_t* slow_list = nullptr;   // [nloc]
+    uint2* vitems = nullptr;         // merge verify work units
+    uint32_t* rank_lo = nullptr;     // [world] first tuple index of each rank
+    const uint8_t** bases = nullptr; // [world] arena base of each rank (peer ones IPC-mapped)
+    uint32_t* n_slow = nullptr;
+    uint64_t* sort_keys_in = nullptr;
+    uint64_t* sort_keys_out = nullptr;
+    uint32_t* sort_vals_in = nullptr;
+    uint32_t* order = nullptr;       // [M] tuple indices sorted by gid (slow path)
+    void* sort_tmp = nullptr;
+    size_t sort_tmp_bytes = 0;
+    uint64_t n_cap = 0, m_cap = 0, t_cap = 0, l_cap = 0, v_cap = 0, w_cap = 0;
+};
+
 struct Params {
     uint64_t digest_mask;
     uint64_t refine_mask;
@@ -80,9 +115,22 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
 int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out,
                  uint64_t* ben_out, cudaStream_t st);
 uint32_t label_hist_rows(int num_sms);
+int launch_site_reduce(const uint64_t* part, uint32_t rows, uint32_t n_sites, uint64_t* ben, cudaStream_t st);
+// shard.cu
+int launch_rep_export(const DevLog& L, Work& W, ShardWork& S, const Params& P, RepTuple* out, cudaStream_t st);
+int launch_merge(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
+                 uint32_t lo, uint32_t nloc, int world, int rank, uint64_t cap, cudaStream_t st);
+int launch_sort_prep(ShardWork& S, const RepTuple* T, uint32_t M, cudaStream_t st);
+size_t sort_tmp_bytes(uint32_t M);
+int launch_merge_slow(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
+                      uint32_t lo, int world, int rank, uint32_t n_slow, cudaStream_t st);
+int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
+                       uint64_t* ben_out, cudaStream_t st);
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 size_t cub_scan_bytes(uint64_t n);
+uint32_t blocks_for(uint64_t threads, uint32_t bs = 256);
+uint32_t resident_grid(const void* kernel, int num_sms, int block = 256);
 
 }  // namespace ffm
 
@@ -127,6 +175,13 @@ struct ffm_log {
     uint64_t ring_arena_start = 0;  // arena offset corresponding to ring[cur][0]
     uint64_t ring_fill = 0;         // bytes used in ring[cur]
     bool ring_pending = false;
+
+    // sharded runs
+    ffm::ShardWork shard;
+    uint64_t n_reps = 0;            // representatives exported by the last ffm_shard_local
+    bool reps_valid = false;
+    std::vector<void*> peer_ptr;    // IPC-mapped peer arenas (index = rank)
+    std::vector<std::string> peer_handle;
 
     // gather descriptors for device payloads
     uint64_t* d_desc = nullptr;

@@ -17,6 +17,7 @@
 #include <unordered_map>
 
 #include "ffm_internal.h"
+#include "digest.cuh"
 
 namespace ffm {
 
@@ -56,69 +57,6 @@ __host__ __device__ constexpr uint32_t kDA(int j) {
 
 __constant__ NHKeys c_nh = make_nh_keys();
 
-__host__ __device__ __forceinline__ uint64_t fmix64(uint64_t k) {
-    k ^= k >> 33;
-    k *= 0xff51afd7ed558ccdull;
-    k ^= k >> 33;
-    k *= 0xc4ceb9fe1a85ec53ull;
-    k ^= k >> 33;
-    return k;
-}
-
-__device__ __forceinline__ uint64_t finalize_digest(uint64_t A, uint64_t B, uint64_t n) {
-    return fmix64(A ^ fmix64(B ^ (n * 0x9E3779B97F4A7C15ull)));
-}
-
-__device__ __forceinline__ uint64_t not_empty(uint64_t k) { return k == kEmptyKey ? k - 1 : k; }
-
-__device__ __forceinline__ uint64_t group_key(uint64_t digest, uint64_t n, uint64_t mask) {
-    return not_empty(fmix64((digest & mask) ^ fmix64(n + 0x632BE59BD9B4E019ull)));
-}
-
-// 32-byte block = two 16-byte words.
-struct Blk {
-    uint32_t v[8];
-};
-
-// Streamed payload bytes: read once, do not pollute L1, evict first from L2.
-__device__ __forceinline__ Blk ld_stream(const uint8_t* p) {
-    Blk r;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::evict_first.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-                 : "=r"(r.v[0]), "=r"(r.v[1]), "=r"(r.v[2]), "=r"(r.v[3]), "=r"(r.v[4]), "=r"(r.v[5]),
-                   "=r"(r.v[6]), "=r"(r.v[7])
-                 : "l"(p));
-    return r;
-}
-
-// Leader bytes during verify: re-read by every member of the class -> keep in L2.
-__device__ __forceinline__ Blk ld_keep(const uint8_t* p) {
-    Blk r;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::evict_last.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-                 : "=r"(r.v[0]), "=r"(r.v[1]), "=r"(r.v[2]), "=r"(r.v[3]), "=r"(r.v[4]), "=r"(r.v[5]),
-                   "=r"(r.v[6]), "=r"(r.v[7])
-                 : "l"(p));
-    return r;
-}
-
-__device__ __forceinline__ Blk zero_blk() {
-    Blk r;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) r.v[i] = 0;
-    return r;
-}
-
-// Zero the bytes of block b at or beyond n (only the record's last block is partial).
-__device__ __forceinline__ void mask_tail(Blk& x, uint64_t n, uint64_t b) {
-    int64_t valid = (int64_t)n - (int64_t)(32 * b);
-    if (valid >= 32) return;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) {
-        int64_t vb = valid - 4 * i;
-        uint32_t m = vb >= 4 ? 0xFFFFFFFFu : (vb <= 0 ? 0u : ((1u << (8 * vb)) - 1u));
-        x.v[i] &= m;
-    }
-}
-
 struct LaneKeys {
     uint32_t k[2][6];
 };
@@ -155,28 +93,6 @@ __device__ __forceinline__ void nh_blk(const Blk& x, const LaneKeys& K, uint64_t
     nh_word(x.v[0], x.v[1], x.v[2], x.v[3], K.k[0], A, B);
     if (32 * b + 16 < n) nh_word(x.v[4], x.v[5], x.v[6], x.v[7], K.k[1], A, B);
 }
-
-// Each warp scans 32 consecutive list entries, ballots the ones that need work and
-// then serves them one at a time with all 32 lanes (cheap skipping of small records).
-#define FFM_WARP_COMPACT(n_list, list, PRED, ...)                                         \
-    {                                                                                      \
-        const int lane_ = threadIdx.x & 31;                                                \
-        const uint32_t i_ = blockIdx.x * blockDim.x + threadIdx.x;                         \
-        uint32_t r_ = 0;                                                                   \
-        bool act_ = false;                                                                 \
-        if (i_ < (n_list)) {                                                               \
-            r_ = (list) ? (list)[i_] : i_;                                                 \
-            act_ = (PRED);                                                                 \
-        }                                                                                  \
-        unsigned bal_ = __ballot_sync(0xFFFFFFFFu, act_);                                  \
-        while (bal_) {                                                                     \
-            const int src_ = __ffs(bal_) - 1;                                              \
-            bal_ &= bal_ - 1;                                                              \
-            const uint32_t rec = __shfl_sync(0xFFFFFFFFu, r_, src_);                       \
-            const int lane = lane_;                                                        \
-            __VA_ARGS__                                                                    \
-        }                                                                                  \
-    }
 
 // ----------------------------------------------------------------------------
 // H1a: payloads <= small_bytes, one 8-lane group ("octet") per record.  Lane g
@@ -631,12 +547,12 @@ __global__ void k_gather(const uint64_t* __restrict__ desc, uint32_t n, uint8_t*
 // ----------------------------------------------------------------------------
 // Launchers
 // ----------------------------------------------------------------------------
-static inline uint32_t blocks_for(uint64_t threads, uint32_t bs = 256) {
+uint32_t blocks_for(uint64_t threads, uint32_t bs) {
     return (uint32_t)((threads + bs - 1) / bs);
 }
 
 // Persistent launch: exactly the resident blocks (num_sms x occupancy), one wave.
-static uint32_t resident_grid(const void* kernel, int num_sms, int block = 256) {
+uint32_t resident_grid(const void* kernel, int num_sms, int block) {
     static std::mutex mu;
     static std::unordered_map<const void*, int> cache;
     std::lock_guard<std::mutex> g(mu);
@@ -769,6 +685,12 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
 
 uint32_t label_hist_rows(int num_sms) { return (uint32_t)num_sms * 2; }
 
+int launch_site_reduce(const uint64_t* part, uint32_t rows, uint32_t n_sites, uint64_t* ben, cudaStream_t st) {
+    k_site_reduce<<<blocks_for(n_sites), 256, 0, st>>>(part, rows, n_sites, ben);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
 int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out, uint64_t* ben_out,
                  cudaStream_t st) {
     if (L.n == 0) return cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * sizeof(uint64_t), st) == cudaSuccess ? 0 : -1;
@@ -784,8 +706,7 @@ int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, in
         const uint32_t rows = label_hist_rows(P.num_sms);
         k_label_hist<<<rows, 512, smem, st>>>(L, W.leader, n_sites, dup_out, W.label_part);
         FFM_LAUNCH_CHECK();
-        k_site_reduce<<<blocks_for(n_sites), 256, 0, st>>>(W.label_part, rows, n_sites, ben_out);
-        FFM_LAUNCH_CHECK();
+        if (launch_site_reduce(W.label_part, rows, n_sites, ben_out, st) < 0) return -1;
         return 2;
     }
     if (cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * sizeof(uint64_t), st) != cudaSuccess) return -1;

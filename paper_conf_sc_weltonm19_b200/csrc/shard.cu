@@ -1,0 +1,351 @@
+// shard.cu -- multi-GPU (sharded log) kernels, SURVEY.md 8(e) / DESIGN.md §9.
+//
+// Exact byte equality is transitive, so after H1-H4 on its own records each rank
+// holds exact local classes.  One representative per local class (its min local
+// gid) is exported as a tuple; ranks all-gather the tuples (NCCL over NVLink, done
+// by the caller), then every rank resolves ITS OWN representatives:
+//   global leader G(x) = min gid over representatives with bytes equal to x's.
+// The global group-by gives the min-gid representative with x's key; a remote
+// candidate is confirmed by a byte compare that loads the candidate's bytes straight
+// from the owning GPU's arena (CUDA-IPC-mapped peer memory over NVLink) -- the
+// transfer is fused into the verify kernel, there is no staging copy.  A
+// representative whose candidate is local (same key, different exact local class)
+// or fails the compare takes the slow path: scan same-key representatives in gid
+// order and byte-compare the remote ones until the first equal one.
+#include <cub/cub.cuh>
+
+#include "digest.cuh"
+#include "ffm_internal.h"
+
+namespace ffm {
+
+enum : uint32_t { kDone = 0, kVerify = 1, kSlow = 2 };
+
+__device__ __forceinline__ int owner_of(uint32_t t, const uint32_t* __restrict__ rank_lo, int world) {
+    int o = 0;
+    for (int r = 1; r < world; ++r) o += (t >= rank_lo[r]);
+    return o;
+}
+
+// ---- export --------------------------------------------------------------------
+__global__ void k_rep_flag(DevLog L, const uint32_t* __restrict__ leader, uint32_t* __restrict__ flag) {
+    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r > L.n) return;
+    flag[r] = (r < L.n && leader[r] == r) ? 1u : 0u;
+}
+
+__global__ void k_rep_export(DevLog L, Work W, const uint32_t* __restrict__ rep_idx, uint64_t digest_mask,
+                             RepTuple* __restrict__ out) {
+    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= L.n || W.leader[r] != r) return;
+    uint64_t n = L.size[r];
+    RepTuple t;
+    t.key = group_key(W.digest[r], n, digest_mask);
+    t.size = n;
+    t.gid = L.gid[r];
+    t.off = L.off[r];
+    out[rep_idx[r]] = t;
+}
+
+// ---- global group-by over all representatives ----------------------------------
+__global__ void k_merge_insert(const RepTuple* __restrict__ T, uint32_t M, uint64_t cap_mask, uint64_t* tkey,
+                               uint64_t* tgid, uint32_t* __restrict__ tslot) {
+    uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= M) return;
+    const uint64_t key = T[t].key;
+    uint64_t h = key & cap_mask;
+    while (true) {
+        unsigned long long prev =
+            atomicCAS((unsigned long long*)&tkey[h], (unsigned long long)kEmptyKey, (unsigned long long)key);
+        if (prev == kEmptyKey || prev == key) break;
+        h = (h + 1) & cap_mask;
+    }
+    atomicMin((unsigned long long*)&tgid[h], (unsigned long long)T[t].gid);
+    tslot[t] = (uint32_t)h;
+}
+
+__global__ void k_merge_index(const RepTuple* __restrict__ T, uint32_t M, const uint64_t* __restrict__ tgid,
+                              const uint32_t* __restrict__ tslot, uint32_t* __restrict__ tidx) {
+    uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= M) return;
+    uint32_t h = tslot[t];
+    if (T[t].gid == tgid[h]) tidx[h] = t;
+}
+
+// Classify this rank's representatives; count verify work units for remote candidates.
+__global__ void k_merge_classify(const RepTuple* __restrict__ T, uint32_t lo, uint32_t nloc,
+                                 const uint32_t* __restrict__ tslot, const uint32_t* __restrict__ tidx,
+                                 const uint32_t* __restrict__ rank_lo, int world, int rank, uint32_t chunk_bytes,
+                                 ShardWork S) {
+    uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j > nloc) return;
+    if (j == nloc) {
+        S.vcount[j] = 0;
+        return;
+    }
+    const uint32_t t = lo + j;
+    const uint32_t c = tidx[tslot[t]];
+    uint32_t st, cnt = 0;
+    if (c == t) {
+        st = kDone;
+        S.G[j] = T[t].gid;
+    } else if (owner_of(c, rank_lo, world) == rank || T[c].size != T[t].size) {
+        st = kSlow;     // same key, different exact local class (or size): not equal
+    } else {
+        st = kVerify;
+        S.cand[j] = c;
+        uint64_t n = T[t].size;
+        cnt = n == 0 ? 1u : (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
+    }
+    S.state[j] = st;
+    S.vcount[j] = cnt;
+}
+
+__global__ void k_merge_fill(uint32_t nloc, ShardWork S) {
+    const uint32_t* nolist = nullptr;
+    FFM_WARP_COMPACT(nloc, nolist, (S.vcount[r_] != 0), {
+        const uint32_t s0 = S.vstart[rec], c_n = S.vcount[rec];
+        for (uint32_t c = lane; c < c_n; c += 32) S.vitems[s0 + c] = make_uint2(rec, c);
+    })
+}
+
+// Byte-compare a local representative with its remote candidate, chunk by chunk.
+// The candidate's bytes are loaded from the peer GPU's arena over NVLink.
+__global__ void __launch_bounds__(256) k_merge_verify(const RepTuple* __restrict__ T, uint32_t lo,
+                                                      const uint32_t* __restrict__ rank_lo, int world, int rank,
+                                                      const uint8_t* const* __restrict__ bases, uint32_t chunk_bytes,
+                                                      const uint32_t* __restrict__ n_items_ptr, ShardWork S) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    const uint32_t n_items = *n_items_ptr;
+    const uint32_t cblk = chunk_bytes >> 5;
+    for (uint32_t it = warp; it < n_items; it += nwarps) {
+        const uint2 w = S.vitems[it];
+        const uint32_t j = w.x;
+        const uint32_t x = lo + j, y = S.cand[j];
+        const uint64_t n = T[x].size;
+        const uint8_t* px = bases[rank] + T[x].off;
+        const uint8_t* py = bases[owner_of(y, rank_lo, world)] + T[y].off;
+        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
+        const uint32_t bb = w.y * cblk, be = min(bb + cblk, nblk);
+        bool diff = false;
+        for (uint32_t b = bb + lane; b < be; b += 32) {
+            Blk a = ld_stream(px + 32ull * b);
+            Blk r = ld_remote(py + 32ull * b);
+            mask_tail(a, n, b);
+            mask_tail(r, n, b);
+            diff |= !blk_equal(a, r);
+        }
+        if (__any_sync(0xFFFFFFFFu, diff) && lane == 0) atomicExch(&S.state[j], (uint32_t)kSlow);
+    }
+}
+
+__global__ void k_merge_finish(const RepTuple* __restrict__ T, uint32_t nloc, ShardWork S, uint32_t* n_slow) {
+    uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
+    bool slow = false;
+    if (j < nloc) {
+        uint32_t st = S.state[j];
+        if (st == kVerify) S.G[j] = T[S.cand[j]].gid;
+        slow = st == kSlow;
+        if (slow) S.slow_list[atomicAdd(n_slow, 1u)] = j;
+    }
+}
+
+// Slow path (digest collisions only): scan all representatives in gid order; the first
+// remote one with the same key and equal bytes is the global leader.  One warp per
+// slow representative; 32 candidates tested per step, lowest gid first.
+__global__ void __launch_bounds__(256) k_merge_slow(const RepTuple* __restrict__ T, uint32_t M, uint32_t lo,
+                                                    const uint32_t* __restrict__ order,
+                                                    const uint32_t* __restrict__ rank_lo, int world, int rank,
+                                                    const uint8_t* const* __restrict__ bases, uint32_t n_slow,
+                                                    ShardWork S) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t q = warp; q < n_slow; q += nwarps) {
+        const uint32_t j = S.slow_list[q];
+        const uint32_t x = lo + j;
+        const RepTuple tx = T[x];
+        const uint64_t nblk = (tx.size + 31) >> 5;
+        const uint8_t* px = bases[rank] + tx.off;
+        uint64_t G = tx.gid;
+        bool found = false;
+        for (uint32_t s0 = 0; s0 < M && !found; s0 += 32) {
+            uint32_t s = s0 + lane;
+            uint32_t y = s < M ? order[s] : 0;
+            bool earlier = s < M && T[y].gid < tx.gid;
+            bool cand = earlier && T[y].key == tx.key && T[y].size == tx.size && owner_of(y, rank_lo, world) != rank;
+            unsigned any_earlier = __ballot_sync(0xFFFFFFFFu, earlier);
+            unsigned cm = __ballot_sync(0xFFFFFFFFu, cand);
+            while (cm) {
+                const int src = __ffs(cm) - 1;
+                cm &= cm - 1;
+                const uint32_t yy = __shfl_sync(0xFFFFFFFFu, y, src);
+                const uint8_t* py = bases[owner_of(yy, rank_lo, world)] + T[yy].off;
+                bool diff = false;
+                for (uint64_t b = lane; b < nblk; b += 32) {
+                    Blk a = ld_stream(px + 32 * b);
+                    Blk r = ld_remote(py + 32 * b);
+                    mask_tail(a, tx.size, b);
+                    mask_tail(r, tx.size, b);
+                    diff |= !blk_equal(a, r);
+                }
+                if (!__any_sync(0xFFFFFFFFu, diff)) {
+                    G = T[yy].gid;
+                    found = true;
+                    break;
+                }
+            }
+            if (any_earlier != 0xFFFFFFFFu) break;    // sorted by gid: nothing earlier beyond here
+        }
+        if (lane == 0) S.G[j] = G;
+    }
+}
+
+// H5 + H6 for a shard: record r's class representative is its local leader; the
+// class's global leader G comes from the merge.  Benefit partial per rank.
+__global__ void __launch_bounds__(512) k_merge_label(DevLog L, const uint32_t* __restrict__ leader,
+                                                     const uint32_t* __restrict__ rep_idx,
+                                                     const uint64_t* __restrict__ G, uint32_t n_sites,
+                                                     int64_t* __restrict__ dup_out, uint64_t* __restrict__ part,
+                                                     uint64_t* __restrict__ ben_global) {
+    extern __shared__ unsigned long long sben[];
+    const bool hist = part != nullptr;
+    if (hist) {
+        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) sben[s] = 0;
+        __syncthreads();
+    }
+    for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < L.n; r += gridDim.x * blockDim.x) {
+        uint64_t g = G[rep_idx[leader[r]]];
+        int64_t d = g == L.gid[r] ? -1 : (int64_t)g;
+        dup_out[r] = d;
+        if (d >= 0) {
+            if (hist)
+                atomicAdd(&sben[L.site[r]], (unsigned long long)L.dur[r]);
+            else
+                atomicAdd((unsigned long long*)&ben_global[L.site[r]], (unsigned long long)L.dur[r]);
+        }
+    }
+    if (hist) {
+        __syncthreads();
+        uint64_t* row = part + (uint64_t)blockIdx.x * n_sites;
+        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) row[s] = sben[s];
+    }
+}
+
+// ---- launchers -------------------------------------------------------------------
+#define SHARD_CHECK()                                     \
+    do {                                                  \
+        if (cudaGetLastError() != cudaSuccess) return -1; \
+    } while (0)
+
+int launch_rep_export(const DevLog& L, Work& W, ShardWork& S, const Params& P, RepTuple* out, cudaStream_t st) {
+    k_rep_flag<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, W.leader, S.flag);
+    SHARD_CHECK();
+    size_t bytes = W.cub_tmp_bytes;
+    if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, S.flag, S.rep_idx, (int)(L.n + 1), st) != cudaSuccess)
+        return -1;
+    if (L.n) {
+        k_rep_export<<<blocks_for(L.n), 256, 0, st>>>(L, W, S.rep_idx, P.digest_mask, out);
+        SHARD_CHECK();
+    }
+    return 3;
+}
+
+int launch_merge(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
+                 uint32_t lo, uint32_t nloc, int world, int rank, uint64_t cap, cudaStream_t st) {
+    int k = 0;
+    if (cudaMemsetAsync(S.tkey, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(S.tgid, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    if (M) {
+        k_merge_insert<<<blocks_for(M), 256, 0, st>>>(T, M, cap - 1, S.tkey, S.tgid, S.tslot);
+        SHARD_CHECK();
+        k_merge_index<<<blocks_for(M), 256, 0, st>>>(T, M, S.tgid, S.tslot, S.tidx);
+        SHARD_CHECK();
+        k += 2;
+    }
+    k_merge_classify<<<blocks_for((uint64_t)nloc + 1), 256, 0, st>>>(T, lo, nloc, S.tslot, S.tidx, S.rank_lo, world,
+                                                                      rank, P.chunk_bytes, S);
+    SHARD_CHECK();
+    size_t bytes = W.cub_tmp_bytes;
+    if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, S.vcount, S.vstart, (int)(nloc + 1), st) != cudaSuccess)
+        return -1;
+    k += 2;
+    if (nloc) {
+        k_merge_fill<<<blocks_for(nloc), 256, 0, st>>>(nloc, S);
+        SHARD_CHECK();
+        uint32_t grid = resident_grid((const void*)k_merge_verify, P.num_sms);
+        k_merge_verify<<<grid, 256, 0, st>>>(T, lo, S.rank_lo, world, rank, S.bases, P.chunk_bytes, S.vstart + nloc,
+                                             S);
+        SHARD_CHECK();
+        k += 2;
+    }
+    if (cudaMemsetAsync(S.n_slow, 0, sizeof(uint32_t), st) != cudaSuccess) return -1;
+    if (nloc) {
+        k_merge_finish<<<blocks_for(nloc), 256, 0, st>>>(T, nloc, S, S.n_slow);
+        SHARD_CHECK();
+        ++k;
+    }
+    return k;
+}
+
+int launch_merge_slow(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
+                      uint32_t lo, int world, int rank, uint32_t n_slow, cudaStream_t st) {
+    // order[] = representatives sorted by gid
+    size_t bytes = S.sort_tmp_bytes;
+    if (cub::DeviceRadixSort::SortPairs(S.sort_tmp, bytes, S.sort_keys_in, S.sort_keys_out, S.sort_vals_in,
+                                        S.order, (int)M, 0, 64, st) != cudaSuccess)
+        return -1;
+    uint32_t grid = resident_grid((const void*)k_merge_slow, P.num_sms);
+    k_merge_slow<<<grid, 256, 0, st>>>(T, M, lo, S.order, S.rank_lo, world, rank, S.bases, n_slow, S);
+    SHARD_CHECK();
+    return 2;
+}
+
+__global__ void k_sort_prep(const RepTuple* __restrict__ T, uint32_t M, uint64_t* keys, uint32_t* vals) {
+    uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= M) return;
+    keys[t] = T[t].gid;
+    vals[t] = t;
+}
+
+int launch_sort_prep(ShardWork& S, const RepTuple* T, uint32_t M, cudaStream_t st) {
+    if (!M) return 0;
+    k_sort_prep<<<blocks_for(M), 256, 0, st>>>(T, M, S.sort_keys_in, S.sort_vals_in);
+    SHARD_CHECK();
+    return 1;
+}
+
+size_t sort_tmp_bytes(uint32_t M) {
+    size_t bytes = 0;
+    cub::DeviceRadixSort::SortPairs(nullptr, bytes, (const uint64_t*)nullptr, (uint64_t*)nullptr,
+                                    (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)M, 0, 64);
+    return bytes;
+}
+
+int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
+                       uint64_t* ben_out, cudaStream_t st) {
+    if (L.n == 0) return cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * 8, st) == cudaSuccess ? 0 : -1;
+    const size_t smem = (size_t)n_sites * sizeof(uint64_t);
+    if (W.label_part && smem <= (size_t)P.max_smem) {
+        static int configured = 0;
+        if (!configured) {
+            if (cudaFuncSetAttribute(k_merge_label, cudaFuncAttributeMaxDynamicSharedMemorySize, P.max_smem) !=
+                cudaSuccess)
+                return -1;
+            configured = 1;
+        }
+        const uint32_t rows = label_hist_rows(P.num_sms);
+        k_merge_label<<<rows, 512, smem, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, W.label_part, nullptr);
+        SHARD_CHECK();
+        return 1 + launch_site_reduce(W.label_part, rows, n_sites, ben_out, st);
+    }
+    if (cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
+    k_merge_label<<<(uint32_t)P.num_sms * 4, 512, 0, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, nullptr,
+                                                           ben_out);
+    SHARD_CHECK();
+    return 1;
+}
+
+}  // namespace ffm
