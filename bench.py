@@ -111,27 +111,40 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
-def make_log(workload, n_scale, size_scale):
+def make_log(workload, n_scale, size_scale, shard=(0, 1)):
+    """The workload's log; with shard=(rank, world) > 1 only that rank's records'
+    contents are materialised (site-affinity LPT plan) -- lg.shard_idx lists them."""
     import loggen
+    import paper_conf_sc_weltonm19_b200 as ffm
     t = time.time()
     lg = loggen.gen_config(workload, n_scale=n_scale, size_scale=size_scale)
-    lg.materialize(nthreads=0)
+    rank, world = shard
+    if world > 1:
+        ranks = ffm.ffm_shard_plan(lg.site, lg.size, lg.n_sites, world, ffm.FFM_SHARD_SITE_LPT)
+        lg.shard_idx = np.nonzero(ranks == rank)[0]
+        lg.materialize(nthreads=0, records=lg.shard_idx)
+    else:
+        lg.shard_idx = np.arange(lg.n)
+        lg.materialize(nthreads=0)
     log_msg(f"[bench] generated {lg.name}: {lg.n} records, {lg.total_bytes / 1e9:.2f} GB payload, "
             f"{lg.distinct_bytes / 1e9:.2f} GB distinct, {time.time() - t:.1f}s")
     return lg
 
 
-def alg_bytes(lg, dup, small_bytes):
-    """Algorithmic bytes per kernel."""
-    size = lg.size.astype(np.int64)
+def alg_bytes(lg, idx, dup, small_bytes):
+    """Algorithmic bytes per kernel for this rank's records idx.
+    dup: this rank's duplicate_of (global gids).  Leaders with >= 1 member are counted
+    once (the other members re-read them from L2); remote leaders are NVLink bytes."""
+    size = lg.size[idx].astype(np.int64)
     n = len(size)
     small = size <= small_bytes
     member = dup >= 0
-    # leaders with >=1 member, counted once (their bytes are re-read from L2 by the others)
     leaders = np.zeros(n, bool)
     if member.any():
-        gid_to_idx = np.arange(n)           # single-GPU: gid == local index
-        leaders[gid_to_idx[dup[member]]] = True
+        pos = np.full(lg.n, -1, np.int64)
+        pos[idx] = np.arange(n)
+        lp = pos[dup[member]]
+        leaders[lp[lp >= 0]] = True
     out = {
         "hash_small": int(size[small].sum()) + 8 * n + 24 * int(small.sum()),
         "hash_large": int(size[~small].sum()) + 40 * int(((size[~small] + 32767) // 32768).sum()),
@@ -155,79 +168,113 @@ def ncu_traffic(kernel):
 
 def run_ours(args):
     import torch
+    import torch.distributed as dist
     import paper_conf_sc_weltonm19_b200 as ffm
+    from paper_conf_sc_weltonm19_b200 import sharded
 
     rank, world, local = dist_env()
-    if world > 1:
-        raise SystemExit("multi-GPU sharded runs: see DESIGN.md 'Multi-GPU' (not enabled in this build)")
+    if os.environ.get("FFM_BENCH_SAME_DEVICE"):      # test hook: several ranks on one GPU
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    lg = make_log(args.workload, args.n_scale, args.size_scale)
-    total = lg.total_bytes
+    if world > 1:
+        backend = os.environ.get("FFM_BENCH_BACKEND", "nccl")   # gloo only to exercise N>1 on one GPU
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+    lg = make_log(args.workload, args.n_scale, args.size_scale, shard=(rank, world))
+    idx = lg.shard_idx
+    total = lg.total_bytes                      # the whole job's payload (strong scaling)
+    my_bytes = int(lg.size[idx].sum())
 
-    # ---- device-resident log: distinct contents uploaded once, records snapshotted by the library
+    # ---- device-resident log: this rank's distinct contents uploaded once, records
+    # snapshotted into the library's HBM arena
     t = time.time()
     content = torch.from_numpy(lg.buf).to(dev)
     ptrs = (lg.c_off[lg.content] + np.uint64(content.data_ptr())).astype(np.uint64)
-    log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=total + 128 * lg.n + (1 << 20),
-                     max_records=lg.n, timing=True)
-    log.append_batch(lg.site, lg.size, ptrs, lg.dur, payload_kind=ffm.FFM_PAYLOAD_DEVICE)
+    log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * len(idx) + (1 << 20),
+                     max_records=len(idx), timing=True, rank=rank, world=world)
+    log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE,
+                   gids=idx if world > 1 else None, idx=idx if world > 1 else None)
     del content
     torch.cuda.synchronize()
     torch.cuda.empty_cache()
-    log_msg(f"[bench] staged {total / 1e9:.2f} GB into the HBM arena in {time.time() - t:.1f}s")
+    if world > 1:
+        sharded.exchange_handles(log)
+    log_msg(f"[bench] rank {rank}: staged {my_bytes / 1e9:.2f} GB ({len(idx)} records) into HBM "
+            f"in {time.time() - t:.1f}s")
 
-    dup = torch.empty(lg.n, dtype=torch.int64, device=dev)
+    dup = torch.empty(max(len(idx), 1), dtype=torch.int64, device=dev)
     ben = torch.empty(lg.n_sites, dtype=torch.int64, device=dev)
+    reps = torch.empty((max(len(idx), 1), ffm.REP_WORDS), dtype=torch.int64, device=dev)
+
+    def step():
+        if world > 1:
+            sharded.dedup_sharded(log, dev, duplicate_of=dup, benefit=ben, reps_buf=reps)
+        else:
+            log.run(dup, ben)
+
     stream = torch.cuda.ExternalStream(log.stream, device=dev)
     for _ in range(args.warmup):
-        log.run(dup, ben)
+        step()
     torch.cuda.synchronize()
-    clocks = ClockSampler(local)
-    clocks.start()
-    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    clocks = ClockSampler(local) if rank == 0 else None
+    if clocks:
+        clocks.start()
+        time.sleep(0.3)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     acc = {}
     torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
     e0.record(stream)
     for _ in range(args.steps):
-        log.run(dup, ben)
+        step()
         for k, v in log.stats().items():
             acc[k] = acc.get(k, 0) + v
     e1.record(stream)
     torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1) / args.steps
-    clk = clocks.stop()
+    ms_local = e0.elapsed_time(e1) / args.steps
+    ms = ms_local
+    if world > 1:
+        t_ms = torch.tensor([ms_local], dtype=torch.float64, device=dev)
+        dist.all_reduce(t_ms, op=dist.ReduceOp.MAX)
+        ms = float(t_ms.item())
+    clk = clocks.stop() if clocks else None
     st = {k: v / args.steps for k, v in acc.items()}
     value = total / (ms * 1e-3) / 1e9
 
-    dup_h = dup.cpu().numpy()
-    ab = alg_bytes(lg, dup_h, 4096)
+    # algorithmic bytes and the dominant kernel on this rank (rank 0 reports)
+    dup_h = dup[:len(idx)].cpu().numpy()
+    ab = alg_bytes(lg, idx, dup_h, 4096)
     peak, peak_src = load_peak()
-    kern_ms = {"hash_small": st["ms_hash_small"], "hash_large": st["ms_hash_large"],
-               "verify": st["ms_verify"]}
-    dom = max(("hash_large", "hash_small"), key=lambda k: kern_ms[k])
-    dom_bytes = ab[dom]
+    kern_ms = {"hash_small": st["ms_hash_small"], "hash_large": st["ms_hash_large"]}
+    dom = max(kern_ms, key=lambda k: kern_ms[k])
     dom_ms = kern_ms[dom]
-    achieved = dom_bytes / (dom_ms * 1e-3) / 1e9 if dom_ms > 0 else 0.0
+    achieved = ab[dom] / (dom_ms * 1e-3) / 1e9 if dom_ms > 0 else 0.0
     kname = {"hash_large": "k_hash_large", "hash_small": "k_hash_small"}[dom]
-    traffic = ncu_traffic(kname)
     roofline = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "traffic": traffic, "alg_bytes": dom_bytes,
-                "ms": round(dom_ms, 4), "peak_source": peak_src}
+                "frac": round(achieved / peak, 4), "traffic": ncu_traffic(kname), "alg_bytes": ab[dom],
+                "ms": round(dom_ms, 4), "peak_source": peak_src,
+                "read_stream_ceiling_gbs": read_ceiling()}
     path_gbs = ab["path"] / (ms * 1e-3) / 1e9
     launches = int(round(st["kernel_launches"])) * args.steps
 
-    # ---- end to end through the public ABI from pinned host buffers
     e2e = None
     if args.e2e_steps > 0:
         del log
         torch.cuda.empty_cache()
-        e2e = run_e2e(args, lg, local)
-
-    # ---- CPU oracle baseline (bounded gid-prefix sample, 1 core)
-    cpu = cpu_baseline(lg, args.cpu_seconds) if args.cpu_seconds > 0 else None
-
+        e2e = run_e2e(args, lg, local, rank, world)
+    cpu = cpu_baseline(lg, args.cpu_seconds) if (args.cpu_seconds > 0 and world == 1) else None
+    if world > 1:
+        dist.barrier()
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
     out = {
         "metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "strong",
@@ -236,47 +283,82 @@ def run_ours(args):
                    "n_sites": lg.n_sites, "seed": "0x5C19D1000%d" % args.workload,
                    "n_scale": args.n_scale, "size_scale": args.size_scale,
                    "l2": "inputs larger than L2 (payload %.1f GB >> 126 MB L2)" % (total / 1e9),
-                   "parallelism": "single GPU" if world == 1 else f"sharded x{world}",
+                   "parallelism": "single GPU" if world == 1 else
+                   f"{world} shards (site-affinity LPT); NCCL all-gather of class representatives, "
+                   "in-kernel peer byte verify over NVLink, NCCL all-reduce of benefit",
                    "chunk_bytes": 32768, "small_bytes": 4096},
         "pct_hbm_roofline_path": round(path_gbs / peak, 4),
         "path_alg_gbs": round(path_gbs, 1),
         "stage_ms": {k: round(st[k], 4) for k in ("ms_hash_small", "ms_hash_large", "ms_group", "ms_verify",
                                                   "ms_resolve", "ms_label", "ms_output", "ms_total")},
         "clocks": clk, "gpu_launches": launches, "roofline": roofline, "e2e": e2e, "cpu_baseline": cpu,
-        "duplicates": int((dup_h >= 0).sum()),
+        "duplicates_rank0": int((dup_h >= 0).sum()),
     }
     print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
 
 
-def run_e2e(args, lg, local):
+def read_ceiling():
+    try:
+        for line in open(os.path.join(ROOT, "profiles", "r01_hbm_ceiling.json")):
+            d = json.loads(line)
+            if d.get("test") == "read_stream_256b":
+                return d["gbs"]
+    except Exception:
+        return None
+
+
+def run_e2e(args, lg, local, rank=0, world=1):
     import torch
+    import torch.distributed as dist
     import paper_conf_sc_weltonm19_b200 as ffm
+    from paper_conf_sc_weltonm19_b200 import sharded
     buf = lg.buf
     cudart = torch.cuda.cudart()
-    reg = cudart.cudaHostRegister(buf.ctypes.data, buf.nbytes, 0)
-    ptrs = lg.payload_ptrs()
-    n = lg.n
-    dup = np.empty(n, np.int64)
-    ben = np.empty(lg.n_sites, np.uint64)
-    dup_pin = torch.empty(n, dtype=torch.int64).pin_memory().numpy()
-    ben_pin = torch.empty(lg.n_sites, dtype=torch.int64).pin_memory().numpy().view(np.uint64)
+    try:
+        reg = int(cudart.cudaHostRegister(buf.ctypes.data, buf.nbytes, 0))
+    except Exception:
+        reg = -1
+    idx = lg.shard_idx
+    ptrs = lg.payload_ptrs()[idx]
+    n = len(idx)
+    my_bytes = int(lg.size[idx].sum())
+    dev = torch.device("cuda", local)
+    dup_pin = torch.empty(max(n, 1), dtype=torch.int64).pin_memory()
+    ben_pin = torch.empty(lg.n_sites, dtype=torch.int64).pin_memory()
     times = []
     for step in range(args.e2e_steps + 1):
         torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
         t0 = time.perf_counter()
-        with ffm.FfmLog(lg.n_sites, device=local, arena_bytes=lg.total_bytes + 128 * n + (1 << 20),
-                        max_records=n) as log:
-            log.append_batch(lg.site, lg.size, ptrs, lg.dur, payload_kind=ffm.FFM_PAYLOAD_HOST)
-            log.run(dup_pin, ben_pin)
+        with ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * n + (1 << 20),
+                        max_records=n, rank=rank, world=world) as log:
+            log.append_batch(lg.site[idx], lg.size[idx], ptrs, lg.dur[idx],
+                             gids=idx if world > 1 else None, payload_kind=ffm.FFM_PAYLOAD_HOST)
+            if world > 1:
+                sharded.exchange_handles(log)
+                d, b = sharded.dedup_sharded(log, dev)
+                dup_pin[:n].copy_(d[:n])
+                ben_pin.copy_(b)
+                dist.barrier()           # peers stop reading this arena before it is freed
+            else:
+                log.run(dup_pin.numpy(), ben_pin.numpy().view(np.uint64))
         t1 = time.perf_counter()
+        sec_step = t1 - t0
+        if world > 1:
+            tt = torch.tensor([sec_step], dtype=torch.float64, device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            sec_step = float(tt.item())
         if step > 0:                     # first step warms up
-            times.append(t1 - t0)
-    if int(reg) == 0:
+            times.append(sec_step)
+    if reg == 0:
         cudart.cudaHostUnregister(buf.ctypes.data)
     sec = statistics.median(times)
-    meta = n * (4 + 8 + 8)
+    meta = lg.n * (4 + 8 + 8) // max(world, 1)
     return {"value": round(lg.total_bytes / sec / 1e9, 3), "unit": UNIT,
-            "h2d_bytes_per_step": int(lg.total_bytes + meta), "d2h_bytes_per_step": int(8 * n + 8 * lg.n_sites),
+            "h2d_bytes_per_step": int(lg.total_bytes + meta * world), "d2h_bytes_per_step": int(8 * lg.n + 8 * lg.n_sites * world),
             "steps": len(times), "s_per_step": round(sec, 4),
             "note": "wall clock per step: create + append (pinned host -> HBM) + run + D2H, median"}
 

@@ -90,11 +90,24 @@ class Log:
         return int(self.c_size.sum())
 
     # ---- materialisation -------------------------------------------------
-    def materialize(self, nthreads: int = 0, buf: np.ndarray | None = None) -> np.ndarray:
-        """Fill every content into one host buffer (16-B aligned slots)."""
+    def needed_contents(self, records: np.ndarray) -> np.ndarray:
+        """Content ids used by `records`, closed under derivation bases."""
+        need = np.zeros(len(self.c_size), bool)
+        need[np.unique(self.content[records])] = True
+        for c in range(len(self.c_base) - 1, -1, -1):       # bases have smaller ids
+            if need[c] and self.c_base[c] >= 0:
+                need[self.c_base[c]] = True
+        return need
+
+    def materialize(self, nthreads: int = 0, buf: np.ndarray | None = None,
+                    records: np.ndarray | None = None) -> np.ndarray:
+        """Fill the contents into one host buffer (16-B aligned slots).  With
+        `records`, only the contents those records use (one shard's share)."""
         if self.buf is not None:
             return self.buf
         sz = self.c_size.astype(np.uint64)
+        if records is not None:
+            sz = np.where(self.needed_contents(records), sz, np.uint64(0)).astype(np.uint64)
         slot = (sz + np.uint64(15)) // np.uint64(16) * np.uint64(16)
         off = np.zeros(len(sz), dtype=np.uint64)
         if len(sz) > 1:

@@ -98,7 +98,7 @@ int loggen_materialize(int64_t m, const int32_t* kind, const uint64_t* seed,
     /* pass 2: derived contents in id order (base < c), copy + flips */
     for (int64_t c = 0; c < m; ++c) {
         int64_t b = base[c];
-        if (b < 0) continue;
+        if (b < 0 || size[c] == 0) continue;     /* size 0: not materialised (subset) */
         if (b >= c || size[b] != size[c]) return -1;
         uint8_t* d = out + off[c];
         const uint8_t* s = out + off[b];
