@@ -327,32 +327,38 @@ def run_e2e(args, lg, local, rank=0, world=1):
     dev = torch.device("cuda", local)
     dup_pin = torch.empty(max(n, 1), dtype=torch.int64).pin_memory()
     ben_pin = torch.empty(lg.n_sites, dtype=torch.int64).pin_memory()
-    times = []
+    times, phases = [], []
     for step in range(args.e2e_steps + 1):
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
-        with ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * n + (1 << 20),
-                        max_records=n, rank=rank, world=world) as log:
-            log.append_batch(lg.site[idx], lg.size[idx], ptrs, lg.dur[idx],
-                             gids=idx if world > 1 else None, payload_kind=ffm.FFM_PAYLOAD_HOST)
-            if world > 1:
-                sharded.exchange_handles(log)
-                d, b = sharded.dedup_sharded(log, dev)
-                dup_pin[:n].copy_(d[:n])
-                ben_pin.copy_(b)
-                dist.barrier()           # peers stop reading this arena before it is freed
-            else:
-                log.run(dup_pin.numpy(), ben_pin.numpy().view(np.uint64))
+        log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * n + (1 << 20),
+                         max_records=n, rank=rank, world=world)
         t1 = time.perf_counter()
-        sec_step = t1 - t0
+        log.append_batch(lg.site[idx], lg.size[idx], ptrs, lg.dur[idx],
+                         gids=idx if world > 1 else None,
+                         payload_kind=ffm.FFM_PAYLOAD_HOST_PINNED if reg == 0 else ffm.FFM_PAYLOAD_HOST)
+        t2 = time.perf_counter()
+        if world > 1:
+            sharded.exchange_handles(log)
+            d, b = sharded.dedup_sharded(log, dev)
+            dup_pin[:n].copy_(d[:n])
+            ben_pin.copy_(b)
+            dist.barrier()           # peers stop reading this arena before it is freed
+        else:
+            log.run(dup_pin.numpy(), ben_pin.numpy().view(np.uint64))
+        t3 = time.perf_counter()
+        log.close()
+        t4 = time.perf_counter()
+        sec_step = t4 - t0
         if world > 1:
             tt = torch.tensor([sec_step], dtype=torch.float64, device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             sec_step = float(tt.item())
         if step > 0:                     # first step warms up
             times.append(sec_step)
+            phases.append((t1 - t0, t2 - t1, t3 - t2, t4 - t3))
     if reg == 0:
         cudart.cudaHostUnregister(buf.ctypes.data)
     sec = statistics.median(times)
@@ -360,6 +366,8 @@ def run_e2e(args, lg, local, rank=0, world=1):
     return {"value": round(lg.total_bytes / sec / 1e9, 3), "unit": UNIT,
             "h2d_bytes_per_step": int(lg.total_bytes + meta * world), "d2h_bytes_per_step": int(8 * lg.n + 8 * lg.n_sites * world),
             "steps": len(times), "s_per_step": round(sec, 4),
+            "phases_s": dict(zip(("create", "append_h2d", "run", "destroy"),
+                                 [round(statistics.median(p), 4) for p in zip(*phases)])),
             "note": "wall clock per step: create + append (pinned host -> HBM) + run + D2H, median"}
 
 

@@ -44,7 +44,11 @@ typedef enum ffm_status {
 typedef struct ffm_log ffm_log;
 
 /* payload_kind for ffm_log_append_batch */
-enum { FFM_PAYLOAD_AUTO = 0, FFM_PAYLOAD_HOST = 1, FFM_PAYLOAD_DEVICE = 2 };
+enum { FFM_PAYLOAD_AUTO = 0,        /* detected per pointer (cudaPointerGetAttributes) */
+       FFM_PAYLOAD_HOST = 1,        /* pageable host memory: copied through a pinned staging ring */
+       FFM_PAYLOAD_DEVICE = 2,      /* device memory on cfg->device: gathered by a kernel / D2D */
+       FFM_PAYLOAD_HOST_PINNED = 3  /* page-locked (cudaHostAlloc / cudaHostRegister) host memory:
+                                       read over PCIe by the gather kernel or the copy engines */ };
 
 /* ffm_config.flags */
 enum { FFM_FLAG_TIMING = 1u /* record per-stage CUDA events (ffm_last_run_stats) */ };
@@ -61,7 +65,7 @@ typedef struct ffm_config {
                               results never change.  0 => group by size alone. */
     uint32_t refine_bits;  /* 64 normally; < 64 weakens the first collision-resolution
                               re-key (test knob for the worst-case resolve path). */
-    uint32_t chunk_bytes;  /* large-payload work unit, multiple of 512; 0 => 32768.
+    uint32_t chunk_bytes;  /* large-payload work unit, multiple of 1024; 0 => 32768.
                               Results never change. */
     uint32_t small_bytes;  /* payloads <= this are hashed/verified one per 8-lane group;
                               multiple of 128; 0 => 4096.  Results never change. */

@@ -20,7 +20,7 @@ from ._build import LIB as _LIB_PATH
 
 FFM_OK, FFM_E_INVAL, FFM_E_RANGE, FFM_E_NOMEM, FFM_E_CUDA, FFM_E_COMM, FFM_E_STATE, FFM_E_NODEV = \
     0, -1, -2, -3, -4, -5, -6, -7
-FFM_PAYLOAD_AUTO, FFM_PAYLOAD_HOST, FFM_PAYLOAD_DEVICE = 0, 1, 2
+FFM_PAYLOAD_AUTO, FFM_PAYLOAD_HOST, FFM_PAYLOAD_DEVICE, FFM_PAYLOAD_HOST_PINNED = 0, 1, 2, 3
 FFM_FLAG_TIMING = 1
 
 # every symbol include/ffm.h declares (checked by tests/test_abi.py)

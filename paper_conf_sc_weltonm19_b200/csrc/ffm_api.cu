@@ -3,6 +3,7 @@
 // poisons the handle.  There is no CPU fallback: without a device, create fails.
 #include <cuda_runtime.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -18,7 +19,7 @@ namespace {
 
 constexpr uint64_t kRingBytes = 16ull << 20;      // per half of the pinned staging ring
 constexpr uint64_t kDirectCopy = 4ull << 20;      // host payloads above this bypass the ring
-constexpr uint64_t kGatherMax = 1ull << 20;       // device payloads up to this use k_gather
+constexpr uint64_t kGatherMaxDefault = 1ull << 20;   // payloads up to this use k_gather (not DMA)
 
 struct LocalRun {
     uint64_t n_members, n_res_total, rounds;
@@ -108,9 +109,10 @@ void ensure_arena(ffm_log* L, uint64_t need) {
 
 void stage_host(ffm_log* L, const void* src, uint64_t size, uint64_t off) {
     if (size > kDirectCopy) {
+        // pageable source: cudaMemcpyAsync returns once the bytes are in the driver's
+        // staging memory, so the snapshot is taken before return without a sync
         ring_flush(L);
         ck(cudaMemcpyAsync(L->arena + off, src, size, cudaMemcpyHostToDevice, L->stage_stream), "H2D");
-        ck(cudaStreamSynchronize(L->stage_stream), "H2D sync");   // snapshot before return
         return;
     }
     if (L->ring_fill && (off < L->ring_arena_start || off + size - L->ring_arena_start > L->ring_bytes))
@@ -118,6 +120,18 @@ void stage_host(ffm_log* L, const void* src, uint64_t size, uint64_t off) {
     if (!L->ring_fill) L->ring_arena_start = off;
     memcpy(L->ring[L->ring_cur] + (off - L->ring_arena_start), src, size);
     L->ring_fill = off + size - L->ring_arena_start;
+}
+
+// FFM_PAYLOAD_DEVICE / _HOST_PINNED / _HOST (pageable) of one pointer.
+int pointer_kind(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return FFM_PAYLOAD_HOST;
+    }
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return FFM_PAYLOAD_DEVICE;
+    if (a.type == cudaMemoryTypeHost) return FFM_PAYLOAD_HOST_PINNED;
+    return FFM_PAYLOAD_HOST;
 }
 
 bool is_device_ptr(const void* p) {
@@ -536,6 +550,11 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
         }
         ck(cudaDeviceGetAttribute(&L->params.num_sms, cudaDevAttrMultiProcessorCount, L->device), "attr");
         ck(cudaDeviceGetAttribute(&L->params.max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, L->device), "attr");
+        int hp = 0;
+        ck(cudaDeviceGetAttribute(&hp, cudaDevAttrCanUseHostPointerForRegisteredMem, L->device), "attr");
+        L->host_ptr_ok = hp != 0;
+        L->gather_max = kGatherMaxDefault;
+        if (const char* e = getenv("FFM_GATHER_MAX")) L->gather_max = strtoull(e, nullptr, 10);   // tuning knob
         L->params.chunk_bytes = chunk;
         L->params.small_bytes = small;
         L->params.digest_mask = cfg->digest_bits >= 64 ? ~0ull : ((1ull << cfg->digest_bits) - 1);
@@ -584,7 +603,7 @@ int ffm_log_append_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const ui
     if (st) return st;
     if (n == 0) return FFM_OK;
     if (!sites || !sizes || !payloads || !durs) return set_err(L, FFM_E_INVAL, "NULL array");
-    if (kind < FFM_PAYLOAD_AUTO || kind > FFM_PAYLOAD_DEVICE) return set_err(L, FFM_E_INVAL, "bad payload_kind");
+    if (kind < FFM_PAYLOAD_AUTO || kind > FFM_PAYLOAD_HOST_PINNED) return set_err(L, FFM_E_INVAL, "bad payload_kind");
     std::vector<uint64_t> offs;
     uint64_t end = 0;
     int rc = plan_batch(L, n, sites, sizes, payloads, gids, offs, end);
@@ -593,22 +612,23 @@ int ffm_log_append_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const ui
         ck(cudaSetDevice(L->device), "cudaSetDevice");
         ensure_arena(L, end);
         std::vector<uint64_t> desc;
-        bool any_device = false;
+        bool need_sync = false;
         for (uint64_t i = 0; i < n; ++i) {
             if (sizes[i] == 0) continue;
-            bool dev = kind == FFM_PAYLOAD_DEVICE || (kind == FFM_PAYLOAD_AUTO && is_device_ptr(payloads[i]));
+            int src = kind;
+            if (kind == FFM_PAYLOAD_AUTO) src = pointer_kind(payloads[i]);
+            const bool ring = src == FFM_PAYLOAD_HOST;        // pageable host: via the pinned ring
             // the ring uploads one contiguous arena range: close it before a record that
             // is written into the arena by another path
-            if (dev && L->ring_fill) ring_flush(L);
-            if (!dev) {
+            if (!ring && L->ring_fill) ring_flush(L);
+            if (ring) {
                 stage_host(L, payloads[i], sizes[i], offs[i]);
-            } else if (sizes[i] > kGatherMax) {
-                any_device = true;
-                ck(cudaMemcpyAsync(L->arena + offs[i], payloads[i], sizes[i], cudaMemcpyDeviceToDevice,
-                                   L->stage_stream),
-                   "D2D");
+            } else if (sizes[i] > L->gather_max || (src == FFM_PAYLOAD_HOST_PINNED && !L->host_ptr_ok)) {
+                need_sync = true;     // async copy engine from caller memory: sync before return
+                ck(cudaMemcpyAsync(L->arena + offs[i], payloads[i], sizes[i], cudaMemcpyDefault, L->stage_stream),
+                   "copy");
             } else {
-                any_device = true;
+                need_sync = true;     // k_gather reads caller memory (HBM, or pinned host over PCIe)
                 desc.push_back((uint64_t)(uintptr_t)payloads[i]);
                 desc.push_back(offs[i]);
                 desc.push_back(sizes[i]);
@@ -629,7 +649,7 @@ int ffm_log_append_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const ui
             if (launch_gather(L->d_desc, (uint32_t)nd, L->arena, L->stage_stream) < 0)
                 throw CudaFail{cudaGetLastError(), "k_gather"};
         }
-        if (any_device) ck(cudaStreamSynchronize(L->stage_stream), "D2D sync");   // snapshot before return
+        if (need_sync) ck(cudaStreamSynchronize(L->stage_stream), "append sync");   // snapshot before return
         push_meta(L, n, sites, sizes, durs, gids, offs, end);
         L->digests_valid = false;
         if (n > 1) upload_meta(L);

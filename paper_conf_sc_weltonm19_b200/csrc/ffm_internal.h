@@ -144,6 +144,8 @@ struct ffm_log {
     cudaEvent_t fork_ev[4] = {};
     bool own_stream = false;
     bool poisoned = false;
+    bool host_ptr_ok = false;      // kernels may dereference registered host pointers
+    uint64_t gather_max = 0;       // payloads up to this are gathered by k_gather, above: DMA
     std::string last_error;
 
     // host metadata (authoritative), program order

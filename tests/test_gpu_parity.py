@@ -167,6 +167,27 @@ def test_single_appends_mixed_host_device(ffm):
     assert_same(lg, dup, ben)
 
 
+@pytest.mark.parametrize("kind", ["pinned", "auto_pinned", "pageable"])
+def test_host_payload_kinds(ffm, kind):
+    import torch
+    lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 16)
+    host = lg.materialize()
+    if kind != "pageable":
+        pinned = torch.from_numpy(host).pin_memory()
+        base = pinned.data_ptr()
+    else:
+        pinned, base = None, host.ctypes.data
+    ptrs = (lg.c_off[lg.content] + np.uint64(base)).astype(np.uint64)
+    pk = {"pinned": ffm.FFM_PAYLOAD_HOST_PINNED, "auto_pinned": ffm.FFM_PAYLOAD_AUTO,
+          "pageable": ffm.FFM_PAYLOAD_HOST}[kind]
+    with ffm.FfmLog(lg.n_sites) as log:
+        log.append_log(lg, ptrs=ptrs, payload_kind=pk)
+        if pinned is not None:
+            pinned.zero_()                       # snapshot taken: later writes are invisible
+        dup, ben = log.run()
+    assert_same(lg, dup, ben)
+
+
 def test_device_outputs(ffm):
     import torch
     lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 64)

@@ -1,0 +1,27 @@
+"""Small logs through every kernel (incl. collision resolve and the gather path), for
+compute-sanitizer memcheck / racecheck / synccheck."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import loggen  # noqa: E402
+import oracle  # noqa: E402
+import paper_conf_sc_weltonm19_b200 as ffm  # noqa: E402
+
+for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (2, 0.001, 1.0)]:
+    lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
+    want = oracle.dedup(lg)
+    for db, rb, dev in [(64, 64, False), (0, 64, True), (0, 0, False)]:
+        with ffm.FfmLog(lg.n_sites, digest_bits=db, refine_bits=rb, chunk_bytes=4096, small_bytes=1024) as log:
+            if dev:
+                buf = torch.from_numpy(lg.materialize()).cuda()
+                ptrs = (lg.c_off[lg.content] + np.uint64(buf.data_ptr())).astype(np.uint64)
+                log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE)
+            else:
+                log.append_log(lg)
+            d, b = log.run()
+            assert np.array_equal(d, want[0]) and np.array_equal(b, want[1]), (k, db, rb)
+print("sanitize smoke ok")
