@@ -147,6 +147,21 @@ typedef struct ffm_run_stats {
 /* Statistics of the last ffm_dedup_run. */
 int ffm_last_run_stats(const ffm_log* log, ffm_run_stats* out);
 
+/* Number of duplicates per call site in the last run ("Number of Transfer Issues",
+   Fig. 6), [n_sites] uint64, host or device.  For a sharded log these are
+   this rank's partial counts (all-reduce them like the benefit). */
+int ffm_site_duplicate_counts(ffm_log* log, uint64_t* counts_out);
+
+/* Folded grouping: group_values_out[g] = sum of site_values[s] over the
+   sites s with site_to_group[s] == g (uint64, mod 2^64), computed by a kernel on the
+   log's device.  site_values [n_sites] and site_to_group [n_sites] (host or device),
+   group_values_out [n_groups] (host or device).  The caller builds site_to_group by
+   folding each site's stack-trace function name: demangled, template parameters
+   discarded (paper_conf_sc_weltonm19_b200/report.py).  Errors: FFM_E_INVAL,
+   FFM_E_RANGE (a group id >= n_groups). */
+int ffm_fold_sites(ffm_log* log, const uint64_t* site_values, const uint32_t* site_to_group, uint32_t n_groups,
+                   uint64_t* group_values_out);
+
 /* Debug / conformance: copy the last run's 64-bit payload digests (host array [n]).
    The digest is specified in DESIGN.md "Digest"; it is an implementation detail
    and never part of the result. */

@@ -28,7 +28,7 @@ EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_appen
            "ffm_dedup_run", "ffm_log_count", "ffm_log_payload_bytes", "ffm_log_stream",
            "ffm_last_run_stats", "ffm_debug_digests", "ffm_log_destroy", "ffm_strerror",
            "ffm_last_error", "ffm_version", "ffm_shard_plan", "ffm_shard_ipc_handle", "ffm_shard_open_peer",
-           "ffm_shard_local", "ffm_shard_merge"]
+           "ffm_shard_local", "ffm_shard_merge", "ffm_site_duplicate_counts", "ffm_fold_sites"]
 FFM_SHARD_SITE_LPT, FFM_SHARD_CONTIGUOUS = 0, 1
 REP_WORDS = 4        # ffm_rep = {key, size, gid, off}, 4 x u64
 
@@ -109,6 +109,10 @@ def lib() -> ctypes.CDLL:
         L.ffm_shard_local.restype = i32
         L.ffm_shard_merge.argtypes = [vp, vp, vp, vp, vp]
         L.ffm_shard_merge.restype = i32
+        L.ffm_site_duplicate_counts.argtypes = [vp, vp]
+        L.ffm_site_duplicate_counts.restype = i32
+        L.ffm_fold_sites.argtypes = [vp, vp, vp, u32, vp]
+        L.ffm_fold_sites.restype = i32
         _lib = L
     return _lib
 
@@ -241,6 +245,23 @@ def ffm_shard_merge(h, all_reps, counts, duplicate_of, benefit_partial):
     _check(h, lib().ffm_shard_merge(h, _addr(all_reps), _addr(c), _addr(duplicate_of), _addr(benefit_partial)))
 
 
+def ffm_site_duplicate_counts(h, n_sites: int, out=None):
+    if out is None:
+        out = np.empty(n_sites, np.uint64)
+    _check(h, lib().ffm_site_duplicate_counts(h, _addr(out)))
+    return out
+
+
+def ffm_fold_sites(h, site_values, site_to_group, n_groups: int, out=None):
+    sv = site_values if not isinstance(site_values, np.ndarray) else np.ascontiguousarray(site_values, np.uint64)
+    mp = site_to_group if not isinstance(site_to_group, np.ndarray) else \
+        np.ascontiguousarray(site_to_group, np.uint32)
+    if out is None:
+        out = np.empty(n_groups, np.uint64)
+    _check(h, lib().ffm_fold_sites(h, _addr(sv), _addr(mp), n_groups, _addr(out)))
+    return out
+
+
 # ---- convenience wrapper ----------------------------------------------------
 class FfmLog:
     """Owns one ffm_log handle."""
@@ -301,6 +322,12 @@ class FfmLog:
 
     def digests(self):
         return ffm_debug_digests(self.h)
+
+    def site_counts(self, out=None):
+        return ffm_site_duplicate_counts(self.h, self.n_sites, out)
+
+    def fold(self, site_values, site_to_group, n_groups, out=None):
+        return ffm_fold_sites(self.h, site_values, site_to_group, n_groups, out)
 
     def close(self):
         if self.h:

@@ -269,8 +269,11 @@ void ensure_work(ffm_log* L, uint64_t n) {
     }
     if (L->cfg.n_sites > W.site_cap) {
         dev_alloc(W.ben, L->cfg.n_sites);
-        if ((uint64_t)L->cfg.n_sites * 8 <= (uint64_t)L->params.max_smem)
+        dev_alloc(W.cnt, L->cfg.n_sites);
+        if (label_smem_bytes(L->cfg.n_sites) <= (uint64_t)L->params.max_smem) {
             dev_alloc(W.label_part, (uint64_t)label_hist_rows(L->params.num_sms) * L->cfg.n_sites);
+            dev_alloc(W.label_cpart, (uint64_t)label_hist_rows(L->params.num_sms) * L->cfg.n_sites);
+        }
         W.site_cap = L->cfg.n_sites;
     }
 }
@@ -319,7 +322,7 @@ void run_prologue(ffm_log* L) {
 // leader (the min local index of its exact byte class).  With `label` the H5/H6
 // kernels are queued before the first sync (single-GPU fast path: one sync when
 // there are no digest collisions) and re-run after collision resolution.
-LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup, uint64_t* d_ben) {
+LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup) {
     const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
     const uint64_t n = L->h_size.size();
     Work& W = L->work;
@@ -355,7 +358,7 @@ LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup, u
                        L->fork_ev[2], L->fork_ev[3]));
     if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
     // H5 + H6 (speculative: valid unless H3 found residuals)
-    if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, d_ben, s));
+    if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, s));
     if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
     ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
     ck(cudaStreamSynchronize(s), "run sync");
@@ -380,7 +383,7 @@ LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup, u
             R.n_res_total += nres;
             cur ^= 1;
         }
-        if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, d_ben, s));
+        if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, s));
         if (timing) ck(cudaEventRecord(L->ev[7], s), "event");
     }
     return R;
@@ -690,16 +693,17 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         bool dup_dev = dup_out && is_device_ptr(dup_out);
         bool ben_dev = ben_out && is_device_ptr(ben_out);
         int64_t* d_dup = dup_dev ? dup_out : W.dup;
-        uint64_t* d_ben = ben_dev ? ben_out : W.ben;
         uint64_t launches = 0;
-        LocalRun R = run_local(L, launches, true, d_dup, d_ben);
+        LocalRun R = run_local(L, launches, true, d_dup);
         // H7 return
         const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
         if (timing) ck(cudaEventRecord(L->ev[9], s), "event");
         if (!dup_dev && n)
             ck(cudaMemcpyAsync(dup_out, d_dup, n * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
-        if (ben_out && !ben_dev)
-            ck(cudaMemcpyAsync(ben_out, d_ben, ns * sizeof(uint64_t), cudaMemcpyDeviceToHost, s), "D2H ben");
+        if (ben_out)
+            ck(cudaMemcpyAsync(ben_out, W.ben, ns * sizeof(uint64_t),
+                               ben_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s),
+               "copy ben");
         if (timing) ck(cudaEventRecord(L->ev[5], s), "event");
         ck(cudaStreamSynchronize(s), "output sync");
         ck(cudaGetLastError(), "run");
@@ -765,7 +769,7 @@ int ffm_shard_local(ffm_log* L, ffm_rep* reps_out, uint64_t cap, uint64_t* n_rep
     try {
         run_prologue(L);
         uint64_t launches = 0;
-        LocalRun R = run_local(L, launches, false, nullptr, nullptr);
+        LocalRun R = run_local(L, launches, false, nullptr);
         ensure_shard(L, n, 1, 1, 1, std::max(L->cfg.world, 1));
         DevLog D = dev_view(L);
         cudaStream_t s = L->stream;
@@ -840,13 +844,12 @@ int ffm_shard_merge(ffm_log* L, const ffm_rep* all_reps, const uint64_t* counts,
         bool dup_dev = dup_out && is_device_ptr(dup_out);
         bool ben_dev = is_device_ptr(ben_out);
         int64_t* d_dup = dup_dev ? dup_out : W.dup;
-        uint64_t* d_ben = ben_dev ? ben_out : W.ben;
-        LCHK(launch_merge_label(D, W, S, L->params, L->cfg.n_sites, d_dup, d_ben, s));
+        LCHK(launch_merge_label(D, W, S, L->params, L->cfg.n_sites, d_dup, s));
         if (!dup_dev && n)
             ck(cudaMemcpyAsync(dup_out, d_dup, n * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
-        if (!ben_dev)
-            ck(cudaMemcpyAsync(ben_out, d_ben, L->cfg.n_sites * sizeof(uint64_t), cudaMemcpyDeviceToHost, s),
-               "D2H ben");
+        ck(cudaMemcpyAsync(ben_out, W.ben, L->cfg.n_sites * sizeof(uint64_t),
+                           ben_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s),
+           "copy ben");
         if (timing) ck(cudaEventRecord(L->ev[14], s), "event");
         ck(cudaStreamSynchronize(s), "merge output sync");
         ck(cudaGetLastError(), "merge");
@@ -856,6 +859,59 @@ int ffm_shard_merge(ffm_log* L, const ffm_rep* all_reps, const uint64_t* counts,
             L->stats.ms_output = ev_ms(L->ev[13], L->ev[14]);
             L->stats.ms_total = ev_ms(L->ev[0], L->ev[14]);
         }
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    } catch (const std::bad_alloc&) {
+        return set_err(L, FFM_E_NOMEM, "host allocation failed");
+    }
+    return FFM_OK;
+}
+
+int ffm_site_duplicate_counts(ffm_log* L, uint64_t* counts_out) {
+    int st = check_state(L);
+    if (st) return st;
+    if (!counts_out) return FFM_E_INVAL;
+    if (!L->digests_valid || !L->work.cnt) return set_err(L, FFM_E_STATE, "no run since the last append");
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        ck(cudaMemcpyAsync(counts_out, L->work.cnt, L->cfg.n_sites * sizeof(uint64_t), cudaMemcpyDefault,
+                           L->stream),
+           "copy counts");
+        ck(cudaStreamSynchronize(L->stream), "sync");
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    }
+    return FFM_OK;
+}
+
+int ffm_fold_sites(ffm_log* L, const uint64_t* site_values, const uint32_t* site_to_group, uint32_t n_groups,
+                   uint64_t* group_values_out) {
+    int st = check_state(L);
+    if (st) return st;
+    const uint32_t ns = L->cfg.n_sites;
+    if (!site_values || !site_to_group || !group_values_out || n_groups == 0) return FFM_E_INVAL;
+    std::vector<uint32_t> map(ns);
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        cudaStream_t s = L->stream;
+        ck(cudaMemcpy(map.data(), site_to_group, ns * sizeof(uint32_t), cudaMemcpyDefault), "copy map");
+        for (uint32_t i = 0; i < ns; ++i)
+            if (map[i] >= n_groups) return set_err(L, FFM_E_RANGE, "site_to_group[s] >= n_groups");
+        uint64_t need = (uint64_t)ns * 8 + (uint64_t)ns * 4 + (uint64_t)n_groups * 8;
+        if (need > L->fold_cap) {
+            if (L->fold_buf) ck(cudaFree(L->fold_buf), "cudaFree");
+            L->fold_buf = nullptr;
+            ck(cudaMalloc(&L->fold_buf, need), "cudaMalloc(fold)");
+            L->fold_cap = need;
+        }
+        uint64_t* d_vals = (uint64_t*)L->fold_buf;
+        uint64_t* d_out = d_vals + ns;
+        uint32_t* d_map = (uint32_t*)(d_out + n_groups);
+        ck(cudaMemcpyAsync(d_vals, site_values, ns * 8, cudaMemcpyDefault, s), "copy vals");
+        ck(cudaMemcpyAsync(d_map, map.data(), ns * 4, cudaMemcpyHostToDevice, s), "copy map");
+        if (launch_fold(d_vals, d_map, ns, d_out, n_groups, s) < 0) throw CudaFail{cudaGetLastError(), "k_fold"};
+        ck(cudaMemcpyAsync(group_values_out, d_out, (uint64_t)n_groups * 8, cudaMemcpyDefault, s), "copy out");
+        ck(cudaStreamSynchronize(s), "fold sync");
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
     } catch (const std::bad_alloc&) {
@@ -887,11 +943,12 @@ int ffm_log_destroy(ffm_log* L) {
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
                     W.lcount, W.lstart, W.gcount, W.pos, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
-                    W.dup, W.ben, W.label_part, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid,
+                    W.dup, W.ben, W.cnt, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid,
                     L->arena, L->d_desc};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     free_shard(L->shard);
+    if (L->fold_buf) cudaFree(L->fold_buf);
     for (void* p : L->peer_ptr)
         if (p) cudaIpcCloseMemHandle(p);
     for (int i = 0; i < 2; ++i) {

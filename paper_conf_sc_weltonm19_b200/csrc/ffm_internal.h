@@ -51,6 +51,8 @@ struct Work {
     int64_t* dup = nullptr;        // [n] output staging
     uint64_t* ben = nullptr;       // [n_sites]
     uint64_t* label_part = nullptr; // [label_hist_rows * n_sites] per-block benefit partials
+    uint32_t* label_cpart = nullptr; // [label_hist_rows * n_sites] per-block duplicate counts
+    uint64_t* cnt = nullptr;       // [n_sites] duplicates per site (last run)
     uint32_t* counters = nullptr;  // device counters: [0] nres, [1] n_members, [2..] misc
     void* cub_tmp = nullptr;
     size_t cub_tmp_bytes = 0;
@@ -112,10 +114,13 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
 int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
                   uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st, cudaStream_t side, cudaEvent_t ev_fork,
                   cudaEvent_t ev_join);
-int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out,
-                 uint64_t* ben_out, cudaStream_t st);
+int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out, cudaStream_t st);
+size_t label_smem_bytes(uint32_t n_sites);
+int launch_fold(const uint64_t* site_vals, const uint32_t* site_to_group, uint32_t n_sites, uint64_t* group_vals,
+                uint32_t n_groups, cudaStream_t st);
 uint32_t label_hist_rows(int num_sms);
-int launch_site_reduce(const uint64_t* part, uint32_t rows, uint32_t n_sites, uint64_t* ben, cudaStream_t st);
+int launch_site_reduce(const uint64_t* part, const uint32_t* cpart, uint32_t rows, uint32_t n_sites, uint64_t* ben,
+                       uint64_t* cnt, cudaStream_t st);
 // shard.cu
 int launch_rep_export(const DevLog& L, Work& W, ShardWork& S, const Params& P, RepTuple* out, cudaStream_t st);
 int launch_merge(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
@@ -125,7 +130,7 @@ size_t sort_tmp_bytes(uint32_t M);
 int launch_merge_slow(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
                       uint32_t lo, int world, int rank, uint32_t n_slow, cudaStream_t st);
 int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
-                       uint64_t* ben_out, cudaStream_t st);
+                       cudaStream_t st);
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 size_t cub_scan_bytes(uint64_t n);
@@ -184,6 +189,10 @@ struct ffm_log {
     bool reps_valid = false;
     std::vector<void*> peer_ptr;    // IPC-mapped peer arenas (index = rank)
     std::vector<std::string> peer_handle;
+
+    // folded grouping scratch
+    void* fold_buf = nullptr;
+    uint64_t fold_cap = 0;
 
     // gather descriptors for device payloads
     uint64_t* d_desc = nullptr;

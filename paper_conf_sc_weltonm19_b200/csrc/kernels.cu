@@ -488,38 +488,68 @@ __global__ void k_refine(DevLog L, Work W, const uint32_t* __restrict__ list, ui
 // 10% of all records on one site) and a second kernel sums the block partials.
 // ----------------------------------------------------------------------------
 __global__ void __launch_bounds__(512) k_label_hist(DevLog L, const uint32_t* __restrict__ leader, uint32_t n_sites,
-                                                    int64_t* __restrict__ dup_out, uint64_t* __restrict__ part) {
+                                                    int64_t* __restrict__ dup_out, uint64_t* __restrict__ part,
+                                                    uint32_t* __restrict__ cpart) {
     extern __shared__ unsigned long long sben[];
-    for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) sben[s] = 0;
+    uint32_t* scnt = (uint32_t*)(sben + n_sites);
+    for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) {
+        sben[s] = 0;
+        scnt[s] = 0;
+    }
     __syncthreads();
     for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < L.n; r += gridDim.x * blockDim.x) {
         uint32_t ld = leader[r];
         int64_t d = ld == r ? -1 : (int64_t)L.gid[ld];
         dup_out[r] = d;
-        if (d >= 0) atomicAdd(&sben[L.site[r]], (unsigned long long)L.dur[r]);
+        if (d >= 0) {
+            const uint32_t s = L.site[r];
+            atomicAdd(&sben[s], (unsigned long long)L.dur[r]);
+            atomicAdd(&scnt[s], 1u);
+        }
     }
     __syncthreads();
     uint64_t* row = part + (uint64_t)blockIdx.x * n_sites;
-    for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) row[s] = sben[s];
+    uint32_t* crow = cpart + (uint64_t)blockIdx.x * n_sites;
+    for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) {
+        row[s] = sben[s];
+        crow[s] = scnt[s];
+    }
 }
 
-__global__ void k_site_reduce(const uint64_t* __restrict__ part, uint32_t rows, uint32_t n_sites,
-                              uint64_t* __restrict__ ben) {
+__global__ void k_site_reduce(const uint64_t* __restrict__ part, const uint32_t* __restrict__ cpart, uint32_t rows,
+                              uint32_t n_sites, uint64_t* __restrict__ ben, uint64_t* __restrict__ cnt) {
     uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= n_sites) return;
-    uint64_t acc = 0;
-    for (uint32_t b = 0; b < rows; ++b) acc += part[(uint64_t)b * n_sites + s];
+    uint64_t acc = 0, c = 0;
+    for (uint32_t b = 0; b < rows; ++b) {
+        acc += part[(uint64_t)b * n_sites + s];
+        c += cpart[(uint64_t)b * n_sites + s];
+    }
     ben[s] = acc;
+    cnt[s] = c;
 }
 
 __global__ void __launch_bounds__(256) k_label_global(DevLog L, const uint32_t* __restrict__ leader,
-                                                      int64_t* __restrict__ dup_out, uint64_t* __restrict__ ben) {
+                                                      int64_t* __restrict__ dup_out, uint64_t* __restrict__ ben,
+                                                      uint64_t* __restrict__ cnt) {
     for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < L.n; r += gridDim.x * blockDim.x) {
         uint32_t ld = leader[r];
         int64_t d = ld == r ? -1 : (int64_t)L.gid[ld];
         dup_out[r] = d;
-        if (d >= 0) atomicAdd((unsigned long long*)&ben[L.site[r]], (unsigned long long)L.dur[r]);
+        if (d >= 0) {
+            atomicAdd((unsigned long long*)&ben[L.site[r]], (unsigned long long)L.dur[r]);
+            atomicAdd((unsigned long long*)&cnt[L.site[r]], 1ull);
+        }
     }
+}
+
+// Folded grouping (S8(f) #1): per-group sums of per-site values.
+__global__ void k_fold(const uint64_t* __restrict__ site_vals, const uint32_t* __restrict__ site_to_group,
+                       uint32_t n_sites, uint64_t* __restrict__ group_vals) {
+    uint32_t s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n_sites) return;
+    uint64_t v = site_vals[s];
+    if (v) atomicAdd((unsigned long long*)&group_vals[site_to_group[s]], (unsigned long long)v);
 }
 
 // ----------------------------------------------------------------------------
@@ -685,34 +715,49 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
 
 uint32_t label_hist_rows(int num_sms) { return (uint32_t)num_sms * 2; }
 
-int launch_site_reduce(const uint64_t* part, uint32_t rows, uint32_t n_sites, uint64_t* ben, cudaStream_t st) {
-    k_site_reduce<<<blocks_for(n_sites), 256, 0, st>>>(part, rows, n_sites, ben);
+int launch_site_reduce(const uint64_t* part, const uint32_t* cpart, uint32_t rows, uint32_t n_sites, uint64_t* ben,
+                       uint64_t* cnt, cudaStream_t st) {
+    k_site_reduce<<<blocks_for(n_sites), 256, 0, st>>>(part, cpart, rows, n_sites, ben, cnt);
     FFM_LAUNCH_CHECK();
     return 1;
 }
 
-int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out, uint64_t* ben_out,
-                 cudaStream_t st) {
-    if (L.n == 0) return cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * sizeof(uint64_t), st) == cudaSuccess ? 0 : -1;
-    const size_t smem = (size_t)n_sites * sizeof(uint64_t);
+size_t label_smem_bytes(uint32_t n_sites) { return (size_t)n_sites * (sizeof(uint64_t) + sizeof(uint32_t)); }
+
+int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out, cudaStream_t st) {
+    if (L.n == 0) {
+        if (cudaMemsetAsync(W.ben, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
+        return cudaMemsetAsync(W.cnt, 0, (uint64_t)n_sites * 8, st) == cudaSuccess ? 0 : -1;
+    }
+    const size_t smem = label_smem_bytes(n_sites);
     if (W.label_part && smem <= (size_t)P.max_smem) {
         static int configured_smem = 0;
-        if ((int)smem > configured_smem) {
+        if (!configured_smem) {
             if (cudaFuncSetAttribute(k_label_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, P.max_smem) !=
                 cudaSuccess)
                 return -1;
-            configured_smem = P.max_smem;
+            configured_smem = 1;
         }
         const uint32_t rows = label_hist_rows(P.num_sms);
-        k_label_hist<<<rows, 512, smem, st>>>(L, W.leader, n_sites, dup_out, W.label_part);
+        k_label_hist<<<rows, 512, smem, st>>>(L, W.leader, n_sites, dup_out, W.label_part, W.label_cpart);
         FFM_LAUNCH_CHECK();
-        if (launch_site_reduce(W.label_part, rows, n_sites, ben_out, st) < 0) return -1;
+        if (launch_site_reduce(W.label_part, W.label_cpart, rows, n_sites, W.ben, W.cnt, st) < 0) return -1;
         return 2;
     }
-    if (cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(W.ben, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(W.cnt, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
     uint32_t grid = blocks_for(L.n);
     if (grid > (uint32_t)P.num_sms * 8) grid = (uint32_t)P.num_sms * 8;
-    k_label_global<<<grid, 256, 0, st>>>(L, W.leader, dup_out, ben_out);
+    k_label_global<<<grid, 256, 0, st>>>(L, W.leader, dup_out, W.ben, W.cnt);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
+int launch_fold(const uint64_t* site_vals, const uint32_t* site_to_group, uint32_t n_sites, uint64_t* group_vals,
+                uint32_t n_groups, cudaStream_t st) {
+    if (cudaMemsetAsync(group_vals, 0, (uint64_t)n_groups * 8, st) != cudaSuccess) return -1;
+    if (n_sites == 0) return 0;
+    k_fold<<<blocks_for(n_sites), 256, 0, st>>>(site_vals, site_to_group, n_sites, group_vals);
     FFM_LAUNCH_CHECK();
     return 1;
 }

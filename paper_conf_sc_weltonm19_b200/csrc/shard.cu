@@ -204,16 +204,21 @@ __global__ void __launch_bounds__(256) k_merge_slow(const RepTuple* __restrict__
 }
 
 // H5 + H6 for a shard: record r's class representative is its local leader; the
-// class's global leader G comes from the merge.  Benefit partial per rank.
+// class's global leader G comes from the merge.  Benefit / count partials per rank.
 __global__ void __launch_bounds__(512) k_merge_label(DevLog L, const uint32_t* __restrict__ leader,
                                                      const uint32_t* __restrict__ rep_idx,
                                                      const uint64_t* __restrict__ G, uint32_t n_sites,
                                                      int64_t* __restrict__ dup_out, uint64_t* __restrict__ part,
-                                                     uint64_t* __restrict__ ben_global) {
+                                                     uint32_t* __restrict__ cpart, uint64_t* __restrict__ ben_global,
+                                                     uint64_t* __restrict__ cnt_global) {
     extern __shared__ unsigned long long sben[];
+    uint32_t* scnt = (uint32_t*)(sben + n_sites);
     const bool hist = part != nullptr;
     if (hist) {
-        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) sben[s] = 0;
+        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) {
+            sben[s] = 0;
+            scnt[s] = 0;
+        }
         __syncthreads();
     }
     for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < L.n; r += gridDim.x * blockDim.x) {
@@ -221,16 +226,24 @@ __global__ void __launch_bounds__(512) k_merge_label(DevLog L, const uint32_t* _
         int64_t d = g == L.gid[r] ? -1 : (int64_t)g;
         dup_out[r] = d;
         if (d >= 0) {
-            if (hist)
-                atomicAdd(&sben[L.site[r]], (unsigned long long)L.dur[r]);
-            else
-                atomicAdd((unsigned long long*)&ben_global[L.site[r]], (unsigned long long)L.dur[r]);
+            const uint32_t s = L.site[r];
+            if (hist) {
+                atomicAdd(&sben[s], (unsigned long long)L.dur[r]);
+                atomicAdd(&scnt[s], 1u);
+            } else {
+                atomicAdd((unsigned long long*)&ben_global[s], (unsigned long long)L.dur[r]);
+                atomicAdd((unsigned long long*)&cnt_global[s], 1ull);
+            }
         }
     }
     if (hist) {
         __syncthreads();
         uint64_t* row = part + (uint64_t)blockIdx.x * n_sites;
-        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) row[s] = sben[s];
+        uint32_t* crow = cpart + (uint64_t)blockIdx.x * n_sites;
+        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) {
+            row[s] = sben[s];
+            crow[s] = scnt[s];
+        }
     }
 }
 
@@ -325,9 +338,12 @@ size_t sort_tmp_bytes(uint32_t M) {
 }
 
 int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
-                       uint64_t* ben_out, cudaStream_t st) {
-    if (L.n == 0) return cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * 8, st) == cudaSuccess ? 0 : -1;
-    const size_t smem = (size_t)n_sites * sizeof(uint64_t);
+                       cudaStream_t st) {
+    if (L.n == 0) {
+        if (cudaMemsetAsync(W.ben, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
+        return cudaMemsetAsync(W.cnt, 0, (uint64_t)n_sites * 8, st) == cudaSuccess ? 0 : -1;
+    }
+    const size_t smem = label_smem_bytes(n_sites);
     if (W.label_part && smem <= (size_t)P.max_smem) {
         static int configured = 0;
         if (!configured) {
@@ -337,13 +353,15 @@ int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, 
             configured = 1;
         }
         const uint32_t rows = label_hist_rows(P.num_sms);
-        k_merge_label<<<rows, 512, smem, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, W.label_part, nullptr);
+        k_merge_label<<<rows, 512, smem, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, W.label_part,
+                                               W.label_cpart, nullptr, nullptr);
         SHARD_CHECK();
-        return 1 + launch_site_reduce(W.label_part, rows, n_sites, ben_out, st);
+        return 1 + launch_site_reduce(W.label_part, W.label_cpart, rows, n_sites, W.ben, W.cnt, st);
     }
-    if (cudaMemsetAsync(ben_out, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(W.ben, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(W.cnt, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
     k_merge_label<<<(uint32_t)P.num_sms * 4, 512, 0, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, nullptr,
-                                                           ben_out);
+                                                           nullptr, W.ben, W.cnt);
     SHARD_CHECK();
     return 1;
 }

@@ -13,7 +13,7 @@ import torch
 import torch.distributed as dist
 
 from . import (REP_WORDS, ffm_log_count, ffm_shard_ipc_handle, ffm_shard_local, ffm_shard_merge,
-               ffm_shard_open_peer)
+               ffm_shard_open_peer, ffm_site_duplicate_counts)
 
 
 def _on_nccl(group=None) -> bool:
@@ -59,6 +59,13 @@ def allreduce_benefit(ben: torch.Tensor, group=None) -> torch.Tensor:
     dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
     ben.copy_(h)
     return ben
+
+
+def site_counts_sharded(log, device, group=None) -> torch.Tensor:
+    """All-reduced duplicates per call site of the last sharded run (int64 [n_sites])."""
+    c = torch.empty(log.n_sites, dtype=torch.int64, device=device)
+    ffm_site_duplicate_counts(log.h, log.n_sites, c)
+    return allreduce_benefit(c, group)
 
 
 def dedup_sharded(log, device, group=None, duplicate_of=None, benefit=None, reps_buf=None):

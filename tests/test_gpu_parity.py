@@ -249,3 +249,30 @@ def test_full_size_configs_1_to_3(ffm, k):
         np.testing.assert_array_equal(dup0, dup)
         np.testing.assert_array_equal(ben0, ben)
         assert st0["n_residual"] > 0
+
+
+def test_site_counts_and_fold(ffm):
+    from paper_conf_sc_weltonm19_b200 import report
+    lg = loggen.gen_config(5, n_scale=0.003, size_scale=1 / 32)
+    want_dup, want_ben = oracle.dedup(lg)
+    want_cnt = np.bincount(lg.site[want_dup >= 0].astype(np.int64), minlength=lg.n_sites).astype(np.uint64)
+    rng = np.random.default_rng(1)
+    gmap = rng.integers(0, 37, lg.n_sites).astype(np.uint32)
+    with ffm.FfmLog(lg.n_sites) as log:
+        log.append_log(lg)
+        dup, ben = log.run()
+        cnt = log.site_counts()
+        np.testing.assert_array_equal(cnt, want_cnt)
+        g = log.fold(ben, gmap, 37)
+        np.testing.assert_array_equal(log.fold(ben, np.arange(lg.n_sites, dtype=np.uint32), lg.n_sites), ben)
+        np.testing.assert_array_equal(log.fold(ben, np.zeros(lg.n_sites, np.uint32), 1),
+                                      [int(ben.sum(dtype=np.uint64))])
+        names = [f"site{s}" for s in range(lg.n_sites)]
+        funcs = [f"ns::fn{s % 7}<T{s % 3}>(int)" for s in range(lg.n_sites)]
+        rep = report.ranked_report(ben, names, cnt, funcs, fold=log.fold, exec_time_ns=10**12)
+    want_g = np.zeros(37, np.uint64)
+    np.add.at(want_g, gmap.astype(np.int64), want_ben)
+    np.testing.assert_array_equal(g, want_g)
+    assert rep["total"]["benefit_ns"] == int(want_ben.sum(dtype=np.uint64))
+    assert len(rep["folded_function"]) <= 7
+    assert sum(r["benefit_ns"] for r in rep["folded_function"]) == rep["total"]["benefit_ns"]

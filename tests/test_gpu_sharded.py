@@ -62,9 +62,10 @@ def _worker(rank, world, port, out_dir, case, policy, digest_bits, device_payloa
         for _ in range(2):                                   # re-runnable
             dup, ben = sharded.dedup_sharded(log, torch.device("cuda", 0))
             outs.append((dup.cpu().numpy().copy(), ben.cpu().numpy().view(np.uint64).copy()))
+        cnt = sharded.site_counts_sharded(log, torch.device("cuda", 0)).cpu().numpy()
         dist.barrier()            # peers must not unmap while others still read their arenas
         np.savez(os.path.join(out_dir, f"r{rank}.npz"), idx=idx, dup=outs[0][0], ben=outs[0][1],
-                 dup2=outs[1][0], ben2=outs[1][1])
+                 dup2=outs[1][0], ben2=outs[1][1], cnt=cnt)
         dist.barrier()
         log.close()
     finally:
@@ -85,6 +86,9 @@ def _run(tmp_path, world, case, policy, digest_bits=64, device_payloads=False):
         np.testing.assert_array_equal(z["dup2"], z["dup"])
         np.testing.assert_array_equal(z["ben2"], z["ben"])
     np.testing.assert_array_equal(got, want_dup)
+    want_cnt = np.bincount(lg.site[want_dup >= 0].astype(np.int64), minlength=lg.n_sites)
+    for r in range(world):
+        np.testing.assert_array_equal(np.load(tmp_path / f"r{r}.npz")["cnt"], want_cnt)
     return lg, got
 
 
