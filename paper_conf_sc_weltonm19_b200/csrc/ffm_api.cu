@@ -165,6 +165,32 @@ void upload_meta(ffm_log* L) {
     ck(cudaMemcpyAsync(L->d_site + a, L->h_site.data() + a, k * 4, cudaMemcpyHostToDevice, s), "meta H2D");
     ck(cudaMemcpyAsync(L->d_dur + a, L->h_dur.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
     ck(cudaMemcpyAsync(L->d_gid + a, L->h_gid.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
+    // small records ordered by block count, largest first (counting sort): the four
+    // 8-lane groups of a warp then get payloads of near-equal length (no idle lanes)
+    {
+        const uint32_t nb = (L->params.small_bytes + 31) / 32 + 1;
+        std::vector<uint32_t> cnt(nb + 1, 0);
+        uint64_t ns = 0;
+        for (uint64_t i = 0; i < n; ++i)
+            if (L->h_size[i] <= L->params.small_bytes) {
+                cnt[nb - 1 - (uint32_t)((L->h_size[i] + 31) / 32)]++;
+                ++ns;
+            }
+        std::vector<uint32_t> start(nb + 1, 0);
+        for (uint32_t b = 0; b < nb; ++b) start[b + 1] = start[b] + cnt[b];
+        std::vector<uint32_t> order(std::max<uint64_t>(ns, 1));
+        for (uint64_t i = 0; i < n; ++i)
+            if (L->h_size[i] <= L->params.small_bytes)
+                order[start[nb - 1 - (uint32_t)((L->h_size[i] + 31) / 32)]++] = (uint32_t)i;
+        if (ns > L->d_small_cap) {
+            if (L->d_small_order) ck(cudaFree(L->d_small_order), "cudaFree");
+            L->d_small_order = nullptr;
+            L->d_small_cap = std::max<uint64_t>(ns, 2 * L->d_small_cap);
+            ck(cudaMalloc(&L->d_small_order, L->d_small_cap * sizeof(uint32_t)), "cudaMalloc(order)");
+        }
+        if (ns) ck(cudaMemcpyAsync(L->d_small_order, order.data(), ns * 4, cudaMemcpyHostToDevice, s), "order H2D");
+        L->n_small = ns;
+    }
     ck(cudaStreamSynchronize(s), "meta sync");
     L->d_meta_n = n;
 }
@@ -287,6 +313,8 @@ DevLog dev_view(const ffm_log* L) {
     d.dur = L->d_dur;
     d.gid = L->d_gid;
     d.n = (uint32_t)L->h_size.size();
+    d.small_order = L->d_small_order;
+    d.n_small = (uint32_t)L->n_small;
     return d;
 }
 
@@ -351,7 +379,7 @@ LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup) {
     if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
     // H2 group-by (round 0, all records)
     uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
-    LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, s));
+    LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, W.res[0], s));
     if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
     // H3 verify
     LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], L->n_large_chunks ? W.vitem_cap : 0, s, side,
@@ -374,7 +402,7 @@ LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup) {
             if (R.rounds > n + 2) throw CudaFail{cudaErrorUnknown, "collision resolution did not converge"};
             ck(cudaMemsetAsync(W.counters, 0, sizeof(uint32_t), s), "memset");
             uint64_t capr = std::max<uint64_t>(1024, pow2_at_least(2 * nres));
-            LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)R.rounds, s));
+            LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)R.rounds, W.res[cur ^ 1], s));
             LCHK(launch_verify(D, W, L->params, W.res[cur], (uint32_t)nres, W.res[cur ^ 1],
                                L->n_large_chunks ? W.vitem_cap : 0, s, nullptr, nullptr, nullptr));
             ck(cudaMemcpyAsync(L->h_counters, W.counters, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
@@ -944,7 +972,7 @@ int ffm_log_destroy(ffm_log* L) {
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
                     W.lcount, W.lstart, W.gcount, W.pos, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
                     W.dup, W.ben, W.cnt, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid,
-                    L->arena, L->d_desc};
+                    L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     free_shard(L->shard);

@@ -24,6 +24,8 @@ struct DevLog {
     const uint64_t* dur;     // [n]
     const uint64_t* gid;     // [n]
     uint32_t n;
+    const uint32_t* small_order;  // records <= small_bytes, sorted by block count (descending)
+    uint32_t n_small;
 };
 
 // Scratch of one run (grown on demand, reused across runs).
@@ -110,7 +112,7 @@ int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st)
 int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st);
 int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
-                 uint64_t cap, int round, cudaStream_t st);
+                 uint64_t cap, int round, uint32_t* res_out, cudaStream_t st);
 int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
                   uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st, cudaStream_t side, cudaEvent_t ev_fork,
                   cudaEvent_t ev_join);
@@ -169,6 +171,8 @@ struct ffm_log {
     uint64_t* d_gid = nullptr;
     uint64_t d_meta_cap = 0;       // records
     uint64_t d_meta_n = 0;         // records uploaded
+    uint32_t* d_small_order = nullptr;   // small records by size class (built at upload)
+    uint64_t d_small_cap = 0, n_small = 0;
 
     // HBM arena
     uint8_t* arena = nullptr;

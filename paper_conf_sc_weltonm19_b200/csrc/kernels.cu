@@ -108,9 +108,9 @@ __global__ void __launch_bounds__(256, 4) k_hash_small(DevLog L, uint32_t small_
     const unsigned omask = 0xFFu << (threadIdx.x & 24);
     LaneKeys K0;
     load_keys(K0, 2 * g, 0);
-    for (uint32_t r = oct; r < L.n; r += noct) {
+    for (uint32_t i = oct; i < L.n_small; i += noct) {
+        const uint32_t r = L.small_order[i];
         const uint64_t n = L.size[r];
-        if (n > small_bytes) continue;
         const uint8_t* base = L.arena + L.off[r];
         const uint32_t nblk = (uint32_t)((n + 31) >> 5);
         LaneKeys K = K0;
@@ -282,7 +282,7 @@ __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ li
 // lstart[leader] + c * gcount[leader] + p -- all members read leader chunk c back
 // to back, so the leader streams from HBM once and is re-read from L2.
 __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list, uint32_t small_bytes,
-                         uint32_t chunk_bytes) {
+                         uint32_t chunk_bytes, uint32_t* __restrict__ res_out) {
     uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     bool member = false;
     if (i < n_list) {
@@ -291,9 +291,16 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
         W.leader[r] = ld;
         if (ld != r) {
             member = true;
-            W.eq[r] = 1;
-            W.mis[r] = ~0ull;
             uint64_t n = L.size[r];
+            if (L.size[ld] != n) {
+                // a key collision across sizes: not equal, first word differs by definition
+                W.eq[r] = 0;
+                W.mis[r] = 0;
+                res_out[atomicAdd(&W.counters[0], 1u)] = r;
+            } else {
+                W.eq[r] = 1;
+                W.mis[r] = ~0ull;
+            }
             if (n > small_bytes && L.size[ld] == n) {
                 atomicAdd(&W.lcount[ld], (uint32_t)((n + chunk_bytes - 1) / chunk_bytes));
                 W.pos[r] = atomicAdd(&W.gcount[ld], 1u);
@@ -352,12 +359,9 @@ __global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const
         const uint32_t ld = W.leader[m];
         if (ld == m) continue;
         const uint64_t n = L.size[m];
-        const bool size_differs = L.size[ld] != n;     // (any size: large ones are not laid out)
-        if (n > small_bytes && !size_differs) continue;
+        if (n > small_bytes || L.size[ld] != n) continue;   // large path / resolved by k_leader
         uint64_t word = ~0ull;
-        if (size_differs) {
-            word = 0;
-        } else {
+        {
             const uint8_t* pm = L.arena + L.off[m];
             const uint8_t* pl = L.arena + L.off[ld];
             const uint32_t nblk = (uint32_t)((n + 31) >> 5);
@@ -487,7 +491,7 @@ __global__ void k_refine(DevLog L, Work W, const uint32_t* __restrict__ list, ui
 // histogram (no global atomic contention on hot call sites -- Zipf-skewed logs put
 // 10% of all records on one site) and a second kernel sums the block partials.
 // ----------------------------------------------------------------------------
-__global__ void __launch_bounds__(512) k_label_hist(DevLog L, const uint32_t* __restrict__ leader, uint32_t n_sites,
+__global__ void __launch_bounds__(1024) k_label_hist(DevLog L, const uint32_t* __restrict__ leader, uint32_t n_sites,
                                                     int64_t* __restrict__ dup_out, uint64_t* __restrict__ part,
                                                     uint32_t* __restrict__ cpart) {
     extern __shared__ unsigned long long sben[];
@@ -614,8 +618,9 @@ size_t cub_scan_bytes(uint64_t n) {
 
 int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
     if (L.n == 0) return 0;
+    if (L.n_small == 0) return 0;
     uint32_t grid = resident_grid((const void*)k_hash_small, P.num_sms);
-    uint32_t need = blocks_for((uint64_t)L.n * 8);
+    uint32_t need = blocks_for((uint64_t)L.n_small * 8);
     k_hash_small<<<need < grid ? need : grid, 256, 0, st>>>(L, P.small_bytes, W.accA, W.accB);
     FFM_LAUNCH_CHECK();
     return 1;
@@ -653,7 +658,7 @@ int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t 
 }
 
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list, uint64_t cap,
-                 int round, cudaStream_t st) {
+                 int round, uint32_t* res_out, cudaStream_t st) {
     if (n_list == 0) return 0;
     int k = 0;
     if (round > 0) {
@@ -667,7 +672,7 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
     if (cudaMemsetAsync(W.gcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
     k_group_insert<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, cap - 1, P.digest_mask, round);
     FFM_LAUNCH_CHECK();
-    k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes);
+    k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes, res_out);
     FFM_LAUNCH_CHECK();
     return k + 2;
 }
@@ -684,11 +689,17 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
         if (cudaEventRecord(ev_fork, st) != cudaSuccess || cudaStreamWaitEvent(side, ev_fork, 0) != cudaSuccess)
             return -1;
     }
-    uint32_t grid_s = resident_grid((const void*)k_verify_small, P.num_sms);
-    uint32_t need = blocks_for((uint64_t)n_list * 8);
-    k_verify_small<<<need < grid_s ? need : grid_s, 256, 0, ss>>>(L, W, list, n_list, P.small_bytes, res_out);
-    FFM_LAUNCH_CHECK();
-    ++k;
+    // main pass: the size-ordered small records; resolve rounds: the residual list
+    const uint32_t* slist = list ? list : L.small_order;
+    const uint32_t sn = list ? n_list : L.n_small;
+    uint32_t need = 0;
+    if (sn) {
+        uint32_t grid_s = resident_grid((const void*)k_verify_small, P.num_sms);
+        need = blocks_for((uint64_t)sn * 8);
+        k_verify_small<<<need < grid_s ? need : grid_s, 256, 0, ss>>>(L, W, slist, sn, P.small_bytes, res_out);
+        FFM_LAUNCH_CHECK();
+        ++k;
+    }
     if (vitem_cap) {
         // large members: chunk-major groups per leader (scan of lcount) then scatter work units
         size_t bytes = W.cub_tmp_bytes;
@@ -713,7 +724,7 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
     return k;
 }
 
-uint32_t label_hist_rows(int num_sms) { return (uint32_t)num_sms * 2; }
+uint32_t label_hist_rows(int num_sms) { return (uint32_t)num_sms; }
 
 int launch_site_reduce(const uint64_t* part, const uint32_t* cpart, uint32_t rows, uint32_t n_sites, uint64_t* ben,
                        uint64_t* cnt, cudaStream_t st) {
@@ -739,7 +750,7 @@ int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, in
             configured_smem = 1;
         }
         const uint32_t rows = label_hist_rows(P.num_sms);
-        k_label_hist<<<rows, 512, smem, st>>>(L, W.leader, n_sites, dup_out, W.label_part, W.label_cpart);
+        k_label_hist<<<rows, 1024, smem, st>>>(L, W.leader, n_sites, dup_out, W.label_part, W.label_cpart);
         FFM_LAUNCH_CHECK();
         if (launch_site_reduce(W.label_part, W.label_cpart, rows, n_sites, W.ben, W.cnt, st) < 0) return -1;
         return 2;

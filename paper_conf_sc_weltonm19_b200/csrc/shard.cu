@@ -205,7 +205,7 @@ __global__ void __launch_bounds__(256) k_merge_slow(const RepTuple* __restrict__
 
 // H5 + H6 for a shard: record r's class representative is its local leader; the
 // class's global leader G comes from the merge.  Benefit / count partials per rank.
-__global__ void __launch_bounds__(512) k_merge_label(DevLog L, const uint32_t* __restrict__ leader,
+__global__ void __launch_bounds__(1024) k_merge_label(DevLog L, const uint32_t* __restrict__ leader,
                                                      const uint32_t* __restrict__ rep_idx,
                                                      const uint64_t* __restrict__ G, uint32_t n_sites,
                                                      int64_t* __restrict__ dup_out, uint64_t* __restrict__ part,
@@ -353,7 +353,7 @@ int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, 
             configured = 1;
         }
         const uint32_t rows = label_hist_rows(P.num_sms);
-        k_merge_label<<<rows, 512, smem, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, W.label_part,
+        k_merge_label<<<rows, 1024, smem, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, W.label_part,
                                                W.label_cpart, nullptr, nullptr);
         SHARD_CHECK();
         return 1 + launch_site_reduce(W.label_part, W.label_cpart, rows, n_sites, W.ben, W.cnt, st);
