@@ -276,3 +276,28 @@ def test_site_counts_and_fold(ffm):
     assert rep["total"]["benefit_ns"] == int(want_ben.sum(dtype=np.uint64))
     assert len(rep["folded_function"]) <= 7
     assert sum(r["benefit_ns"] for r in rep["folded_function"]) == rep["total"]["benefit_ns"]
+
+
+@pytest.mark.parametrize("k", [4, 5])
+def test_full_size_configs_4_5(ffm, k):
+    """Full BASELINE sizes (config 4: 40.9 GB, config 5: 63.4 GB) in bench.py's launch
+    configuration (default chunk / small sizes, device-resident payloads), against
+    the full oracle run on the host (~10-20 s single core)."""
+    import torch
+    lg = loggen.gen_config(k)
+    buf_h = lg.materialize(nthreads=0)
+    want_dup, want_ben = oracle.dedup(lg)
+    dev = torch.from_numpy(buf_h).cuda()
+    ptrs = (lg.c_off[lg.content] + np.uint64(dev.data_ptr())).astype(np.uint64)
+    with ffm.FfmLog(lg.n_sites, arena_bytes=lg.total_bytes + 32 * lg.n + (1 << 20), max_records=lg.n) as log:
+        log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE)
+        del dev
+        torch.cuda.empty_cache()
+        d = torch.empty(lg.n, dtype=torch.int64, device="cuda")
+        b = torch.empty(lg.n_sites, dtype=torch.int64, device="cuda")
+        log.run(d, b)
+        dup = d.cpu().numpy()
+        ben = b.cpu().numpy().view(np.uint64)
+    np.testing.assert_array_equal(dup, want_dup)
+    np.testing.assert_array_equal(ben, want_ben)
+    np.testing.assert_array_equal(dup, lg.planted_duplicate_of())
