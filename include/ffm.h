@@ -162,6 +162,23 @@ int ffm_site_duplicate_counts(ffm_log* log, uint64_t* counts_out);
 int ffm_fold_sites(ffm_log* log, const uint64_t* site_values, const uint32_t* site_to_group, uint32_t n_groups,
                    uint64_t* group_values_out);
 
+/* ---------------------------------------------------------------------------
+ * Online (streaming) mode -- the paper's per-call semantics: each new
+ * transfer is "hashed and then compared to the stored hashes from prior transfers".
+ * ffm_online_step labels every record appended since the previous step (a window):
+ * H1..H4 on the window, then each window class is matched against the stored
+ * representatives of all earlier classes (byte-verified), and new classes are
+ * stored.  Labels of earlier records never change, so the concatenated windows
+ * equal ffm_dedup_run over the whole log, bit for bit.
+ *   duplicate_of [window records] (host or device): gids, or -1
+ *   benefit_ns   [n_sites] (may be NULL): cumulative per-site benefit so far
+ *   *n_window    (may be NULL): records labelled by this step
+ * Single-log only (world == 1). */
+int ffm_online_step(ffm_log* log, int64_t* duplicate_of, uint64_t* benefit_ns, uint64_t* n_window);
+
+/* Records labelled by online steps so far. */
+uint64_t ffm_online_done(const ffm_log* log);
+
 /* Debug / conformance: copy the last run's 64-bit payload digests (host array [n]).
    The digest is specified in DESIGN.md "Digest"; it is an implementation detail
    and never part of the result. */

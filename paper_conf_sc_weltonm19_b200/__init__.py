@@ -28,7 +28,8 @@ EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_appen
            "ffm_dedup_run", "ffm_log_count", "ffm_log_payload_bytes", "ffm_log_stream",
            "ffm_last_run_stats", "ffm_debug_digests", "ffm_log_destroy", "ffm_strerror",
            "ffm_last_error", "ffm_version", "ffm_shard_plan", "ffm_shard_ipc_handle", "ffm_shard_open_peer",
-           "ffm_shard_local", "ffm_shard_merge", "ffm_site_duplicate_counts", "ffm_fold_sites"]
+           "ffm_shard_local", "ffm_shard_merge", "ffm_site_duplicate_counts", "ffm_fold_sites",
+           "ffm_online_step", "ffm_online_done"]
 FFM_SHARD_SITE_LPT, FFM_SHARD_CONTIGUOUS = 0, 1
 REP_WORDS = 4        # ffm_rep = {key, size, gid, off}, 4 x u64
 
@@ -113,6 +114,10 @@ def lib() -> ctypes.CDLL:
         L.ffm_site_duplicate_counts.restype = i32
         L.ffm_fold_sites.argtypes = [vp, vp, vp, u32, vp]
         L.ffm_fold_sites.restype = i32
+        L.ffm_online_step.argtypes = [vp, vp, vp, ctypes.POINTER(u64)]
+        L.ffm_online_step.restype = i32
+        L.ffm_online_done.argtypes = [vp]
+        L.ffm_online_done.restype = u64
         _lib = L
     return _lib
 
@@ -262,6 +267,17 @@ def ffm_fold_sites(h, site_values, site_to_group, n_groups: int, out=None):
     return out
 
 
+def ffm_online_step(h, duplicate_of, benefit_ns=None) -> int:
+    """Label the records appended since the previous step; returns how many."""
+    n = ctypes.c_uint64()
+    _check(h, lib().ffm_online_step(h, _addr(duplicate_of), _addr(benefit_ns), ctypes.byref(n)))
+    return int(n.value)
+
+
+def ffm_online_done(h) -> int:
+    return int(lib().ffm_online_done(h))
+
+
 # ---- convenience wrapper ----------------------------------------------------
 class FfmLog:
     """Owns one ffm_log handle."""
@@ -322,6 +338,16 @@ class FfmLog:
 
     def digests(self):
         return ffm_debug_digests(self.h)
+
+    def online_step(self, duplicate_of=None, benefit_ns=None):
+        """Online mode: label the records appended since the last step."""
+        pending = self.count - ffm_online_done(self.h)
+        if duplicate_of is None:
+            duplicate_of = np.empty(max(pending, 1), np.int64)
+        if benefit_ns is None:
+            benefit_ns = np.empty(self.n_sites, np.uint64)
+        k = ffm_online_step(self.h, duplicate_of, benefit_ns)
+        return (duplicate_of[:k] if isinstance(duplicate_of, np.ndarray) else duplicate_of), benefit_ns
 
     def site_counts(self, out=None):
         return ffm_site_duplicate_counts(self.h, self.n_sites, out)

@@ -143,6 +143,38 @@ bool is_device_ptr(const void* p) {
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// Records in [begin, end) with size <= small_bytes, as indices relative to begin,
+// ordered by 32-byte block count, largest first (stable counting sort).
+void build_small_order(const ffm_log* L, uint64_t begin, uint64_t end, std::vector<uint32_t>& order) {
+    const uint32_t nb = (L->params.small_bytes + 31) / 32 + 1;
+    std::vector<uint32_t> start(nb + 1, 0);
+    uint64_t ns = 0;
+    for (uint64_t i = begin; i < end; ++i)
+        if (L->h_size[i] <= L->params.small_bytes) {
+            start[nb - (uint32_t)((L->h_size[i] + 31) / 32)]++;
+            ++ns;
+        }
+    for (uint32_t b = 1; b <= nb; ++b) start[b] += start[b - 1];
+    // start[c] now counts classes < c; class c = nb-1-blocks  ->  cursor = start[c]
+    std::vector<uint32_t> cur(nb, 0);
+    for (uint32_t c = 0; c < nb; ++c) cur[c] = c ? start[c] : 0;
+    order.assign(ns, 0);
+    for (uint64_t i = begin; i < end; ++i)
+        if (L->h_size[i] <= L->params.small_bytes)
+            order[cur[nb - 1 - (uint32_t)((L->h_size[i] + 31) / 32)]++] = (uint32_t)(i - begin);
+}
+
+void upload_order(ffm_log* L, const std::vector<uint32_t>& order, uint32_t*& dptr, uint64_t& cap, cudaStream_t s) {
+    uint64_t ns = order.size();
+    if (ns > cap || !dptr) {
+        if (dptr) ck(cudaFree(dptr), "cudaFree");
+        dptr = nullptr;
+        cap = std::max<uint64_t>(std::max<uint64_t>(ns, 2 * cap), 1024);
+        ck(cudaMalloc(&dptr, cap * sizeof(uint32_t)), "cudaMalloc(order)");
+    }
+    if (ns) ck(cudaMemcpyAsync(dptr, order.data(), ns * 4, cudaMemcpyHostToDevice, s), "order H2D");
+}
+
 void upload_meta(ffm_log* L) {
     uint64_t n = L->h_size.size();
     if (L->d_meta_n == n) return;
@@ -168,28 +200,10 @@ void upload_meta(ffm_log* L) {
     // small records ordered by block count, largest first (counting sort): the four
     // 8-lane groups of a warp then get payloads of near-equal length (no idle lanes)
     {
-        const uint32_t nb = (L->params.small_bytes + 31) / 32 + 1;
-        std::vector<uint32_t> cnt(nb + 1, 0);
-        uint64_t ns = 0;
-        for (uint64_t i = 0; i < n; ++i)
-            if (L->h_size[i] <= L->params.small_bytes) {
-                cnt[nb - 1 - (uint32_t)((L->h_size[i] + 31) / 32)]++;
-                ++ns;
-            }
-        std::vector<uint32_t> start(nb + 1, 0);
-        for (uint32_t b = 0; b < nb; ++b) start[b + 1] = start[b] + cnt[b];
-        std::vector<uint32_t> order(std::max<uint64_t>(ns, 1));
-        for (uint64_t i = 0; i < n; ++i)
-            if (L->h_size[i] <= L->params.small_bytes)
-                order[start[nb - 1 - (uint32_t)((L->h_size[i] + 31) / 32)]++] = (uint32_t)i;
-        if (ns > L->d_small_cap) {
-            if (L->d_small_order) ck(cudaFree(L->d_small_order), "cudaFree");
-            L->d_small_order = nullptr;
-            L->d_small_cap = std::max<uint64_t>(ns, 2 * L->d_small_cap);
-            ck(cudaMalloc(&L->d_small_order, L->d_small_cap * sizeof(uint32_t)), "cudaMalloc(order)");
-        }
-        if (ns) ck(cudaMemcpyAsync(L->d_small_order, order.data(), ns * 4, cudaMemcpyHostToDevice, s), "order H2D");
-        L->n_small = ns;
+        std::vector<uint32_t> order;
+        build_small_order(L, 0, n, order);
+        upload_order(L, order, L->d_small_order, L->d_small_cap, s);
+        L->n_small = order.size();
     }
     ck(cudaStreamSynchronize(s), "meta sync");
     L->d_meta_n = n;
@@ -350,12 +364,11 @@ void run_prologue(ffm_log* L) {
 // leader (the min local index of its exact byte class).  With `label` the H5/H6
 // kernels are queued before the first sync (single-GPU fast path: one sync when
 // there are no digest collisions) and re-run after collision resolution.
-LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup) {
+LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& launches, bool label, int64_t* d_dup) {
     const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
-    const uint64_t n = L->h_size.size();
+    const uint64_t n = D.n;
     Work& W = L->work;
     cudaStream_t s = L->stream;
-    DevLog D = dev_view(L);
     const uint32_t ns = L->cfg.n_sites;
     LocalRun R{};
     if (timing) ck(cudaEventRecord(L->ev[0], s), "event");
@@ -368,10 +381,10 @@ LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup) {
     LCHK(launch_hash_small(D, W, L->params, side));
     if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
     ck(cudaEventRecord(L->fork_ev[1], side), "event");
-    if (L->n_large_chunks) {
+    if (n_large) {
         LCHK(launch_hash_plan(D, W, L->params, s));
         if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
-        LCHK(launch_hash_large(D, W, L->params, L->n_large_chunks, s));
+        LCHK(launch_hash_large(D, W, L->params, n_large, s));
         if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
         LCHK(launch_hash_combine(D, W, L->params, s));
     }
@@ -382,7 +395,7 @@ LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup) {
     LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, W.res[0], s));
     if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
     // H3 verify
-    LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], L->n_large_chunks ? W.vitem_cap : 0, s, side,
+    LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], n_large ? W.vitem_cap : 0, s, side,
                        L->fork_ev[2], L->fork_ev[3]));
     if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
     // H5 + H6 (speculative: valid unless H3 found residuals)
@@ -404,7 +417,7 @@ LocalRun run_local(ffm_log* L, uint64_t& launches, bool label, int64_t* d_dup) {
             uint64_t capr = std::max<uint64_t>(1024, pow2_at_least(2 * nres));
             LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)R.rounds, W.res[cur ^ 1], s));
             LCHK(launch_verify(D, W, L->params, W.res[cur], (uint32_t)nres, W.res[cur ^ 1],
-                               L->n_large_chunks ? W.vitem_cap : 0, s, nullptr, nullptr, nullptr));
+                               n_large ? W.vitem_cap : 0, s, nullptr, nullptr, nullptr));
             ck(cudaMemcpyAsync(L->h_counters, W.counters, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
             ck(cudaStreamSynchronize(s), "round sync");
             nres = L->h_counters[0];
@@ -722,7 +735,7 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         bool ben_dev = ben_out && is_device_ptr(ben_out);
         int64_t* d_dup = dup_dev ? dup_out : W.dup;
         uint64_t launches = 0;
-        LocalRun R = run_local(L, launches, true, d_dup);
+        LocalRun R = run_local(L, dev_view(L), L->n_large_chunks, launches, true, d_dup);
         // H7 return
         const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
         if (timing) ck(cudaEventRecord(L->ev[9], s), "event");
@@ -797,7 +810,7 @@ int ffm_shard_local(ffm_log* L, ffm_rep* reps_out, uint64_t cap, uint64_t* n_rep
     try {
         run_prologue(L);
         uint64_t launches = 0;
-        LocalRun R = run_local(L, launches, false, nullptr);
+        LocalRun R = run_local(L, dev_view(L), L->n_large_chunks, launches, false, nullptr);
         ensure_shard(L, n, 1, 1, 1, std::max(L->cfg.world, 1));
         DevLog D = dev_view(L);
         cudaStream_t s = L->stream;
@@ -948,6 +961,121 @@ int ffm_fold_sites(ffm_log* L, const uint64_t* site_values, const uint32_t* site
     return FFM_OK;
 }
 
+uint64_t ffm_online_done(const ffm_log* L) { return L ? L->online_done : 0; }
+
+int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n_out) {
+    int st = check_state(L);
+    if (st) return st;
+    if (L->cfg.world > 1) return set_err(L, FFM_E_STATE, "online mode is single-log (world == 1)");
+    const uint64_t n = L->h_size.size(), w0 = L->online_done, nw = n - w0;
+    if (nw && !dup_out) return set_err(L, FFM_E_INVAL, "duplicate_of is NULL");
+    const uint32_t ns = L->cfg.n_sites;
+    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
+    try {
+        run_prologue(L);
+        Work& W = L->work;
+        ShardWork& S = L->shard;
+        cudaStream_t s = L->stream;
+        if (!L->online_ben) {
+            ck(cudaMalloc(&L->online_ben, ns * sizeof(uint64_t)), "cudaMalloc(online)");
+            ck(cudaMalloc(&L->online_cnt, ns * sizeof(uint64_t)), "cudaMalloc(online)");
+            ck(cudaMemsetAsync(L->online_ben, 0, ns * sizeof(uint64_t), s), "memset");
+            ck(cudaMemsetAsync(L->online_cnt, 0, ns * sizeof(uint64_t), s), "memset");
+        }
+        uint64_t launches = 0;
+        LocalRun R{};
+        uint64_t n_slow = 0;
+        if (nw) {
+            // the window view: records [w0, n) as a log of their own (indices relative to w0)
+            DevLog D = dev_view(L);
+            D.off += w0;
+            D.size += w0;
+            D.site += w0;
+            D.dur += w0;
+            D.gid += w0;
+            D.n = (uint32_t)nw;
+            std::vector<uint32_t> order;
+            build_small_order(L, w0, n, order);
+            upload_order(L, order, L->d_win_order, L->d_win_cap, s);
+            D.small_order = L->d_win_order;
+            D.n_small = (uint32_t)order.size();
+            uint64_t n_large = 0;
+            for (uint64_t i = w0; i < n; ++i) n_large += large_chunks(L, L->h_size[i]);
+            // H1..H4 on the window: exact window-local classes
+            R = run_local(L, D, n_large, launches, false, nullptr);
+            // window representatives appended after the prior ones
+            const uint64_t np = L->online_np;
+            if (np + nw > L->online_cap) {
+                uint64_t c = std::max<uint64_t>(np + nw, 2 * L->online_cap);
+                ffm::RepTuple* t = nullptr;
+                ck(cudaMalloc(&t, c * sizeof(ffm::RepTuple)), "cudaMalloc(online)");
+                if (np) ck(cudaMemcpyAsync(t, L->online_T, np * sizeof(ffm::RepTuple), cudaMemcpyDeviceToDevice, s),
+                           "copy");
+                ck(cudaStreamSynchronize(s), "sync");
+                if (L->online_T) ck(cudaFree(L->online_T), "cudaFree");
+                if (L->online_tmp) ck(cudaFree(L->online_tmp), "cudaFree");
+                L->online_T = t;
+                ck(cudaMalloc(&L->online_tmp, c * sizeof(ffm::RepTuple)), "cudaMalloc(online)");
+                L->online_cap = c;
+            }
+            ensure_shard(L, nw, np + nw, nw, nw + n_large + 64, 2);
+            LCHK(launch_rep_export(D, W, S, L->params, L->online_T + np, s));
+            ck(cudaMemcpyAsync(L->h_counters, S.rep_idx + nw, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+            ck(cudaStreamSynchronize(s), "online sync");
+            const uint64_t nloc = L->h_counters[0], M = np + nloc;
+            // "compared to the stored hashes from prior transfers": the prior
+            // classes play the part of a peer shard living in the same arena
+            const uint32_t rank_lo[2] = {0u, (uint32_t)np};
+            const uint8_t* bases[2] = {L->arena, L->arena};
+            ck(cudaMemcpyAsync(S.rank_lo, rank_lo, sizeof(rank_lo), cudaMemcpyHostToDevice, s), "H2D");
+            ck(cudaMemcpyAsync((void*)S.bases, bases, sizeof(bases), cudaMemcpyHostToDevice, s), "H2D");
+            uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(M, 1)));
+            LCHK(launch_merge(D, W, S, L->params, L->online_T, (uint32_t)M, (uint32_t)np, (uint32_t)nloc, 2, 1, cap, s));
+            ck(cudaMemcpyAsync(L->h_counters, S.n_slow, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+            ck(cudaStreamSynchronize(s), "online merge sync");
+            n_slow = L->h_counters[0];
+            if (n_slow) {
+                LCHK(launch_sort_prep(S, L->online_T, (uint32_t)M, s));
+                LCHK(launch_merge_slow(D, W, S, L->params, L->online_T, (uint32_t)M, (uint32_t)np, 2, 1,
+                                       (uint32_t)n_slow, s));
+            }
+            const bool dup_dev = is_device_ptr(dup_out);
+            int64_t* d_dup = dup_dev ? dup_out : W.dup;
+            LCHK(launch_merge_label(D, W, S, L->params, ns, d_dup, s));
+            LCHK(launch_vec_add(L->online_ben, W.ben, ns, s));
+            LCHK(launch_vec_add(L->online_cnt, W.cnt, ns, s));
+            // new classes join the stored representatives
+            LCHK(launch_online_newreps(W, S, L->online_T + np, (uint32_t)nloc, L->online_tmp, s));
+            ck(cudaMemcpyAsync(L->h_counters, S.vstart + nloc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+            if (!dup_dev)
+                ck(cudaMemcpyAsync(dup_out, d_dup, nw * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
+            ck(cudaStreamSynchronize(s), "online new reps sync");
+            const uint64_t n_new = L->h_counters[0];
+            if (n_new)
+                ck(cudaMemcpyAsync(L->online_T + np, L->online_tmp, n_new * sizeof(ffm::RepTuple),
+                                   cudaMemcpyDeviceToDevice, s),
+                   "copy reps");
+            L->online_np = np + n_new;
+        }
+        if (ben_out)
+            ck(cudaMemcpyAsync(ben_out, L->online_ben, ns * sizeof(uint64_t), cudaMemcpyDefault, s), "copy ben");
+        ck(cudaStreamSynchronize(s), "online sync");
+        ck(cudaGetLastError(), "online step");
+        L->online_done = n;
+        fill_stats(L, R, launches, false);
+        L->stats.n_residual += n_slow;
+        L->stats.n_records = nw;
+        L->digests_valid = false;
+        (void)timing;
+        if (n_out) *n_out = nw;
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    } catch (const std::bad_alloc&) {
+        return set_err(L, FFM_E_NOMEM, "host allocation failed");
+    }
+    return FFM_OK;
+}
+
 int ffm_debug_digests(ffm_log* L, uint64_t* out) {
     int st = check_state(L);
     if (st) return st;
@@ -977,6 +1105,9 @@ int ffm_log_destroy(ffm_log* L) {
         if (p) cudaFree(p);
     free_shard(L->shard);
     if (L->fold_buf) cudaFree(L->fold_buf);
+    void* op[] = {L->online_T, L->online_tmp, L->online_ben, L->online_cnt, L->d_win_order};
+    for (void* p : op)
+        if (p) cudaFree(p);
     for (void* p : L->peer_ptr)
         if (p) cudaIpcCloseMemHandle(p);
     for (int i = 0; i < 2; ++i) {

@@ -131,6 +131,8 @@ int launch_sort_prep(ShardWork& S, const RepTuple* T, uint32_t M, cudaStream_t s
 size_t sort_tmp_bytes(uint32_t M);
 int launch_merge_slow(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
                       uint32_t lo, int world, int rank, uint32_t n_slow, cudaStream_t st);
+int launch_online_newreps(Work& W, ShardWork& S, RepTuple* Tw, uint32_t nloc, RepTuple* tmp, cudaStream_t st);
+int launch_vec_add(uint64_t* a, const uint64_t* b, uint32_t n, cudaStream_t st);
 int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
                        cudaStream_t st);
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
@@ -193,6 +195,16 @@ struct ffm_log {
     bool reps_valid = false;
     std::vector<void*> peer_ptr;    // IPC-mapped peer arenas (index = rank)
     std::vector<std::string> peer_handle;
+
+    // online (streaming) mode: representatives of every class seen so far
+    uint64_t online_done = 0;        // records already labelled online
+    ffm::RepTuple* online_T = nullptr;   // [online_np prior reps | window reps]
+    ffm::RepTuple* online_tmp = nullptr;
+    uint64_t online_np = 0, online_cap = 0;
+    uint64_t* online_ben = nullptr;  // cumulative per-site benefit / duplicate counts
+    uint64_t* online_cnt = nullptr;
+    uint32_t* d_win_order = nullptr;
+    uint64_t d_win_cap = 0;
 
     // folded grouping scratch
     void* fold_buf = nullptr;
