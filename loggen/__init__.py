@@ -75,6 +75,7 @@ class Log:
     flip_xor: np.ndarray        # uint8  [F]
     name: str = ""
     buf: np.ndarray | None = field(default=None, repr=False)   # materialised bytes
+    channel: np.ndarray | None = None   # uint64 [N] direction/destination id (S8(f) #3), or None
     c_off: np.ndarray | None = field(default=None, repr=False)
 
     @property
@@ -146,10 +147,13 @@ class Log:
 
     # ---- planted ground truth ---------------------------------------------
     def planted_duplicate_of(self) -> np.ndarray:
-        """dup_of from content ids alone: first earlier record with the same id."""
-        first: dict[int, int] = {}
+        """dup_of from content ids (and channels, if any) alone: first earlier record
+        with the same id."""
+        first: dict = {}
         out = np.full(self.n, -1, dtype=np.int64)
-        for i, c in enumerate(self.content.tolist()):
+        keys = self.content.tolist() if self.channel is None else \
+            list(zip(self.content.tolist(), self.channel.tolist()))
+        for i, c in enumerate(keys):
             j = first.get(c)
             if j is None:
                 first[c] = i
@@ -170,6 +174,7 @@ class Log:
                  self.c_kind, self.c_seed, self.c_size, self.c_base, self.c_flip_start,
                  self.flip_pos, self.flip_xor, name or self.name + "/subset")
         lg.buf, lg.c_off = self.buf, self.c_off
+        lg.channel = None if self.channel is None else self.channel[idx]
         return lg
 
 
@@ -467,7 +472,8 @@ def gen_config(k: int, seed: int | None = None, n_scale: float = 1.0, size_scale
     return CONFIGS[k](seed=seed, n_scale=n_scale, size_scale=size_scale)
 
 
-def from_payloads(payloads: list[bytes], sites=None, durs=None, n_sites: int | None = None) -> Log:
+def from_payloads(payloads: list[bytes], sites=None, durs=None, n_sites: int | None = None,
+                  channels=None) -> Log:
     """A log from explicit byte strings (tiny / adversarial tests).  Content ids
     are assigned by exact byte equality, so planted truth is exact."""
     n = len(payloads)
@@ -494,4 +500,5 @@ def from_payloads(payloads: list[bytes], sites=None, durs=None, n_sites: int | N
         o = int(off[c])
         buf[o:o + len(b)] = np.frombuffer(b, np.uint8) if len(b) else buf[o:o]
     lg.buf, lg.c_off = buf, off
+    lg.channel = None if channels is None else np.asarray(channels, np.uint64)
     return lg

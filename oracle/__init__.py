@@ -43,12 +43,12 @@ def _get():
         build()
         _lib = ctypes.CDLL(_LIB)
         vp = ctypes.c_void_p
-        _lib.oracle_dedup.argtypes = [ctypes.c_uint64, vp, vp, vp, vp, ctypes.c_uint32,
+        _lib.oracle_dedup.argtypes = [ctypes.c_uint64, vp, vp, vp, vp, vp, ctypes.c_uint32,
                                       ctypes.c_int, vp, vp]
         _lib.oracle_dedup.restype = ctypes.c_int
-        _lib.oracle_brute.argtypes = [ctypes.c_uint64, vp, vp, vp, vp, ctypes.c_uint32, vp, vp]
+        _lib.oracle_brute.argtypes = [ctypes.c_uint64, vp, vp, vp, vp, vp, ctypes.c_uint32, vp, vp]
         _lib.oracle_brute.restype = ctypes.c_int
-        _lib.oracle_dup_of_one.argtypes = [ctypes.c_uint64, vp, vp]
+        _lib.oracle_dup_of_one.argtypes = [ctypes.c_uint64, vp, vp, vp]
         _lib.oracle_dup_of_one.restype = ctypes.c_int64
     return _lib
 
@@ -61,8 +61,13 @@ def _arrays(log):
     return site, size, dur, ptrs
 
 
+def _chan(log):
+    ch = getattr(log, "channel", None)
+    return None if ch is None else np.ascontiguousarray(ch, dtype=np.uint64)
+
+
 def _p(a):
-    return ctypes.c_void_p(a.ctypes.data)
+    return None if a is None else ctypes.c_void_p(a.ctypes.data)
 
 
 def dedup(log, hash_bits: int = 64):
@@ -71,17 +76,17 @@ def dedup(log, hash_bits: int = 64):
     n = len(site)
     dup = np.empty(max(n, 1), np.int64)
     ben = np.empty(max(log.n_sites, 1), np.uint64)
-    rc = _get().oracle_dedup(n, _p(site), _p(size), _p(ptrs), _p(dur), log.n_sites,
+    rc = _get().oracle_dedup(n, _p(site), _p(size), _p(ptrs), _p(dur), _p(_chan(log)), log.n_sites,
                              hash_bits, _p(dup), _p(ben))
     if rc != 0:
         raise ValueError(f"oracle_dedup failed: {rc}")
     return dup[:n], ben[:log.n_sites]
 
 
-def dedup_raw(n, site, size, ptrs, dur, n_sites, hash_bits=64):
+def dedup_raw(n, site, size, ptrs, dur, n_sites, hash_bits=64, channel=None):
     dup = np.empty(max(n, 1), np.int64)
     ben = np.empty(max(n_sites, 1), np.uint64)
-    rc = _get().oracle_dedup(n, _p(site), _p(size), _p(ptrs), _p(dur), n_sites, hash_bits,
+    rc = _get().oracle_dedup(n, _p(site), _p(size), _p(ptrs), _p(dur), _p(channel), n_sites, hash_bits,
                              _p(dup), _p(ben))
     if rc != 0:
         raise ValueError(f"oracle_dedup failed: {rc}")
@@ -93,7 +98,7 @@ def brute(log):
     n = len(site)
     dup = np.empty(max(n, 1), np.int64)
     ben = np.empty(max(log.n_sites, 1), np.uint64)
-    rc = _get().oracle_brute(n, _p(site), _p(size), _p(ptrs), _p(dur), log.n_sites,
+    rc = _get().oracle_brute(n, _p(site), _p(size), _p(ptrs), _p(dur), _p(_chan(log)), log.n_sites,
                              _p(dup), _p(ben))
     if rc != 0:
         raise ValueError(f"oracle_brute failed: {rc}")
@@ -103,17 +108,18 @@ def brute(log):
 def dup_of_one(log, i: int) -> int:
     _, size, _, ptrs = _arrays(log) if not hasattr(log, "_oracle_cache") else log._oracle_cache
     log._oracle_cache = (None, size, None, ptrs)
-    return int(_get().oracle_dup_of_one(i, _p(size), _p(ptrs)))
+    return int(_get().oracle_dup_of_one(i, _p(size), _p(ptrs), _p(_chan(log))))
 
 
-def brute_py(payloads, sites, durs, n_sites):
+def brute_py(payloads, sites, durs, n_sites, channels=None):
     """The plain definition in pure Python (tiny logs only)."""
     n = len(payloads)
+    ch = channels if channels is not None else [0] * n
     dup = [-1] * n
     ben = [0] * n_sites
     for i in range(n):
         for j in range(i):
-            if len(payloads[j]) == len(payloads[i]) and payloads[j] == payloads[i]:
+            if len(payloads[j]) == len(payloads[i]) and ch[j] == ch[i] and payloads[j] == payloads[i]:
                 dup[i] = j
                 break
         if dup[i] >= 0:

@@ -39,9 +39,35 @@ def test_golden_fixture(name, hash_bits):
     pay = [bytes.fromhex(r["hex"]) for r in fx["records"]]
     sites = [r["site"] for r in fx["records"]]
     durs = [r["dur"] for r in fx["records"]]
-    dup, ben = _run(pay, sites, durs, fx["n_sites"], hash_bits)
+    chans = [r["channel"] for r in fx["records"]] if "channel" in fx["records"][0] else None
+    lg = loggen.from_payloads(pay, sites, durs, fx["n_sites"], channels=chans)
+    dup, ben = oracle.dedup(lg, hash_bits=hash_bits)
     assert dup.tolist() == fx["expect_duplicate_of"]
     assert ben.tolist() == fx["expect_benefit_ns"]
+    if "expect_content_only" in fx:
+        lg.channel = None
+        dup, ben = oracle.dedup(lg, hash_bits=hash_bits)
+        assert dup.tolist() == fx["expect_content_only"]["duplicate_of"]
+        assert ben.tolist() == fx["expect_content_only"]["benefit_ns"]
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_channels_vs_python_brute(seed):
+    """Destination-aware variant (S8(f) #3) against the plain definition."""
+    rng = np.random.default_rng(5000 + seed)
+    n = int(rng.integers(1, 150))
+    pay, sites, durs, ns = _random_log(rng, n, int(rng.integers(1, 8)), int(rng.integers(0, 40)))
+    chans = rng.integers(0, int(rng.integers(1, 4)), n).tolist()
+    want = oracle.brute_py(pay, sites, durs, ns, chans)
+    lg = loggen.from_payloads(pay, sites, durs, ns, channels=chans)
+    for hb in (64, 0):
+        d, b = oracle.dedup(lg, hash_bits=hb)
+        assert d.tolist() == want[0] and b.tolist() == want[1]
+    d, b = oracle.brute(lg)
+    assert d.tolist() == want[0]
+    # a single channel reduces to the content-only result
+    lg1 = loggen.from_payloads(pay, sites, durs, ns, channels=[7] * n)
+    assert oracle.dedup(lg1)[0].tolist() == oracle.brute_py(pay, sites, durs, ns)[0]
 
 
 def _random_log(rng, n, alphabet_size, max_len):
