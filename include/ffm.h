@@ -107,6 +107,16 @@ int ffm_log_append_batch(ffm_log* log, uint64_t n, const uint32_t* call_sites,
                          const uint64_t* durations_ns, const uint64_t* gids,
                          int payload_kind);
 
+/* ffm_log_append_batch with an optional per-record channel id (S8(f) #3, the
+   destination-aware variant: "retransfer the same data to the same destination",
+   P:1194-1197; direction "to and from the GPU").  A record then
+   duplicates only an earlier record with equal size, bytes AND channel.  channels
+   NULL (or all equal) is the content-only reading R5. */
+int ffm_log_append_batch_ex(ffm_log* log, uint64_t n, const uint32_t* call_sites,
+                            const uint64_t* sizes, const void* const* payloads,
+                            const uint64_t* durations_ns, const uint64_t* gids,
+                            const uint64_t* channels, int payload_kind);
+
 /* Run the hot path over the whole log (H1 hash, H2 group-by, H3 verify,
    H4 collision resolve, H5 label, H6 per-site benefit, H7 return):
      duplicate_of[n_local]  int64  gid of the earliest byte-identical record, or -1
@@ -202,10 +212,11 @@ int ffm_debug_digests(ffm_log* log, uint64_t* digests_out);
  * outputs (after the last append) and call ffm_shard_open_peer for every other rank.
  * ------------------------------------------------------------------------- */
 typedef struct ffm_rep {
-    uint64_t key;    /* group key of the payload digest (identical function on every rank) */
+    uint64_t key;    /* group key of (digest, size, channel) (identical function on every rank) */
     uint64_t size;   /* payload bytes */
     uint64_t gid;    /* global gid of the class's first record on the owning rank */
     uint64_t off;    /* arena offset on the owning rank */
+    uint64_t chan;   /* channel id (0 unless ffm_log_append_batch_ex gave one) */
 } ffm_rep;
 
 enum { FFM_SHARD_SITE_LPT = 0,     /* whole call sites, bin-packed by bytes (largest first) */

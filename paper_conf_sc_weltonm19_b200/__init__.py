@@ -24,14 +24,14 @@ FFM_PAYLOAD_AUTO, FFM_PAYLOAD_HOST, FFM_PAYLOAD_DEVICE, FFM_PAYLOAD_HOST_PINNED 
 FFM_FLAG_TIMING = 1
 
 # every symbol include/ffm.h declares (checked by tests/test_abi.py)
-EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_append_batch",
+EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_append_batch", "ffm_log_append_batch_ex",
            "ffm_dedup_run", "ffm_log_count", "ffm_log_payload_bytes", "ffm_log_stream",
            "ffm_last_run_stats", "ffm_debug_digests", "ffm_log_destroy", "ffm_strerror",
            "ffm_last_error", "ffm_version", "ffm_shard_plan", "ffm_shard_ipc_handle", "ffm_shard_open_peer",
            "ffm_shard_local", "ffm_shard_merge", "ffm_site_duplicate_counts", "ffm_fold_sites",
            "ffm_online_step", "ffm_online_done"]
 FFM_SHARD_SITE_LPT, FFM_SHARD_CONTIGUOUS = 0, 1
-REP_WORDS = 4        # ffm_rep = {key, size, gid, off}, 4 x u64
+REP_WORDS = 5        # ffm_rep = {key, size, gid, off, chan}, 5 x u64
 
 
 class FfmConfig(ctypes.Structure):
@@ -80,6 +80,8 @@ def lib() -> ctypes.CDLL:
         L.ffm_log_append.restype = i32
         L.ffm_log_append_batch.argtypes = [vp, u64, vp, vp, vp, vp, vp, i32]
         L.ffm_log_append_batch.restype = i32
+        L.ffm_log_append_batch_ex.argtypes = [vp, u64, vp, vp, vp, vp, vp, vp, i32]
+        L.ffm_log_append_batch_ex.restype = i32
         L.ffm_dedup_run.argtypes = [vp, vp, vp]
         L.ffm_dedup_run.restype = i32
         L.ffm_log_count.argtypes = [vp]
@@ -171,16 +173,23 @@ def _addr(a):
 
 def ffm_log_append_batch(h, call_sites, sizes, payload_ptrs, durations_ns, gids=None,
                          payload_kind: int = FFM_PAYLOAD_AUTO):
+    ffm_log_append_batch_ex(h, call_sites, sizes, payload_ptrs, durations_ns, gids, None, payload_kind)
+
+
+def ffm_log_append_batch_ex(h, call_sites, sizes, payload_ptrs, durations_ns, gids=None, channels=None,
+                            payload_kind: int = FFM_PAYLOAD_AUTO):
     sites = np.ascontiguousarray(call_sites, dtype=np.uint32)
     sz = np.ascontiguousarray(sizes, dtype=np.uint64)
     pp = np.ascontiguousarray(payload_ptrs, dtype=np.uint64)
     du = np.ascontiguousarray(durations_ns, dtype=np.uint64)
     g = None if gids is None else np.ascontiguousarray(gids, dtype=np.uint64)
+    ch = None if channels is None else np.ascontiguousarray(channels, dtype=np.uint64)
     n = len(sites)
-    if not (len(sz) == len(pp) == len(du) == n) or (g is not None and len(g) != n):
+    if not (len(sz) == len(pp) == len(du) == n) or (g is not None and len(g) != n) or \
+            (ch is not None and len(ch) != n):
         raise ValueError("array lengths differ")
-    _check(h, lib().ffm_log_append_batch(h, n, _addr(sites), _addr(sz), _addr(pp), _addr(du),
-                                         _addr(g), payload_kind))
+    _check(h, lib().ffm_log_append_batch_ex(h, n, _addr(sites), _addr(sz), _addr(pp), _addr(du),
+                                            _addr(g), _addr(ch), payload_kind))
 
 
 def ffm_dedup_run(h, duplicate_of, benefit_ns):
@@ -299,18 +308,20 @@ class FfmLog:
         ffm_log_append(self.h, call_site, size, payload_ptr, duration_ns)
 
     def append_batch(self, call_sites, sizes, payload_ptrs, durations_ns, gids=None,
-                     payload_kind=FFM_PAYLOAD_AUTO):
-        ffm_log_append_batch(self.h, call_sites, sizes, payload_ptrs, durations_ns, gids, payload_kind)
+                     payload_kind=FFM_PAYLOAD_AUTO, channels=None):
+        ffm_log_append_batch_ex(self.h, call_sites, sizes, payload_ptrs, durations_ns, gids, channels,
+                                payload_kind)
 
     def append_log(self, log, ptrs=None, payload_kind=FFM_PAYLOAD_HOST, gids=None, idx=None):
         """Append a log object with site/size/dur arrays and payload_ptrs() (host payloads by
         default, or the device addresses `ptrs`)."""
         p = log.payload_ptrs() if ptrs is None else ptrs
+        ch = getattr(log, "channel", None)
         if idx is None:
-            self.append_batch(log.site, log.size, p, log.dur, gids, payload_kind)
+            self.append_batch(log.site, log.size, p, log.dur, gids, payload_kind, ch)
         else:
             self.append_batch(log.site[idx], log.size[idx], np.asarray(p)[idx], log.dur[idx],
-                              gids, payload_kind)
+                              gids, payload_kind, None if ch is None else ch[idx])
 
     def run(self, duplicate_of=None, benefit_ns=None):
         n = self.count

@@ -23,8 +23,11 @@ __device__ __forceinline__ uint64_t finalize_digest(uint64_t A, uint64_t B, uint
 
 __device__ __forceinline__ uint64_t not_empty(uint64_t k) { return k == kEmptyKey ? k - 1 : k; }
 
-__device__ __forceinline__ uint64_t group_key(uint64_t digest, uint64_t n, uint64_t mask) {
-    return not_empty(fmix64((digest & mask) ^ fmix64(n + 0x632BE59BD9B4E019ull)));
+// Group key of (digest, size, channel).  Equal bytes, size and channel => equal key;
+// digest_bits truncation (mask) forces collisions without changing results.
+__device__ __forceinline__ uint64_t group_key(uint64_t digest, uint64_t n, uint64_t mask, uint64_t chan) {
+    return not_empty(fmix64((digest & mask) ^ fmix64(n + 0x632BE59BD9B4E019ull) ^
+                            fmix64(chan ^ 0x2545F4914F6CDD1Dull)));
 }
 
 // 32-byte block = two 16-byte words.

@@ -189,6 +189,8 @@ void upload_meta(ffm_log* L) {
     dev_grow(L->d_dur, cap, n, keep, L->stage_stream);
     cap = c0;
     dev_grow(L->d_gid, cap, n, keep, L->stage_stream);
+    cap = c0;
+    dev_grow(L->d_chan, cap, n, keep, L->stage_stream);
     L->d_meta_cap = cap;
     uint64_t a = L->d_meta_n, k = n - a;
     cudaStream_t s = L->stage_stream;
@@ -197,6 +199,7 @@ void upload_meta(ffm_log* L) {
     ck(cudaMemcpyAsync(L->d_site + a, L->h_site.data() + a, k * 4, cudaMemcpyHostToDevice, s), "meta H2D");
     ck(cudaMemcpyAsync(L->d_dur + a, L->h_dur.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
     ck(cudaMemcpyAsync(L->d_gid + a, L->h_gid.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
+    ck(cudaMemcpyAsync(L->d_chan + a, L->h_chan.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
     // small records ordered by block count, largest first (counting sort): the four
     // 8-lane groups of a warp then get payloads of near-equal length (no idle lanes)
     {
@@ -246,13 +249,14 @@ int plan_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* si
 }
 
 void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes, const uint64_t* durs,
-               const uint64_t* gids, const std::vector<uint64_t>& offs, uint64_t arena_end) {
+               const uint64_t* gids, const uint64_t* chans, const std::vector<uint64_t>& offs, uint64_t arena_end) {
     bool any = !L->h_gid.empty();
     for (uint64_t i = 0; i < n; ++i) {
         L->h_site.push_back(sites[i]);
         L->h_size.push_back(sizes[i]);
         L->h_off.push_back(offs[i]);
         L->h_dur.push_back(durs[i]);
+        L->h_chan.push_back(chans ? chans[i] : 0);
         uint64_t g = gids ? gids[i] : (any ? L->last_gid + 1 : 0);
         L->h_gid.push_back(g);
         L->last_gid = g;
@@ -326,6 +330,7 @@ DevLog dev_view(const ffm_log* L) {
     d.site = L->d_site;
     d.dur = L->d_dur;
     d.gid = L->d_gid;
+    d.chan = L->d_chan;
     d.n = (uint32_t)L->h_size.size();
     d.small_order = L->d_small_order;
     d.n_small = (uint32_t)L->n_small;
@@ -627,6 +632,7 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
             L->h_off.reserve(cfg->max_records);
             L->h_dur.reserve(cfg->max_records);
             L->h_gid.reserve(cfg->max_records);
+            L->h_chan.reserve(cfg->max_records);
         }
     } catch (const CudaFail& f) {
         int code = (f.e == cudaErrorMemoryAllocation) ? FFM_E_NOMEM : FFM_E_CUDA;
@@ -643,6 +649,12 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
 
 int ffm_log_append_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes,
                          const void* const* payloads, const uint64_t* durs, const uint64_t* gids, int kind) {
+    return ffm_log_append_batch_ex(L, n, sites, sizes, payloads, durs, gids, nullptr, kind);
+}
+
+int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes,
+                            const void* const* payloads, const uint64_t* durs, const uint64_t* gids,
+                            const uint64_t* channels, int kind) {
     int st = check_state(L);
     if (st) return st;
     if (n == 0) return FFM_OK;
@@ -694,7 +706,7 @@ int ffm_log_append_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const ui
                 throw CudaFail{cudaGetLastError(), "k_gather"};
         }
         if (need_sync) ck(cudaStreamSynchronize(L->stage_stream), "append sync");   // snapshot before return
-        push_meta(L, n, sites, sizes, durs, gids, offs, end);
+        push_meta(L, n, sites, sizes, durs, gids, channels, offs, end);
         L->digests_valid = false;
         if (n > 1) upload_meta(L);
     } catch (const CudaFail& f) {
@@ -993,6 +1005,7 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
             D.site += w0;
             D.dur += w0;
             D.gid += w0;
+            D.chan += w0;
             D.n = (uint32_t)nw;
             std::vector<uint32_t> order;
             build_small_order(L, w0, n, order);
@@ -1099,7 +1112,7 @@ int ffm_log_destroy(ffm_log* L) {
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
                     W.lcount, W.lstart, W.gcount, W.pos, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
-                    W.dup, W.ben, W.cnt, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid,
+                    W.dup, W.ben, W.cnt, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
                     L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)
         if (p) cudaFree(p);

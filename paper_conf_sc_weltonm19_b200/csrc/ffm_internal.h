@@ -23,6 +23,7 @@ struct DevLog {
     const uint32_t* site;    // [n]
     const uint64_t* dur;     // [n]
     const uint64_t* gid;     // [n]
+    const uint64_t* chan;    // [n] channel (direction / destination) id, 0 = content only
     uint32_t n;
     const uint32_t* small_order;  // records <= small_bytes, sorted by block count (descending)
     uint32_t n_small;
@@ -68,6 +69,7 @@ struct RepTuple {
     uint64_t size;
     uint64_t gid;    // global gid of the class's first local record
     uint64_t off;    // arena offset on the owning rank
+    uint64_t chan;   // channel id (destination-aware variant), 0 = content only
 };
 
 struct ShardWork {
@@ -159,7 +161,7 @@ struct ffm_log {
 
     // host metadata (authoritative), program order
     std::vector<uint32_t> h_site;
-    std::vector<uint64_t> h_size, h_off, h_dur, h_gid;
+    std::vector<uint64_t> h_size, h_off, h_dur, h_gid, h_chan;
     uint64_t payload_bytes = 0;
     uint64_t n_large_chunks = 0;   // sum over size > small of ceil(size / chunk)
     uint64_t last_gid = 0;
@@ -171,6 +173,7 @@ struct ffm_log {
     uint32_t* d_site = nullptr;
     uint64_t* d_dur = nullptr;
     uint64_t* d_gid = nullptr;
+    uint64_t* d_chan = nullptr;
     uint64_t d_meta_cap = 0;       // records
     uint64_t d_meta_n = 0;         // records uploaded
     uint32_t* d_small_order = nullptr;   // small records by size class (built at upload)

@@ -260,7 +260,7 @@ __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ li
         uint64_t n = L.size[r];
         uint64_t d = finalize_digest(W.accA[r], W.accB[r], n);
         W.digest[r] = d;
-        key = group_key(d, n, digest_mask);
+        key = group_key(d, n, digest_mask, L.chan[r]);
         W.key[r] = key;
     } else {
         key = W.key[r];
@@ -292,8 +292,8 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
         if (ld != r) {
             member = true;
             uint64_t n = L.size[r];
-            if (L.size[ld] != n) {
-                // a key collision across sizes: not equal, first word differs by definition
+            if (L.size[ld] != n || L.chan[ld] != L.chan[r]) {
+                // a key collision across sizes / channels: not equal by definition
                 W.eq[r] = 0;
                 W.mis[r] = 0;
                 res_out[atomicAdd(&W.counters[0], 1u)] = r;
@@ -301,7 +301,7 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
                 W.eq[r] = 1;
                 W.mis[r] = ~0ull;
             }
-            if (n > small_bytes && L.size[ld] == n) {
+            if (n > small_bytes && L.size[ld] == n && L.chan[ld] == L.chan[r]) {
                 atomicAdd(&W.lcount[ld], (uint32_t)((n + chunk_bytes - 1) / chunk_bytes));
                 W.pos[r] = atomicAdd(&W.gcount[ld], 1u);
             }
@@ -314,7 +314,8 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
 __global__ void k_verify_fill(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
                               uint32_t small_bytes, uint32_t chunk_bytes) {
     FFM_WARP_COMPACT(n_list, list,
-                     (W.leader[r_] != r_ && L.size[r_] > small_bytes && L.size[W.leader[r_]] == L.size[r_]), {
+                     (W.leader[r_] != r_ && L.size[r_] > small_bytes && L.size[W.leader[r_]] == L.size[r_] &&
+                      L.chan[W.leader[r_]] == L.chan[r_]), {
         const uint32_t ld = W.leader[rec];
         const uint64_t n = L.size[rec];
         const uint32_t c_n = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
@@ -359,7 +360,7 @@ __global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const
         const uint32_t ld = W.leader[m];
         if (ld == m) continue;
         const uint64_t n = L.size[m];
-        if (n > small_bytes || L.size[ld] != n) continue;   // large path / resolved by k_leader
+        if (n > small_bytes || L.size[ld] != n || L.chan[ld] != L.chan[m]) continue;   // large / k_leader
         uint64_t word = ~0ull;
         {
             const uint8_t* pm = L.arena + L.off[m];

@@ -40,10 +40,11 @@ __global__ void k_rep_export(DevLog L, Work W, const uint32_t* __restrict__ rep_
     if (r >= L.n || W.leader[r] != r) return;
     uint64_t n = L.size[r];
     RepTuple t;
-    t.key = group_key(W.digest[r], n, digest_mask);
+    t.key = group_key(W.digest[r], n, digest_mask, L.chan[r]);
     t.size = n;
     t.gid = L.gid[r];
     t.off = L.off[r];
+    t.chan = L.chan[r];
     out[rep_idx[r]] = t;
 }
 
@@ -89,8 +90,8 @@ __global__ void k_merge_classify(const RepTuple* __restrict__ T, uint32_t lo, ui
     if (c == t) {
         st = kDone;
         S.G[j] = T[t].gid;
-    } else if (owner_of(c, rank_lo, world) == rank || T[c].size != T[t].size) {
-        st = kSlow;     // same key, different exact local class (or size): not equal
+    } else if (owner_of(c, rank_lo, world) == rank || T[c].size != T[t].size || T[c].chan != T[t].chan) {
+        st = kSlow;     // same key, different exact local class (or size / channel): not equal
     } else {
         st = kVerify;
         S.cand[j] = c;
@@ -175,7 +176,8 @@ __global__ void __launch_bounds__(256) k_merge_slow(const RepTuple* __restrict__
             uint32_t s = s0 + lane;
             uint32_t y = s < M ? order[s] : 0;
             bool earlier = s < M && T[y].gid < tx.gid;
-            bool cand = earlier && T[y].key == tx.key && T[y].size == tx.size && owner_of(y, rank_lo, world) != rank;
+            bool cand = earlier && T[y].key == tx.key && T[y].size == tx.size && T[y].chan == tx.chan &&
+                        owner_of(y, rank_lo, world) != rank;
             unsigned any_earlier = __ballot_sync(0xFFFFFFFFu, earlier);
             unsigned cm = __ballot_sync(0xFFFFFFFFu, cand);
             while (cm) {

@@ -27,7 +27,8 @@ def _online(ffm, lg, cuts, **kw):
         for c in list(cuts) + [lg.n]:
             if c > prev:
                 sl = slice(prev, c)
-                log.append_batch(lg.site[sl], lg.size[sl], ptrs[sl], lg.dur[sl])
+                log.append_batch(lg.site[sl], lg.size[sl], ptrs[sl], lg.dur[sl],
+                                 channels=None if lg.channel is None else lg.channel[sl])
             d, b = log.online_step()
             dups.append(d.copy())
             bens.append((c, b.copy()))
@@ -62,3 +63,13 @@ def test_online_single_record_windows_and_empty_steps(ffm):
     with ffm.FfmLog(2) as log:                # a step with nothing pending
         d, b = log.online_step()
         assert len(d) == 0 and b.tolist() == [0, 0]
+
+
+def test_online_with_channels(ffm):
+    lg = loggen.gen_config(2, n_scale=0.01)
+    lg.channel = (lg.site.astype(np.uint64) % np.uint64(3))
+    want_d, want_b = oracle.dedup(lg)
+    got_d, bens, bd, bb = _online(ffm, lg, [100, 2000, 7000], digest_bits=8)
+    np.testing.assert_array_equal(got_d, want_d)
+    np.testing.assert_array_equal(bd, want_d)
+    np.testing.assert_array_equal(bb, want_b)

@@ -52,6 +52,8 @@ def test_golden(ffm, name, digest_bits):
     lg = loggen.from_payloads([bytes.fromhex(r["hex"]) for r in fx["records"]],
                               [r["site"] for r in fx["records"]], [r["dur"] for r in fx["records"]],
                               fx["n_sites"])
+    if "channel" in fx["records"][0]:
+        lg.channel = np.asarray([r["channel"] for r in fx["records"]], np.uint64)
     dup, ben, _ = gpu_dedup(ffm, lg, digest_bits=digest_bits)
     assert dup.tolist() == fx["expect_duplicate_of"]
     assert ben.tolist() == fx["expect_benefit_ns"]
@@ -301,3 +303,19 @@ def test_full_size_configs_4_5(ffm, k):
     np.testing.assert_array_equal(dup, want_dup)
     np.testing.assert_array_equal(ben, want_ben)
     np.testing.assert_array_equal(dup, lg.planted_duplicate_of())
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_channels_destination_aware(ffm, seed, digest_bits):
+    """S8(f) #3: a record duplicates only an earlier one with equal bytes AND channel."""
+    lg = _rand_log(100 + seed, 300, 10, 600)
+    rng = np.random.default_rng(seed)
+    lg.channel = rng.integers(0, 3, lg.n).astype(np.uint64)
+    dup, ben, _ = gpu_dedup(ffm, lg, digest_bits=digest_bits, chunk_bytes=1024, small_bytes=128)
+    assert_same(lg, dup, ben)
+    big = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 32)
+    big.channel = (big.site.astype(np.uint64) * np.uint64(7) + rng.integers(0, 2, big.n).astype(np.uint64)) \
+        % np.uint64(5)
+    dup, ben, _ = gpu_dedup(ffm, big, digest_bits=digest_bits)
+    assert_same(big, dup, ben)

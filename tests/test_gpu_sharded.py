@@ -32,8 +32,11 @@ CASES = {
 
 
 def _make(case):
-    c = CASES[case]
-    return loggen.gen_config(c["k"], n_scale=c["n_scale"], size_scale=c["size_scale"])
+    c = CASES[case.replace("+ch", "")]
+    lg = loggen.gen_config(c["k"], n_scale=c["n_scale"], size_scale=c["size_scale"])
+    if case.endswith("+ch"):        # destination-aware variant (S8(f) #3)
+        lg.channel = np.random.default_rng(3).integers(0, 2, lg.n).astype(np.uint64)
+    return lg
 
 
 def _worker(rank, world, port, out_dir, case, policy, digest_bits, device_payloads):
@@ -114,3 +117,8 @@ def test_forced_collisions_sharded(tmp_path, digest_bits):
 
 def test_four_ranks_device_payloads(tmp_path):
     _run(tmp_path, 4, "c5", 0, device_payloads=True)
+
+
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_sharded_with_channels(tmp_path, digest_bits):
+    _run(tmp_path, 3, "c5+ch", 1, digest_bits=digest_bits)
