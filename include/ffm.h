@@ -51,7 +51,12 @@ enum { FFM_PAYLOAD_AUTO = 0,        /* detected per pointer (cudaPointerGetAttri
                                        read over PCIe by the gather kernel or the copy engines */ };
 
 /* ffm_config.flags */
-enum { FFM_FLAG_TIMING = 1u /* record per-stage CUDA events (ffm_last_run_stats) */ };
+enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_stats) */
+       FFM_FLAG_PREFILTER = 2u   /* S8(f) #4: ffm_dedup_run hashes only the first chunk of a large
+                                    payload whose (size, first-chunk NH, channel) is unique in the log
+                                    -- it cannot equal any other payload.  Same results, fewer bytes.
+                                    Ignored by ffm_shard_* and ffm_online_step (uniqueness within one
+                                    shard / window says nothing about the others). */ };
 
 typedef struct ffm_config {
     uint32_t n_sites;      /* call_site must be < n_sites.  Sites are caller-interned stack
@@ -152,6 +157,7 @@ typedef struct ffm_run_stats {
     uint64_t kernel_launches;   /* kernels this library launched in the last run */
     uint64_t hash_items;        /* large-payload hash work units */
     uint64_t verify_items;      /* large-payload verify work units */
+    uint64_t prefilter_rest_bytes; /* FFM_FLAG_PREFILTER: bytes hashed beyond first chunks */
 } ffm_run_stats;
 
 /* Statistics of the last ffm_dedup_run. */

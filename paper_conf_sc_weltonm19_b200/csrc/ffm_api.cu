@@ -22,7 +22,7 @@ constexpr uint64_t kDirectCopy = 4ull << 20;      // host payloads above this by
 constexpr uint64_t kGatherMaxDefault = 1ull << 20;   // payloads up to this use k_gather (not DMA)
 
 struct LocalRun {
-    uint64_t n_members, n_res_total, rounds;
+    uint64_t n_members, n_res_total, rounds, prefilter_rest;
 };
 
 struct CudaFail {
@@ -369,7 +369,8 @@ void run_prologue(ffm_log* L) {
 // leader (the min local index of its exact byte class).  With `label` the H5/H6
 // kernels are queued before the first sync (single-GPU fast path: one sync when
 // there are no digest collisions) and re-run after collision resolution.
-LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& launches, bool label, int64_t* d_dup) {
+LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& launches, bool label, int64_t* d_dup,
+                   bool prefilter = false) {
     const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
     const uint64_t n = D.n;
     Work& W = L->work;
@@ -389,9 +390,17 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     if (n_large) {
         LCHK(launch_hash_plan(D, W, L->params, s));
         if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
-        LCHK(launch_hash_large(D, W, L->params, n_large, s));
+        if (prefilter) {
+            // S8(f) #4: first chunks, prefix keys, then the rest of non-unique payloads only
+            LCHK(launch_hash_large(D, W, L->params, n_large, s, 1));
+            uint64_t capp = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
+            LCHK(launch_prefilter(D, W, L->params, capp, s));
+            LCHK(launch_hash_large(D, W, L->params, n_large, s, 2));
+        } else {
+            LCHK(launch_hash_large(D, W, L->params, n_large, s));
+        }
         if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
-        LCHK(launch_hash_combine(D, W, L->params, s));
+        LCHK(launch_hash_combine(D, W, L->params, s, prefilter));
     }
     ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
     if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
@@ -409,6 +418,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
     ck(cudaStreamSynchronize(s), "run sync");
     R.n_members = L->h_counters[1];
+    R.prefilter_rest = (uint64_t)L->h_counters[4] | ((uint64_t)L->h_counters[5] << 32);
     uint64_t nres = L->h_counters[0];
     R.n_res_total = nres;
     if (nres) {
@@ -446,6 +456,7 @@ void fill_stats(ffm_log* L, const LocalRun& R, uint64_t launches, bool single) {
     S.resolve_rounds = R.rounds;
     S.kernel_launches = launches;
     S.hash_items = L->n_large_chunks;
+    S.prefilter_rest_bytes = R.prefilter_rest;
     if (timing) {
         S.ms_hash_small = ev_ms(L->ev[12], L->ev[8]);
         S.ms_hash_large = L->n_large_chunks ? ev_ms(L->ev[10], L->ev[11]) : 0.0;
@@ -747,7 +758,8 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         bool ben_dev = ben_out && is_device_ptr(ben_out);
         int64_t* d_dup = dup_dev ? dup_out : W.dup;
         uint64_t launches = 0;
-        LocalRun R = run_local(L, dev_view(L), L->n_large_chunks, launches, true, d_dup);
+        const bool prefilter = (L->cfg.flags & FFM_FLAG_PREFILTER) != 0;
+        LocalRun R = run_local(L, dev_view(L), L->n_large_chunks, launches, true, d_dup, prefilter);
         // H7 return
         const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
         if (timing) ck(cudaEventRecord(L->ev[9], s), "event");

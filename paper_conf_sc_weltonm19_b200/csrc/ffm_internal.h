@@ -111,8 +111,9 @@ struct Params {
 // number of kernels it launched (for the launch count), or -1 on launch error.
 int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
-int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st);
-int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
+int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st, int phase = 0);
+int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st, bool prefiltered = false);
+int launch_prefilter(const DevLog& L, Work& W, const Params& P, uint64_t cap, cudaStream_t st);
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
                  uint64_t cap, int round, uint32_t* res_out, cudaStream_t st);
 int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,

@@ -151,9 +151,12 @@ __global__ void __launch_bounds__(256, 4) k_hash_small(DevLog L, uint32_t small_
 // ----------------------------------------------------------------------------
 constexpr int kLargeU = 4;
 
+// phase 0: every unit; phase 1: first chunks only; phase 2: the other chunks of
+// records that are not prefix-singletons (S8(f) #4 pre-filter, `single` flags).
 __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __restrict__ items,
                                                     const uint32_t* __restrict__ n_items_ptr, uint32_t chunk_bytes,
-                                                    uint64_t* __restrict__ part) {
+                                                    uint64_t* __restrict__ part, int phase,
+                                                    const uint32_t* __restrict__ single) {
     const int lane = threadIdx.x & 31;
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -162,6 +165,8 @@ __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __
     for (uint32_t it = warp; it < n_items; it += nwarps) {
         const uint2 w = items[it];
         const uint32_t r = w.x;
+        if (phase == 1 && w.y != 0) continue;
+        if (phase == 2 && (w.y == 0 || single[r])) continue;
         const uint64_t n = L.size[r];
         const uint8_t* base = L.arena + L.off[r];
         const uint32_t nblk = (uint32_t)((n + 31) >> 5);
@@ -203,10 +208,11 @@ __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __
 // accumulators are the sums of its chunks' -- no atomics, deterministic).
 __global__ void k_hash_combine(DevLog L, uint32_t small_bytes, const uint32_t* __restrict__ start,
                                const uint64_t* __restrict__ part, uint64_t* __restrict__ accA,
-                               uint64_t* __restrict__ accB) {
+                               uint64_t* __restrict__ accB, const uint32_t* __restrict__ single) {
     const uint32_t* nolist = nullptr;
     FFM_WARP_COMPACT(L.n, nolist, (L.size[r_] > small_bytes), {
-        const uint32_t s0 = start[rec], e0 = start[rec + 1];
+        const uint32_t s0 = start[rec];
+        const uint32_t e0 = (single && single[rec]) ? s0 + 1 : start[rec + 1];   // pre-filter: prefix only
         uint64_t A = 0, B = 0;
         for (uint32_t it = s0 + lane; it < e0; it += 32) {
             A += part[2ull * it];
@@ -641,19 +647,71 @@ int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st)
     return 3;
 }
 
-int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st) {
+int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st, int phase) {
     if (n_items == 0) return 0;
     uint32_t grid = resident_grid((const void*)k_hash_large, P.num_sms);
     uint32_t need = blocks_for(n_items * 32);
-    k_hash_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W.hitems, W.hstart + L.n, P.chunk_bytes, W.hpart);
+    k_hash_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W.hitems, W.hstart + L.n, P.chunk_bytes, W.hpart,
+                                                            phase, W.eq);
     FFM_LAUNCH_CHECK();
     return 1;
 }
 
-int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
+// S8(f) #4 size / prefix pre-filter: key every large payload by (size, NH of its first
+// chunk, channel) and count; a payload whose prefix key is unique cannot equal any
+// other payload of the log (equal payloads have equal sizes and first chunks), so its
+// remaining chunks are never read.  Single-log batch runs only.
+__global__ void k_prefix_insert(DevLog L, Work W, uint32_t small_bytes, uint64_t cap_mask) {
+    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= L.n) return;
+    const uint64_t n = L.size[r];
+    if (n <= small_bytes) return;
+    const uint32_t it = W.hstart[r];
+    const uint64_t pk = not_empty(fmix64(W.hpart[2ull * it] ^ fmix64(W.hpart[2ull * it + 1] ^ fmix64(n)) ^
+                                         fmix64(L.chan[r] + 0x51ED270B27F4A4A5ull)));
+    uint64_t h = pk & cap_mask;
+    while (true) {
+        unsigned long long prev =
+            atomicCAS((unsigned long long*)&W.tkey[h], (unsigned long long)kEmptyKey, (unsigned long long)pk);
+        if (prev == kEmptyKey || prev == pk) break;
+        h = (h + 1) & cap_mask;
+    }
+    atomicAdd(&W.tval[h], 1u);
+    W.slot[r] = (uint32_t)h;
+}
+
+__global__ void k_prefix_flag(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes) {
+    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+    uint64_t rest = 0;
+    if (r < L.n) {
+        const uint64_t n = L.size[r];
+        uint32_t single = 0;
+        if (n > small_bytes) {
+            single = W.tval[W.slot[r]] == 1u;
+            if (!single && n > chunk_bytes) rest = n - chunk_bytes;
+        }
+        W.eq[r] = single;
+    }
+    // bytes the second phase will hash (for the roofline accounting)
+    for (int o = 16; o; o >>= 1) rest += __shfl_xor_sync(0xFFFFFFFFu, rest, o);
+    if ((threadIdx.x & 31) == 0 && rest) atomicAdd((unsigned long long*)(W.counters + 4), (unsigned long long)rest);
+}
+
+int launch_prefilter(const DevLog& L, Work& W, const Params& P, uint64_t cap, cudaStream_t st) {
+    if (L.n == 0) return 0;
+    if (cudaMemsetAsync(W.tkey, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(W.tval, 0, cap * sizeof(uint32_t), st) != cudaSuccess) return -1;
+    k_prefix_insert<<<blocks_for(L.n), 256, 0, st>>>(L, W, P.small_bytes, cap - 1);
+    FFM_LAUNCH_CHECK();
+    k_prefix_flag<<<blocks_for(L.n), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes);
+    FFM_LAUNCH_CHECK();
+    return 2;
+}
+
+int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st, bool prefiltered) {
     if (L.n == 0) return 0;
     k_hash_combine<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, P.small_bytes, W.hstart, W.hpart, W.accA,
-                                                                     W.accB);
+                                                                     W.accB, prefiltered ? W.eq : nullptr);
     FFM_LAUNCH_CHECK();
     return 1;
 }

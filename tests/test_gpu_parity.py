@@ -319,3 +319,25 @@ def test_channels_destination_aware(ffm, seed, digest_bits):
         % np.uint64(5)
     dup, ben, _ = gpu_dedup(ffm, big, digest_bits=digest_bits)
     assert_same(big, dup, ben)
+
+
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_prefilter_same_results(ffm, digest_bits):
+    """S8(f) #4: skipping the rest of payloads with a unique (size, first chunk) prefix
+    changes no output -- near-duplicates (configs 3, 4) share prefixes and still resolve."""
+    for k, ns, ss in [(1, 0.5, 0.25), (3, 0.03, 1 / 16), (4, 0.1, 1 / 64), (5, 0.003, 1 / 32)]:
+        lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
+        dup, ben, st = gpu_dedup(ffm, lg, prefilter=True, digest_bits=digest_bits, chunk_bytes=4096)
+        assert_same(lg, dup, ben)
+        large = lg.size > 4096
+        assert st["prefilter_rest_bytes"] <= int((lg.size[large] - 4096).clip(0).sum())
+
+
+def test_prefilter_full_size_config5(ffm):
+    lg = loggen.gen_config(5)
+    lg.materialize(nthreads=0)
+    want_dup, want_ben = oracle.dedup(lg)
+    dup, ben, st = gpu_dedup(ffm, lg, prefilter=True)
+    np.testing.assert_array_equal(dup, want_dup)
+    np.testing.assert_array_equal(ben, want_ben)
+    assert st["prefilter_rest_bytes"] < 0.8 * lg.total_bytes
