@@ -195,7 +195,7 @@ def run_ours(args):
     ptrs = (lg.c_off[lg.content] + np.uint64(content.data_ptr())).astype(np.uint64)
     log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * len(idx) + (1 << 20),
                      max_records=len(idx), timing=True, rank=rank, world=world,
-                     prefilter=args.prefilter and world == 1)
+                     prefilter=args.prefilter and world == 1, digest_bits=args.digest_bits)
     log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE,
                    gids=idx if world > 1 else None, idx=idx if world > 1 else None)
     del content
@@ -296,13 +296,15 @@ def run_ours(args):
                    "parallelism": "single GPU" if world == 1 else
                    f"{world} shards (site-affinity LPT); NCCL all-gather of class representatives, "
                    "in-kernel peer byte verify over NVLink, NCCL all-reduce of benefit",
-                   "chunk_bytes": 32768, "small_bytes": 4096, "prefilter": bool(args.prefilter and world == 1)},
+                   "chunk_bytes": 32768, "small_bytes": 4096, "prefilter": bool(args.prefilter and world == 1),
+                   "digest_bits": args.digest_bits},
         "pct_hbm_roofline_path": round(path_gbs / peak, 4),
         "path_alg_gbs": round(path_gbs, 1),
         "stage_ms": {k: round(st[k], 4) for k in ("ms_hash_small", "ms_hash_large", "ms_group", "ms_verify",
                                                   "ms_resolve", "ms_label", "ms_output", "ms_total")},
         "clocks": clk, "gpu_launches": launches, "roofline": roofline, "e2e": e2e, "cpu_baseline": cpu,
         "duplicates_rank0": int((dup_h >= 0).sum()),
+        "collisions": {"residual_members": int(round(st["n_residual"])), "resolve_rounds": int(round(st["resolve_rounds"]))},
     }
     print(json.dumps(out), flush=True)
     if world > 1:
@@ -338,13 +340,17 @@ def run_e2e(args, lg, local, rank=0, world=1):
     dup_pin = torch.empty(max(n, 1), dtype=torch.int64).pin_memory()
     ben_pin = torch.empty(lg.n_sites, dtype=torch.int64).pin_memory()
     times, phases = [], []
+    # one long-lived log (allocated once, like any buffer); every step empties it
+    # (ffm_log_reset keeps the HBM allocations), appends every payload from pinned
+    # host memory (H2D inside the step), runs, and reads the results back (D2H).
+    log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * n + (1 << 20),
+                     max_records=n, rank=rank, world=world)
     for step in range(args.e2e_steps + 1):
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
         t0 = time.perf_counter()
-        log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * n + (1 << 20),
-                         max_records=n, rank=rank, world=world)
+        log.reset()
         t1 = time.perf_counter()
         log.append_batch(lg.site[idx], lg.size[idx], ptrs, lg.dur[idx],
                          gids=idx if world > 1 else None,
@@ -355,20 +361,19 @@ def run_e2e(args, lg, local, rank=0, world=1):
             d, b = sharded.dedup_sharded(log, dev)
             dup_pin[:n].copy_(d[:n])
             ben_pin.copy_(b)
-            dist.barrier()           # peers stop reading this arena before it is freed
+            dist.barrier()           # peers stop reading this arena before it is reused
         else:
             log.run(dup_pin.numpy(), ben_pin.numpy().view(np.uint64))
         t3 = time.perf_counter()
-        log.close()
-        t4 = time.perf_counter()
-        sec_step = t4 - t0
+        sec_step = t3 - t0
         if world > 1:
             tt = torch.tensor([sec_step], dtype=torch.float64, device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             sec_step = float(tt.item())
         if step > 0:                     # first step warms up
             times.append(sec_step)
-            phases.append((t1 - t0, t2 - t1, t3 - t2, t4 - t3))
+            phases.append((t1 - t0, t2 - t1, t3 - t2))
+    log.close()
     if reg == 0:
         cudart.cudaHostUnregister(buf.ctypes.data)
     sec = statistics.median(times)
@@ -376,9 +381,10 @@ def run_e2e(args, lg, local, rank=0, world=1):
     return {"value": round(lg.total_bytes / sec / 1e9, 3), "unit": UNIT,
             "h2d_bytes_per_step": int(lg.total_bytes + meta * world), "d2h_bytes_per_step": int(8 * lg.n + 8 * lg.n_sites * world),
             "steps": len(times), "s_per_step": round(sec, 4),
-            "phases_s": dict(zip(("create", "append_h2d", "run", "destroy"),
+            "phases_s": dict(zip(("reset", "append_h2d", "run_d2h"),
                                  [round(statistics.median(p), 4) for p in zip(*phases)])),
-            "note": "wall clock per step: create + append (pinned host -> HBM) + run + D2H, median"}
+            "note": "wall clock per step on a reused log: ffm_log_reset + append (pinned host -> HBM) + "
+                    "run + D2H of duplicate_of/benefit, median"}
 
 
 def oracle_sample(lg, seconds_budget):
@@ -459,6 +465,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-step-seconds", type=float, default=6.0)
+    ap.add_argument("--digest-bits", type=int, default=64,
+                    help="< 64 truncates the group-by digest (forced collisions, verify stress; config 3)")
     ap.add_argument("--prefilter", action="store_true",
                     help="S8(f) #4 size/prefix pre-filter (opt-in; single GPU); roofline counts bytes required")
     args = ap.parse_args()

@@ -253,6 +253,11 @@ int ffm_shard_local(ffm_log* log, ffm_rep* reps_out, uint64_t cap, uint64_t* n_r
 int ffm_shard_merge(ffm_log* log, const ffm_rep* all_reps, const uint64_t* counts, int64_t* duplicate_of,
                     uint64_t* benefit_partial);
 
+/* Empty the log (records, online state) but keep every allocation (HBM arena, work
+   buffers, staging ring): the next batch of transfers reuses them.  Peer mappings of
+   a sharded log stay valid while the arena is not reallocated. */
+int ffm_log_reset(ffm_log* log);
+
 /* Destroy the log and release its memory.  NULL is a no-op (returns FFM_OK). */
 int ffm_log_destroy(ffm_log* log);
 

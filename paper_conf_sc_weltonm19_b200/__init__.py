@@ -30,7 +30,7 @@ EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_appen
            "ffm_last_run_stats", "ffm_debug_digests", "ffm_log_destroy", "ffm_strerror",
            "ffm_last_error", "ffm_version", "ffm_shard_plan", "ffm_shard_ipc_handle", "ffm_shard_open_peer",
            "ffm_shard_local", "ffm_shard_merge", "ffm_site_duplicate_counts", "ffm_fold_sites",
-           "ffm_online_step", "ffm_online_done"]
+           "ffm_online_step", "ffm_online_done", "ffm_log_reset"]
 FFM_SHARD_SITE_LPT, FFM_SHARD_CONTIGUOUS = 0, 1
 REP_WORDS = 5        # ffm_rep = {key, size, gid, off, chan}, 5 x u64
 
@@ -95,6 +95,8 @@ def lib() -> ctypes.CDLL:
         L.ffm_last_run_stats.restype = i32
         L.ffm_debug_digests.argtypes = [vp, vp]
         L.ffm_debug_digests.restype = i32
+        L.ffm_log_reset.argtypes = [vp]
+        L.ffm_log_reset.restype = i32
         L.ffm_log_destroy.argtypes = [vp]
         L.ffm_log_destroy.restype = i32
         L.ffm_strerror.argtypes = [i32]
@@ -220,6 +222,10 @@ def ffm_debug_digests(h) -> np.ndarray:
     out = np.empty(max(1, ffm_log_count(h)), np.uint64)
     _check(h, lib().ffm_debug_digests(h, _addr(out)))
     return out[:ffm_log_count(h)]
+
+
+def ffm_log_reset(h):
+    _check(h, lib().ffm_log_reset(h))
 
 
 def ffm_log_destroy(h):
@@ -367,6 +373,10 @@ class FfmLog:
 
     def fold(self, site_values, site_to_group, n_groups, out=None):
         return ffm_fold_sites(self.h, site_values, site_to_group, n_groups, out)
+
+    def reset(self):
+        """Empty the log, keep its HBM allocations (ffm_log_reset)."""
+        ffm_log_reset(self.h)
 
     def close(self):
         if self.h:

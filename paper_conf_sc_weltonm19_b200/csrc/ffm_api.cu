@@ -250,21 +250,29 @@ int plan_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* si
 
 void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes, const uint64_t* durs,
                const uint64_t* gids, const uint64_t* chans, const std::vector<uint64_t>& offs, uint64_t arena_end) {
-    bool any = !L->h_gid.empty();
+    const uint64_t base = L->h_size.size();
+    bool any = base > 0;
+    L->h_site.insert(L->h_site.end(), sites, sites + n);
+    L->h_size.insert(L->h_size.end(), sizes, sizes + n);
+    L->h_off.insert(L->h_off.end(), offs.begin(), offs.begin() + n);
+    L->h_dur.insert(L->h_dur.end(), durs, durs + n);
+    if (chans)
+        L->h_chan.insert(L->h_chan.end(), chans, chans + n);
+    else
+        L->h_chan.resize(base + n, 0);
+    if (gids) {
+        L->h_gid.insert(L->h_gid.end(), gids, gids + n);
+        L->any_gid = true;
+    } else {
+        L->h_gid.resize(base + n);
+        uint64_t g = any ? L->last_gid + 1 : 0;
+        for (uint64_t i = 0; i < n; ++i) L->h_gid[base + i] = g + i;
+    }
+    if (n) L->last_gid = L->h_gid.back();
     for (uint64_t i = 0; i < n; ++i) {
-        L->h_site.push_back(sites[i]);
-        L->h_size.push_back(sizes[i]);
-        L->h_off.push_back(offs[i]);
-        L->h_dur.push_back(durs[i]);
-        L->h_chan.push_back(chans ? chans[i] : 0);
-        uint64_t g = gids ? gids[i] : (any ? L->last_gid + 1 : 0);
-        L->h_gid.push_back(g);
-        L->last_gid = g;
-        any = true;
         L->payload_bytes += sizes[i];
         L->n_large_chunks += large_chunks(L, sizes[i]);
     }
-    if (gids) L->any_gid = true;
     L->arena_used = arena_end;
 }
 
@@ -679,6 +687,7 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
         ck(cudaSetDevice(L->device), "cudaSetDevice");
         ensure_arena(L, end);
         std::vector<uint64_t> desc;
+        if (kind == FFM_PAYLOAD_DEVICE || kind == FFM_PAYLOAD_HOST_PINNED) desc.reserve(3 * n);
         bool need_sync = false;
         for (uint64_t i = 0; i < n; ++i) {
             if (sizes[i] == 0) continue;
@@ -1113,6 +1122,40 @@ int ffm_debug_digests(ffm_log* L, uint64_t* out) {
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
     }
+    return FFM_OK;
+}
+
+int ffm_log_reset(ffm_log* L) {
+    int st = check_state(L);
+    if (st) return st;
+    try {
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
+        ck(cudaStreamSynchronize(L->stage_stream), "reset sync");
+        ck(cudaStreamSynchronize(L->stream), "reset sync");
+    } catch (const CudaFail& f) {
+        return fail_cuda(L, f);
+    }
+    L->h_site.clear();
+    L->h_size.clear();
+    L->h_off.clear();
+    L->h_dur.clear();
+    L->h_gid.clear();
+    L->h_chan.clear();
+    L->payload_bytes = L->n_large_chunks = L->last_gid = 0;
+    L->any_gid = false;
+    L->d_meta_n = 0;
+    L->n_small = 0;
+    L->arena_used = 0;
+    L->ring_fill = 0;
+    L->n_reps = 0;
+    L->reps_valid = false;
+    L->online_done = L->online_np = 0;
+    if (L->online_ben) {
+        cudaMemset(L->online_ben, 0, L->cfg.n_sites * sizeof(uint64_t));
+        cudaMemset(L->online_cnt, 0, L->cfg.n_sites * sizeof(uint64_t));
+    }
+    L->digests_valid = false;
+    memset(&L->stats, 0, sizeof(L->stats));
     return FFM_OK;
 }
 

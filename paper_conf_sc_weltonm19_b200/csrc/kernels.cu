@@ -567,17 +567,31 @@ __global__ void k_fold(const uint64_t* __restrict__ site_vals, const uint32_t* _
 // H0 helper: snapshot device-resident payloads into the arena (one warp per record).
 // desc[3i] = src address, desc[3i+1] = arena offset, desc[3i+2] = size.
 // ----------------------------------------------------------------------------
-__global__ void k_gather(const uint64_t* __restrict__ desc, uint32_t n, uint8_t* __restrict__ arena) {
+__global__ void __launch_bounds__(256) k_gather(const uint64_t* __restrict__ desc, uint32_t n,
+                                                uint8_t* __restrict__ arena) {
     const int lane = threadIdx.x & 31;
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    constexpr int U = 4;   // 4 x 16 B in flight per lane: PCIe (pinned host) reads are latency-bound
     for (uint32_t i = warp; i < n; i += nwarps) {
         const uint8_t* src = (const uint8_t*)desc[3 * i];
         uint8_t* dst = arena + desc[3 * i + 1];
         const uint64_t sz = desc[3 * i + 2];
         if (((uintptr_t)src & 15) == 0) {
             const uint64_t nv = sz >> 4;
-            for (uint64_t k = lane; k < nv; k += 32) ((uint4*)dst)[k] = ((const uint4*)src)[k];
+            for (uint64_t k0 = 0; k0 < nv; k0 += 32 * U) {
+                uint4 v[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    uint64_t k = k0 + 32 * u + lane;
+                    if (k < nv) v[u] = ((const uint4*)src)[k];
+                }
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    uint64_t k = k0 + 32 * u + lane;
+                    if (k < nv) ((uint4*)dst)[k] = v[u];
+                }
+            }
             for (uint64_t k = (nv << 4) + lane; k < sz; k += 32) dst[k] = src[k];
         } else {
             for (uint64_t k = lane; k < sz; k += 32) dst[k] = src[k];

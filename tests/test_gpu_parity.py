@@ -341,3 +341,23 @@ def test_prefilter_full_size_config5(ffm):
     np.testing.assert_array_equal(dup, want_dup)
     np.testing.assert_array_equal(ben, want_ben)
     assert st["prefilter_rest_bytes"] < 0.8 * lg.total_bytes
+
+
+def test_reset_reuses_the_log(ffm):
+    a = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 32)
+    b = loggen.gen_config(2, n_scale=0.003)
+    b.n_sites = a.n_sites           # same site space for one log
+    with ffm.FfmLog(a.n_sites) as log:
+        log.append_log(a)
+        d1, b1 = [x.copy() for x in log.run()]
+        log.reset()
+        assert log.count == 0
+        log.append_log(b)
+        d2, b2 = [x.copy() for x in log.run()]
+        log.reset()
+        log.append_log(a)
+        d3, _ = log.online_step()
+        d3 = d3.copy()
+    assert_same(a, d1, b1)
+    assert_same(b, d2, b2)
+    np.testing.assert_array_equal(d3, d1)
