@@ -53,8 +53,8 @@ enum { FFM_PAYLOAD_AUTO = 0,        /* detected per pointer (cudaPointerGetAttri
 /* ffm_config.flags */
 enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_stats) */
        FFM_FLAG_PREFILTER = 2u   /* S8(f) #4: ffm_dedup_run hashes only the first chunk of a large
-                                    payload whose (size, first-chunk NH, channel) is unique in the log
-                                    -- it cannot equal any other payload.  Same results, fewer bytes.
+                                    payload whose (size, first-chunk digest, channel) is unique in the
+                                    log -- it cannot equal any other payload.  Same results, fewer bytes.
                                     Ignored by ffm_shard_* and ffm_online_step (uniqueness within one
                                     shard / window says nothing about the others). */ };
 
@@ -147,7 +147,7 @@ typedef struct ffm_run_stats {
     double   ms_resolve;        /* H4: collision-resolution rounds */
     double   ms_label;          /* H5+H6: label + benefit */
     double   ms_output;         /* H7: output copies */
-    double   ms_hash_large;     /* the large-payload hash kernel alone */
+    double   ms_hash_large;     /* the large-payload prefix-pass kernel alone (first chunks) */
     double   ms_hash_small;     /* the small-payload hash kernel alone */
     uint64_t n_records;
     uint64_t payload_bytes;     /* sum of sizes */
@@ -157,7 +157,8 @@ typedef struct ffm_run_stats {
     uint64_t kernel_launches;   /* kernels this library launched in the last run */
     uint64_t hash_items;        /* large-payload hash work units */
     uint64_t verify_items;      /* large-payload verify work units */
-    uint64_t prefilter_rest_bytes; /* FFM_FLAG_PREFILTER: bytes hashed beyond first chunks */
+    uint64_t prefilter_rest_bytes; /* bytes hashed beyond first chunks by the fused pass */
+    double   ms_fused;          /* the fused hash + compare kernel alone (large payloads) */
 } ffm_run_stats;
 
 /* Statistics of the last ffm_dedup_run. */

@@ -49,7 +49,8 @@ class FfmRunStats(ctypes.Structure):
                                                  "ms_label", "ms_output", "ms_hash_large", "ms_hash_small")] + \
                [(k, ctypes.c_uint64) for k in ("n_records", "payload_bytes", "n_members", "n_residual",
                                                 "resolve_rounds", "kernel_launches", "hash_items",
-                                                "verify_items", "prefilter_rest_bytes")]
+                                                "verify_items", "prefilter_rest_bytes")] + \
+               [("ms_fused", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -296,6 +296,7 @@ void ensure_work(ffm_log* L, uint64_t n) {
         dev_alloc(W.lstart, c + 1);
         dev_alloc(W.gcount, c + 1);
         dev_alloc(W.pos, c);
+        dev_alloc(W.fhead, c);
         dev_alloc(W.hcount, c + 1);
         dev_alloc(W.hstart, c + 1);
         dev_alloc(W.dup, c);
@@ -396,29 +397,28 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
     ck(cudaEventRecord(L->fork_ev[1], side), "event");
     if (n_large) {
+        // prefix pass: the first chunk of every large payload
         LCHK(launch_hash_plan(D, W, L->params, s));
         if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
-        if (prefilter) {
-            // S8(f) #4: first chunks, prefix keys, then the rest of non-unique payloads only
-            LCHK(launch_hash_large(D, W, L->params, n_large, s, 1));
-            uint64_t capp = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
-            LCHK(launch_prefilter(D, W, L->params, capp, s));
-            LCHK(launch_hash_large(D, W, L->params, n_large, s, 2));
-        } else {
-            LCHK(launch_hash_large(D, W, L->params, n_large, s));
-        }
+        LCHK(launch_hash_large(D, W, L->params, n_large, s, 1));
         if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
-        LCHK(launch_hash_combine(D, W, L->params, s, prefilter));
     }
     ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
     if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
-    // H2 group-by (round 0, all records)
+    // H2 group-by (round 0): small payloads by full digest, large ones by first-chunk digest
     uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
     LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, W.res[0], s));
     if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
-    // H3 verify
-    LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], n_large ? W.vitem_cap : 0, s, side,
-                       L->fork_ev[2], L->fork_ev[3]));
+    // H3: small members verified on the side stream while the fused pass hashes the rest
+    // of every large payload and byte-compares each large member with its group leader
+    ck(cudaEventRecord(L->fork_ev[2], s), "event");
+    ck(cudaStreamWaitEvent(side, L->fork_ev[2], 0), "fork");
+    LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], 0, side, nullptr, nullptr, nullptr));
+    ck(cudaEventRecord(L->fork_ev[3], side), "event");
+    if (n_large)
+        LCHK(launch_fused(D, W, L->params, n_large, prefilter, W.res[0], s, timing ? L->ev[16] : nullptr,
+                          timing ? L->ev[17] : nullptr));
+    ck(cudaStreamWaitEvent(s, L->fork_ev[3], 0), "join");
     if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
     // H5 + H6 (speculative: valid unless H3 found residuals)
     if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, s));
@@ -468,6 +468,7 @@ void fill_stats(ffm_log* L, const LocalRun& R, uint64_t launches, bool single) {
     if (timing) {
         S.ms_hash_small = ev_ms(L->ev[12], L->ev[8]);
         S.ms_hash_large = L->n_large_chunks ? ev_ms(L->ev[10], L->ev[11]) : 0.0;
+        S.ms_fused = L->n_large_chunks ? ev_ms(L->ev[16], L->ev[17]) : 0.0;
         S.ms_hash = ev_ms(L->ev[0], L->ev[1]);
         S.ms_group = ev_ms(L->ev[1], L->ev[2]);
         S.ms_verify = ev_ms(L->ev[2], L->ev[3]);
@@ -1166,7 +1167,7 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->stage_stream) cudaStreamSynchronize(L->stage_stream);
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
-                    W.lcount, W.lstart, W.gcount, W.pos, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
+                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
                     W.dup, W.ben, W.cnt, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
                     L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)

@@ -43,7 +43,8 @@ struct Work {
     uint32_t* lcount = nullptr;    // [n+1] per-leader verify chunk counts
     uint32_t* lstart = nullptr;    // [n+1] exclusive scan of lcount: group base of each leader
     uint32_t* gcount = nullptr;    // [n+1] large members per leader (chunk-major stride)
-    uint32_t* pos = nullptr;       // [n] position of a large member within its leader's group
+    uint32_t* pos = nullptr;       // [n] position of a large record within its fused / verify group
+    uint32_t* fhead = nullptr;     // [n] round 0: head (leader) of a large record's fused group
     uint2* hitems = nullptr;       // large-payload hash work units (record, chunk)
     uint2* vitems = nullptr;       // large-payload verify work units (member, chunk)
     uint32_t* hcount = nullptr;    // [n+1] per-record hash chunk counts
@@ -112,8 +113,8 @@ struct Params {
 int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st, int phase = 0);
-int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st, bool prefiltered = false);
-int launch_prefilter(const DevLog& L, Work& W, const Params& P, uint64_t cap, cudaStream_t st);
+int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
+                 cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b);
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
                  uint64_t cap, int round, uint32_t* res_out, cudaStream_t st);
 int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
@@ -222,7 +223,7 @@ struct ffm_log {
     ffm::Work work;
     ffm::Params params{};
     uint32_t* h_counters = nullptr;   // pinned mirror
-    cudaEvent_t ev[16] = {};
+    cudaEvent_t ev[20] = {};
     ffm_run_stats stats{};
     bool digests_valid = false;
 };

@@ -19,6 +19,26 @@
 #include "ffm_internal.h"
 #include "digest.cuh"
 
+// tuning knobs of the fused pass (defaults = the measured best)
+#ifndef FFM_FUSED_CMP_U
+#define FFM_FUSED_CMP_U 2
+#endif
+#ifndef FFM_FUSED_LEADER_FIRST
+#define FFM_FUSED_LEADER_FIRST 1
+#endif
+#ifndef FFM_FUSED_KEEP_OWN
+#define FFM_FUSED_KEEP_OWN 0
+#endif
+#ifndef FFM_FUSED_DEMOTE
+#define FFM_FUSED_DEMOTE 0
+#endif
+#ifndef FFM_FUSED_SKEW
+#define FFM_FUSED_SKEW 0x7FFFFFFF   /* measured: leader-first (no skew) is best */
+#endif
+#ifndef FFM_FUSED_Y_POLICY
+#define FFM_FUSED_Y_POLICY 1
+#endif
+
 namespace ffm {
 
 // ----------------------------------------------------------------------------
@@ -94,6 +114,27 @@ __device__ __forceinline__ void nh_blk(const Blk& x, const LaneKeys& K, uint64_t
     if (32 * b + 16 < n) nh_word(x.v[4], x.v[5], x.v[6], x.v[7], K.k[1], A, B);
 }
 
+// H3 helpers (byte comparison, mismatch reporting)
+__device__ __forceinline__ int blk_diff(const Blk& x, const Blk& y) {
+    // -1: equal; 0: first word differs; 1: only second word differs
+    uint32_t d0 = (x.v[0] ^ y.v[0]) | (x.v[1] ^ y.v[1]) | (x.v[2] ^ y.v[2]) | (x.v[3] ^ y.v[3]);
+    uint32_t d1 = (x.v[4] ^ y.v[4]) | (x.v[5] ^ y.v[5]) | (x.v[6] ^ y.v[6]) | (x.v[7] ^ y.v[7]);
+    return d0 ? 0 : (d1 ? 1 : -1);
+}
+
+__device__ __forceinline__ void report_mismatch(Work& W, uint32_t m, uint64_t word, uint32_t* res_out, bool atomic) {
+    if (atomic) {
+        atomicMin((unsigned long long*)&W.mis[m], (unsigned long long)word);
+        if (atomicExch(&W.eq[m], 0u) == 1u) res_out[atomicAdd(&W.counters[0], 1u)] = m;
+    } else {
+        W.mis[m] = word;
+        W.eq[m] = 0;
+        res_out[atomicAdd(&W.counters[0], 1u)] = m;
+    }
+}
+
+constexpr int kVerifyU = 2;
+
 // ----------------------------------------------------------------------------
 // H1a: payloads <= small_bytes, one 8-lane group ("octet") per record.  Lane g
 // reads 32-B block g of each 256-B stripe: positions 2g, 2g+1.
@@ -151,12 +192,10 @@ __global__ void __launch_bounds__(256, 4) k_hash_small(DevLog L, uint32_t small_
 // ----------------------------------------------------------------------------
 constexpr int kLargeU = 4;
 
-// phase 0: every unit; phase 1: first chunks only; phase 2: the other chunks of
-// records that are not prefix-singletons (S8(f) #4 pre-filter, `single` flags).
+// phase 0: every unit; phase 1: first chunks only (the prefix pass of round 0).
 __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __restrict__ items,
                                                     const uint32_t* __restrict__ n_items_ptr, uint32_t chunk_bytes,
-                                                    uint64_t* __restrict__ part, int phase,
-                                                    const uint32_t* __restrict__ single) {
+                                                    uint64_t* __restrict__ part, int phase) {
     const int lane = threadIdx.x & 31;
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -166,7 +205,6 @@ __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __
         const uint2 w = items[it];
         const uint32_t r = w.x;
         if (phase == 1 && w.y != 0) continue;
-        if (phase == 2 && (w.y == 0 || single[r])) continue;
         const uint64_t n = L.size[r];
         const uint8_t* base = L.arena + L.off[r];
         const uint32_t nblk = (uint32_t)((n + 31) >> 5);
@@ -204,31 +242,6 @@ __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __
     }
 }
 
-// Combine the chunk partial sums of large records (NH is a plain sum, so the record's
-// accumulators are the sums of its chunks' -- no atomics, deterministic).
-__global__ void k_hash_combine(DevLog L, uint32_t small_bytes, const uint32_t* __restrict__ start,
-                               const uint64_t* __restrict__ part, uint64_t* __restrict__ accA,
-                               uint64_t* __restrict__ accB, const uint32_t* __restrict__ single) {
-    const uint32_t* nolist = nullptr;
-    FFM_WARP_COMPACT(L.n, nolist, (L.size[r_] > small_bytes), {
-        const uint32_t s0 = start[rec];
-        const uint32_t e0 = (single && single[rec]) ? s0 + 1 : start[rec + 1];   // pre-filter: prefix only
-        uint64_t A = 0, B = 0;
-        for (uint32_t it = s0 + lane; it < e0; it += 32) {
-            A += part[2ull * it];
-            B += part[2ull * it + 1];
-        }
-        for (int o = 16; o; o >>= 1) {
-            A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
-            B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
-        }
-        if (lane == 0) {
-            accA[rec] = A;
-            accB[rec] = B;
-        }
-    })
-}
-
 // Work-unit planning for H1b / H3b: counts -> exclusive scan -> scatter.
 __global__ void k_hash_count(DevLog L, uint32_t small_bytes, uint32_t chunk_bytes, uint32_t* __restrict__ cnt) {
     uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
@@ -257,16 +270,25 @@ __global__ void k_hash_fill(DevLog L, uint32_t small_bytes, uint32_t chunk_bytes
 // resolve rounds re-key residual lists (k_refine) and reuse this kernel.
 // ----------------------------------------------------------------------------
 __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
-                               uint64_t cap_mask, uint64_t digest_mask, int round) {
+                               uint64_t cap_mask, uint64_t digest_mask, int round, uint32_t small_bytes) {
     uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n_list) return;
     uint32_t r = list ? list[i] : i;
     uint64_t key;
     if (round == 0) {
         uint64_t n = L.size[r];
-        uint64_t d = finalize_digest(W.accA[r], W.accB[r], n);
-        W.digest[r] = d;
-        key = group_key(d, n, digest_mask, L.chan[r]);
+        if (n <= small_bytes) {
+            // small payload: its full digest
+            uint64_t d = finalize_digest(W.accA[r], W.accB[r], n);
+            W.digest[r] = d;
+            key = group_key(d, n, digest_mask, L.chan[r]);
+        } else {
+            // large payload: the digest of its FIRST chunk (computed by the prefix pass);
+            // equal payloads have equal first chunks, so every candidate still shares a group
+            const uint32_t it = W.hstart[r];
+            uint64_t pd = finalize_digest(W.hpart[2ull * it], W.hpart[2ull * it + 1], n);
+            key = group_key(pd, n, digest_mask, L.chan[r]);
+        }
         W.key[r] = key;
     } else {
         key = W.key[r];
@@ -317,6 +339,234 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
     if ((threadIdx.x & 31) == 0 && b) atomicAdd(&W.counters[1], (uint32_t)__popc(b));
 }
 
+// Round 0 leader lookup.  Small payloads as in k_leader.  A large payload joins the
+// fused pass's group of its leader (same size and channel): the group's work is laid
+// out chunk-major, (chunk c, position p) at lstart[head] + c * (gcount[head] + 1) + p,
+// with the leader itself at p = 0 -- the leader's chunk c is read from HBM once, by
+// its own hashing unit, and re-read from L2 by every member comparing against it.
+__global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, uint32_t chunk_bytes,
+                          uint32_t* __restrict__ res_out) {
+    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+    bool member = false;
+    if (r < n) {
+        const uint32_t ld = W.tval[W.slot[r]];
+        W.leader[r] = ld;
+        const uint64_t sz = L.size[r];
+        const bool same = L.size[ld] == sz && L.chan[ld] == L.chan[r];
+        if (ld != r) {
+            member = true;
+            if (!same) {
+                W.eq[r] = 0;            // key collision across sizes / channels: not equal
+                W.mis[r] = 0;
+                res_out[atomicAdd(&W.counters[0], 1u)] = r;
+            } else {
+                W.eq[r] = 1;
+                W.mis[r] = ~0ull;
+            }
+        }
+        if (sz > small_bytes) {
+            uint32_t head = r, p = 0;
+            if (ld != r && same) {
+                head = ld;
+                p = 1u + atomicAdd(&W.gcount[ld], 1u);
+            }
+            W.fhead[r] = head;
+            W.pos[r] = p;
+            atomicAdd(&W.lcount[head], (uint32_t)((sz + chunk_bytes - 1) / chunk_bytes));
+        }
+    }
+    unsigned b = __ballot_sync(0xFFFFFFFFu, member);
+    if ((threadIdx.x & 31) == 0 && b) atomicAdd(&W.counters[1], (uint32_t)__popc(b));
+}
+
+__global__ void k_fused_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes) {
+    const uint32_t* nolist = nullptr;
+    FFM_WARP_COMPACT(L.n, nolist, (L.size[r_] > small_bytes), {
+        const uint32_t h = W.fhead[rec];
+        const uint32_t k = W.gcount[h] + 1, p = W.pos[rec], base = W.lstart[h];
+        const uint32_t c_n = (uint32_t)((L.size[rec] + chunk_bytes - 1) / chunk_bytes);
+#if FFM_FUSED_LEADER_FIRST
+        // skewed chunk-major layout: the leader runs D chunks ahead of its members, so a
+        // member compares against a leader chunk fetched a little earlier -- an L2 hit,
+        // not a wait on the same in-flight miss, and not yet evicted.  Step t holds the
+        // leader's chunk t and the members' chunk t - D; no holes:
+        //   [0, D) leader only | [D, nch) leader + members | [nch, nch + D) members only
+        const uint32_t D = min((uint32_t)FFM_FUSED_SKEW, c_n);
+        for (uint32_t c = lane; c < c_n; c += 32) {
+            uint32_t at;
+            if (p == 0) {
+                at = c < D ? c : D + (c - D) * k;
+            } else {
+                const uint32_t t = c + D;
+                at = t < c_n ? D + c * k + p : D + (c_n - D) * k + (t - c_n) * (k - 1) + (p - 1);
+            }
+            W.vitems[base + at] = make_uint2(rec, c);
+        }
+#else
+        for (uint32_t c = lane; c < c_n; c += 32) W.vitems[base + c * k + p] = make_uint2(rec, c);
+#endif
+    })
+}
+
+// With FFM_FLAG_PREFILTER a leader whose fused group has no member has a unique
+// (size, first chunk, channel): it cannot equal any other payload, so its remaining
+// chunks are not read.
+__device__ __forceinline__ bool prefix_unique(const Work& W, uint32_t r) {
+    return W.fhead[r] == r && W.gcount[r] == 0 && W.leader[r] == r;
+}
+
+// H1 + H3 fused for large payloads (round 0): one pass over every chunk c >= 1 hashes
+// it (chunk 0 was hashed by the prefix pass) and, for a member, byte-compares it with
+// the leader's chunk c (L2-resident: the group's units run back to back); members
+// also compare chunk 0.  A member's first mismatching word is the exact minimum (a
+// chunk's compare is skipped only when a lower mismatch is known); failures go to the
+// residual list and are resolved exactly (H4) with their full digests.
+template <int U, bool kCmp>
+__device__ __forceinline__ void fused_chunk(const uint8_t* pr, const uint8_t* ph, uint64_t n, uint32_t bb,
+                                            uint32_t be, int lane, bool hashc, bool keep_own, LaneKeys& K,
+                                            uint64_t& A, uint64_t& B, uint64_t& found) {
+    for (uint32_t b0 = bb; b0 < be; b0 += 32 * U) {
+        Blk x[U], y[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint32_t b = b0 + 32 * u + lane;
+            // a group leader's own chunk is re-read by its members: keep it in L2
+            x[u] = b < be ? (keep_own ? ld_keep(pr + 32ull * b) : ld_stream(pr + 32ull * b)) : zero_blk();
+#if FFM_FUSED_Y_POLICY == 0
+            if (kCmp) y[u] = b < be ? ld_remote(ph + 32ull * b) : zero_blk();   // default L2 policy
+#elif FFM_FUSED_Y_POLICY == 2
+            if (kCmp) y[u] = b < be ? ld_stream(ph + 32ull * b) : zero_blk();
+#else
+            if (kCmp) y[u] = b < be ? ld_keep(ph + 32ull * b) : zero_blk();
+#endif
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint32_t b = b0 + 32 * u + lane;
+            if (b < be) {
+                mask_tail(x[u], n, b);
+                if (hashc) nh_blk(x[u], K, n, b, A, B);
+                if (kCmp) {
+                    mask_tail(y[u], n, b);
+                    int d = blk_diff(x[u], y[u]);
+                    if (d >= 0 && found == ~0ull) found = 2ull * b + d;
+                }
+            }
+            advance<4>(K);
+        }
+    }
+}
+
+#ifndef FFM_FUSED_MINB
+#define FFM_FUSED_MINB 3
+#endif
+__global__ void __launch_bounds__(256, FFM_FUSED_MINB) k_fused(DevLog L, Work W, const uint32_t* __restrict__ n_items_ptr,
+                                                  uint32_t chunk_bytes, int prefilter, uint32_t* res_out) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    const uint32_t n_items = *n_items_ptr;
+    const uint32_t cblk = chunk_bytes >> 5;
+    for (uint32_t it = warp; it < n_items; it += nwarps) {
+        const uint2 w = W.vitems[it];
+        const uint32_t r = w.x, c = w.y;
+        const uint32_t h = W.fhead[r];
+        const bool hashc = c > 0 && !(prefilter && prefix_unique(W, r));
+        bool cmp = h != r;
+        if (cmp) {
+            uint64_t known = lane == 0 ? *((volatile uint64_t*)&W.mis[r]) : 0;
+            known = __shfl_sync(0xFFFFFFFFu, known, 0);
+            cmp = 2ull * c * cblk < known;         // no lower mismatch known yet
+        }
+        if (!hashc && !cmp) continue;
+        const uint64_t n = L.size[r];
+        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
+        const uint32_t bb = c * cblk, be = min(bb + cblk, nblk);
+        const uint8_t* pr = L.arena + L.off[r];
+        const uint8_t* ph = L.arena + L.off[h];
+        const bool keep_own = FFM_FUSED_KEEP_OWN && h == r && W.gcount[r] > 0;
+        LaneKeys K;
+        load_keys(K, 2 * (lane & 7), (bb + lane) >> 3);
+        uint64_t A = 0, B = 0, found = ~0ull;
+        if (cmp)
+            fused_chunk<FFM_FUSED_CMP_U, true>(pr, ph, n, bb, be, lane, hashc, keep_own, K, A, B, found);
+        else
+            fused_chunk<4, false>(pr, ph, n, bb, be, lane, hashc, keep_own, K, A, B, found);
+#if FFM_FUSED_DEMOTE
+        // the group's last member hands the leader's chunk back to normal L2 priority
+        // (it was loaded evict_last so that every member hits it)
+        if (h != r && W.pos[r] == W.gcount[h]) {
+            for (uint32_t b = bb + 4 * lane; b < be; b += 128)
+                asm volatile("applypriority.global.L2::evict_normal [%0], 128;" ::"l"(ph + 32ull * b));
+        }
+#endif
+        if (hashc) {
+#pragma unroll
+            for (int o = 16; o; o >>= 1) {
+                A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
+                B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
+            }
+            if (lane == 0) {
+                const uint64_t slot = W.hstart[r] + c;
+                W.hpart[2 * slot] = A;
+                W.hpart[2 * slot + 1] = B;
+            }
+        }
+        if (cmp && __any_sync(0xFFFFFFFFu, found != ~0ull)) {
+#pragma unroll
+            for (int o = 16; o; o >>= 1) {
+                uint64_t other = __shfl_xor_sync(0xFFFFFFFFu, found, o);
+                found = other < found ? other : found;
+            }
+            if (lane == 0) report_mismatch(W, r, found, res_out, true);
+        }
+    }
+}
+
+// Combine the chunk partial sums of large records (NH is a plain sum, so the record's
+// accumulators are the sums of its chunks' -- no atomics, deterministic) and finish
+// their digests.  Also totals the bytes hashed beyond first chunks (roofline stats).
+__global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes,
+                                                      int prefilter) {
+    __shared__ unsigned long long s_rest[8];
+    const int lane = threadIdx.x & 31;
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    const bool act = i < L.n && L.size[i] > small_bytes;
+    unsigned bal = __ballot_sync(0xFFFFFFFFu, act);
+    unsigned long long rest = 0;
+    while (bal) {
+        const int src = __ffs(bal) - 1;
+        bal &= bal - 1;
+        const uint32_t rec = __shfl_sync(0xFFFFFFFFu, i, src);
+        const uint32_t s0 = W.hstart[rec];
+        const bool skip = prefilter && prefix_unique(W, rec);
+        const uint32_t e0 = skip ? s0 + 1 : W.hstart[rec + 1];
+        uint64_t A = 0, B = 0;
+        for (uint32_t it = s0 + lane; it < e0; it += 32) {
+            A += W.hpart[2ull * it];
+            B += W.hpart[2ull * it + 1];
+        }
+        for (int o = 16; o; o >>= 1) {
+            A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
+            B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
+        }
+        const uint64_t n = L.size[rec];
+        if (lane == 0) {
+            W.accA[rec] = A;
+            W.accB[rec] = B;
+            W.digest[rec] = finalize_digest(A, B, n);
+            if (!skip && n > chunk_bytes) rest += n - chunk_bytes;
+        }
+    }
+    if (lane == 0) s_rest[threadIdx.x >> 5] = rest;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long t = 0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s_rest[w];
+        if (t) atomicAdd((unsigned long long*)(W.counters + 4), t);
+    }
+}
+
 __global__ void k_verify_fill(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
                               uint32_t small_bytes, uint32_t chunk_bytes) {
     FFM_WARP_COMPACT(n_list, list,
@@ -335,25 +585,6 @@ __global__ void k_verify_fill(DevLog L, Work W, const uint32_t* __restrict__ lis
 // first mismatching 16-B word (exact minimum: a chunk is skipped only when a
 // mismatch at a lower word is already known), and appends failures to a residual list.
 // ----------------------------------------------------------------------------
-__device__ __forceinline__ int blk_diff(const Blk& x, const Blk& y) {
-    // -1: equal; 0: first word differs; 1: only second word differs
-    uint32_t d0 = (x.v[0] ^ y.v[0]) | (x.v[1] ^ y.v[1]) | (x.v[2] ^ y.v[2]) | (x.v[3] ^ y.v[3]);
-    uint32_t d1 = (x.v[4] ^ y.v[4]) | (x.v[5] ^ y.v[5]) | (x.v[6] ^ y.v[6]) | (x.v[7] ^ y.v[7]);
-    return d0 ? 0 : (d1 ? 1 : -1);
-}
-
-__device__ __forceinline__ void report_mismatch(Work& W, uint32_t m, uint64_t word, uint32_t* res_out, bool atomic) {
-    if (atomic) {
-        atomicMin((unsigned long long*)&W.mis[m], (unsigned long long)word);
-        if (atomicExch(&W.eq[m], 0u) == 1u) res_out[atomicAdd(&W.counters[0], 1u)] = m;
-    } else {
-        W.mis[m] = word;
-        W.eq[m] = 0;
-        res_out[atomicAdd(&W.counters[0], 1u)] = m;
-    }
-}
-
-constexpr int kVerifyU = 2;
 
 __global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const uint32_t* __restrict__ list,
                                                       uint32_t n_list, uint32_t small_bytes, uint32_t* res_out) {
@@ -666,68 +897,36 @@ int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_item
     uint32_t grid = resident_grid((const void*)k_hash_large, P.num_sms);
     uint32_t need = blocks_for(n_items * 32);
     k_hash_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W.hitems, W.hstart + L.n, P.chunk_bytes, W.hpart,
-                                                            phase, W.eq);
+                                                            phase);
     FFM_LAUNCH_CHECK();
     return 1;
 }
 
-// S8(f) #4 size / prefix pre-filter: key every large payload by (size, NH of its first
-// chunk, channel) and count; a payload whose prefix key is unique cannot equal any
-// other payload of the log (equal payloads have equal sizes and first chunks), so its
-// remaining chunks are never read.  Single-log batch runs only.
-__global__ void k_prefix_insert(DevLog L, Work W, uint32_t small_bytes, uint64_t cap_mask) {
-    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-    if (r >= L.n) return;
-    const uint64_t n = L.size[r];
-    if (n <= small_bytes) return;
-    const uint32_t it = W.hstart[r];
-    const uint64_t pk = not_empty(fmix64(W.hpart[2ull * it] ^ fmix64(W.hpart[2ull * it + 1] ^ fmix64(n)) ^
-                                         fmix64(L.chan[r] + 0x51ED270B27F4A4A5ull)));
-    uint64_t h = pk & cap_mask;
-    while (true) {
-        unsigned long long prev =
-            atomicCAS((unsigned long long*)&W.tkey[h], (unsigned long long)kEmptyKey, (unsigned long long)pk);
-        if (prev == kEmptyKey || prev == pk) break;
-        h = (h + 1) & cap_mask;
-    }
-    atomicAdd(&W.tval[h], 1u);
-    W.slot[r] = (uint32_t)h;
-}
-
-__global__ void k_prefix_flag(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes) {
-    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-    uint64_t rest = 0;
-    if (r < L.n) {
-        const uint64_t n = L.size[r];
-        uint32_t single = 0;
-        if (n > small_bytes) {
-            single = W.tval[W.slot[r]] == 1u;
-            if (!single && n > chunk_bytes) rest = n - chunk_bytes;
-        }
-        W.eq[r] = single;
-    }
-    // bytes the second phase will hash (for the roofline accounting)
-    for (int o = 16; o; o >>= 1) rest += __shfl_xor_sync(0xFFFFFFFFu, rest, o);
-    if ((threadIdx.x & 31) == 0 && rest) atomicAdd((unsigned long long*)(W.counters + 4), (unsigned long long)rest);
-}
-
-int launch_prefilter(const DevLog& L, Work& W, const Params& P, uint64_t cap, cudaStream_t st) {
-    if (L.n == 0) return 0;
-    if (cudaMemsetAsync(W.tkey, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
-    if (cudaMemsetAsync(W.tval, 0, cap * sizeof(uint32_t), st) != cudaSuccess) return -1;
-    k_prefix_insert<<<blocks_for(L.n), 256, 0, st>>>(L, W, P.small_bytes, cap - 1);
+// Round 0, large payloads: fused groups (scan of lcount), work units, the fused
+// hash + compare pass, then the per-record combine of chunk partial sums.
+int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
+                 cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b) {
+    if (L.n == 0 || n_units == 0) return 0;
+    int k = 0;
+    size_t bytes = W.cub_tmp_bytes;
+    if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.lcount, W.lstart, (int)(L.n + 1), st) != cudaSuccess)
+        return -1;
+    ++k;
+    k_fused_fill<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes);
     FFM_LAUNCH_CHECK();
-    k_prefix_flag<<<blocks_for(L.n), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes);
+    ++k;
+    if (ev_a && cudaEventRecord(ev_a, st) != cudaSuccess) return -1;
+    uint32_t grid = resident_grid((const void*)k_fused, P.num_sms);
+    uint32_t need = blocks_for(n_units * 32);
+    k_fused<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.lstart + L.n, P.chunk_bytes, prefilter ? 1 : 0,
+                                                       res_out);
     FFM_LAUNCH_CHECK();
-    return 2;
-}
-
-int launch_hash_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st, bool prefiltered) {
-    if (L.n == 0) return 0;
-    k_hash_combine<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, P.small_bytes, W.hstart, W.hpart, W.accA,
-                                                                     W.accB, prefiltered ? W.eq : nullptr);
+    ++k;
+    if (ev_b && cudaEventRecord(ev_b, st) != cudaSuccess) return -1;
+    k_hash_combine<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes,
+                                                              prefilter ? 1 : 0);
     FFM_LAUNCH_CHECK();
-    return 1;
+    return k + 1;
 }
 
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list, uint64_t cap,
@@ -743,9 +942,13 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
     if (cudaMemsetAsync(W.tval, 0xFF, cap * sizeof(uint32_t), st) != cudaSuccess) return -1;
     if (cudaMemsetAsync(W.lcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
     if (cudaMemsetAsync(W.gcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
-    k_group_insert<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, cap - 1, P.digest_mask, round);
+    k_group_insert<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, cap - 1, P.digest_mask, round,
+                                                        P.small_bytes);
     FFM_LAUNCH_CHECK();
-    k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes, res_out);
+    if (round == 0)
+        k_leader0<<<blocks_for(n_list), 256, 0, st>>>(L, W, n_list, P.small_bytes, P.chunk_bytes, res_out);
+    else
+        k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes, res_out);
     FFM_LAUNCH_CHECK();
     return k + 2;
 }
