@@ -131,10 +131,14 @@ def make_log(workload, n_scale, size_scale, shard=(0, 1)):
     return lg
 
 
-def alg_bytes(lg, idx, dup, small_bytes):
-    """Algorithmic bytes per kernel for this rank's records idx.
-    dup: this rank's duplicate_of (global gids).  Leaders with >= 1 member are counted
-    once (the other members re-read them from L2); remote leaders are NVLink bytes."""
+def alg_bytes(lg, idx, dup, small_bytes, chunk=32768):
+    """Algorithmic bytes per kernel for this rank's records idx: every
+    payload byte is hashed once; a member payload's bytes are compared once against its
+    leader, whose chunks (after the first) are shared through L2 by the group.
+      prefix (k_hash_large, first chunks):  sum over large payloads of c0 = min(size, chunk)
+      fused  (k_fused):  sum over large (size - c0) + members' c0 + their leaders' c0
+      small  (k_hash_small / k_verify_small): sizes / members + leaders
+    dup: this rank's duplicate_of (global gids)."""
     size = lg.size[idx].astype(np.int64)
     n = len(size)
     small = size <= small_bytes
@@ -145,11 +149,15 @@ def alg_bytes(lg, idx, dup, small_bytes):
         pos[idx] = np.arange(n)
         lp = pos[dup[member]]
         leaders[lp[lp >= 0]] = True
+    big = ~small
+    c0 = np.minimum(size, chunk)
+    units = int(((size[big] + chunk - 1) // chunk).sum())
     out = {
         "hash_small": int(size[small].sum()) + 8 * n + 24 * int(small.sum()),
-        "hash_large": int(size[~small].sum()) + 40 * int(((size[~small] + 32767) // 32768).sum()),
+        "prefix": int(c0[big].sum()) + 40 * int(big.sum()),
+        "fused": int((size[big] - c0[big]).sum()) + int(c0[big & member].sum()) + int(c0[big & leaders].sum())
+        + 40 * units,
         "verify_small": int(size[small & member].sum()) + int(size[small & leaders].sum()) + 4 * n,
-        "verify_large": int(size[~small & member].sum()) + int(size[~small & leaders].sum()),
     }
     out["path"] = sum(out.values()) + 64 * n    # + group-by / label metadata
     return out
@@ -195,7 +203,8 @@ def run_ours(args):
     ptrs = (lg.c_off[lg.content] + np.uint64(content.data_ptr())).astype(np.uint64)
     log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * len(idx) + (1 << 20),
                      max_records=len(idx), timing=True, rank=rank, world=world,
-                     prefilter=args.prefilter and world == 1, digest_bits=args.digest_bits)
+                     prefilter=args.prefilter and world == 1, digest_bits=args.digest_bits,
+                     two_pass=args.two_pass)
     log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE,
                    gids=idx if world > 1 else None, idx=idx if world > 1 else None)
     del content
@@ -252,24 +261,35 @@ def run_ours(args):
     dup_h = dup[:len(idx)].cpu().numpy()
     ab = alg_bytes(lg, idx, dup_h, 4096)
     if args.prefilter and world == 1:
-        # only the bytes the pre-filtered path must read: first chunks + the rest of
-        # payloads whose prefix is not unique (reported by the library)
+        # only the bytes the pre-filtered path must read: the library reports the bytes it
+        # hashed beyond first chunks (prefix-unique payloads skip theirs)
         sz = lg.size[idx].astype(np.int64)
-        lg_ = sz > 4096
-        first = int(np.minimum(sz[lg_], 32768).sum())
-        ab["hash_large"] = first + int(st["prefilter_rest_bytes"]) + 40 * int(((sz[lg_] + 32767) // 32768).sum())
+        big = sz > 4096
+        mem = dup_h >= 0
+        c0 = np.minimum(sz, 32768)
+        ab["fused"] = int(st["prefilter_rest_bytes"]) + int(c0[big & mem].sum()) + 40 * int(((sz[big] + 32767) // 32768).sum())
         ab["path"] = sum(v for k, v in ab.items() if k != "path") + 64 * len(idx)
     peak, peak_src = load_peak()
-    kern_ms = {"hash_small": st["ms_hash_small"], "hash_large": st["ms_hash_large"]}
+    if args.two_pass:
+        # two-pass round 0: k_hash_large hashes every large byte, then verify (members +
+        # each class leader once) -- the "fused" slot times the verify stage
+        sz = lg.size[idx].astype(np.int64)
+        big = sz > 4096
+        mem = dup_h >= 0
+        ab["prefix"] = int(sz[big].sum()) + 40 * int(((sz[big] + 32767) // 32768).sum())
+        ab["fused"] = int(sz[big & mem].sum()) + int(ab["fused"] - (sz[big] - np.minimum(sz[big], 32768)).sum()
+                                                      - np.minimum(sz[big & mem], 32768).sum())
+    kern_ms = {"hash_small": st["ms_hash_small"], "prefix": st["ms_hash_large"], "fused": st["ms_fused"]}
     dom = max(kern_ms, key=lambda k: kern_ms[k])
     dom_ms = kern_ms[dom]
     achieved = ab[dom] / (dom_ms * 1e-3) / 1e9 if dom_ms > 0 else 0.0
-    kname = {"hash_large": "k_hash_large", "hash_small": "k_hash_small"}[dom]
+    kname = {"hash_small": "k_hash_small", "prefix": "k_hash_large", "fused": "k_fused"}[dom]
     traffic = None if args.prefilter else ncu_traffic(kname)   # committed ncu summary is of the default path
     roofline = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic, "alg_bytes": ab[dom],
                 "ms": round(dom_ms, 4), "peak_source": peak_src,
-                "read_stream_ceiling_gbs": read_ceiling()}
+                "read_stream_ceiling_gbs": read_ceiling(),
+                "note": "traffic = ncu dram__bytes_read+write of this kernel on config 5 (profiles/ncu_summary.json)"}
     path_gbs = ab["path"] / (ms * 1e-3) / 1e9
     launches = int(round(st["kernel_launches"])) * args.steps
 
@@ -297,11 +317,11 @@ def run_ours(args):
                    f"{world} shards (site-affinity LPT); NCCL all-gather of class representatives, "
                    "in-kernel peer byte verify over NVLink, NCCL all-reduce of benefit",
                    "chunk_bytes": 32768, "small_bytes": 4096, "prefilter": bool(args.prefilter and world == 1),
-                   "digest_bits": args.digest_bits},
+                   "digest_bits": args.digest_bits, "round0": "two-pass" if args.two_pass else "fused"},
         "pct_hbm_roofline_path": round(path_gbs / peak, 4),
         "path_alg_gbs": round(path_gbs, 1),
         "stage_ms": {k: round(st[k], 4) for k in ("ms_hash_small", "ms_hash_large", "ms_group", "ms_verify",
-                                                  "ms_resolve", "ms_label", "ms_output", "ms_total")},
+                                                  "ms_fused", "ms_resolve", "ms_label", "ms_output", "ms_total")},
         "clocks": clk, "gpu_launches": launches, "roofline": roofline, "e2e": e2e, "cpu_baseline": cpu,
         "duplicates_rank0": int((dup_h >= 0).sum()),
         "collisions": {"residual_members": int(round(st["n_residual"])), "resolve_rounds": int(round(st["resolve_rounds"]))},
@@ -467,6 +487,8 @@ def main():
     ap.add_argument("--ref-step-seconds", type=float, default=6.0)
     ap.add_argument("--digest-bits", type=int, default=64,
                     help="< 64 truncates the group-by digest (forced collisions, verify stress; config 3)")
+    ap.add_argument("--two-pass", action="store_true",
+                    help="round 0 as hash-all then verify (better for near-duplicate-heavy logs, config 3)")
     ap.add_argument("--prefilter", action="store_true",
                     help="S8(f) #4 size/prefix pre-filter (opt-in; single GPU); roofline counts bytes required")
     args = ap.parse_args()

@@ -52,11 +52,17 @@ enum { FFM_PAYLOAD_AUTO = 0,        /* detected per pointer (cudaPointerGetAttri
 
 /* ffm_config.flags */
 enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_stats) */
-       FFM_FLAG_PREFILTER = 2u   /* S8(f) #4: ffm_dedup_run hashes only the first chunk of a large
+       FFM_FLAG_PREFILTER = 2u,  /* S8(f) #4: ffm_dedup_run hashes only the first chunk of a large
                                     payload whose (size, first-chunk digest, channel) is unique in the
                                     log -- it cannot equal any other payload.  Same results, fewer bytes.
                                     Ignored by ffm_shard_* and ffm_online_step (uniqueness within one
-                                    shard / window says nothing about the others). */ };
+                                    shard / window says nothing about the others). */
+       FFM_FLAG_TWO_PASS = 4u    /* round 0 of H1-H3 as two passes: hash every payload fully, group by
+                                    the full digest, then byte-verify members (chunk-major per class).
+                                    Default is fused: group large payloads by their first chunk and hash
+                                    + compare in one pass -- fewer bytes when duplicates are exact, more
+                                    when most candidates are near-duplicates (BASELINE config 3).  Same
+                                    results either way. */ };
 
 typedef struct ffm_config {
     uint32_t n_sites;      /* call_site must be < n_sites.  Sites are caller-interned stack

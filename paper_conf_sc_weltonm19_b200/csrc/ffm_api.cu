@@ -396,29 +396,39 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     LCHK(launch_hash_small(D, W, L->params, side));
     if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
     ck(cudaEventRecord(L->fork_ev[1], side), "event");
+    const bool two_pass = (L->cfg.flags & FFM_FLAG_TWO_PASS) != 0;
     if (n_large) {
-        // prefix pass: the first chunk of every large payload
         LCHK(launch_hash_plan(D, W, L->params, s));
         if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
-        LCHK(launch_hash_large(D, W, L->params, n_large, s, 1));
+        // fused: the prefix pass (first chunks); two-pass: every chunk, then the combine
+        LCHK(launch_hash_large(D, W, L->params, n_large, s, two_pass ? 0 : 1));
         if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
+        if (two_pass) LCHK(launch_combine(D, W, L->params, s));
     }
     ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
     if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
     // H2 group-by (round 0): small payloads by full digest, large ones by first-chunk digest
     uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
-    LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, 0, W.res[0], s));
+    LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, two_pass ? -1 : 0, W.res[0], s));
     if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
-    // H3: small members verified on the side stream while the fused pass hashes the rest
-    // of every large payload and byte-compares each large member with its group leader
-    ck(cudaEventRecord(L->fork_ev[2], s), "event");
-    ck(cudaStreamWaitEvent(side, L->fork_ev[2], 0), "fork");
-    LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], 0, side, nullptr, nullptr, nullptr));
-    ck(cudaEventRecord(L->fork_ev[3], side), "event");
-    if (n_large)
-        LCHK(launch_fused(D, W, L->params, n_large, prefilter, W.res[0], s, timing ? L->ev[16] : nullptr,
-                          timing ? L->ev[17] : nullptr));
-    ck(cudaStreamWaitEvent(s, L->fork_ev[3], 0), "join");
+    if (two_pass) {
+        // H3 (two-pass): every member byte-verified against its full-digest candidate
+        if (timing) ck(cudaEventRecord(L->ev[16], s), "event");
+        LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], n_large ? W.vitem_cap : 0, s, side,
+                           L->fork_ev[2], L->fork_ev[3]));
+        if (timing) ck(cudaEventRecord(L->ev[17], s), "event");
+    } else {
+        // H3: small members verified on the side stream while the fused pass hashes the rest
+        // of every large payload and byte-compares each large member with its group leader
+        ck(cudaEventRecord(L->fork_ev[2], s), "event");
+        ck(cudaStreamWaitEvent(side, L->fork_ev[2], 0), "fork");
+        LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], 0, side, nullptr, nullptr, nullptr));
+        ck(cudaEventRecord(L->fork_ev[3], side), "event");
+        if (n_large)
+            LCHK(launch_fused(D, W, L->params, n_large, prefilter, W.res[0], s, timing ? L->ev[16] : nullptr,
+                              timing ? L->ev[17] : nullptr));
+        ck(cudaStreamWaitEvent(s, L->fork_ev[3], 0), "join");
+    }
     if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
     // H5 + H6 (speculative: valid unless H3 found residuals)
     if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, s));

@@ -113,6 +113,7 @@ struct Params {
 int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st, int phase = 0);
+int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
                  cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b);
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,

@@ -19,7 +19,11 @@
 #include "ffm_internal.h"
 #include "digest.cuh"
 
-// tuning knobs of the fused pass (defaults = the measured best)
+// Tuning knobs of the fused pass; defaults are the measured best on B200 (config 5 / 4,
+// profiles/r01_fused_variants.md): leader-first layout, members' compare loads
+// L2::evict_last, everyone's own loads L2::evict_first (evict_last or normal priority on
+// the leaders' own loads measured 12-13% slower), 2 loads in flight per lane when
+// comparing, 3 CTAs/SM.
 #ifndef FFM_FUSED_CMP_U
 #define FFM_FUSED_CMP_U 2
 #endif
@@ -28,9 +32,6 @@
 #endif
 #ifndef FFM_FUSED_KEEP_OWN
 #define FFM_FUSED_KEEP_OWN 0
-#endif
-#ifndef FFM_FUSED_DEMOTE
-#define FFM_FUSED_DEMOTE 0
 #endif
 #ifndef FFM_FUSED_SKEW
 #define FFM_FUSED_SKEW 0x7FFFFFFF   /* measured: leader-first (no skew) is best */
@@ -275,9 +276,9 @@ __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ li
     if (i >= n_list) return;
     uint32_t r = list ? list[i] : i;
     uint64_t key;
-    if (round == 0) {
+    if (round <= 0) {                 // 0: fused round 0 (prefix keys); -1: two-pass round 0
         uint64_t n = L.size[r];
-        if (n <= small_bytes) {
+        if (n <= small_bytes || round < 0) {
             // small payload: its full digest
             uint64_t d = finalize_digest(W.accA[r], W.accB[r], n);
             W.digest[r] = d;
@@ -492,14 +493,6 @@ __global__ void __launch_bounds__(256, FFM_FUSED_MINB) k_fused(DevLog L, Work W,
             fused_chunk<FFM_FUSED_CMP_U, true>(pr, ph, n, bb, be, lane, hashc, keep_own, K, A, B, found);
         else
             fused_chunk<4, false>(pr, ph, n, bb, be, lane, hashc, keep_own, K, A, B, found);
-#if FFM_FUSED_DEMOTE
-        // the group's last member hands the leader's chunk back to normal L2 priority
-        // (it was loaded evict_last so that every member hits it)
-        if (h != r && W.pos[r] == W.gcount[h]) {
-            for (uint32_t b = bb + 4 * lane; b < be; b += 128)
-                asm volatile("applypriority.global.L2::evict_normal [%0], 128;" ::"l"(ph + 32ull * b));
-        }
-#endif
         if (hashc) {
 #pragma unroll
             for (int o = 16; o; o >>= 1) {
@@ -904,6 +897,13 @@ int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_item
 
 // Round 0, large payloads: fused groups (scan of lcount), work units, the fused
 // hash + compare pass, then the per-record combine of chunk partial sums.
+int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
+    if (L.n == 0) return 0;
+    k_hash_combine<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 0);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
 int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
                  cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b) {
     if (L.n == 0 || n_units == 0) return 0;
@@ -947,6 +947,8 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
     FFM_LAUNCH_CHECK();
     if (round == 0)
         k_leader0<<<blocks_for(n_list), 256, 0, st>>>(L, W, n_list, P.small_bytes, P.chunk_bytes, res_out);
+    else if (round < 0)
+        k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, nullptr, n_list, P.small_bytes, P.chunk_bytes, res_out);
     else
         k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes, res_out);
     FFM_LAUNCH_CHECK();

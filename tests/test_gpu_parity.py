@@ -361,3 +361,12 @@ def test_reset_reuses_the_log(ffm):
     assert_same(a, d1, b1)
     assert_same(b, d2, b2)
     np.testing.assert_array_equal(d3, d1)
+
+
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_two_pass_round0(ffm, digest_bits):
+    """FFM_FLAG_TWO_PASS (hash all, group by full digest, verify) gives the same results."""
+    for k, ns, ss in [(3, 0.03, 1 / 16), (4, 0.1, 1 / 64), (5, 0.003, 1 / 32)]:
+        lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
+        dup, ben, st = gpu_dedup(ffm, lg, two_pass=True, digest_bits=digest_bits, chunk_bytes=4096)
+        assert_same(lg, dup, ben)
