@@ -131,7 +131,7 @@ def make_log(workload, n_scale, size_scale, shard=(0, 1)):
     return lg
 
 
-def alg_bytes(lg, idx, dup, small_bytes, chunk=32768):
+def alg_bytes(lg, idx, dup, small_bytes, chunk=32768, two_pass=False):
     """Algorithmic bytes per kernel for this rank's records idx: every
     payload byte is hashed once; a member payload's bytes are compared once against its
     leader, whose chunks (after the first) are shared through L2 by the group.
@@ -159,6 +159,11 @@ def alg_bytes(lg, idx, dup, small_bytes, chunk=32768):
         + 40 * units,
         "verify_small": int(size[small & member].sum()) + int(size[small & leaders].sum()) + 4 * n,
     }
+    if two_pass:
+        # hash every large byte (k_hash_large), then verify members against their class
+        # leader, each leader read once per class (the "fused" slot times the verify stage)
+        out["prefix"] = int(size[big].sum()) + 40 * units
+        out["fused"] = int(size[big & member].sum()) + int(size[big & leaders].sum())
     out["path"] = sum(out.values()) + 64 * n    # + group-by / label metadata
     return out
 
@@ -259,7 +264,7 @@ def run_ours(args):
 
     # algorithmic bytes and the dominant kernel on this rank (rank 0 reports)
     dup_h = dup[:len(idx)].cpu().numpy()
-    ab = alg_bytes(lg, idx, dup_h, 4096)
+    ab = alg_bytes(lg, idx, dup_h, 4096, two_pass=args.two_pass)
     if args.prefilter and world == 1:
         # only the bytes the pre-filtered path must read: the library reports the bytes it
         # hashed beyond first chunks (prefix-unique payloads skip theirs)
@@ -270,15 +275,6 @@ def run_ours(args):
         ab["fused"] = int(st["prefilter_rest_bytes"]) + int(c0[big & mem].sum()) + 40 * int(((sz[big] + 32767) // 32768).sum())
         ab["path"] = sum(v for k, v in ab.items() if k != "path") + 64 * len(idx)
     peak, peak_src = load_peak()
-    if args.two_pass:
-        # two-pass round 0: k_hash_large hashes every large byte, then verify (members +
-        # each class leader once) -- the "fused" slot times the verify stage
-        sz = lg.size[idx].astype(np.int64)
-        big = sz > 4096
-        mem = dup_h >= 0
-        ab["prefix"] = int(sz[big].sum()) + 40 * int(((sz[big] + 32767) // 32768).sum())
-        ab["fused"] = int(sz[big & mem].sum()) + int(ab["fused"] - (sz[big] - np.minimum(sz[big], 32768)).sum()
-                                                      - np.minimum(sz[big & mem], 32768).sum())
     kern_ms = {"hash_small": st["ms_hash_small"], "prefix": st["ms_hash_large"], "fused": st["ms_fused"]}
     dom = max(kern_ms, key=lambda k: kern_ms[k])
     dom_ms = kern_ms[dom]
