@@ -264,7 +264,7 @@ def run_ours(args):
 
     # algorithmic bytes and the dominant kernel on this rank (rank 0 reports)
     dup_h = dup[:len(idx)].cpu().numpy()
-    ab = alg_bytes(lg, idx, dup_h, 4096, two_pass=args.two_pass)
+    ab = alg_bytes(lg, idx, dup_h, 4096, two_pass=args.two_pass or st.get("two_pass", 0) >= 0.5)
     if args.prefilter and world == 1:
         # only the bytes the pre-filtered path must read: the library reports the bytes it
         # hashed beyond first chunks (prefix-unique payloads skip theirs)
@@ -313,7 +313,9 @@ def run_ours(args):
                    f"{world} shards (site-affinity LPT); NCCL all-gather of class representatives, "
                    "in-kernel peer byte verify over NVLink, NCCL all-reduce of benefit",
                    "chunk_bytes": 32768, "small_bytes": 4096, "prefilter": bool(args.prefilter and world == 1),
-                   "digest_bits": args.digest_bits, "round0": "two-pass" if args.two_pass else "fused"},
+                   "digest_bits": args.digest_bits,
+                   "round0": "two-pass (forced)" if args.two_pass else
+                   ("two-pass (adaptive)" if st.get("two_pass", 0) >= 0.5 else "fused")},
         "pct_hbm_roofline_path": round(path_gbs / peak, 4),
         "path_alg_gbs": round(path_gbs, 1),
         "stage_ms": {k: round(st[k], 4) for k in ("ms_hash_small", "ms_hash_large", "ms_group", "ms_verify",

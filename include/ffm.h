@@ -57,12 +57,15 @@ enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_s
                                     log -- it cannot equal any other payload.  Same results, fewer bytes.
                                     Ignored by ffm_shard_* and ffm_online_step (uniqueness within one
                                     shard / window says nothing about the others). */
-       FFM_FLAG_TWO_PASS = 4u    /* round 0 of H1-H3 as two passes: hash every payload fully, group by
+       FFM_FLAG_TWO_PASS = 4u,   /* round 0 of H1-H3 as two passes: hash every payload fully, group by
                                     the full digest, then byte-verify members (chunk-major per class).
                                     Default is fused: group large payloads by their first chunk and hash
                                     + compare in one pass -- fewer bytes when duplicates are exact, more
                                     when most candidates are near-duplicates (BASELINE config 3).  Same
-                                    results either way. */ };
+                                    results either way.  With neither flag the mode is adaptive: a log
+                                    whose fused run found more than half of its candidates to mismatch
+                                    uses two-pass on later runs. */
+       FFM_FLAG_FUSED = 8u       /* force the fused round 0 (no adaptation) */ };
 
 typedef struct ffm_config {
     uint32_t n_sites;      /* call_site must be < n_sites.  Sites are caller-interned stack
@@ -165,6 +168,7 @@ typedef struct ffm_run_stats {
     uint64_t verify_items;      /* large-payload verify work units */
     uint64_t prefilter_rest_bytes; /* bytes hashed beyond first chunks by the fused pass */
     double   ms_fused;          /* the fused hash + compare kernel alone (large payloads) */
+    uint64_t two_pass;          /* 1 if the last run used the two-pass round 0 */
 } ffm_run_stats;
 
 /* Statistics of the last ffm_dedup_run. */

@@ -24,6 +24,7 @@ FFM_PAYLOAD_AUTO, FFM_PAYLOAD_HOST, FFM_PAYLOAD_DEVICE, FFM_PAYLOAD_HOST_PINNED 
 FFM_FLAG_TIMING = 1
 FFM_FLAG_PREFILTER = 2
 FFM_FLAG_TWO_PASS = 4
+FFM_FLAG_FUSED = 8
 
 # every symbol include/ffm.h declares (checked by tests/test_abi.py)
 EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_append_batch", "ffm_log_append_batch_ex",
@@ -51,7 +52,7 @@ class FfmRunStats(ctypes.Structure):
                [(k, ctypes.c_uint64) for k in ("n_records", "payload_bytes", "n_members", "n_residual",
                                                 "resolve_rounds", "kernel_launches", "hash_items",
                                                 "verify_items", "prefilter_rest_bytes")] + \
-               [("ms_fused", ctypes.c_double)]
+               [("ms_fused", ctypes.c_double), ("two_pass", ctypes.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -303,14 +304,14 @@ class FfmLog:
     def __init__(self, n_sites: int, device: int = 0, *, arena_bytes: int = 0, max_records: int = 0,
                  digest_bits: int = 64, refine_bits: int = 64, chunk_bytes: int = 0, small_bytes: int = 0,
                  timing: bool = False, stream: int = 0, rank: int = 0, world: int = 1,
-                 prefilter: bool = False, two_pass: bool = False):
+                 prefilter: bool = False, two_pass: bool = False, fused: bool = False):
         cfg = ffm_config_init()
         cfg.n_sites, cfg.device, cfg.rank, cfg.world = n_sites, device, rank, world
         cfg.arena_bytes, cfg.max_records = arena_bytes, max_records
         cfg.digest_bits, cfg.refine_bits = digest_bits, refine_bits
         cfg.chunk_bytes, cfg.small_bytes = chunk_bytes, small_bytes
         cfg.flags = (FFM_FLAG_TIMING if timing else 0) | (FFM_FLAG_PREFILTER if prefilter else 0) | \
-            (FFM_FLAG_TWO_PASS if two_pass else 0)
+            (FFM_FLAG_TWO_PASS if two_pass else 0) | (FFM_FLAG_FUSED if fused else 0)
         cfg.stream = stream or None
         self.n_sites = n_sites
         self.h = ffm_log_create(cfg)

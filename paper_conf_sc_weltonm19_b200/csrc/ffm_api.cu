@@ -23,6 +23,7 @@ constexpr uint64_t kGatherMaxDefault = 1ull << 20;   // payloads up to this use 
 
 struct LocalRun {
     uint64_t n_members, n_res_total, rounds, prefilter_rest;
+    bool two_pass;
 };
 
 struct CudaFail {
@@ -396,7 +397,10 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     LCHK(launch_hash_small(D, W, L->params, side));
     if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
     ck(cudaEventRecord(L->fork_ev[1], side), "event");
-    const bool two_pass = (L->cfg.flags & FFM_FLAG_TWO_PASS) != 0;
+    // round-0 mode: forced by a flag, else adaptive -- a log whose fused run found most
+    // large candidates to be near-duplicate mismatches uses the two-pass round 0 next time
+    const bool two_pass = (L->cfg.flags & FFM_FLAG_TWO_PASS) != 0 ||
+                          (!(L->cfg.flags & FFM_FLAG_FUSED) && L->prefer_two_pass);
     if (n_large) {
         LCHK(launch_hash_plan(D, W, L->params, s));
         if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
@@ -436,6 +440,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
     ck(cudaStreamSynchronize(s), "run sync");
     R.n_members = L->h_counters[1];
+    R.two_pass = two_pass;
     R.prefilter_rest = (uint64_t)L->h_counters[4] | ((uint64_t)L->h_counters[5] << 32);
     uint64_t nres = L->h_counters[0];
     R.n_res_total = nres;
@@ -475,6 +480,7 @@ void fill_stats(ffm_log* L, const LocalRun& R, uint64_t launches, bool single) {
     S.kernel_launches = launches;
     S.hash_items = L->n_large_chunks;
     S.prefilter_rest_bytes = R.prefilter_rest;
+    S.two_pass = R.two_pass ? 1 : 0;
     if (timing) {
         S.ms_hash_small = ev_ms(L->ev[12], L->ev[8]);
         S.ms_hash_large = L->n_large_chunks ? ev_ms(L->ev[10], L->ev[11]) : 0.0;
@@ -793,6 +799,9 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         ck(cudaStreamSynchronize(s), "output sync");
         ck(cudaGetLastError(), "run");
         fill_stats(L, R, launches, true);
+        // adaptive round 0: more than half of the candidates failed the fused compare
+        // (near-duplicates sharing first chunks) -> hash-all-then-verify is cheaper
+        if (!R.two_pass && R.n_members >= 64 && 2 * R.n_res_total > R.n_members) L->prefer_two_pass = true;
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
     } catch (const std::bad_alloc&) {
@@ -1166,6 +1175,7 @@ int ffm_log_reset(ffm_log* L) {
         cudaMemset(L->online_cnt, 0, L->cfg.n_sites * sizeof(uint64_t));
     }
     L->digests_valid = false;
+    L->prefer_two_pass = false;
     memset(&L->stats, 0, sizeof(L->stats));
     return FFM_OK;
 }

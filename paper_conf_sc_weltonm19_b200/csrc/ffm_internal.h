@@ -159,6 +159,7 @@ struct ffm_log {
     bool own_stream = false;
     bool poisoned = false;
     bool host_ptr_ok = false;      // kernels may dereference registered host pointers
+    bool prefer_two_pass = false;  // adaptive round 0 (see run_local)
     uint64_t gather_max = 0;       // payloads up to this are gathered by k_gather, above: DMA
     std::string last_error;
 

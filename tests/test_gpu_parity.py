@@ -370,3 +370,25 @@ def test_two_pass_round0(ffm, digest_bits):
         lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
         dup, ben, st = gpu_dedup(ffm, lg, two_pass=True, digest_bits=digest_bits, chunk_bytes=4096)
         assert_same(lg, dup, ben)
+
+
+def test_adaptive_round0(ffm):
+    """Near-duplicates sharing first chunks make the fused round 0 mismatch: the log
+    switches itself to two-pass after one run; outputs never change."""
+    lg = loggen.gen_config(3, n_scale=0.05, size_scale=1 / 8)
+    want = oracle.dedup(lg)
+    with ffm.FfmLog(lg.n_sites, timing=True) as log:
+        log.append_log(lg)
+        d1, b1 = [x.copy() for x in log.run()]
+        s1 = log.stats()
+        d2, b2 = [x.copy() for x in log.run()]
+        s2 = log.stats()
+    assert s1["two_pass"] == 0 and s2["two_pass"] == 1
+    for d, b in ((d1, b1), (d2, b2)):
+        np.testing.assert_array_equal(d, want[0])
+        np.testing.assert_array_equal(b, want[1])
+    with ffm.FfmLog(lg.n_sites, fused=True) as log:       # forced: no adaptation
+        log.append_log(lg)
+        log.run()
+        log.run()
+        assert log.stats()["two_pass"] == 0
