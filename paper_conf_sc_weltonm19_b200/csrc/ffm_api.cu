@@ -89,6 +89,9 @@ void ring_flush(ffm_log* L) {
 }
 
 void ensure_arena(ffm_log* L, uint64_t need) {
+    // slack: kernels load a record's last, partial 32-byte block whole (and mask it in
+    // registers), so the allocation must extend to the 32-byte boundary past the end
+    need = align_up(need, kArenaAlign) + 64;
     if (need <= L->arena_cap) return;
     ring_flush(L);
     ck(cudaStreamSynchronize(L->stage_stream), "arena sync");

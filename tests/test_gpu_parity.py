@@ -392,3 +392,12 @@ def test_adaptive_round0(ffm):
         log.run()
         log.run()
         assert log.stats()["two_pass"] == 0
+
+
+def test_benefit_linear_in_durations(ffm):
+    """Scaling every duration by k scales every per-site benefit by k (mod 2^64)."""
+    lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 32)
+    _, b1, _ = gpu_dedup(ffm, lg)
+    lg.dur = lg.dur * np.uint64(7)
+    _, b7, _ = gpu_dedup(ffm, lg)
+    np.testing.assert_array_equal(b7, b1 * np.uint64(7))

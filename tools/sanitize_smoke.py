@@ -1,5 +1,6 @@
-"""Small logs through every kernel (incl. collision resolve and the gather path), for
-compute-sanitizer memcheck / racecheck / synccheck."""
+"""Small logs through every kernel (fused and two-pass round 0, pre-filter, collision
+resolve, online windows, device-payload gather), for compute-sanitizer memcheck /
+racecheck / synccheck."""
 import os
 import sys
 
@@ -11,11 +12,14 @@ import loggen  # noqa: E402
 import oracle  # noqa: E402
 import paper_conf_sc_weltonm19_b200 as ffm  # noqa: E402
 
-for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (2, 0.001, 1.0)]:
+for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (4, 0.04, 1 / 512), (2, 0.001, 1.0)]:
     lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
     want = oracle.dedup(lg)
-    for db, rb, dev in [(64, 64, False), (0, 64, True), (0, 0, False)]:
-        with ffm.FfmLog(lg.n_sites, digest_bits=db, refine_bits=rb, chunk_bytes=4096, small_bytes=1024) as log:
+    for db, rb, dev, extra in [(64, 64, False, {}), (0, 64, True, {}), (0, 0, False, {}),
+                               (64, 64, False, {"two_pass": True}), (64, 64, False, {"prefilter": True}),
+                               (8, 64, True, {"fused": True})]:
+        with ffm.FfmLog(lg.n_sites, digest_bits=db, refine_bits=rb, chunk_bytes=4096, small_bytes=1024,
+                        **extra) as log:
             if dev:
                 buf = torch.from_numpy(lg.materialize()).cuda()
                 ptrs = (lg.c_off[lg.content] + np.uint64(buf.data_ptr())).astype(np.uint64)
@@ -23,5 +27,13 @@ for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (2, 0.001, 1.0)]:
             else:
                 log.append_log(lg)
             d, b = log.run()
-            assert np.array_equal(d, want[0]) and np.array_equal(b, want[1]), (k, db, rb)
+            assert np.array_equal(d, want[0]) and np.array_equal(b, want[1]), (k, db, rb, extra)
+    # online windows
+    with ffm.FfmLog(lg.n_sites, digest_bits=8, chunk_bytes=4096) as log:
+        ptrs = lg.payload_ptrs()
+        got = []
+        for a, e in ((0, lg.n // 3), (lg.n // 3, lg.n)):
+            log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e])
+            got.append(log.online_step()[0].copy())
+        assert np.array_equal(np.concatenate(got), want[0]), ("online", k)
 print("sanitize smoke ok")
