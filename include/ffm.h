@@ -51,7 +51,8 @@ enum { FFM_PAYLOAD_AUTO = 0,        /* detected per pointer (cudaPointerGetAttri
                                        read over PCIe by the gather kernel or the copy engines */ };
 
 /* ffm_config.flags */
-enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_stats) */
+enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_stats); such runs
+                                    launch their kernels directly (no graph replay) */
        FFM_FLAG_PREFILTER = 2u,  /* S8(f) #4: ffm_dedup_run hashes only the first chunk of a large
                                     payload whose (size, first-chunk digest, channel) is unique in the
                                     log -- it cannot equal any other payload.  Same results, fewer bytes.
@@ -65,7 +66,9 @@ enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_s
                                     results either way.  With neither flag the mode is adaptive: a log
                                     whose fused run found more than half of its candidates to mismatch
                                     uses two-pass on later runs. */
-       FFM_FLAG_FUSED = 8u       /* force the fused round 0 (no adaptation) */ };
+       FFM_FLAG_FUSED = 8u,      /* force the fused round 0 (no adaptation) */
+       FFM_FLAG_NO_GRAPH = 16u   /* launch every kernel directly instead of replaying the captured
+                                    CUDA graph of a run (default: graph while the log is unchanged) */ };
 
 typedef struct ffm_config {
     uint32_t n_sites;      /* call_site must be < n_sites.  Sites are caller-interned stack
@@ -263,6 +266,10 @@ int ffm_shard_local(ffm_log* log, ffm_rep* reps_out, uint64_t cap, uint64_t* n_r
    [n_sites] receives this rank's partial sums (all-reduce them). */
 int ffm_shard_merge(ffm_log* log, const ffm_rep* all_reps, const uint64_t* counts, int64_t* duplicate_of,
                     uint64_t* benefit_partial);
+
+/* Replace cfg.flags of a live log (e.g. toggle FFM_FLAG_TIMING between measured and
+   instrumented runs).  Takes effect at the next run. */
+int ffm_log_set_flags(ffm_log* log, uint32_t flags);
 
 /* Empty the log (records, online state) but keep every allocation (HBM arena, work
    buffers, staging ring): the next batch of transfers reuses them.  Peer mappings of

@@ -25,6 +25,7 @@ FFM_FLAG_TIMING = 1
 FFM_FLAG_PREFILTER = 2
 FFM_FLAG_TWO_PASS = 4
 FFM_FLAG_FUSED = 8
+FFM_FLAG_NO_GRAPH = 16
 
 # every symbol include/ffm.h declares (checked by tests/test_abi.py)
 EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_append_batch", "ffm_log_append_batch_ex",
@@ -32,7 +33,7 @@ EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_appen
            "ffm_last_run_stats", "ffm_debug_digests", "ffm_log_destroy", "ffm_strerror",
            "ffm_last_error", "ffm_version", "ffm_shard_plan", "ffm_shard_ipc_handle", "ffm_shard_open_peer",
            "ffm_shard_local", "ffm_shard_merge", "ffm_site_duplicate_counts", "ffm_fold_sites",
-           "ffm_online_step", "ffm_online_done", "ffm_log_reset"]
+           "ffm_online_step", "ffm_online_done", "ffm_log_reset", "ffm_log_set_flags"]
 FFM_SHARD_SITE_LPT, FFM_SHARD_CONTIGUOUS = 0, 1
 REP_WORDS = 5        # ffm_rep = {key, size, gid, off, chan}, 5 x u64
 
@@ -98,6 +99,8 @@ def lib() -> ctypes.CDLL:
         L.ffm_last_run_stats.restype = i32
         L.ffm_debug_digests.argtypes = [vp, vp]
         L.ffm_debug_digests.restype = i32
+        L.ffm_log_set_flags.argtypes = [vp, u32]
+        L.ffm_log_set_flags.restype = i32
         L.ffm_log_reset.argtypes = [vp]
         L.ffm_log_reset.restype = i32
         L.ffm_log_destroy.argtypes = [vp]
@@ -227,6 +230,10 @@ def ffm_debug_digests(h) -> np.ndarray:
     return out[:ffm_log_count(h)]
 
 
+def ffm_log_set_flags(h, flags: int):
+    _check(h, lib().ffm_log_set_flags(h, flags))
+
+
 def ffm_log_reset(h):
     _check(h, lib().ffm_log_reset(h))
 
@@ -304,16 +311,19 @@ class FfmLog:
     def __init__(self, n_sites: int, device: int = 0, *, arena_bytes: int = 0, max_records: int = 0,
                  digest_bits: int = 64, refine_bits: int = 64, chunk_bytes: int = 0, small_bytes: int = 0,
                  timing: bool = False, stream: int = 0, rank: int = 0, world: int = 1,
-                 prefilter: bool = False, two_pass: bool = False, fused: bool = False):
+                 prefilter: bool = False, two_pass: bool = False, fused: bool = False,
+                 graph: bool = True):
         cfg = ffm_config_init()
         cfg.n_sites, cfg.device, cfg.rank, cfg.world = n_sites, device, rank, world
         cfg.arena_bytes, cfg.max_records = arena_bytes, max_records
         cfg.digest_bits, cfg.refine_bits = digest_bits, refine_bits
         cfg.chunk_bytes, cfg.small_bytes = chunk_bytes, small_bytes
         cfg.flags = (FFM_FLAG_TIMING if timing else 0) | (FFM_FLAG_PREFILTER if prefilter else 0) | \
-            (FFM_FLAG_TWO_PASS if two_pass else 0) | (FFM_FLAG_FUSED if fused else 0)
+            (FFM_FLAG_TWO_PASS if two_pass else 0) | (FFM_FLAG_FUSED if fused else 0) | \
+            (0 if graph else FFM_FLAG_NO_GRAPH)
         cfg.stream = stream or None
         self.n_sites = n_sites
+        self.flags = cfg.flags
         self.h = ffm_log_create(cfg)
 
     def append(self, call_site, size, payload_ptr, duration_ns):
@@ -377,6 +387,11 @@ class FfmLog:
 
     def fold(self, site_values, site_to_group, n_groups, out=None):
         return ffm_fold_sites(self.h, site_values, site_to_group, n_groups, out)
+
+    def set_timing(self, on: bool):
+        """Per-stage CUDA events on (direct launches) or off (graph replay)."""
+        self.flags = (self.flags | FFM_FLAG_TIMING) if on else (self.flags & ~FFM_FLAG_TIMING)
+        ffm_log_set_flags(self.h, self.flags)
 
     def reset(self):
         """Empty the log, keep its HBM allocations (ffm_log_reset)."""

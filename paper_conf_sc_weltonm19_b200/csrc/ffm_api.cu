@@ -109,6 +109,7 @@ void ensure_arena(ffm_log* L, uint64_t need) {
     if (L->arena) ck(cudaFree(L->arena), "cudaFree(arena)");
     L->arena = na;
     L->arena_cap = nc;
+    ++L->epoch;
 }
 
 void stage_host(ffm_log* L, const void* src, uint64_t size, uint64_t off) {
@@ -278,6 +279,7 @@ void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* si
         L->n_large_chunks += large_chunks(L, sizes[i]);
     }
     L->arena_used = arena_end;
+    ++L->epoch;
 }
 
 // ---------------------------------------------------------------- work buffers
@@ -285,6 +287,7 @@ void ensure_work(ffm_log* L, uint64_t n) {
     Work& W = L->work;
     uint64_t tcap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
     if (n > W.n_cap || W.accA == nullptr) {
+        ++L->epoch;
         uint64_t c = std::max<uint64_t>(n, 1024);
         dev_alloc(W.accA, c);
         dev_alloc(W.accB, c);
@@ -313,11 +316,13 @@ void ensure_work(ffm_log* L, uint64_t n) {
         W.n_cap = c;
     }
     if (tcap > W.t_cap) {
+        ++L->epoch;
         dev_alloc(W.tkey, tcap);
         dev_alloc(W.tval, tcap);
         W.t_cap = tcap;
     }
     if (L->n_large_chunks > W.hitem_cap) {
+        ++L->epoch;
         uint64_t c = L->n_large_chunks + L->n_large_chunks / 4 + 64;
         dev_alloc(W.hitems, c);
         dev_alloc(W.vitems, c);
@@ -325,6 +330,7 @@ void ensure_work(ffm_log* L, uint64_t n) {
         W.hitem_cap = W.vitem_cap = c;
     }
     if (L->cfg.n_sites > W.site_cap) {
+        ++L->epoch;
         dev_alloc(W.ben, L->cfg.n_sites);
         dev_alloc(W.cnt, L->cfg.n_sites);
         if (label_smem_bytes(L->cfg.n_sites) <= (uint64_t)L->params.max_smem) {
@@ -390,57 +396,95 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     cudaStream_t s = L->stream;
     const uint32_t ns = L->cfg.n_sites;
     LocalRun R{};
-    if (timing) ck(cudaEventRecord(L->ev[0], s), "event");
-    if (launch_zero_counters(W, s) < 0) throw CudaFail{cudaGetLastError(), "zero counters"};
-    // H1 hash: small payloads on the side stream, concurrently with the large path
     cudaStream_t side = L->side_stream;
-    ck(cudaEventRecord(L->fork_ev[0], s), "event");
-    ck(cudaStreamWaitEvent(side, L->fork_ev[0], 0), "fork");
-    if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
-    LCHK(launch_hash_small(D, W, L->params, side));
-    if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
-    ck(cudaEventRecord(L->fork_ev[1], side), "event");
     // round-0 mode: forced by a flag, else adaptive -- a log whose fused run found most
     // large candidates to be near-duplicate mismatches uses the two-pass round 0 next time
     const bool two_pass = (L->cfg.flags & FFM_FLAG_TWO_PASS) != 0 ||
                           (!(L->cfg.flags & FFM_FLAG_FUSED) && L->prefer_two_pass);
-    if (n_large) {
-        LCHK(launch_hash_plan(D, W, L->params, s));
-        if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
-        // fused: the prefix pass (first chunks); two-pass: every chunk, then the combine
-        LCHK(launch_hash_large(D, W, L->params, n_large, s, two_pass ? 0 : 1));
-        if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
-        if (two_pass) LCHK(launch_combine(D, W, L->params, s));
-    }
-    ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
-    if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
-    // H2 group-by (round 0): small payloads by full digest, large ones by first-chunk digest
-    uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
-    LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, two_pass ? -1 : 0, W.res[0], s));
-    if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
-    if (two_pass) {
-        // H3 (two-pass): every member byte-verified against its full-digest candidate
-        if (timing) ck(cudaEventRecord(L->ev[16], s), "event");
-        LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], n_large ? W.vitem_cap : 0, s, side,
-                           L->fork_ev[2], L->fork_ev[3]));
-        if (timing) ck(cudaEventRecord(L->ev[17], s), "event");
+    // segment A: everything up to the first host sync (H1, H2, H3, speculative H5/H6 and
+    // the counters read-back) -- ~30 launches on two streams, no host dependency
+    auto segment_a = [&]() {
+        if (timing) ck(cudaEventRecord(L->ev[0], s), "event");
+        if (launch_zero_counters(W, s) < 0) throw CudaFail{cudaGetLastError(), "zero counters"};
+        // H1 hash: small payloads on the side stream, concurrently with the large path
+        ck(cudaEventRecord(L->fork_ev[0], s), "event");
+        ck(cudaStreamWaitEvent(side, L->fork_ev[0], 0), "fork");
+        if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
+        LCHK(launch_hash_small(D, W, L->params, side));
+        if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
+        ck(cudaEventRecord(L->fork_ev[1], side), "event");
+        if (n_large) {
+            LCHK(launch_hash_plan(D, W, L->params, s));
+            if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
+            // fused: the prefix pass (first chunks); two-pass: every chunk, then the combine
+            LCHK(launch_hash_large(D, W, L->params, n_large, s, two_pass ? 0 : 1));
+            if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
+            if (two_pass) LCHK(launch_combine(D, W, L->params, s));
+        }
+        ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
+        if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
+        // H2 group-by (round 0): small payloads by full digest, large ones by first-chunk digest
+        uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
+        LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, two_pass ? -1 : 0, W.res[0], s));
+        if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
+        if (two_pass) {
+            // H3 (two-pass): every member byte-verified against its full-digest candidate
+            if (timing) ck(cudaEventRecord(L->ev[16], s), "event");
+            LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], n_large ? W.vitem_cap : 0, s, side,
+                               L->fork_ev[2], L->fork_ev[3]));
+            if (timing) ck(cudaEventRecord(L->ev[17], s), "event");
+        } else {
+            // H3: small members verified on the side stream while the fused pass hashes the rest
+            // of every large payload and byte-compares each large member with its group leader
+            ck(cudaEventRecord(L->fork_ev[2], s), "event");
+            ck(cudaStreamWaitEvent(side, L->fork_ev[2], 0), "fork");
+            LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], 0, side, nullptr, nullptr, nullptr));
+            ck(cudaEventRecord(L->fork_ev[3], side), "event");
+            if (n_large)
+                LCHK(launch_fused(D, W, L->params, n_large, prefilter, W.res[0], s, timing ? L->ev[16] : nullptr,
+                                  timing ? L->ev[17] : nullptr));
+            ck(cudaStreamWaitEvent(s, L->fork_ev[3], 0), "join");
+        }
+        if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
+        // H5 + H6 (speculative: valid unless H3 found residuals)
+        if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, s));
+        if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
+        ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+    };
+    // (per-stage timing needs directly recorded events: FFM_FLAG_TIMING runs launch directly)
+    const bool graph = label && !(L->cfg.flags & FFM_FLAG_NO_GRAPH) && !timing;
+    if (graph) {
+        // replay a CUDA graph of segment A while the log, its buffers and the run mode are
+        // unchanged: one launch instead of ~30 (launch-bound small logs)
+        const GraphKey key{L->epoch, d_dup, two_pass, prefilter, timing};
+        if (!L->graph_exec || !(key == L->graph_key)) {
+            if (L->graph_exec) cudaGraphExecDestroy(L->graph_exec);
+            L->graph_exec = nullptr;
+            uint64_t before = launches;
+            ck(cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed), "begin capture");
+            try {
+                segment_a();
+            } catch (...) {
+                cudaGraph_t g = nullptr;
+                cudaStreamEndCapture(s, &g);
+                if (g) cudaGraphDestroy(g);
+                cudaGetLastError();
+                throw;
+            }
+            cudaGraph_t g = nullptr;
+            ck(cudaStreamEndCapture(s, &g), "end capture");
+            cudaError_t e = cudaGraphInstantiate(&L->graph_exec, g, 0);
+            cudaGraphDestroy(g);
+            ck(e, "graph instantiate");
+            L->graph_key = key;
+            L->graph_launches = launches - before;
+            launches = before;
+        }
+        ck(cudaGraphLaunch(L->graph_exec, s), "graph launch");
+        launches += L->graph_launches;
     } else {
-        // H3: small members verified on the side stream while the fused pass hashes the rest
-        // of every large payload and byte-compares each large member with its group leader
-        ck(cudaEventRecord(L->fork_ev[2], s), "event");
-        ck(cudaStreamWaitEvent(side, L->fork_ev[2], 0), "fork");
-        LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], 0, side, nullptr, nullptr, nullptr));
-        ck(cudaEventRecord(L->fork_ev[3], side), "event");
-        if (n_large)
-            LCHK(launch_fused(D, W, L->params, n_large, prefilter, W.res[0], s, timing ? L->ev[16] : nullptr,
-                              timing ? L->ev[17] : nullptr));
-        ck(cudaStreamWaitEvent(s, L->fork_ev[3], 0), "join");
+        segment_a();
     }
-    if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
-    // H5 + H6 (speculative: valid unless H3 found residuals)
-    if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, s));
-    if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
-    ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
     ck(cudaStreamSynchronize(s), "run sync");
     R.n_members = L->h_counters[1];
     R.two_pass = two_pass;
@@ -1148,6 +1192,13 @@ int ffm_debug_digests(ffm_log* L, uint64_t* out) {
     return FFM_OK;
 }
 
+int ffm_log_set_flags(ffm_log* L, uint32_t flags) {
+    int st = check_state(L);
+    if (st) return st;
+    L->cfg.flags = flags;
+    return FFM_OK;
+}
+
 int ffm_log_reset(ffm_log* L) {
     int st = check_state(L);
     if (st) return st;
@@ -1179,6 +1230,7 @@ int ffm_log_reset(ffm_log* L) {
     }
     L->digests_valid = false;
     L->prefer_two_pass = false;
+    ++L->epoch;
     memset(&L->stats, 0, sizeof(L->stats));
     return FFM_OK;
 }
@@ -1213,6 +1265,7 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->side_stream) cudaStreamDestroy(L->side_stream);
     for (auto e : L->fork_ev)
         if (e) cudaEventDestroy(e);
+    if (L->graph_exec) cudaGraphExecDestroy(L->graph_exec);
     if (L->own_stream && L->stream) cudaStreamDestroy(L->stream);
     cudaGetLastError();
     delete L;

@@ -145,8 +145,20 @@ int launch_zero_counters(Work& W, cudaStream_t st);
 size_t cub_scan_bytes(uint64_t n);
 uint32_t blocks_for(uint64_t threads, uint32_t bs = 256);
 uint32_t resident_grid(const void* kernel, int num_sms, int block = 256);
+bool smem_configured(const void* kernel, int bytes);
 
 }  // namespace ffm
+
+// What a captured run graph depends on.
+struct GraphKey {
+    uint64_t epoch = ~0ull;
+    const void* dup = nullptr;
+    bool two_pass = false, prefilter = false, timing = false;
+    bool operator==(const GraphKey& o) const {
+        return epoch == o.epoch && dup == o.dup && two_pass == o.two_pass && prefilter == o.prefilter &&
+               timing == o.timing;
+    }
+};
 
 // The opaque handle.
 struct ffm_log {
@@ -160,6 +172,10 @@ struct ffm_log {
     bool poisoned = false;
     bool host_ptr_ok = false;      // kernels may dereference registered host pointers
     bool prefer_two_pass = false;  // adaptive round 0 (see run_local)
+    uint64_t epoch = 0;            // bumped whenever records or device buffers change
+    cudaGraphExec_t graph_exec = nullptr;   // captured run segment A (see run_local)
+    GraphKey graph_key;
+    uint64_t graph_launches = 0;
     uint64_t gather_max = 0;       // payloads up to this are gathered by k_gather, above: DMA
     std::string last_error;
 

@@ -830,6 +830,21 @@ uint32_t blocks_for(uint64_t threads, uint32_t bs) {
     return (uint32_t)((threads + bs - 1) / bs);
 }
 
+// Opt-in dynamic shared memory for a kernel, once per (device, kernel).
+bool smem_configured(const void* kernel, int bytes) {
+    static std::mutex mu;
+    static std::unordered_map<uint64_t, int> done;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return false;
+    const uint64_t key = (uint64_t)(uintptr_t)kernel * 131 + (uint64_t)dev;
+    std::lock_guard<std::mutex> g(mu);
+    auto it = done.find(key);
+    if (it != done.end() && it->second >= bytes) return true;
+    if (cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess) return false;
+    done[key] = bytes;
+    return true;
+}
+
 // Persistent launch: exactly the resident blocks (num_sms x occupancy), one wave.
 uint32_t resident_grid(const void* kernel, int num_sms, int block) {
     static std::mutex mu;
@@ -1020,13 +1035,7 @@ int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, in
     }
     const size_t smem = label_smem_bytes(n_sites);
     if (W.label_part && smem <= (size_t)P.max_smem) {
-        static int configured_smem = 0;
-        if (!configured_smem) {
-            if (cudaFuncSetAttribute(k_label_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, P.max_smem) !=
-                cudaSuccess)
-                return -1;
-            configured_smem = 1;
-        }
+        if (!smem_configured((const void*)k_label_hist, P.max_smem)) return -1;
         const uint32_t rows = label_hist_rows(P.num_sms);
         k_label_hist<<<rows, 1024, smem, st>>>(L, W.leader, n_sites, dup_out, W.label_part, W.label_cpart);
         FFM_LAUNCH_CHECK();

@@ -347,13 +347,7 @@ int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, 
     }
     const size_t smem = label_smem_bytes(n_sites);
     if (W.label_part && smem <= (size_t)P.max_smem) {
-        static int configured = 0;
-        if (!configured) {
-            if (cudaFuncSetAttribute(k_merge_label, cudaFuncAttributeMaxDynamicSharedMemorySize, P.max_smem) !=
-                cudaSuccess)
-                return -1;
-            configured = 1;
-        }
+        if (!smem_configured((const void*)k_merge_label, P.max_smem)) return -1;
         const uint32_t rows = label_hist_rows(P.num_sms);
         k_merge_label<<<rows, 1024, smem, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, W.label_part,
                                                W.label_cpart, nullptr, nullptr);

@@ -401,3 +401,60 @@ def test_benefit_linear_in_durations(ffm):
     lg.dur = lg.dur * np.uint64(7)
     _, b7, _ = gpu_dedup(ffm, lg)
     np.testing.assert_array_equal(b7, b1 * np.uint64(7))
+
+
+def test_sharded_api_errors(ffm):
+    """Call-order and consistency errors of the sharded / online API (one process)."""
+    import torch
+    x = np.frombuffer(b"abcdefgh" * 8, np.uint8).copy()
+    with ffm.FfmLog(2, rank=0, world=2) as log:
+        log.append_batch([0, 1], [64, 64], [x.ctypes.data] * 2, [1, 2], gids=[0, 3])
+        with pytest.raises(ffm.FfmError) as e:
+            log.run()                                   # a sharded log has no single-log run
+        assert e.value.code == ffm.FFM_E_STATE
+        with pytest.raises(ffm.FfmError) as e:
+            log.online_step()
+        assert e.value.code == ffm.FFM_E_STATE
+        reps = torch.empty((4, ffm.REP_WORDS), dtype=torch.int64, device="cuda")
+        dup = torch.empty(2, dtype=torch.int64, device="cuda")
+        ben = torch.empty(2, dtype=torch.int64, device="cuda")
+        with pytest.raises(ffm.FfmError) as e:          # merge before local
+            ffm.ffm_shard_merge(log.h, reps, [1, 0], dup, ben)
+        assert e.value.code == ffm.FFM_E_STATE
+        n = ffm.ffm_shard_local(log.h, reps, 4)
+        assert n == 1                                   # two equal payloads: one class
+        with pytest.raises(ffm.FfmError) as e:          # counts disagree with this rank
+            ffm.ffm_shard_merge(log.h, reps, [2, 0], dup, ben)
+        assert e.value.code == ffm.FFM_E_COMM
+        with pytest.raises(ffm.FfmError) as e:          # a peer with reps but no mapping
+            ffm.ffm_shard_merge(log.h, reps, [1, 1], dup, ben)
+        assert e.value.code == ffm.FFM_E_STATE
+        ffm.ffm_shard_merge(log.h, reps, [1, 0], dup, ben)   # alone: duplicates stay local
+        assert dup.cpu().tolist() == [-1, 0] and ben.cpu().tolist() == [0, 2]
+
+
+def test_graph_replay_matches_direct_launches(ffm):
+    """Runs replay a captured CUDA graph while the log is unchanged; appends, output
+    buffer changes and mode changes re-capture.  Same results as direct launches."""
+    import torch
+    lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 32)
+    want = oracle.dedup(lg)
+    half = lg.n // 2
+    ptrs = lg.payload_ptrs()
+    for graph in (True, False):
+        with ffm.FfmLog(lg.n_sites, graph=graph, timing=True) as log:
+            log.append_batch(lg.site[:half], lg.size[:half], ptrs[:half], lg.dur[:half])
+            for _ in range(3):
+                d, b = log.run()
+            np.testing.assert_array_equal(d, oracle.dedup(lg.subset(np.arange(half)))[0])
+            log.append_batch(lg.site[half:], lg.size[half:], ptrs[half:], lg.dur[half:])
+            for _ in range(2):
+                d, b = log.run()
+                np.testing.assert_array_equal(d, want[0])
+                np.testing.assert_array_equal(b, want[1])
+            dd = torch.empty(lg.n, dtype=torch.int64, device="cuda")
+            bb = torch.empty(lg.n_sites, dtype=torch.int64, device="cuda")
+            for _ in range(2):
+                log.run(dd, bb)
+                np.testing.assert_array_equal(dd.cpu().numpy(), want[0])
+                np.testing.assert_array_equal(bb.cpu().numpy().view(np.uint64), want[1])
