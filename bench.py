@@ -134,10 +134,13 @@ def make_log(workload, n_scale, size_scale, shard=(0, 1)):
 def alg_bytes(lg, idx, dup, small_bytes, chunk=32768, two_pass=False):
     """Algorithmic bytes per kernel for this rank's records idx: every
     payload byte is hashed once; a member payload's bytes are compared once against its
-    leader, whose chunks (after the first) are shared through L2 by the group.
+    leader, whose bytes are read once per class.
       prefix (k_hash_large, first chunks):  sum over large payloads of c0 = min(size, chunk)
-      fused  (k_fused):  sum over large (size - c0) + members' c0 + their leaders' c0
-      small  (k_hash_small / k_verify_small): sizes / members + leaders
+      fused  (k_fused_fx):  sum over large (size - c0) + members' c0 + their leaders' c0
+      small  (k_fused_small): small sizes + leaders of small members
+    two-pass: k_hash_large hashes every large byte, then members and their class leaders
+    are read once more (verify); small: k_hash_small, then k_verify_small (side stream,
+    concurrent with the large verify).
     dup: this rank's duplicate_of (global gids)."""
     size = lg.size[idx].astype(np.int64)
     n = len(size)
@@ -153,27 +156,27 @@ def alg_bytes(lg, idx, dup, small_bytes, chunk=32768, two_pass=False):
     c0 = np.minimum(size, chunk)
     units = int(((size[big] + chunk - 1) // chunk).sum())
     out = {
-        "hash_small": int(size[small].sum()) + 8 * n + 24 * int(small.sum()),
+        "small": int(size[small].sum()) + int(size[small & leaders].sum()) + 40 * int(small.sum()),
         "prefix": int(c0[big].sum()) + 40 * int(big.sum()),
         "fused": int((size[big] - c0[big]).sum()) + int(c0[big & member].sum()) + int(c0[big & leaders].sum())
-        + 40 * units,
-        "verify_small": int(size[small & member].sum()) + int(size[small & leaders].sum()) + 4 * n,
+        + 32 * units,
     }
     if two_pass:
-        # hash every large byte (k_hash_large), then verify members against their class
-        # leader, each leader read once per class (the "fused" slot times the verify stage)
+        out["small"] = int(size[small].sum()) + 32 * int(small.sum())      # k_hash_small only
+        out["verify_small"] = int(size[small & member].sum()) + int(size[small & leaders].sum())
         out["prefix"] = int(size[big].sum()) + 40 * units
         out["fused"] = int(size[big & member].sum()) + int(size[big & leaders].sum())
     out["path"] = sum(out.values()) + 64 * n    # + group-by / label metadata
     return out
 
 
-def ncu_traffic(kernel):
-    """dram bytes per launch of `kernel` from the committed ncu --set full summary."""
+def ncu_traffic(kernel, capture):
+    """dram bytes per launch of `kernel` from the committed ncu --set full capture of the
+    same workload and round-0 mode (profiles/ncu_summary.json), else None."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         d = json.load(open(p))
-        k = d["kernels"].get(kernel)
+        k = d["captures"][capture]["kernels"].get(kernel)
         return None if k is None else float(k["dram_bytes_per_launch"])
     except Exception:
         return None
@@ -285,17 +288,24 @@ def run_ours(args):
         ab["fused"] = int(st["prefilter_rest_bytes"]) + int(c0[big & mem].sum()) + 40 * int(((sz[big] + 32767) // 32768).sum())
         ab["path"] = sum(v for k, v in ab.items() if k != "path") + 64 * len(idx)
     peak, peak_src = load_peak()
-    kern_ms = {"hash_small": st["ms_hash_small"], "prefix": st["ms_hash_large"], "fused": st["ms_fused"]}
+    kern_ms = {"small": st["ms_hash_small"], "prefix": st["ms_hash_large"], "fused": st["ms_fused"]}
     dom = max(kern_ms, key=lambda k: kern_ms[k])
     dom_ms = kern_ms[dom]
     achieved = ab[dom] / (dom_ms * 1e-3) / 1e9 if dom_ms > 0 else 0.0
-    kname = {"hash_small": "k_hash_small", "prefix": "k_hash_large", "fused": "k_fused"}[dom]
-    traffic = None if args.prefilter else ncu_traffic(kname)   # committed ncu summary is of the default path
+    two_pass = args.two_pass or st.get("two_pass", 0) >= 0.5
+    fused_k = "k_fused" if os.environ.get("FFM_FUSED_IMPL", "0") == "1" else "k_fused_fx"
+    kname = {"small": "k_hash_small" if two_pass else "k_fused_small", "prefix": "k_hash_large",
+             "fused": "k_verify_large" if two_pass else fused_k}[dom]
+    mode = "two-pass" if two_pass else ("fused" if fused_k == "k_fused_fx" else "fused-l2")
+    capture = f"config{args.workload}/{mode}" + ("/prefilter" if args.prefilter else "") + \
+        (f"/digest_bits{args.digest_bits}" if args.digest_bits < 64 else "")
+    traffic = ncu_traffic(kname, capture) if world == 1 and args.n_scale == 1 and args.size_scale == 1 else None
     roofline = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic, "alg_bytes": ab[dom],
                 "ms": round(dom_ms, 4), "peak_source": peak_src,
                 "read_stream_ceiling_gbs": read_ceiling(),
-                "note": "traffic = ncu dram__bytes_read+write of this kernel on config 5 (profiles/ncu_summary.json)"}
+                "traffic_source": f"profiles/ncu_summary.json captures[{capture}] (ncu --set full, same workload and mode)"
+                if traffic is not None else "no committed ncu capture of this workload/mode"}
     path_gbs = ab["path"] / (ms * 1e-3) / 1e9
 
     e2e = None

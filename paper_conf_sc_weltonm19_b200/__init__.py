@@ -16,7 +16,10 @@ import os
 
 import numpy as np
 
-from ._build import LIB as _LIB_PATH
+from ._build import LIB as _LIB_DEFAULT
+
+# FFM_LIB: a tuning-variant build of the same sources (tools/build_variants.sh)
+_LIB_PATH = os.environ.get("FFM_LIB") or _LIB_DEFAULT
 
 FFM_OK, FFM_E_INVAL, FFM_E_RANGE, FFM_E_NOMEM, FFM_E_CUDA, FFM_E_COMM, FFM_E_STATE, FFM_E_NODEV = \
     0, -1, -2, -3, -4, -5, -6, -7

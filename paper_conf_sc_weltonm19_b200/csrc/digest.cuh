@@ -114,4 +114,19 @@ __device__ __forceinline__ bool blk_equal(const Blk& x, const Blk& y) {
         }                                                                                  \
     }
 
+// One warp per item (grid-stride over warps): item w is record REC_EXPR (may use w_);
+// the body runs with all 32 lanes when PRED(rec) holds.  For per-record planning work
+// whose size varies by orders of magnitude (a few records of ~1000 chunks each, or
+// millions of single-chunk ones).
+#define FFM_WARP_EACH(COUNT, REC_EXPR, PRED, ...)                                         \
+    {                                                                                      \
+        const int lane = threadIdx.x & 31;                                                 \
+        const uint32_t nw_ = (gridDim.x * blockDim.x) >> 5;                                \
+        for (uint32_t w_ = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; w_ < (COUNT); w_ += nw_) { \
+            const uint32_t rec = (REC_EXPR);                                               \
+            if (!(PRED)) continue;                                                         \
+            __VA_ARGS__                                                                    \
+        }                                                                                  \
+    }
+
 }  // namespace ffm

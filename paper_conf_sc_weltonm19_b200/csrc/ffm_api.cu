@@ -148,9 +148,11 @@ bool is_device_ptr(const void* p) {
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
-// Records in [begin, end) with size <= small_bytes, as indices relative to begin,
-// ordered by 32-byte block count, largest first (stable counting sort).
-void build_small_order(const ffm_log* L, uint64_t begin, uint64_t end, std::vector<uint32_t>& order) {
+// Records in [begin, end) as indices relative to begin: first those with size <=
+// small_bytes, ordered by 32-byte block count, largest first (stable counting sort);
+// then the large ones in index order (one warp per large record in the planning
+// kernels).  Returns the number of small records.
+uint64_t build_small_order(const ffm_log* L, uint64_t begin, uint64_t end, std::vector<uint32_t>& order) {
     const uint32_t nb = (L->params.small_bytes + 31) / 32 + 1;
     std::vector<uint32_t> start(nb + 1, 0);
     uint64_t ns = 0;
@@ -167,6 +169,9 @@ void build_small_order(const ffm_log* L, uint64_t begin, uint64_t end, std::vect
     for (uint64_t i = begin; i < end; ++i)
         if (L->h_size[i] <= L->params.small_bytes)
             order[cur[nb - 1 - (uint32_t)((L->h_size[i] + 31) / 32)]++] = (uint32_t)(i - begin);
+    for (uint64_t i = begin; i < end; ++i)
+        if (L->h_size[i] > L->params.small_bytes) order.push_back((uint32_t)(i - begin));
+    return ns;
 }
 
 void upload_order(ffm_log* L, const std::vector<uint32_t>& order, uint32_t*& dptr, uint64_t& cap, cudaStream_t s) {
@@ -209,9 +214,9 @@ void upload_meta(ffm_log* L) {
     // 8-lane groups of a warp then get payloads of near-equal length (no idle lanes)
     {
         std::vector<uint32_t> order;
-        build_small_order(L, 0, n, order);
+        L->n_small = build_small_order(L, 0, n, order);
+        L->n_large_rec = order.size() - L->n_small;
         upload_order(L, order, L->d_small_order, L->d_small_cap, s);
-        L->n_small = order.size();
     }
     ck(cudaStreamSynchronize(s), "meta sync");
     L->d_meta_n = n;
@@ -329,6 +334,13 @@ void ensure_work(ffm_log* L, uint64_t n) {
         dev_alloc(W.hpart, 2 * c);
         W.hitem_cap = W.vitem_cap = c;
     }
+    const uint64_t fcap = fx_entry_cap(L->n_large_chunks, L->params.chunk_bytes);
+    if (fcap > W.fitem_cap) {
+        ++L->epoch;
+        const uint64_t c = fcap + fcap / 4;
+        dev_alloc(W.fitems, 2 * c);   // 32-byte descriptors
+        W.fitem_cap = c;
+    }
     if (L->cfg.n_sites > W.site_cap) {
         ++L->epoch;
         dev_alloc(W.ben, L->cfg.n_sites);
@@ -353,6 +365,8 @@ DevLog dev_view(const ffm_log* L) {
     d.n = (uint32_t)L->h_size.size();
     d.small_order = L->d_small_order;
     d.n_small = (uint32_t)L->n_small;
+    d.large_order = L->d_small_order ? L->d_small_order + L->n_small : nullptr;
+    d.n_large = (uint32_t)L->n_large_rec;
     return d;
 }
 
@@ -406,13 +420,16 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     auto segment_a = [&]() {
         if (timing) ck(cudaEventRecord(L->ev[0], s), "event");
         if (launch_zero_counters(W, s) < 0) throw CudaFail{cudaGetLastError(), "zero counters"};
-        // H1 hash: small payloads on the side stream, concurrently with the large path
-        ck(cudaEventRecord(L->fork_ev[0], s), "event");
-        ck(cudaStreamWaitEvent(side, L->fork_ev[0], 0), "fork");
-        if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
-        LCHK(launch_hash_small(D, W, L->params, side));
-        if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
-        ck(cudaEventRecord(L->fork_ev[1], side), "event");
+        // two-pass H1 of small payloads on the side stream, concurrently with the large path
+        // (fused: small payloads are grouped by their first 32 bytes, hashed after H2)
+        if (two_pass) {
+            ck(cudaEventRecord(L->fork_ev[0], s), "event");
+            ck(cudaStreamWaitEvent(side, L->fork_ev[0], 0), "fork");
+            if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
+            LCHK(launch_hash_small(D, W, L->params, side));
+            if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
+            ck(cudaEventRecord(L->fork_ev[1], side), "event");
+        }
         if (n_large) {
             LCHK(launch_hash_plan(D, W, L->params, s));
             if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
@@ -421,9 +438,10 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
             if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
             if (two_pass) LCHK(launch_combine(D, W, L->params, s));
         }
-        ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
+        if (two_pass) ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
         if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
-        // H2 group-by (round 0): small payloads by full digest, large ones by first-chunk digest
+        // H2 group-by (round 0): two-pass -- every payload by its full digest; fused -- small
+        // payloads by their first 32 bytes, large ones by their first-chunk digest
         uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
         LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, two_pass ? -1 : 0, W.res[0], s));
         if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
@@ -434,11 +452,14 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
                                L->fork_ev[2], L->fork_ev[3]));
             if (timing) ck(cudaEventRecord(L->ev[17], s), "event");
         } else {
-            // H3: small members verified on the side stream while the fused pass hashes the rest
-            // of every large payload and byte-compares each large member with its group leader
+            // H1 + H3 of small payloads on the side stream (hash each, byte-compare members
+            // with their prefix-group leader) while the fused pass hashes the rest of every
+            // large payload and byte-compares each large member with its group leader
             ck(cudaEventRecord(L->fork_ev[2], s), "event");
             ck(cudaStreamWaitEvent(side, L->fork_ev[2], 0), "fork");
-            LCHK(launch_verify(D, W, L->params, nullptr, D.n, W.res[0], 0, side, nullptr, nullptr, nullptr));
+            if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
+            LCHK(launch_fused_small(D, W, L->params, W.res[0], side));
+            if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
             ck(cudaEventRecord(L->fork_ev[3], side), "event");
             if (n_large)
                 LCHK(launch_fused(D, W, L->params, n_large, prefilter, W.res[0], s, timing ? L->ev[16] : nullptr,
@@ -687,6 +708,8 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
         L->host_ptr_ok = hp != 0;
         L->gather_max = kGatherMaxDefault;
         if (const char* e = getenv("FFM_GATHER_MAX")) L->gather_max = strtoull(e, nullptr, 10);   // tuning knob
+        L->params.fused_impl = 0;
+        if (const char* e = getenv("FFM_FUSED_IMPL")) L->params.fused_impl = atoi(e);   // A/B knob (same results)
         L->params.chunk_bytes = chunk;
         L->params.small_bytes = small;
         L->params.digest_mask = cfg->digest_bits >= 64 ? ~0ull : ((1ull << cfg->digest_bits) - 1);
@@ -1096,10 +1119,12 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
             D.chan += w0;
             D.n = (uint32_t)nw;
             std::vector<uint32_t> order;
-            build_small_order(L, w0, n, order);
+            const uint64_t nsw = build_small_order(L, w0, n, order);
             upload_order(L, order, L->d_win_order, L->d_win_cap, s);
             D.small_order = L->d_win_order;
-            D.n_small = (uint32_t)order.size();
+            D.n_small = (uint32_t)nsw;
+            D.large_order = L->d_win_order + nsw;
+            D.n_large = (uint32_t)(order.size() - nsw);
             uint64_t n_large = 0;
             for (uint64_t i = w0; i < n; ++i) n_large += large_chunks(L, L->h_size[i]);
             // H1..H4 on the window: exact window-local classes
@@ -1219,6 +1244,7 @@ int ffm_log_reset(ffm_log* L) {
     L->any_gid = false;
     L->d_meta_n = 0;
     L->n_small = 0;
+    L->n_large_rec = 0;
     L->arena_used = 0;
     L->ring_fill = 0;
     L->n_reps = 0;
@@ -1242,7 +1268,7 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->stage_stream) cudaStreamSynchronize(L->stage_stream);
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
-                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.vitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
+                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.vitems, W.fitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
                     W.dup, W.ben, W.cnt, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
                     L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)

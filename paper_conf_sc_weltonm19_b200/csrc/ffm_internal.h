@@ -27,6 +27,8 @@ struct DevLog {
     uint32_t n;
     const uint32_t* small_order;  // records <= small_bytes, sorted by block count (descending)
     uint32_t n_small;
+    const uint32_t* large_order;  // records > small_bytes, ascending
+    uint32_t n_large;
 };
 
 // Scratch of one run (grown on demand, reused across runs).
@@ -47,6 +49,7 @@ struct Work {
     uint32_t* fhead = nullptr;     // [n] round 0: head (leader) of a large record's fused group
     uint2* hitems = nullptr;       // large-payload hash work units (record, chunk)
     uint2* vitems = nullptr;       // large-payload verify work units (member, chunk)
+    uint4* fitems = nullptr;       // pipelined fused pass stage descriptors (2 x uint4 each)
     uint32_t* hcount = nullptr;    // [n+1] per-record hash chunk counts
     uint32_t* hstart = nullptr;    // [n+1] exclusive scan of hcount
     uint64_t* hpart = nullptr;     // [2 * hitem_cap] per-unit partial NH sums (A, B)
@@ -60,7 +63,7 @@ struct Work {
     uint32_t* counters = nullptr;  // device counters: [0] nres, [1] n_members, [2..] misc
     void* cub_tmp = nullptr;
     size_t cub_tmp_bytes = 0;
-    uint64_t n_cap = 0, t_cap = 0, hitem_cap = 0, vitem_cap = 0, site_cap = 0;
+    uint64_t n_cap = 0, t_cap = 0, hitem_cap = 0, vitem_cap = 0, site_cap = 0, fitem_cap = 0;
 };
 
 // One representative per exact local class, exported for the cross-shard merge.
@@ -106,11 +109,13 @@ struct Params {
     uint32_t small_bytes;
     int num_sms;
     int max_smem;      // opt-in dynamic shared memory per block (bytes)
+    int fused_impl;    // round-0 fused pass: 0 = pipelined (k_fused_fx), 1 = L2 leader-first (k_fused)
 };
 
 // ---- kernel launchers (kernels.cu).  All asynchronous on `st`; each returns the
 // number of kernels it launched (for the launch count), or -1 on launch error.
 int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
+int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_out, cudaStream_t st);
 int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st, int phase = 0);
 int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
@@ -143,6 +148,7 @@ int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, 
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 size_t cub_scan_bytes(uint64_t n);
+uint64_t fx_entry_cap(uint64_t n_large_chunks, uint32_t chunk_bytes);
 uint32_t blocks_for(uint64_t threads, uint32_t bs = 256);
 uint32_t resident_grid(const void* kernel, int num_sms, int block = 256);
 bool smem_configured(const void* kernel, int bytes);
@@ -197,7 +203,7 @@ struct ffm_log {
     uint64_t d_meta_cap = 0;       // records
     uint64_t d_meta_n = 0;         // records uploaded
     uint32_t* d_small_order = nullptr;   // small records by size class (built at upload)
-    uint64_t d_small_cap = 0, n_small = 0;
+    uint64_t d_small_cap = 0, n_small = 0, n_large_rec = 0;
 
     // HBM arena
     uint8_t* arena = nullptr;

@@ -257,8 +257,7 @@ __global__ void k_hash_count(DevLog L, uint32_t small_bytes, uint32_t chunk_byte
 
 __global__ void k_hash_fill(DevLog L, uint32_t small_bytes, uint32_t chunk_bytes, const uint32_t* __restrict__ start,
                             uint2* __restrict__ items) {
-    const uint32_t* nolist = nullptr;
-    FFM_WARP_COMPACT(L.n, nolist, (L.size[r_] > small_bytes), {
+    FFM_WARP_EACH(L.n_large, L.large_order[w_], true, {
         const uint32_t c_n = start[rec + 1] - start[rec];
         const uint32_t s0 = start[rec];
         for (uint32_t c = lane; c < c_n; c += 32) items[s0 + c] = make_uint2(rec, c);
@@ -278,11 +277,23 @@ __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ li
     uint64_t key;
     if (round <= 0) {                 // 0: fused round 0 (prefix keys); -1: two-pass round 0
         uint64_t n = L.size[r];
-        if (n <= small_bytes || round < 0) {
-            // small payload: its full digest
+        if (round < 0) {
+            // two-pass round 0: every payload by its full digest
             uint64_t d = finalize_digest(W.accA[r], W.accB[r], n);
-            W.digest[r] = d;
+            if (n <= small_bytes) W.digest[r] = d;
             key = group_key(d, n, digest_mask, L.chan[r]);
+        } else if (n <= small_bytes) {
+            // fused round 0, small payload: its first 32 bytes (equal payloads have equal
+            // prefixes; k_fused_small hashes and byte-compares the rest)
+            Blk x = zero_blk();
+            if (n) {
+                x = ld_stream(L.arena + L.off[r]);
+                mask_tail(x, n, 0);
+            }
+            uint64_t pd = 0x5851F42D4C957F2Dull;
+#pragma unroll
+            for (int i = 0; i < 8; i += 2) pd = fmix64(pd ^ ((uint64_t)x.v[i + 1] << 32 | x.v[i]));
+            key = group_key(pd, n, digest_mask, L.chan[r]);
         } else {
             // large payload: the digest of its FIRST chunk (computed by the prefix pass);
             // equal payloads have equal first chunks, so every candidate still shares a group
@@ -381,8 +392,7 @@ __global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, ui
 }
 
 __global__ void k_fused_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes) {
-    const uint32_t* nolist = nullptr;
-    FFM_WARP_COMPACT(L.n, nolist, (L.size[r_] > small_bytes), {
+    FFM_WARP_EACH(L.n_large, L.large_order[w_], true, {
         const uint32_t h = W.fhead[rec];
         const uint32_t k = W.gcount[h] + 1, p = W.pos[rec], base = W.lstart[h];
         const uint32_t c_n = (uint32_t)((L.size[rec] + chunk_bytes - 1) / chunk_bytes);
@@ -516,29 +526,531 @@ __global__ void __launch_bounds__(256, FFM_FUSED_MINB) k_fused(DevLog L, Work W,
     }
 }
 
+// ----------------------------------------------------------------------------
+// H1 + H3 fused, pipelined (round 0, large payloads; the default).  Every byte of the
+// pass is read from HBM exactly once (the prefix-chunk compares aside), with no
+// reliance on L2 for the leaders' bytes:
+//
+//   * the pass works on pieces of <= kFxPiece bytes (a chunk, or an equal split of a
+//     larger chunk); a task is (group head h, piece t) with all of the group's members:
+//     stages [leader piece, member 1 piece, ..., member k-1 piece];
+//   * k_fx_fill writes one self-contained 32-byte descriptor per (record, piece), laid
+//     out task by task; one producer warp per CTA takes segments of kFxSeg descriptors
+//     (dynamic scheduling), prefetches them a batch ahead and streams every stage into
+//     a ring of kFxStages shared-memory buffers with cp.async.bulk (TMA engine, mbarrier
+//     complete_tx, L2 evict_first);
+//   * eight consumer warps own the piece word by word: the leader's words are hashed
+//     (outside chunk 0, which the prefix pass hashed) and kept in registers for the
+//     whole task, and every member's words are compared against them -- no member byte
+//     is hashed.
+//
+// A member's NH sums follow from its leader's: NH is a plain positional sum, so over
+// a chunk the member's partial equals the leader's plus, for each differing word,
+// nh(member word) - nh(leader word) (mod 2^64).  Those deltas (zero for a duplicate)
+// are added into the member's chunk slot; k_hash_combine forms
+// acc[m] = acc_prefix[m] + sum_{c>=1} (part[h][c] + delta[m][c]).  The first
+// mismatching word is the exact minimum (every word is compared).
+// ----------------------------------------------------------------------------
+#ifndef FFM_FX_PIECE
+#define FFM_FX_PIECE 32768
+#endif
+#ifndef FFM_FX_STAGES
+#define FFM_FX_STAGES 3
+#endif
+#ifndef FFM_FX_CTAS
+#define FFM_FX_CTAS 2
+#endif
+constexpr int kFxConsumers = 8;                       // consumer warps
+constexpr int kFxThreads = 32 * (kFxConsumers + 1);   // + one producer warp
+constexpr uint32_t kFxPiece = FFM_FX_PIECE;           // bytes per stage (max)
+constexpr int kFxWords = kFxPiece / 16 / (32 * kFxConsumers);   // 16-B words per consumer thread per stage
+constexpr int kFxStages = FFM_FX_STAGES;
+constexpr uint32_t kFxSeg = 64;                       // descriptors per scheduler grab
+
+enum : uint32_t { kFxLeader = 1u, kFxHash = 2u, kFxDelta = 4u, kFxReduce = 8u, kFxSkip = 16u, kFxDone = 32u };
+
+// one stage of the pipelined pass (descriptor in HBM, meta in shared memory)
+struct FxDesc {
+    uint64_t src;     // arena offset of the piece
+    uint32_t rec;     // record
+    uint32_t lenf;    // piece bytes (bits 0-23) | kFx* flags << 24
+    uint32_t w0;      // first 16-B word of the piece (record-relative)
+    uint32_t slot;    // the record's hpart slot of the piece's chunk
+    uint32_t k;       // on a task's first descriptor: the task's length (entries); else 0
+    uint32_t pad;
+};
+
+constexpr size_t kFxSmem = (size_t)kFxStages * kFxPiece + (size_t)kFxStages * sizeof(FxDesc) +
+                           2 * kFxStages * sizeof(uint64_t) + 2 * kFxConsumers * 2 * sizeof(uint64_t);
+
+// pieces of a record of n bytes: chunks of chunk_bytes, each split into ppc pieces of ps
+struct FxSplit {
+    uint32_t chunk, ppc, ps;
+};
+__host__ __device__ __forceinline__ FxSplit fx_split(uint32_t chunk_bytes) {
+    FxSplit f;
+    f.chunk = chunk_bytes;
+    f.ppc = (chunk_bytes + kFxPiece - 1) / kFxPiece;
+    f.ps = ((chunk_bytes + f.ppc - 1) / f.ppc + 1023u) & ~1023u;
+    return f;
+}
+__host__ __device__ __forceinline__ uint32_t fx_pieces(const FxSplit& f, uint64_t n) {
+    const uint64_t full = n / f.chunk, rem = n % f.chunk;
+    return (uint32_t)(full * f.ppc + (rem + f.ps - 1) / f.ps);
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "FFM_WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra FFM_WAIT_%=;\n}" ::"r"(bar),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+            dst),
+        "l"(src), "r"(bytes), "r"(bar), "l"(pol)
+        : "memory");
+}
+
+// keep the first `valid` bytes of a 16-B word, zero the rest
+__device__ __forceinline__ void mask_word(uint4& w, int32_t valid) {
+    if (valid >= 16) return;
+    uint32_t* v = reinterpret_cast<uint32_t*>(&w);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int32_t vb = valid - 4 * i;
+        v[i] &= vb >= 4 ? 0xFFFFFFFFu : (vb <= 0 ? 0u : ((1u << (8 * vb)) - 1u));
+    }
+}
+
+// NH keys of word q: position q mod 16 (fixed per consumer thread), stripe q div 16.
+__device__ __forceinline__ void word_keys(uint32_t* k, const uint32_t* ka, uint32_t s) {
+#pragma unroll
+    for (int j = 0; j < 6; ++j) k[j] = ka[j] + s * kDA(j);
+}
+
+// Task layout.  Head h's group (k = members + 1 records) becomes, per piece t, S =
+// ceil((k - 1) / (kFxMaxK - 1)) sub-tasks (at least 1) of <= kFxMaxK entries: a copy of
+// the head's descriptor, then up to kFxMaxK - 1 members.  Long groups thus spread over
+// CTAs (a leader piece is re-staged once per kFxMaxK - 1 members, hashed only in
+// sub-task 0).  Entries of a head: pieces x (k - 1 + S), contiguous from lstart[h].
+constexpr uint32_t kFxMaxK = 64;
+
+__device__ __forceinline__ uint32_t fx_subtasks(uint32_t k) {
+    return k <= 1 ? 1u : (k - 1 + kFxMaxK - 2) / (kFxMaxK - 1);
+}
+
+// verify = 0: round-0 fused groups (every large head, singletons included);
+// verify = 1: verify groups of k_leader (leaders with >= 1 large member).
+__global__ void k_fx_count(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes, int verify) {
+    const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r > L.n) return;
+    uint32_t c = 0;
+    if (r < L.n && L.size[r] > small_bytes && (verify ? W.gcount[r] > 0 : W.fhead[r] == r)) {
+        const uint32_t k = W.gcount[r] + 1;
+        c = fx_pieces(fx_split(chunk_bytes), L.size[r]) * (k - 1 + fx_subtasks(k));
+    }
+    W.lcount[r] = c;
+}
+
+// Verify-only descriptors (two-pass round 0 and resolve rounds): each large member of
+// `list` whose leader has its size and channel, at position pos + 1 of its leader's
+// group; the member at pos 0 also writes the leader's copies.  No hashing: the
+// digests are final.
+__global__ void k_fx_vfill(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
+                           uint32_t small_bytes, uint32_t chunk_bytes, FxDesc* __restrict__ items) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) W.counters[8] = 0;   // segment scheduler
+    const FxSplit f = fx_split(chunk_bytes);
+    FFM_WARP_EACH(list ? n_list : L.n_large, list ? list[w_] : L.large_order[w_],
+                  (W.leader[rec] != rec && L.size[rec] > small_bytes && L.size[W.leader[rec]] == L.size[rec] &&
+                   L.chan[W.leader[rec]] == L.chan[rec]), {
+        const uint32_t ld = W.leader[rec];
+        const uint32_t k = W.gcount[ld] + 1, p = W.pos[rec] + 1, base = W.lstart[ld];
+        const uint32_t S = fx_subtasks(k), K = k - 1 + S;
+        const uint64_t n = L.size[rec];
+        const uint32_t np = fx_pieces(f, n);
+        for (uint32_t t = lane; t < np; t += 32) {
+            const uint32_t c = t / f.ppc, j = t - c * f.ppc;
+            const uint64_t st = (uint64_t)c * f.chunk + (uint64_t)j * f.ps;
+            const uint64_t en = min(min(st + f.ps, (uint64_t)(c + 1) * f.chunk), n);
+            const uint64_t pb = base + (uint64_t)t * K;
+            FxDesc d;
+            d.w0 = (uint32_t)(st >> 4);
+            d.slot = 0;
+            d.pad = 0;
+            d.lenf = (uint32_t)(en - st);
+            const uint32_t q = (p - 1) / (kFxMaxK - 1), i = (p - 1) - q * (kFxMaxK - 1) + 1;
+            d.src = L.off[rec] + st;
+            d.rec = rec;
+            d.k = 0;
+            items[pb + (uint64_t)q * kFxMaxK + i] = d;
+            if (p == 1) {
+                d.src = L.off[ld] + st;
+                d.rec = ld;
+                d.lenf |= kFxLeader << 24;
+                for (uint32_t qq = 0; qq < S; ++qq) {
+                    d.k = qq + 1 < S ? kFxMaxK : k - qq * (kFxMaxK - 1);
+                    items[pb + (uint64_t)qq * kFxMaxK] = d;
+                }
+            }
+        }
+    })
+}
+
+// One descriptor per (record, piece, sub-task copy); also zeroes the chunk slots (>= 1)
+// the pass accumulates into.
+__global__ void k_fx_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes, int prefilter,
+                          FxDesc* __restrict__ items) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) W.counters[8] = 0;   // segment scheduler
+    const FxSplit f = fx_split(chunk_bytes);
+    FFM_WARP_EACH(L.n_large, L.large_order[w_], true, {
+        const uint32_t h = W.fhead[rec];
+        const uint32_t k = W.gcount[h] + 1, p = W.pos[rec], base = W.lstart[h];
+        const uint32_t S = fx_subtasks(k), K = k - 1 + S;   // sub-tasks, entries per piece
+        const uint64_t n = L.size[rec], off = L.off[rec];
+        const uint32_t np = fx_pieces(f, n), hs = W.hstart[rec];
+        const bool skip_all = prefilter && prefix_unique(W, rec);
+        const uint32_t last0 = min(k - 1, kFxMaxK - 1);      // position ending sub-task 0
+        for (uint32_t t = lane; t < np; t += 32) {
+            const uint32_t c = t / f.ppc, j = t - c * f.ppc;
+            const uint64_t st = (uint64_t)c * f.chunk + (uint64_t)j * f.ps;
+            const uint64_t en = min(min(st + f.ps, (uint64_t)(c + 1) * f.chunk), n);
+            FxDesc d;
+            d.src = off + st;
+            d.rec = rec;
+            d.w0 = (uint32_t)(st >> 4);
+            d.slot = hs + c;
+            d.pad = 0;
+            const uint64_t pb = base + (uint64_t)t * K;
+            if (p == 0) {
+                for (uint32_t q = 0; q < S; ++q) {
+                    uint32_t fl = kFxLeader;
+                    if (q == 0 && c > 0) fl |= kFxHash;
+                    if ((k == 1 && c == 0) || skip_all) fl |= kFxSkip;
+                    if (q == 0 && last0 == 0 && c > 0) fl |= kFxReduce;
+                    d.lenf = (uint32_t)(en - st) | (fl << 24);
+                    d.k = q + 1 < S ? kFxMaxK : k - q * (kFxMaxK - 1);
+                    items[pb + (uint64_t)q * kFxMaxK] = d;
+                }
+            } else {
+                const uint32_t q = (p - 1) / (kFxMaxK - 1), i = (p - 1) - q * (kFxMaxK - 1) + 1;
+                uint32_t fl = c > 0 ? kFxDelta : 0u;
+                if (p == last0 && c > 0) fl |= kFxReduce;
+                d.lenf = (uint32_t)(en - st) | (fl << 24);
+                d.k = 0;
+                items[pb + (uint64_t)q * kFxMaxK + i] = d;
+            }
+            if (c > 0 && j == 0) {
+                W.hpart[2ull * (hs + c)] = 0;
+                W.hpart[2ull * (hs + c) + 1] = 0;
+            }
+        }
+    })
+}
+
+__global__ void __launch_bounds__(kFxThreads, FFM_FX_CTAS) k_fused_fx(DevLog L, Work W,
+                                                                      const FxDesc* __restrict__ items,
+                                                                      const uint32_t* __restrict__ n_items_ptr,
+                                                                      uint32_t* res_out) {
+    extern __shared__ __align__(128) uint8_t fx_smem[];
+    uint8_t* bufs = fx_smem;
+    FxDesc* meta = reinterpret_cast<FxDesc*>(fx_smem + (size_t)kFxStages * kFxPiece);
+    uint64_t* full = reinterpret_cast<uint64_t*>(meta + kFxStages);
+    uint64_t* empty = full + kFxStages;
+    uint64_t* red = empty + kFxStages;   // [2][kFxConsumers][2]
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kFxStages; ++s) {
+            mbar_init(smem_u32(&full[s]), 1);
+            mbar_init(smem_u32(&empty[s]), kFxConsumers);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+    __syncthreads();
+
+    if (warp == kFxConsumers) {
+        // ------------------------------------------------------------ producer
+        uint64_t pol;
+        asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+        const uint32_t E = *n_items_ptr;
+        int stage = 0;
+        uint32_t phase = 0;
+        const uint4* raw = reinterpret_cast<const uint4*>(items);
+        // lane-parallel batch of 32 descriptors [bb, bb + 32), the next one prefetched
+        auto load = [&](uint32_t bb, uint4& a, uint4& b) {
+            const uint32_t i = bb + lane;
+            if (i < E) {
+                a = raw[2ull * i];
+                b = raw[2ull * i + 1];
+            } else {
+                a = make_uint4(0, 0, 0, 0);
+                b = make_uint4(0, 0, 0, 0);
+            }
+        };
+        uint32_t seg = 0;
+        if (lane == 0) seg = atomicAdd(&W.counters[8], 1u);
+        seg = __shfl_sync(0xFFFFFFFFu, seg, 0);
+        uint32_t lo = seg * kFxSeg;
+        uint32_t bb = lo;
+        uint4 ca, cb, na, nb;
+        load(bb, ca, cb);
+        load(bb + 32, na, nb);
+        uint32_t rem = 0;          // entries left in the current task
+        bool started = false;      // a task starting in this segment has been seen
+        while (lo < E) {
+            const uint32_t hi = min(E, lo + kFxSeg);
+            // walk descriptors from bb; stop after the last task that starts before hi
+            bool seg_done = false;
+            while (!seg_done) {
+#pragma unroll 1
+                for (int j = 0; j < 32; ++j) {
+                    const uint32_t e = bb + j;
+                    const uint32_t k = __shfl_sync(0xFFFFFFFFu, cb.z, j);
+                    if (rem == 0) {
+                        if (e >= hi || e >= E) {
+                            seg_done = true;
+                            break;
+                        }
+                        if (k == 0) {   // a member of a task that started in an earlier segment
+                            if (started) {
+                                seg_done = true;   // cannot happen: tasks are contiguous
+                                break;
+                            }
+                            continue;
+                        }
+                        rem = k;
+                        started = true;
+                    }
+                    --rem;
+                    const uint32_t s_lo = __shfl_sync(0xFFFFFFFFu, ca.x, j);
+                    const uint32_t s_hi = __shfl_sync(0xFFFFFFFFu, ca.y, j);
+                    const uint32_t rec = __shfl_sync(0xFFFFFFFFu, ca.z, j);
+                    const uint32_t lenf = __shfl_sync(0xFFFFFFFFu, ca.w, j);
+                    const uint32_t w0 = __shfl_sync(0xFFFFFFFFu, cb.x, j);
+                    const uint32_t slot = __shfl_sync(0xFFFFFFFFu, cb.y, j);
+                    if ((lenf >> 24) & kFxSkip) continue;
+                    if (lane == 0) {
+                        mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+                        FxDesc& m = meta[stage];
+                        m.rec = rec;
+                        m.lenf = lenf;
+                        m.w0 = w0;
+                        m.slot = slot;
+                        const uint32_t len = lenf & 0xFFFFFFu;
+                        const uint32_t bytes = (len + 15u) & ~15u;
+                        const uint32_t fb = smem_u32(&full[stage]);
+                        mbar_arrive_tx(fb, bytes);
+                        bulk_g2s(smem_u32(bufs + (size_t)stage * kFxPiece),
+                                 L.arena + (((uint64_t)s_hi << 32) | s_lo), bytes, fb, pol);
+                    }
+                    if (++stage == kFxStages) {
+                        stage = 0;
+                        phase ^= 1;
+                    }
+                }
+                if (seg_done) break;
+                bb += 32;
+                ca = na;
+                cb = nb;
+                load(bb + 32, na, nb);
+            }
+            // next segment
+            if (lane == 0) seg = atomicAdd(&W.counters[8], 1u);
+            seg = __shfl_sync(0xFFFFFFFFu, seg, 0);
+            lo = seg * kFxSeg;
+            rem = 0;
+            started = false;
+            if (lo >= E) break;
+            bb = lo;
+            load(bb, ca, cb);
+            load(bb + 32, na, nb);
+        }
+        if (lane == 0) {
+            mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+            meta[stage].lenf = kFxDone << 24;
+            mbar_arrive(smem_u32(&full[stage]));
+        }
+        return;
+    }
+
+    // ---------------------------------------------------------------- consumers
+    const int t = threadIdx.x;                 // 0 .. 32 * kFxConsumers - 1
+    const int g = t & 15;                      // NH position of every word this thread owns
+    uint32_t ka[6];
+#pragma unroll
+    for (int j = 0; j < 6; ++j) ka[j] = c_nh.ka[g][j];
+    uint4 x[kFxWords];                         // the current piece of the leader
+    uint64_t A = 0, B = 0;
+    uint32_t lslot = 0;
+    int stage = 0, rbuf = 0;
+    uint32_t phase = 0;
+    constexpr uint32_t kStride = 32 * kFxConsumers;   // words between a thread's words
+    for (;;) {
+        mbar_wait(smem_u32(&full[stage]), phase);
+        const uint32_t lenf = meta[stage].lenf;
+        const uint32_t flags = lenf >> 24;
+        if (flags & kFxDone) break;
+        const uint32_t w0 = meta[stage].w0, slot = meta[stage].slot, rec = meta[stage].rec;
+        const int32_t len = (int32_t)(lenf & 0xFFFFFFu);
+        const uint8_t* buf = bufs + (size_t)stage * kFxPiece;
+        if (flags & kFxLeader) {
+#pragma unroll
+            for (int u = 0; u < kFxWords; ++u) {
+                const int32_t vb = len - 16 * (int32_t)(t + kStride * u);
+                x[u] = vb > 0 ? *reinterpret_cast<const uint4*>(buf + 16 * (t + kStride * u)) : make_uint4(0, 0, 0, 0);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(smem_u32(&empty[stage]));
+#pragma unroll
+            for (int u = 0; u < kFxWords; ++u) mask_word(x[u], len - 16 * (int32_t)(t + kStride * u));
+            if (flags & kFxHash) {
+                lslot = slot;
+                uint32_t k[6];
+                word_keys(k, ka, (w0 + t) >> 4);
+#pragma unroll
+                for (int u = 0; u < kFxWords; ++u) {
+                    if (len > 16 * (int32_t)(t + kStride * u)) nh_word(x[u].x, x[u].y, x[u].z, x[u].w, k, A, B);
+#pragma unroll
+                    for (int j = 0; j < 6; ++j) k[j] += kDA(j) * (kStride / 16);
+                }
+            }
+        } else {
+            uint4 y[kFxWords];
+#pragma unroll
+            for (int u = 0; u < kFxWords; ++u) {
+                const int32_t vb = len - 16 * (int32_t)(t + kStride * u);
+                y[u] = vb > 0 ? *reinterpret_cast<const uint4*>(buf + 16 * (t + kStride * u)) : make_uint4(0, 0, 0, 0);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(smem_u32(&empty[stage]));
+            uint32_t dmask = 0;
+#pragma unroll
+            for (int u = 0; u < kFxWords; ++u) {
+                mask_word(y[u], len - 16 * (int32_t)(t + kStride * u));
+                if ((y[u].x ^ x[u].x) | (y[u].y ^ x[u].y) | (y[u].z ^ x[u].z) | (y[u].w ^ x[u].w)) dmask |= 1u << u;
+            }
+            if (__any_sync(0xFFFFFFFFu, dmask != 0)) {
+                // rare: a near-duplicate or a collision -- first mismatching word and NH deltas
+                uint64_t found = dmask ? (uint64_t)(w0 + t + kStride * (__ffs(dmask) - 1)) : ~0ull;
+                uint64_t dA = 0, dB = 0;
+                if ((flags & kFxDelta) && dmask) {
+                    uint64_t xA = 0, xB = 0;
+#pragma unroll
+                    for (int u = 0; u < kFxWords; ++u) {
+                        if (dmask & (1u << u)) {
+                            uint32_t k[6];
+                            word_keys(k, ka, (w0 + t + kStride * u) >> 4);
+                            nh_word(y[u].x, y[u].y, y[u].z, y[u].w, k, dA, dB);
+                            nh_word(x[u].x, x[u].y, x[u].z, x[u].w, k, xA, xB);
+                        }
+                    }
+                    dA -= xA;
+                    dB -= xB;
+                }
+#pragma unroll
+                for (int o = 16; o; o >>= 1) {
+                    const uint64_t of = __shfl_xor_sync(0xFFFFFFFFu, found, o);
+                    found = of < found ? of : found;
+                    dA += __shfl_xor_sync(0xFFFFFFFFu, dA, o);
+                    dB += __shfl_xor_sync(0xFFFFFFFFu, dB, o);
+                }
+                if (lane == 0) {
+                    report_mismatch(W, rec, found, res_out, true);
+                    if ((flags & kFxDelta) && (dA | dB)) {
+                        atomicAdd((unsigned long long*)&W.hpart[2ull * slot], (unsigned long long)dA);
+                        atomicAdd((unsigned long long*)&W.hpart[2ull * slot + 1], (unsigned long long)dB);
+                    }
+                }
+            }
+        }
+        if (flags & kFxReduce) {
+            // the leader's piece partial: CTA reduction over the consumer threads, added
+            // into the chunk slot (a chunk may span several pieces)
+#pragma unroll
+            for (int o = 16; o; o >>= 1) {
+                A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
+                B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
+            }
+            if (lane == 0) {
+                red[(rbuf * kFxConsumers + warp) * 2] = A;
+                red[(rbuf * kFxConsumers + warp) * 2 + 1] = B;
+            }
+            asm volatile("bar.sync 1, %0;" ::"n"(32 * kFxConsumers) : "memory");
+            if (t == 0) {
+                uint64_t sA = 0, sB = 0;
+#pragma unroll
+                for (int w = 0; w < kFxConsumers; ++w) {
+                    sA += red[(rbuf * kFxConsumers + w) * 2];
+                    sB += red[(rbuf * kFxConsumers + w) * 2 + 1];
+                }
+                atomicAdd((unsigned long long*)&W.hpart[2ull * lslot], (unsigned long long)sA);
+                atomicAdd((unsigned long long*)&W.hpart[2ull * lslot + 1], (unsigned long long)sB);
+            }
+            rbuf ^= 1;
+            A = B = 0;
+        }
+        if (++stage == kFxStages) {
+            stage = 0;
+            phase ^= 1;
+        }
+    }
+}
+
 // Combine the chunk partial sums of large records (NH is a plain sum, so the record's
 // accumulators are the sums of its chunks' -- no atomics, deterministic) and finish
 // their digests.  Also totals the bytes hashed beyond first chunks (roofline stats).
+// After the pipelined fused pass (fx) a member's chunks >= 1 are its head's partials
+// plus its own deltas.
 __global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes,
-                                                      int prefilter) {
-    __shared__ unsigned long long s_rest[8];
-    const int lane = threadIdx.x & 31;
-    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-    const bool act = i < L.n && L.size[i] > small_bytes;
-    unsigned bal = __ballot_sync(0xFFFFFFFFu, act);
+                                                      int prefilter, int fx) {
     unsigned long long rest = 0;
-    while (bal) {
-        const int src = __ffs(bal) - 1;
-        bal &= bal - 1;
-        const uint32_t rec = __shfl_sync(0xFFFFFFFFu, i, src);
+    FFM_WARP_EACH(L.n_large, L.large_order[w_], true, {
         const uint32_t s0 = W.hstart[rec];
         const bool skip = prefilter && prefix_unique(W, rec);
         const uint32_t e0 = skip ? s0 + 1 : W.hstart[rec + 1];
-        uint64_t A = 0, B = 0;
-        for (uint32_t it = s0 + lane; it < e0; it += 32) {
-            A += W.hpart[2ull * it];
-            B += W.hpart[2ull * it + 1];
+        const uint32_t h = fx ? W.fhead[rec] : rec;
+        const int64_t dh = (int64_t)W.hstart[h] - (int64_t)s0;   // head slot of the same chunk
+        uint64_t A0 = 0, B0 = 0, A1 = 0, B1 = 0;
+        uint32_t it = s0 + lane;
+        for (; it + 32 < e0; it += 64) {
+            A0 += W.hpart[2ull * it];
+            B0 += W.hpart[2ull * it + 1];
+            A1 += W.hpart[2ull * (it + 32)];
+            B1 += W.hpart[2ull * (it + 32) + 1];
+            if (h != rec) {   // member chunks >= 1: head's partial + own delta
+                if (it != s0) {
+                    A0 += W.hpart[2ull * (it + dh)];
+                    B0 += W.hpart[2ull * (it + dh) + 1];
+                }
+                A1 += W.hpart[2ull * (it + 32 + dh)];
+                B1 += W.hpart[2ull * (it + 32 + dh) + 1];
+            }
         }
+        if (it < e0) {
+            A0 += W.hpart[2ull * it];
+            B0 += W.hpart[2ull * it + 1];
+            if (h != rec && it != s0) {
+                A0 += W.hpart[2ull * (it + dh)];
+                B0 += W.hpart[2ull * (it + dh) + 1];
+            }
+        }
+        uint64_t A = A0 + A1, B = B0 + B1;
         for (int o = 16; o; o >>= 1) {
             A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
             B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
@@ -550,21 +1062,15 @@ __global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t
             W.digest[rec] = finalize_digest(A, B, n);
             if (!skip && n > chunk_bytes) rest += n - chunk_bytes;
         }
-    }
-    if (lane == 0) s_rest[threadIdx.x >> 5] = rest;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        unsigned long long t = 0;
-        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s_rest[w];
-        if (t) atomicAdd((unsigned long long*)(W.counters + 4), t);
-    }
+    })
+    if (rest) atomicAdd((unsigned long long*)(W.counters + 4), rest);
 }
 
 __global__ void k_verify_fill(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
                               uint32_t small_bytes, uint32_t chunk_bytes) {
-    FFM_WARP_COMPACT(n_list, list,
-                     (W.leader[r_] != r_ && L.size[r_] > small_bytes && L.size[W.leader[r_]] == L.size[r_] &&
-                      L.chan[W.leader[r_]] == L.chan[r_]), {
+    FFM_WARP_EACH(list ? n_list : L.n_large, list ? list[w_] : L.large_order[w_],
+                  (W.leader[rec] != rec && L.size[rec] > small_bytes && L.size[W.leader[rec]] == L.size[rec] &&
+                   L.chan[W.leader[rec]] == L.chan[rec]), {
         const uint32_t ld = W.leader[rec];
         const uint64_t n = L.size[rec];
         const uint32_t c_n = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
@@ -628,6 +1134,67 @@ __global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const
             }
         }
         if (word != ~0ull && g == 0) report_mismatch(W, m, word, res_out, false);
+    }
+}
+
+// H1 + H3 fused for small payloads (round 0): one 8-lane group per record, records in
+// size-class order.  Each group hashes its whole record (full digest: residuals and the
+// cross-shard / online merges need it) and, for a member of a prefix group, byte-compares
+// it with the group's leader -- re-uploads of one content share their leader, so its
+// bytes are L2-hot; the member's own bytes are read from HBM once.
+__global__ void __launch_bounds__(256, 3) k_fused_small(DevLog L, Work W, uint32_t* res_out) {
+    const int g = threadIdx.x & 7;
+    const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
+    const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
+    const unsigned omask = 0xFFu << (threadIdx.x & 24);
+    LaneKeys K0;
+    load_keys(K0, 2 * g, 0);
+    for (uint32_t i = oct; i < L.n_small; i += noct) {
+        const uint32_t r = L.small_order[i];
+        const uint64_t n = L.size[r];
+        const uint32_t ld = W.leader[r];
+        const uint8_t* base = L.arena + L.off[r];
+        const bool cmp = ld != r && L.size[ld] == n && L.chan[ld] == L.chan[r];
+        const uint8_t* lb = L.arena + L.off[ld];
+        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
+        LaneKeys K = K0;
+        uint64_t A = 0, B = 0, found = ~0ull;
+        for (uint32_t b0 = 0; b0 < nblk; b0 += 8 * kSmallU) {
+            Blk x[kSmallU], y[kSmallU];
+#pragma unroll
+            for (int u = 0; u < kSmallU; ++u) {
+                const uint32_t b = b0 + 8 * u + g;
+                x[u] = b < nblk ? ld_stream(base + 32ull * b) : zero_blk();
+                y[u] = (cmp && b < nblk) ? ld_keep(lb + 32ull * b) : zero_blk();
+            }
+#pragma unroll
+            for (int u = 0; u < kSmallU; ++u) {
+                const uint32_t b = b0 + 8 * u + g;
+                if (b < nblk) {
+                    mask_tail(x[u], n, b);
+                    nh_blk(x[u], K, n, b, A, B);
+                    if (cmp) {
+                        mask_tail(y[u], n, b);
+                        const int d = blk_diff(x[u], y[u]);
+                        if (d >= 0 && found == ~0ull) found = 2ull * b + d;
+                    }
+                }
+                advance<1>(K);
+            }
+        }
+#pragma unroll
+        for (int o = 4; o; o >>= 1) {
+            A += __shfl_xor_sync(omask, A, o);
+            B += __shfl_xor_sync(omask, B, o);
+            const uint64_t of = __shfl_xor_sync(omask, found, o);
+            found = of < found ? of : found;
+        }
+        if (g == 0) {
+            W.accA[r] = A;
+            W.accB[r] = B;
+            W.digest[r] = finalize_digest(A, B, n);
+            if (found != ~0ull) report_mismatch(W, r, found, res_out, false);
+        }
     }
 }
 
@@ -870,6 +1437,12 @@ uint32_t resident_grid(const void* kernel, int num_sms, int block) {
         if (cudaGetLastError() != cudaSuccess) return -1; \
     } while (0)
 
+// grid for one warp per item (FFM_WARP_EACH): at most one resident wave of 256-thread blocks
+static uint32_t warp_grid(uint64_t items, int num_sms) {
+    const uint64_t b = (items * 32 + 255) / 256, cap = (uint64_t)num_sms * 8;
+    return (uint32_t)(b == 0 ? 1 : (b < cap ? b : cap));
+}
+
 size_t cub_scan_bytes(uint64_t n) {
     size_t bytes = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, bytes, (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n);
@@ -886,6 +1459,15 @@ int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st
     return 1;
 }
 
+int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_out, cudaStream_t st) {
+    if (L.n == 0 || L.n_small == 0) return 0;
+    uint32_t grid = resident_grid((const void*)k_fused_small, P.num_sms);
+    uint32_t need = blocks_for((uint64_t)L.n_small * 8);
+    k_fused_small<<<need < grid ? need : grid, 256, 0, st>>>(L, W, res_out);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
 int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
     k_hash_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hcount);
     FFM_LAUNCH_CHECK();
@@ -893,7 +1475,7 @@ int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st)
     if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.hcount, W.hstart, (int)(L.n + 1), st) != cudaSuccess)
         return -1;
     if (L.n) {
-        k_hash_fill<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hstart,
+        k_hash_fill<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hstart,
                                                                     W.hitems);
         FFM_LAUNCH_CHECK();
     }
@@ -914,7 +1496,7 @@ int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_item
 // hash + compare pass, then the per-record combine of chunk partial sums.
 int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
     if (L.n == 0) return 0;
-    k_hash_combine<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 0);
+    k_hash_combine<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 0, 0);
     FFM_LAUNCH_CHECK();
     return 1;
 }
@@ -923,25 +1505,49 @@ int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bo
                  cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b) {
     if (L.n == 0 || n_units == 0) return 0;
     int k = 0;
+    const bool fx = P.fused_impl == 0 && smem_configured((const void*)k_fused_fx, (int)kFxSmem);
+    if (fx) {
+        // entries per head (pieces x (members + sub-task leader copies)), then their scan
+        k_fx_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 0);
+        FFM_LAUNCH_CHECK();
+        ++k;
+    }
     size_t bytes = W.cub_tmp_bytes;
     if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.lcount, W.lstart, (int)(L.n + 1), st) != cudaSuccess)
         return -1;
     ++k;
-    k_fused_fill<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes);
+    if (fx) {
+        k_fx_fill<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, prefilter ? 1 : 0,
+                                                              reinterpret_cast<FxDesc*>(W.fitems));
+    } else {
+        k_fused_fill<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes);
+    }
     FFM_LAUNCH_CHECK();
     ++k;
     if (ev_a && cudaEventRecord(ev_a, st) != cudaSuccess) return -1;
-    uint32_t grid = resident_grid((const void*)k_fused, P.num_sms);
-    uint32_t need = blocks_for(n_units * 32);
-    k_fused<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.lstart + L.n, P.chunk_bytes, prefilter ? 1 : 0,
-                                                       res_out);
+    if (fx) {
+        k_fused_fx<<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
+            L, W, reinterpret_cast<const FxDesc*>(W.fitems), W.lstart + L.n, res_out);
+    } else {
+        uint32_t grid = resident_grid((const void*)k_fused, P.num_sms);
+        uint32_t need = blocks_for(n_units * 32);
+        k_fused<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.lstart + L.n, P.chunk_bytes, prefilter ? 1 : 0,
+                                                           res_out);
+    }
     FFM_LAUNCH_CHECK();
     ++k;
     if (ev_b && cudaEventRecord(ev_b, st) != cudaSuccess) return -1;
-    k_hash_combine<<<blocks_for((uint64_t)L.n), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes,
-                                                              prefilter ? 1 : 0);
+    k_hash_combine<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes,
+                                                              prefilter ? 1 : 0, fx ? 1 : 0);
     FFM_LAUNCH_CHECK();
     return k + 1;
+}
+
+// Capacity (entries) the pipelined fused pass may need beyond the chunk count: pieces
+// smaller than chunks and one leader copy per extra sub-task (host-side bound).
+uint64_t fx_entry_cap(uint64_t n_large_chunks, uint32_t chunk_bytes) {
+    const FxSplit f = fx_split(chunk_bytes);
+    return n_large_chunks * (uint64_t)f.ppc + (n_large_chunks * (uint64_t)f.ppc) / (kFxMaxK - 1) + 64;
 }
 
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list, uint64_t cap,
@@ -994,21 +1600,41 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
         ++k;
     }
     if (vitem_cap) {
-        // large members: chunk-major groups per leader (scan of lcount) then scatter work units
+        // large members: groups per leader (scan of per-leader entry counts), then the
+        // verify work -- the pipelined pass (leader piece in registers, members compared
+        // against it) or the chunk-major L2 kernel
+        const bool fx = P.fused_impl == 0 && smem_configured((const void*)k_fused_fx, (int)kFxSmem);
+        if (fx) {
+            k_fx_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 1);
+            FFM_LAUNCH_CHECK();
+            ++k;
+        }
         size_t bytes = W.cub_tmp_bytes;
         if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.lcount, W.lstart, (int)(L.n + 1), st) != cudaSuccess)
             return -1;
         ++k;
         uint32_t* n_vitems = W.lstart + L.n;   // total large verify work units
-        k_verify_fill<<<blocks_for((uint64_t)n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes,
-                                                                    P.chunk_bytes);
-        FFM_LAUNCH_CHECK();
-        ++k;
-        uint32_t grid = resident_grid((const void*)k_verify_large, P.num_sms);
-        need = blocks_for(vitem_cap * 32);
-        k_verify_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.vitems, n_vitems, P.chunk_bytes, res_out);
-        FFM_LAUNCH_CHECK();
-        ++k;
+        if (fx) {
+            k_fx_vfill<<<warp_grid(list ? n_list : L.n_large, P.num_sms), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes,
+                                                                     reinterpret_cast<FxDesc*>(W.fitems));
+            FFM_LAUNCH_CHECK();
+            ++k;
+            k_fused_fx<<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
+                L, W, reinterpret_cast<const FxDesc*>(W.fitems), n_vitems, res_out);
+            FFM_LAUNCH_CHECK();
+            ++k;
+        } else {
+            k_verify_fill<<<warp_grid(list ? n_list : L.n_large, P.num_sms), 256, 0, st>>>(L, W, list, n_list, P.small_bytes,
+                                                                        P.chunk_bytes);
+            FFM_LAUNCH_CHECK();
+            ++k;
+            uint32_t grid = resident_grid((const void*)k_verify_large, P.num_sms);
+            need = blocks_for(vitem_cap * 32);
+            k_verify_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.vitems, n_vitems, P.chunk_bytes,
+                                                                      res_out);
+            FFM_LAUNCH_CHECK();
+            ++k;
+        }
     }
     if (side) {
         if (cudaEventRecord(ev_join, side) != cudaSuccess || cudaStreamWaitEvent(st, ev_join, 0) != cudaSuccess)

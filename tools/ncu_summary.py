@@ -1,9 +1,10 @@
 #!/usr/bin/env python3
 """Summarise ncu output into profiles/: launch list shares + per-kernel full-set metrics.
 
-usage: ncu_summary.py <launches.csv> <prof.ncu-rep> <out_prefix>
-Writes <out_prefix>_launches.md, <out_prefix>_kernels.md and profiles/ncu_summary.json
-(dram bytes per launch per kernel; bench.py reads it for roofline.traffic).
+usage: ncu_summary.py <launches.csv> <prof.ncu-rep> <out_prefix> <capture key, e.g. config5/fused>
+Writes <out_prefix>_launches.md, <out_prefix>_kernels.md and merges the capture into
+profiles/ncu_summary.json under "captures"/<key> (dram bytes per launch per kernel;
+bench.py reads the capture of its own workload and round-0 mode for roofline.traffic).
 """
 import csv
 import io
@@ -59,7 +60,7 @@ def full(rep):
 
 
 def main():
-    lpath, rep, prefix = sys.argv[1:4]
+    lpath, rep, prefix, key = sys.argv[1:5]
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     agg = launches(lpath)
     tot = sum(sum(v) for v in agg.values())
@@ -85,8 +86,15 @@ def main():
                                       "source": os.path.basename(rep)}
     open(prefix + "_kernels.md", "w").write(
         f"# ncu --set full ({os.path.basename(rep)}; last captured launch per kernel)\n\n" + "\n".join(lines) + "\n")
-    json.dump({"kernels": summ, "note": "ncu --set full --clock-control none; per launch"},
-              open(os.path.join(root, "profiles", "ncu_summary.json"), "w"), indent=1)
+    jpath = os.path.join(root, "profiles", "ncu_summary.json")
+    try:
+        doc = json.load(open(jpath))
+    except Exception:
+        doc = {}
+    caps = doc.get("captures", {})
+    caps[key] = {"kernels": summ}
+    json.dump({"captures": caps, "note": "ncu --set full --clock-control none; per launch; key = config<k>/<round-0 mode>"},
+              open(jpath, "w"), indent=1)
     print(open(prefix + "_launches.md").read())
     print(open(prefix + "_kernels.md").read())
 
