@@ -131,12 +131,13 @@ def make_log(workload, n_scale, size_scale, shard=(0, 1)):
     return lg
 
 
-def alg_bytes(lg, idx, dup, small_bytes, chunk=32768, two_pass=False):
+def alg_bytes(lg, idx, dup, small_bytes, chunk=32768, two_pass=False, prefix=4096):
     """Algorithmic bytes per kernel for this rank's records idx: every
     payload byte is hashed once; a member payload's bytes are compared once against its
     leader, whose bytes are read once per class.
-      prefix (k_hash_large, first chunks):  sum over large payloads of c0 = min(size, chunk)
-      fused  (k_fused_fx):  sum over large (size - c0) + members' c0 + their leaders' c0
+      prefix (k_prefix_hash):  sum over large payloads of p0 = min(size, prefix)
+      fused  (k_fused_fx):  sum over large (size - p0) + members' p0 + their leaders' p0
+                            (a group's first pieces are compared from byte 0)
       small  (k_fused_small): small sizes + leaders of small members
     two-pass: k_hash_large hashes every large byte, then members and their class leaders
     are read once more (verify); small: k_hash_small, then k_verify_small (side stream,
@@ -153,12 +154,12 @@ def alg_bytes(lg, idx, dup, small_bytes, chunk=32768, two_pass=False):
         lp = pos[dup[member]]
         leaders[lp[lp >= 0]] = True
     big = ~small
-    c0 = np.minimum(size, chunk)
+    p0 = np.minimum(size, prefix)
     units = int(((size[big] + chunk - 1) // chunk).sum())
     out = {
         "small": int(size[small].sum()) + int(size[small & leaders].sum()) + 40 * int(small.sum()),
-        "prefix": int(c0[big].sum()) + 40 * int(big.sum()),
-        "fused": int((size[big] - c0[big]).sum()) + int(c0[big & member].sum()) + int(c0[big & leaders].sum())
+        "prefix": int(p0[big].sum()) + 40 * int(big.sum()),
+        "fused": int((size[big] - p0[big]).sum()) + int(p0[big & member].sum()) + int(p0[big & leaders].sum())
         + 32 * units,
     }
     if two_pass:
@@ -284,8 +285,8 @@ def run_ours(args):
         sz = lg.size[idx].astype(np.int64)
         big = sz > 4096
         mem = dup_h >= 0
-        c0 = np.minimum(sz, 32768)
-        ab["fused"] = int(st["prefilter_rest_bytes"]) + int(c0[big & mem].sum()) + 40 * int(((sz[big] + 32767) // 32768).sum())
+        p0 = np.minimum(sz, 4096)
+        ab["fused"] = int(st["prefilter_rest_bytes"]) + int(p0[big & mem].sum()) + 32 * int(((sz[big] + 32767) // 32768).sum())
         ab["path"] = sum(v for k, v in ab.items() if k != "path") + 64 * len(idx)
     peak, peak_src = load_peak()
     kern_ms = {"small": st["ms_hash_small"], "prefix": st["ms_hash_large"], "fused": st["ms_fused"]}
@@ -293,10 +294,11 @@ def run_ours(args):
     dom_ms = kern_ms[dom]
     achieved = ab[dom] / (dom_ms * 1e-3) / 1e9 if dom_ms > 0 else 0.0
     two_pass = args.two_pass or st.get("two_pass", 0) >= 0.5
-    fused_k = "k_fused" if os.environ.get("FFM_FUSED_IMPL", "0") == "1" else "k_fused_fx"
-    kname = {"small": "k_hash_small" if two_pass else "k_fused_small", "prefix": "k_hash_large",
-             "fused": "k_verify_large" if two_pass else fused_k}[dom]
-    mode = "two-pass" if two_pass else ("fused" if fused_k == "k_fused_fx" else "fused-l2")
+    fused_k = "k_fused_fx"
+    kname = {"small": "k_hash_small" if two_pass else "k_fused_small",
+             "prefix": "k_hash_large" if two_pass else "k_prefix_hash",
+             "fused": fused_k}[dom]
+    mode = "two-pass" if two_pass else "fused"
     capture = f"config{args.workload}/{mode}" + ("/prefilter" if args.prefilter else "") + \
         (f"/digest_bits{args.digest_bits}" if args.digest_bits < 64 else "")
     traffic = ncu_traffic(kname, capture) if world == 1 and args.n_scale == 1 and args.size_scale == 1 else None

@@ -153,6 +153,16 @@ bool is_device_ptr(const void* p) {
 // then the large ones in index order (one warp per large record in the planning
 // kernels).  Returns the number of small records.
 uint64_t build_small_order(const ffm_log* L, uint64_t begin, uint64_t end, std::vector<uint32_t>& order) {
+    static const bool gid_order = getenv("FFM_SMALL_GID_ORDER") != nullptr;   // A/B knob (same results)
+    if (gid_order) {
+        order.clear();
+        for (uint64_t i = begin; i < end; ++i)
+            if (L->h_size[i] <= L->params.small_bytes) order.push_back((uint32_t)(i - begin));
+        const uint64_t ns = order.size();
+        for (uint64_t i = begin; i < end; ++i)
+            if (L->h_size[i] > L->params.small_bytes) order.push_back((uint32_t)(i - begin));
+        return ns;
+    }
     const uint32_t nb = (L->params.small_bytes + 31) / 32 + 1;
     std::vector<uint32_t> start(nb + 1, 0);
     uint64_t ns = 0;
@@ -309,6 +319,7 @@ void ensure_work(ffm_log* L, uint64_t n) {
         dev_alloc(W.gcount, c + 1);
         dev_alloc(W.pos, c);
         dev_alloc(W.fhead, c);
+        dev_alloc(W.sdesc, 2 * c);
         dev_alloc(W.hcount, c + 1);
         dev_alloc(W.hstart, c + 1);
         dev_alloc(W.dup, c);
@@ -330,9 +341,8 @@ void ensure_work(ffm_log* L, uint64_t n) {
         ++L->epoch;
         uint64_t c = L->n_large_chunks + L->n_large_chunks / 4 + 64;
         dev_alloc(W.hitems, c);
-        dev_alloc(W.vitems, c);
         dev_alloc(W.hpart, 2 * c);
-        W.hitem_cap = W.vitem_cap = c;
+        W.hitem_cap = W.vitem_cap = c;   // vitem_cap: non-zero enables the large verify
     }
     const uint64_t fcap = fx_entry_cap(L->n_large_chunks, L->params.chunk_bytes);
     if (fcap > W.fitem_cap) {
@@ -431,10 +441,11 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
             ck(cudaEventRecord(L->fork_ev[1], side), "event");
         }
         if (n_large) {
-            LCHK(launch_hash_plan(D, W, L->params, s));
+            LCHK(launch_hash_plan(D, W, L->params, two_pass, s));
             if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
-            // fused: the prefix pass (first chunks); two-pass: every chunk, then the combine
-            LCHK(launch_hash_large(D, W, L->params, n_large, s, two_pass ? 0 : 1));
+            // fused: the prefix pass (first prefix_bytes); two-pass: every chunk, then the combine
+            if (two_pass) LCHK(launch_hash_large(D, W, L->params, n_large, s));
+            else LCHK(launch_prefix(D, W, L->params, s));
             if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
             if (two_pass) LCHK(launch_combine(D, W, L->params, s));
         }
@@ -708,8 +719,11 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
         L->host_ptr_ok = hp != 0;
         L->gather_max = kGatherMaxDefault;
         if (const char* e = getenv("FFM_GATHER_MAX")) L->gather_max = strtoull(e, nullptr, 10);   // tuning knob
-        L->params.fused_impl = 0;
-        if (const char* e = getenv("FFM_FUSED_IMPL")) L->params.fused_impl = atoi(e);   // A/B knob (same results)
+        L->params.prefix_bytes = std::min<uint32_t>(4096, chunk);   // a multiple of 256 (chunk: of 1024)
+        if (const char* e = getenv("FFM_PREFIX_BYTES")) {                // tuning knob (same results)
+            const uint32_t v = (uint32_t)strtoul(e, nullptr, 10);
+            if (v >= 256 && v % 256 == 0) L->params.prefix_bytes = std::min(v, chunk);
+        }
         L->params.chunk_bytes = chunk;
         L->params.small_bytes = small;
         L->params.digest_mask = cfg->digest_bits >= 64 ? ~0ull : ((1ull << cfg->digest_bits) - 1);
@@ -1268,7 +1282,7 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->stage_stream) cudaStreamSynchronize(L->stage_stream);
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
-                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.vitems, W.fitems, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
+                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.fitems, W.sdesc, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
                     W.dup, W.ben, W.cnt, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
                     L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)

@@ -48,7 +48,7 @@ struct Work {
     uint32_t* pos = nullptr;       // [n] position of a large record within its fused / verify group
     uint32_t* fhead = nullptr;     // [n] round 0: head (leader) of a large record's fused group
     uint2* hitems = nullptr;       // large-payload hash work units (record, chunk)
-    uint2* vitems = nullptr;       // large-payload verify work units (member, chunk)
+    uint4* sdesc = nullptr;        // [2 * n] fused round 0: compare descriptors of small records (order position)
     uint4* fitems = nullptr;       // pipelined fused pass stage descriptors (2 x uint4 each)
     uint32_t* hcount = nullptr;    // [n+1] per-record hash chunk counts
     uint32_t* hstart = nullptr;    // [n+1] exclusive scan of hcount
@@ -109,15 +109,16 @@ struct Params {
     uint32_t small_bytes;
     int num_sms;
     int max_smem;      // opt-in dynamic shared memory per block (bytes)
-    int fused_impl;    // round-0 fused pass: 0 = pipelined (k_fused_fx), 1 = L2 leader-first (k_fused)
+    uint32_t prefix_bytes;  // fused round 0: large payloads are grouped by the NH of their first prefix_bytes
 };
 
 // ---- kernel launchers (kernels.cu).  All asynchronous on `st`; each returns the
 // number of kernels it launched (for the launch count), or -1 on launch error.
 int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_out, cudaStream_t st);
-int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
-int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st, int phase = 0);
+int launch_hash_plan(const DevLog& L, Work& W, const Params& P, bool units, cudaStream_t st);
+int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st);
+int launch_prefix(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
                  cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b);

@@ -19,27 +19,6 @@
 #include "ffm_internal.h"
 #include "digest.cuh"
 
-// Tuning knobs of the fused pass; defaults are the measured best on B200 (config 5 / 4,
-// profiles/r01_fused_variants.md): leader-first layout, members' compare loads
-// L2::evict_last, everyone's own loads L2::evict_first (evict_last or normal priority on
-// the leaders' own loads measured 12-13% slower), 2 loads in flight per lane when
-// comparing, 3 CTAs/SM.
-#ifndef FFM_FUSED_CMP_U
-#define FFM_FUSED_CMP_U 2
-#endif
-#ifndef FFM_FUSED_LEADER_FIRST
-#define FFM_FUSED_LEADER_FIRST 1
-#endif
-#ifndef FFM_FUSED_KEEP_OWN
-#define FFM_FUSED_KEEP_OWN 0
-#endif
-#ifndef FFM_FUSED_SKEW
-#define FFM_FUSED_SKEW 0x7FFFFFFF   /* measured: leader-first (no skew) is best */
-#endif
-#ifndef FFM_FUSED_Y_POLICY
-#define FFM_FUSED_Y_POLICY 1
-#endif
-
 namespace ffm {
 
 // ----------------------------------------------------------------------------
@@ -193,10 +172,10 @@ __global__ void __launch_bounds__(256, 4) k_hash_small(DevLog L, uint32_t small_
 // ----------------------------------------------------------------------------
 constexpr int kLargeU = 4;
 
-// phase 0: every unit; phase 1: first chunks only (the prefix pass of round 0).
+// (two-pass round 0: every chunk of every large payload)
 __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __restrict__ items,
                                                     const uint32_t* __restrict__ n_items_ptr, uint32_t chunk_bytes,
-                                                    uint64_t* __restrict__ part, int phase) {
+                                                    uint64_t* __restrict__ part) {
     const int lane = threadIdx.x & 31;
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
@@ -205,7 +184,6 @@ __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __
     for (uint32_t it = warp; it < n_items; it += nwarps) {
         const uint2 w = items[it];
         const uint32_t r = w.x;
-        if (phase == 1 && w.y != 0) continue;
         const uint64_t n = L.size[r];
         const uint8_t* base = L.arena + L.off[r];
         const uint32_t nblk = (uint32_t)((n + 31) >> 5);
@@ -241,6 +219,45 @@ __global__ void __launch_bounds__(256, 3) k_hash_large(DevLog L, const uint2* __
             part[2ull * it + 1] = B;
         }
     }
+}
+
+// Fused round 0, prefix pass: one warp per large payload hashes its first
+// prefix_bytes into accA / accB (the group key of H2; k_hash_combine adds the rest).
+__global__ void __launch_bounds__(256) k_prefix_hash(DevLog L, Work W, uint32_t prefix_bytes) {
+    FFM_WARP_EACH(L.n_large, L.large_order[w_], true, {
+        const uint64_t n = L.size[rec];
+        const uint8_t* base = L.arena + L.off[rec];
+        const uint32_t be = (uint32_t)((min(n, (uint64_t)prefix_bytes) + 31) >> 5);
+        LaneKeys K;
+        load_keys(K, 2 * (lane & 7), (uint32_t)lane >> 3);
+        uint64_t A = 0, B = 0;
+        for (uint32_t b0 = 0; b0 < be; b0 += 32 * kLargeU) {
+            Blk x[kLargeU];
+_Pragma("unroll")
+            for (int u = 0; u < kLargeU; ++u) {
+                const uint32_t b = b0 + 32 * u + lane;
+                x[u] = b < be ? ld_stream(base + 32ull * b) : zero_blk();
+            }
+_Pragma("unroll")
+            for (int u = 0; u < kLargeU; ++u) {
+                const uint32_t b = b0 + 32 * u + lane;
+                if (b < be) {
+                    mask_tail(x[u], n, b);
+                    nh_blk(x[u], K, n, b, A, B);
+                }
+                advance<4>(K);
+            }
+        }
+_Pragma("unroll")
+        for (int o = 16; o; o >>= 1) {
+            A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
+            B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
+        }
+        if (lane == 0) {
+            W.accA[rec] = A;
+            W.accB[rec] = B;
+        }
+    })
 }
 
 // Work-unit planning for H1b / H3b: counts -> exclusive scan -> scatter.
@@ -295,10 +312,9 @@ __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ li
             for (int i = 0; i < 8; i += 2) pd = fmix64(pd ^ ((uint64_t)x.v[i + 1] << 32 | x.v[i]));
             key = group_key(pd, n, digest_mask, L.chan[r]);
         } else {
-            // large payload: the digest of its FIRST chunk (computed by the prefix pass);
-            // equal payloads have equal first chunks, so every candidate still shares a group
-            const uint32_t it = W.hstart[r];
-            uint64_t pd = finalize_digest(W.hpart[2ull * it], W.hpart[2ull * it + 1], n);
+            // large payload: the NH of its first prefix_bytes (the prefix pass); equal
+            // payloads have equal prefixes, so every candidate still shares a group
+            uint64_t pd = finalize_digest(W.accA[r], W.accB[r], n);
             key = group_key(pd, n, digest_mask, L.chan[r]);
         }
         W.key[r] = key;
@@ -356,11 +372,13 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
 // out chunk-major, (chunk c, position p) at lstart[head] + c * (gcount[head] + 1) + p,
 // with the leader itself at p = 0 -- the leader's chunk c is read from HBM once, by
 // its own hashing unit, and re-read from L2 by every member comparing against it.
-__global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, uint32_t chunk_bytes,
-                          uint32_t* __restrict__ res_out) {
-    uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, uint32_t* __restrict__ res_out) {
+    // thread i: record order[i] (small records in size-class order, then large ones), so
+    // a small record's compare descriptor lands at its position in k_fused_small's order
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     bool member = false;
-    if (r < n) {
+    if (i < n) {
+        const uint32_t r = L.small_order[i];
         const uint32_t ld = W.tval[W.slot[r]];
         W.leader[r] = ld;
         const uint64_t sz = L.size[r];
@@ -384,39 +402,14 @@ __global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, ui
             }
             W.fhead[r] = head;
             W.pos[r] = p;
-            atomicAdd(&W.lcount[head], (uint32_t)((sz + chunk_bytes - 1) / chunk_bytes));
+        } else {
+            const uint64_t off = L.off[r], loff = (ld != r && same) ? L.off[ld] : ~0ull;
+            W.sdesc[2ull * i] = make_uint4((uint32_t)off, (uint32_t)(off >> 32), (uint32_t)loff, (uint32_t)(loff >> 32));
+            W.sdesc[2ull * i + 1] = make_uint4((uint32_t)sz, r, 0, 0);
         }
     }
     unsigned b = __ballot_sync(0xFFFFFFFFu, member);
     if ((threadIdx.x & 31) == 0 && b) atomicAdd(&W.counters[1], (uint32_t)__popc(b));
-}
-
-__global__ void k_fused_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes) {
-    FFM_WARP_EACH(L.n_large, L.large_order[w_], true, {
-        const uint32_t h = W.fhead[rec];
-        const uint32_t k = W.gcount[h] + 1, p = W.pos[rec], base = W.lstart[h];
-        const uint32_t c_n = (uint32_t)((L.size[rec] + chunk_bytes - 1) / chunk_bytes);
-#if FFM_FUSED_LEADER_FIRST
-        // skewed chunk-major layout: the leader runs D chunks ahead of its members, so a
-        // member compares against a leader chunk fetched a little earlier -- an L2 hit,
-        // not a wait on the same in-flight miss, and not yet evicted.  Step t holds the
-        // leader's chunk t and the members' chunk t - D; no holes:
-        //   [0, D) leader only | [D, nch) leader + members | [nch, nch + D) members only
-        const uint32_t D = min((uint32_t)FFM_FUSED_SKEW, c_n);
-        for (uint32_t c = lane; c < c_n; c += 32) {
-            uint32_t at;
-            if (p == 0) {
-                at = c < D ? c : D + (c - D) * k;
-            } else {
-                const uint32_t t = c + D;
-                at = t < c_n ? D + c * k + p : D + (c_n - D) * k + (t - c_n) * (k - 1) + (p - 1);
-            }
-            W.vitems[base + at] = make_uint2(rec, c);
-        }
-#else
-        for (uint32_t c = lane; c < c_n; c += 32) W.vitems[base + c * k + p] = make_uint2(rec, c);
-#endif
-    })
 }
 
 // With FFM_FLAG_PREFILTER a leader whose fused group has no member has a unique
@@ -424,106 +417,6 @@ __global__ void k_fused_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t ch
 // chunks are not read.
 __device__ __forceinline__ bool prefix_unique(const Work& W, uint32_t r) {
     return W.fhead[r] == r && W.gcount[r] == 0 && W.leader[r] == r;
-}
-
-// H1 + H3 fused for large payloads (round 0): one pass over every chunk c >= 1 hashes
-// it (chunk 0 was hashed by the prefix pass) and, for a member, byte-compares it with
-// the leader's chunk c (L2-resident: the group's units run back to back); members
-// also compare chunk 0.  A member's first mismatching word is the exact minimum (a
-// chunk's compare is skipped only when a lower mismatch is known); failures go to the
-// residual list and are resolved exactly (H4) with their full digests.
-template <int U, bool kCmp>
-__device__ __forceinline__ void fused_chunk(const uint8_t* pr, const uint8_t* ph, uint64_t n, uint32_t bb,
-                                            uint32_t be, int lane, bool hashc, bool keep_own, LaneKeys& K,
-                                            uint64_t& A, uint64_t& B, uint64_t& found) {
-    for (uint32_t b0 = bb; b0 < be; b0 += 32 * U) {
-        Blk x[U], y[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const uint32_t b = b0 + 32 * u + lane;
-            // a group leader's own chunk is re-read by its members: keep it in L2
-            x[u] = b < be ? (keep_own ? ld_keep(pr + 32ull * b) : ld_stream(pr + 32ull * b)) : zero_blk();
-#if FFM_FUSED_Y_POLICY == 0
-            if (kCmp) y[u] = b < be ? ld_remote(ph + 32ull * b) : zero_blk();   // default L2 policy
-#elif FFM_FUSED_Y_POLICY == 2
-            if (kCmp) y[u] = b < be ? ld_stream(ph + 32ull * b) : zero_blk();
-#else
-            if (kCmp) y[u] = b < be ? ld_keep(ph + 32ull * b) : zero_blk();
-#endif
-        }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const uint32_t b = b0 + 32 * u + lane;
-            if (b < be) {
-                mask_tail(x[u], n, b);
-                if (hashc) nh_blk(x[u], K, n, b, A, B);
-                if (kCmp) {
-                    mask_tail(y[u], n, b);
-                    int d = blk_diff(x[u], y[u]);
-                    if (d >= 0 && found == ~0ull) found = 2ull * b + d;
-                }
-            }
-            advance<4>(K);
-        }
-    }
-}
-
-#ifndef FFM_FUSED_MINB
-#define FFM_FUSED_MINB 3
-#endif
-__global__ void __launch_bounds__(256, FFM_FUSED_MINB) k_fused(DevLog L, Work W, const uint32_t* __restrict__ n_items_ptr,
-                                                  uint32_t chunk_bytes, int prefilter, uint32_t* res_out) {
-    const int lane = threadIdx.x & 31;
-    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
-    const uint32_t n_items = *n_items_ptr;
-    const uint32_t cblk = chunk_bytes >> 5;
-    for (uint32_t it = warp; it < n_items; it += nwarps) {
-        const uint2 w = W.vitems[it];
-        const uint32_t r = w.x, c = w.y;
-        const uint32_t h = W.fhead[r];
-        const bool hashc = c > 0 && !(prefilter && prefix_unique(W, r));
-        bool cmp = h != r;
-        if (cmp) {
-            uint64_t known = lane == 0 ? *((volatile uint64_t*)&W.mis[r]) : 0;
-            known = __shfl_sync(0xFFFFFFFFu, known, 0);
-            cmp = 2ull * c * cblk < known;         // no lower mismatch known yet
-        }
-        if (!hashc && !cmp) continue;
-        const uint64_t n = L.size[r];
-        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
-        const uint32_t bb = c * cblk, be = min(bb + cblk, nblk);
-        const uint8_t* pr = L.arena + L.off[r];
-        const uint8_t* ph = L.arena + L.off[h];
-        const bool keep_own = FFM_FUSED_KEEP_OWN && h == r && W.gcount[r] > 0;
-        LaneKeys K;
-        load_keys(K, 2 * (lane & 7), (bb + lane) >> 3);
-        uint64_t A = 0, B = 0, found = ~0ull;
-        if (cmp)
-            fused_chunk<FFM_FUSED_CMP_U, true>(pr, ph, n, bb, be, lane, hashc, keep_own, K, A, B, found);
-        else
-            fused_chunk<4, false>(pr, ph, n, bb, be, lane, hashc, keep_own, K, A, B, found);
-        if (hashc) {
-#pragma unroll
-            for (int o = 16; o; o >>= 1) {
-                A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
-                B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
-            }
-            if (lane == 0) {
-                const uint64_t slot = W.hstart[r] + c;
-                W.hpart[2 * slot] = A;
-                W.hpart[2 * slot + 1] = B;
-            }
-        }
-        if (cmp && __any_sync(0xFFFFFFFFu, found != ~0ull)) {
-#pragma unroll
-            for (int o = 16; o; o >>= 1) {
-                uint64_t other = __shfl_xor_sync(0xFFFFFFFFu, found, o);
-                found = other < found ? other : found;
-            }
-            if (lane == 0) report_mismatch(W, r, found, res_out, true);
-        }
-    }
 }
 
 // ----------------------------------------------------------------------------
@@ -559,6 +452,12 @@ __global__ void __launch_bounds__(256, FFM_FUSED_MINB) k_fused(DevLog L, Work W,
 #endif
 #ifndef FFM_FX_CTAS
 #define FFM_FX_CTAS 2
+#endif
+#ifndef FFM_FX_MINB          // __launch_bounds__ min blocks (register budget)
+#define FFM_FX_MINB FFM_FX_CTAS
+#endif
+#ifndef FFM_SMALL_OWN_EVICT_FIRST  // k_fused_small: own bytes evict_first (1) or normal L2 policy (0)
+#define FFM_SMALL_OWN_EVICT_FIRST 1
 #endif
 constexpr int kFxConsumers = 8;                       // consumer warps
 constexpr int kFxThreads = 32 * (kFxConsumers + 1);   // + one producer warp
@@ -712,9 +611,11 @@ __global__ void k_fx_vfill(DevLog L, Work W, const uint32_t* __restrict__ list, 
     })
 }
 
-// One descriptor per (record, piece, sub-task copy); also zeroes the chunk slots (>= 1)
-// the pass accumulates into.
-__global__ void k_fx_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes, int prefilter,
+// One descriptor per (record, piece, sub-task copy); also zeroes the chunk slots the
+// pass accumulates into.  The first prefix_bytes of every record were hashed by the
+// prefix pass: a group's pieces still cover them (the members' compares), a
+// singleton's first piece starts after them.
+__global__ void k_fx_fill(DevLog L, Work W, uint32_t chunk_bytes, uint32_t prefix_bytes, int prefilter,
                           FxDesc* __restrict__ items) {
     if (blockIdx.x == 0 && threadIdx.x == 0) W.counters[8] = 0;   // segment scheduler
     const FxSplit f = fx_split(chunk_bytes);
@@ -728,8 +629,14 @@ __global__ void k_fx_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk
         const uint32_t last0 = min(k - 1, kFxMaxK - 1);      // position ending sub-task 0
         for (uint32_t t = lane; t < np; t += 32) {
             const uint32_t c = t / f.ppc, j = t - c * f.ppc;
-            const uint64_t st = (uint64_t)c * f.chunk + (uint64_t)j * f.ps;
+            uint64_t st = (uint64_t)c * f.chunk + (uint64_t)j * f.ps;
             const uint64_t en = min(min(st + f.ps, (uint64_t)(c + 1) * f.chunk), n);
+            const bool hashes = en > prefix_bytes;             // has words beyond the prefix
+            bool skip = skip_all;
+            if (k == 1 && st < prefix_bytes) {                 // singleton: skip the prefix
+                if (!hashes) skip = true;
+                else st = prefix_bytes;
+            }
             FxDesc d;
             d.src = off + st;
             d.rec = rec;
@@ -740,22 +647,22 @@ __global__ void k_fx_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk
             if (p == 0) {
                 for (uint32_t q = 0; q < S; ++q) {
                     uint32_t fl = kFxLeader;
-                    if (q == 0 && c > 0) fl |= kFxHash;
-                    if ((k == 1 && c == 0) || skip_all) fl |= kFxSkip;
-                    if (q == 0 && last0 == 0 && c > 0) fl |= kFxReduce;
+                    if (q == 0 && hashes) fl |= kFxHash;
+                    if (skip) fl |= kFxSkip;
+                    if (q == 0 && last0 == 0 && hashes) fl |= kFxReduce;
                     d.lenf = (uint32_t)(en - st) | (fl << 24);
                     d.k = q + 1 < S ? kFxMaxK : k - q * (kFxMaxK - 1);
                     items[pb + (uint64_t)q * kFxMaxK] = d;
                 }
             } else {
                 const uint32_t q = (p - 1) / (kFxMaxK - 1), i = (p - 1) - q * (kFxMaxK - 1) + 1;
-                uint32_t fl = c > 0 ? kFxDelta : 0u;
-                if (p == last0 && c > 0) fl |= kFxReduce;
+                uint32_t fl = hashes ? kFxDelta : 0u;
+                if (p == last0 && hashes) fl |= kFxReduce;
                 d.lenf = (uint32_t)(en - st) | (fl << 24);
                 d.k = 0;
                 items[pb + (uint64_t)q * kFxMaxK + i] = d;
             }
-            if (c > 0 && j == 0) {
+            if (j == 0) {
                 W.hpart[2ull * (hs + c)] = 0;
                 W.hpart[2ull * (hs + c) + 1] = 0;
             }
@@ -763,10 +670,11 @@ __global__ void k_fx_fill(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk
     })
 }
 
-__global__ void __launch_bounds__(kFxThreads, FFM_FX_CTAS) k_fused_fx(DevLog L, Work W,
+__global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, Work W,
                                                                       const FxDesc* __restrict__ items,
                                                                       const uint32_t* __restrict__ n_items_ptr,
-                                                                      uint32_t* res_out) {
+                                                                      uint32_t pw, uint32_t* res_out) {
+    // pw: words below it were hashed by the prefix pass (not hashed, no deltas here)
     extern __shared__ __align__(128) uint8_t fx_smem[];
     uint8_t* bufs = fx_smem;
     FxDesc* meta = reinterpret_cast<FxDesc*>(fx_smem + (size_t)kFxStages * kFxPiece);
@@ -925,7 +833,8 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_CTAS) k_fused_fx(DevLog L, 
                 word_keys(k, ka, (w0 + t) >> 4);
 #pragma unroll
                 for (int u = 0; u < kFxWords; ++u) {
-                    if (len > 16 * (int32_t)(t + kStride * u)) nh_word(x[u].x, x[u].y, x[u].z, x[u].w, k, A, B);
+                    if (len > 16 * (int32_t)(t + kStride * u) && w0 + t + kStride * u >= pw)
+                        nh_word(x[u].x, x[u].y, x[u].z, x[u].w, k, A, B);
 #pragma unroll
                     for (int j = 0; j < 6; ++j) k[j] += kDA(j) * (kStride / 16);
                 }
@@ -953,7 +862,7 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_CTAS) k_fused_fx(DevLog L, 
                     uint64_t xA = 0, xB = 0;
 #pragma unroll
                     for (int u = 0; u < kFxWords; ++u) {
-                        if (dmask & (1u << u)) {
+                        if ((dmask & (1u << u)) && w0 + t + kStride * u >= pw) {
                             uint32_t k[6];
                             word_keys(k, ka, (w0 + t + kStride * u) >> 4);
                             nh_word(y[u].x, y[u].y, y[u].z, y[u].w, k, dA, dB);
@@ -1013,17 +922,18 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_CTAS) k_fused_fx(DevLog L, 
 }
 
 // Combine the chunk partial sums of large records (NH is a plain sum, so the record's
-// accumulators are the sums of its chunks' -- no atomics, deterministic) and finish
-// their digests.  Also totals the bytes hashed beyond first chunks (roofline stats).
-// After the pipelined fused pass (fx) a member's chunks >= 1 are its head's partials
-// plus its own deltas.
-__global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t small_bytes, uint32_t chunk_bytes,
+// accumulators are the sums of its parts' -- deterministic) and finish their digests.
+// Two-pass: the chunk slots of k_hash_large.  After the pipelined fused pass (fx): the
+// prefix partial + the record's chunk slots, and for a member also its head's chunk
+// slots (its own slots hold NH deltas).  Also totals the bytes hashed beyond the
+// prefixes (roofline stats).
+__global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t chunk_bytes, uint32_t prefix_bytes,
                                                       int prefilter, int fx) {
     unsigned long long rest = 0;
     FFM_WARP_EACH(L.n_large, L.large_order[w_], true, {
         const uint32_t s0 = W.hstart[rec];
-        const bool skip = prefilter && prefix_unique(W, rec);
-        const uint32_t e0 = skip ? s0 + 1 : W.hstart[rec + 1];
+        const bool skip = fx && prefilter && prefix_unique(W, rec);
+        const uint32_t e0 = skip ? s0 : W.hstart[rec + 1];
         const uint32_t h = fx ? W.fhead[rec] : rec;
         const int64_t dh = (int64_t)W.hstart[h] - (int64_t)s0;   // head slot of the same chunk
         uint64_t A0 = 0, B0 = 0, A1 = 0, B1 = 0;
@@ -1033,11 +943,9 @@ __global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t
             B0 += W.hpart[2ull * it + 1];
             A1 += W.hpart[2ull * (it + 32)];
             B1 += W.hpart[2ull * (it + 32) + 1];
-            if (h != rec) {   // member chunks >= 1: head's partial + own delta
-                if (it != s0) {
-                    A0 += W.hpart[2ull * (it + dh)];
-                    B0 += W.hpart[2ull * (it + dh) + 1];
-                }
+            if (h != rec) {   // a member: head's partials + own deltas
+                A0 += W.hpart[2ull * (it + dh)];
+                B0 += W.hpart[2ull * (it + dh) + 1];
                 A1 += W.hpart[2ull * (it + 32 + dh)];
                 B1 += W.hpart[2ull * (it + 32 + dh) + 1];
             }
@@ -1045,7 +953,7 @@ __global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t
         if (it < e0) {
             A0 += W.hpart[2ull * it];
             B0 += W.hpart[2ull * it + 1];
-            if (h != rec && it != s0) {
+            if (h != rec) {
                 A0 += W.hpart[2ull * (it + dh)];
                 B0 += W.hpart[2ull * (it + dh) + 1];
             }
@@ -1056,27 +964,19 @@ __global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t
             B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
         }
         const uint64_t n = L.size[rec];
+        if (fx) {   // + the prefix pass's partial (accA/accB hold it until here)
+            A += W.accA[rec];
+            B += W.accB[rec];
+        }
+        __syncwarp();
         if (lane == 0) {
             W.accA[rec] = A;
             W.accB[rec] = B;
             W.digest[rec] = finalize_digest(A, B, n);
-            if (!skip && n > chunk_bytes) rest += n - chunk_bytes;
+            if (fx && !skip && n > prefix_bytes) rest += n - prefix_bytes;
         }
     })
     if (rest) atomicAdd((unsigned long long*)(W.counters + 4), rest);
-}
-
-__global__ void k_verify_fill(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list,
-                              uint32_t small_bytes, uint32_t chunk_bytes) {
-    FFM_WARP_EACH(list ? n_list : L.n_large, list ? list[w_] : L.large_order[w_],
-                  (W.leader[rec] != rec && L.size[rec] > small_bytes && L.size[W.leader[rec]] == L.size[rec] &&
-                   L.chan[W.leader[rec]] == L.chan[rec]), {
-        const uint32_t ld = W.leader[rec];
-        const uint64_t n = L.size[rec];
-        const uint32_t c_n = (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
-        const uint32_t base = W.lstart[ld], k = W.gcount[ld], p = W.pos[rec];
-        for (uint32_t c = lane; c < c_n; c += 32) W.vitems[base + c * k + p] = make_uint2(rec, c);
-    })
 }
 
 // ----------------------------------------------------------------------------
@@ -1149,13 +1049,24 @@ __global__ void __launch_bounds__(256, 3) k_fused_small(DevLog L, Work W, uint32
     const unsigned omask = 0xFFu << (threadIdx.x & 24);
     LaneKeys K0;
     load_keys(K0, 2 * g, 0);
+    // descriptors of k_leader0 at the record's position in the size-class order:
+    // (own arena offset, leader's offset or ~0 when not compared, size, record)
+    uint4 da = make_uint4(0, 0, 0, 0), db = make_uint4(0, 0, 0, 0);
+    if (oct < L.n_small) {
+        da = W.sdesc[2ull * oct];
+        db = W.sdesc[2ull * oct + 1];
+    }
     for (uint32_t i = oct; i < L.n_small; i += noct) {
-        const uint32_t r = L.small_order[i];
-        const uint64_t n = L.size[r];
-        const uint32_t ld = W.leader[r];
-        const uint8_t* base = L.arena + L.off[r];
-        const bool cmp = ld != r && L.size[ld] == n && L.chan[ld] == L.chan[r];
-        const uint8_t* lb = L.arena + L.off[ld];
+        const uint64_t off = (uint64_t)da.y << 32 | da.x, loff = (uint64_t)da.w << 32 | da.z;
+        const uint64_t n = db.x;
+        const uint32_t r = db.y;
+        if (i + noct < L.n_small) {   // the next record's descriptor, in flight meanwhile
+            da = W.sdesc[2ull * (i + noct)];
+            db = W.sdesc[2ull * (i + noct) + 1];
+        }
+        const bool cmp = loff != ~0ull;
+        const uint8_t* base = L.arena + off;
+        const uint8_t* lb = L.arena + (cmp ? loff : off);
         const uint32_t nblk = (uint32_t)((n + 31) >> 5);
         LaneKeys K = K0;
         uint64_t A = 0, B = 0, found = ~0ull;
@@ -1164,7 +1075,11 @@ __global__ void __launch_bounds__(256, 3) k_fused_small(DevLog L, Work W, uint32
 #pragma unroll
             for (int u = 0; u < kSmallU; ++u) {
                 const uint32_t b = b0 + 8 * u + g;
+#if FFM_SMALL_OWN_EVICT_FIRST
                 x[u] = b < nblk ? ld_stream(base + 32ull * b) : zero_blk();
+#else
+                x[u] = b < nblk ? ld_remote(base + 32ull * b) : zero_blk();
+#endif
                 y[u] = (cmp && b < nblk) ? ld_keep(lb + 32ull * b) : zero_blk();
             }
 #pragma unroll
@@ -1195,65 +1110,6 @@ __global__ void __launch_bounds__(256, 3) k_fused_small(DevLog L, Work W, uint32
             W.digest[r] = finalize_digest(A, B, n);
             if (found != ~0ull) report_mismatch(W, r, found, res_out, false);
         }
-    }
-}
-
-__global__ void __launch_bounds__(256, 3) k_verify_large(DevLog L, Work W, const uint2* __restrict__ items,
-                                                      const uint32_t* __restrict__ n_items_ptr, uint32_t chunk_bytes,
-                                                      uint32_t* res_out) {
-    const int lane = threadIdx.x & 31;
-    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
-    const uint32_t n_items = *n_items_ptr;
-    const uint32_t cblk = chunk_bytes >> 5;
-    for (uint32_t it = warp; it < n_items; it += nwarps) {
-        const uint2 w = items[it];
-        const uint32_t m = w.x;
-        const uint32_t ld = W.leader[m];
-        const uint64_t n = L.size[m];
-        if (L.size[ld] != n) {
-            if (lane == 0) report_mismatch(W, m, 0, res_out, true);
-            continue;
-        }
-        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
-        const uint32_t bb = w.y * cblk;
-        const uint32_t be = min(bb + cblk, nblk);
-        uint64_t known = lane == 0 ? *((volatile uint64_t*)&W.mis[m]) : 0;
-        known = __shfl_sync(0xFFFFFFFFu, known, 0);
-        if (2 * bb >= known) continue;   // a mismatch at a lower word is already known
-        const uint8_t* pm = L.arena + L.off[m];
-        const uint8_t* pl = L.arena + L.off[ld];
-        uint64_t word = ~0ull;
-        for (uint32_t b0 = bb; b0 < be; b0 += 32 * kVerifyU) {
-            Blk x[kVerifyU], y[kVerifyU];
-#pragma unroll
-            for (int u = 0; u < kVerifyU; ++u) {
-                uint32_t b = b0 + 32 * u + lane;
-                x[u] = b < be ? ld_stream(pm + 32ull * b) : zero_blk();
-                y[u] = b < be ? ld_keep(pl + 32ull * b) : zero_blk();
-            }
-            uint64_t found = ~0ull;
-#pragma unroll
-            for (int u = 0; u < kVerifyU; ++u) {
-                uint32_t b = b0 + 32 * u + lane;
-                if (b < be) {
-                    mask_tail(x[u], n, b);
-                    mask_tail(y[u], n, b);
-                    int d = blk_diff(x[u], y[u]);
-                    if (d >= 0 && found == ~0ull) found = 2ull * b + d;
-                }
-            }
-            if (__any_sync(0xFFFFFFFFu, found != ~0ull)) {
-#pragma unroll
-                for (int o = 16; o; o >>= 1) {
-                    uint64_t other = __shfl_xor_sync(0xFFFFFFFFu, found, o);
-                    found = other < found ? other : found;
-                }
-                word = found;
-                break;
-            }
-        }
-        if (word != ~0ull && lane == 0) report_mismatch(W, m, word, res_out, true);
     }
 }
 
@@ -1461,6 +1317,8 @@ int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st
 
 int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_out, cudaStream_t st) {
     if (L.n == 0 || L.n_small == 0) return 0;
+    // (measured: capping its grid so that it co-resides with the persistent large pass
+    // slowed that pass more than it hid -- profiles/r01b/README.md)
     uint32_t grid = resident_grid((const void*)k_fused_small, P.num_sms);
     uint32_t need = blocks_for((uint64_t)L.n_small * 8);
     k_fused_small<<<need < grid ? need : grid, 256, 0, st>>>(L, W, res_out);
@@ -1468,26 +1326,35 @@ int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_
     return 1;
 }
 
-int launch_hash_plan(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
+// Chunk slots of large payloads (count -> scan); two-pass also scatters the
+// (record, chunk) work units of k_hash_large.
+int launch_hash_plan(const DevLog& L, Work& W, const Params& P, bool units, cudaStream_t st) {
     k_hash_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hcount);
     FFM_LAUNCH_CHECK();
     size_t bytes = W.cub_tmp_bytes;
     if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.hcount, W.hstart, (int)(L.n + 1), st) != cudaSuccess)
         return -1;
-    if (L.n) {
+    if (units && L.n_large) {
         k_hash_fill<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, P.small_bytes, P.chunk_bytes, W.hstart,
-                                                                    W.hitems);
+                                                                     W.hitems);
         FFM_LAUNCH_CHECK();
+        return 3;
     }
-    return 3;
+    return 2;
 }
 
-int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st, int phase) {
+int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_items, cudaStream_t st) {
     if (n_items == 0) return 0;
     uint32_t grid = resident_grid((const void*)k_hash_large, P.num_sms);
     uint32_t need = blocks_for(n_items * 32);
-    k_hash_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W.hitems, W.hstart + L.n, P.chunk_bytes, W.hpart,
-                                                            phase);
+    k_hash_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W.hitems, W.hstart + L.n, P.chunk_bytes, W.hpart);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
+int launch_prefix(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
+    if (L.n_large == 0) return 0;
+    k_prefix_hash<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.prefix_bytes);
     FFM_LAUNCH_CHECK();
     return 1;
 }
@@ -1496,49 +1363,35 @@ int launch_hash_large(const DevLog& L, Work& W, const Params& P, uint64_t n_item
 // hash + compare pass, then the per-record combine of chunk partial sums.
 int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
     if (L.n == 0) return 0;
-    k_hash_combine<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 0, 0);
+    k_hash_combine<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.chunk_bytes, P.prefix_bytes, 0, 0);
     FFM_LAUNCH_CHECK();
     return 1;
 }
 
 int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
                  cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b) {
-    if (L.n == 0 || n_units == 0) return 0;
+    if (L.n == 0 || n_units == 0 || L.n_large == 0) return 0;
+    if (!smem_configured((const void*)k_fused_fx, (int)kFxSmem)) return -1;
     int k = 0;
-    const bool fx = P.fused_impl == 0 && smem_configured((const void*)k_fused_fx, (int)kFxSmem);
-    if (fx) {
-        // entries per head (pieces x (members + sub-task leader copies)), then their scan
-        k_fx_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 0);
-        FFM_LAUNCH_CHECK();
-        ++k;
-    }
+    // entries per head (pieces x (members + sub-task leader copies)), their scan, the
+    // stage descriptors, the pipelined pass, the per-record combine
+    k_fx_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 0);
+    FFM_LAUNCH_CHECK();
     size_t bytes = W.cub_tmp_bytes;
     if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.lcount, W.lstart, (int)(L.n + 1), st) != cudaSuccess)
         return -1;
-    ++k;
-    if (fx) {
-        k_fx_fill<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, prefilter ? 1 : 0,
-                                                              reinterpret_cast<FxDesc*>(W.fitems));
-    } else {
-        k_fused_fill<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes);
-    }
+    k_fx_fill<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.chunk_bytes, P.prefix_bytes,
+                                                               prefilter ? 1 : 0, reinterpret_cast<FxDesc*>(W.fitems));
     FFM_LAUNCH_CHECK();
-    ++k;
+    k += 3;
     if (ev_a && cudaEventRecord(ev_a, st) != cudaSuccess) return -1;
-    if (fx) {
-        k_fused_fx<<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
-            L, W, reinterpret_cast<const FxDesc*>(W.fitems), W.lstart + L.n, res_out);
-    } else {
-        uint32_t grid = resident_grid((const void*)k_fused, P.num_sms);
-        uint32_t need = blocks_for(n_units * 32);
-        k_fused<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.lstart + L.n, P.chunk_bytes, prefilter ? 1 : 0,
-                                                           res_out);
-    }
+    k_fused_fx<<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
+        L, W, reinterpret_cast<const FxDesc*>(W.fitems), W.lstart + L.n, P.prefix_bytes >> 4, res_out);
     FFM_LAUNCH_CHECK();
     ++k;
     if (ev_b && cudaEventRecord(ev_b, st) != cudaSuccess) return -1;
-    k_hash_combine<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes,
-                                                              prefilter ? 1 : 0, fx ? 1 : 0);
+    k_hash_combine<<<warp_grid(L.n_large, P.num_sms), 256, 0, st>>>(L, W, P.chunk_bytes, P.prefix_bytes,
+                                                                   prefilter ? 1 : 0, 1);
     FFM_LAUNCH_CHECK();
     return k + 1;
 }
@@ -1567,7 +1420,7 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
                                                         P.small_bytes);
     FFM_LAUNCH_CHECK();
     if (round == 0)
-        k_leader0<<<blocks_for(n_list), 256, 0, st>>>(L, W, n_list, P.small_bytes, P.chunk_bytes, res_out);
+        k_leader0<<<blocks_for(n_list), 256, 0, st>>>(L, W, n_list, P.small_bytes, res_out);
     else if (round < 0)
         k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, nullptr, n_list, P.small_bytes, P.chunk_bytes, res_out);
     else
@@ -1599,42 +1452,22 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
         FFM_LAUNCH_CHECK();
         ++k;
     }
-    if (vitem_cap) {
+    if (vitem_cap && L.n_large) {
         // large members: groups per leader (scan of per-leader entry counts), then the
-        // verify work -- the pipelined pass (leader piece in registers, members compared
-        // against it) or the chunk-major L2 kernel
-        const bool fx = P.fused_impl == 0 && smem_configured((const void*)k_fused_fx, (int)kFxSmem);
-        if (fx) {
-            k_fx_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 1);
-            FFM_LAUNCH_CHECK();
-            ++k;
-        }
+        // pipelined pass in verify mode (leader piece in registers, members compared)
+        if (!smem_configured((const void*)k_fused_fx, (int)kFxSmem)) return -1;
+        k_fx_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 1);
+        FFM_LAUNCH_CHECK();
         size_t bytes = W.cub_tmp_bytes;
         if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, W.lcount, W.lstart, (int)(L.n + 1), st) != cudaSuccess)
             return -1;
-        ++k;
-        uint32_t* n_vitems = W.lstart + L.n;   // total large verify work units
-        if (fx) {
-            k_fx_vfill<<<warp_grid(list ? n_list : L.n_large, P.num_sms), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes,
-                                                                     reinterpret_cast<FxDesc*>(W.fitems));
-            FFM_LAUNCH_CHECK();
-            ++k;
-            k_fused_fx<<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
-                L, W, reinterpret_cast<const FxDesc*>(W.fitems), n_vitems, res_out);
-            FFM_LAUNCH_CHECK();
-            ++k;
-        } else {
-            k_verify_fill<<<warp_grid(list ? n_list : L.n_large, P.num_sms), 256, 0, st>>>(L, W, list, n_list, P.small_bytes,
-                                                                        P.chunk_bytes);
-            FFM_LAUNCH_CHECK();
-            ++k;
-            uint32_t grid = resident_grid((const void*)k_verify_large, P.num_sms);
-            need = blocks_for(vitem_cap * 32);
-            k_verify_large<<<need < grid ? need : grid, 256, 0, st>>>(L, W, W.vitems, n_vitems, P.chunk_bytes,
-                                                                      res_out);
-            FFM_LAUNCH_CHECK();
-            ++k;
-        }
+        k_fx_vfill<<<warp_grid(list ? n_list : L.n_large, P.num_sms), 256, 0, st>>>(
+            L, W, list, n_list, P.small_bytes, P.chunk_bytes, reinterpret_cast<FxDesc*>(W.fitems));
+        FFM_LAUNCH_CHECK();
+        k_fused_fx<<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
+            L, W, reinterpret_cast<const FxDesc*>(W.fitems), W.lstart + L.n, 0xFFFFFFFFu, res_out);
+        FFM_LAUNCH_CHECK();
+        k += 4;
     }
     if (side) {
         if (cudaEventRecord(ev_join, side) != cudaSuccess || cudaStreamWaitEvent(st, ev_join, 0) != cudaSuccess)
