@@ -11,14 +11,14 @@
 
 namespace ffm {
 
-constexpr uint32_t kArenaAlign = 128;        // record slots in the HBM arena
+constexpr uint32_t kArenaAlign = 32;         // record slots in the HBM arena (consecutive small records are contiguous)
 constexpr uint64_t kEmptyKey = ~0ull;         // group-by table: empty slot
 constexpr uint32_t kNoRecord = 0xFFFFFFFFu;
 
 // Device-side views handed to the kernel launchers.
 struct DevLog {
     const uint8_t* arena;
-    const uint64_t* off;     // [n] arena offset of record i (128-B aligned)
+    const uint64_t* off;     // [n] arena offset of record i (32-B aligned)
     const uint64_t* size;    // [n]
     const uint32_t* site;    // [n]
     const uint64_t* dur;     // [n]
@@ -110,6 +110,7 @@ struct Params {
     int num_sms;
     int max_smem;      // opt-in dynamic shared memory per block (bytes)
     uint32_t prefix_bytes;  // fused round 0: large payloads are grouped by the NH of their first prefix_bytes
+    int small_pipe;         // fused round 0: small payloads through k_small_fx (1) or k_fused_small (0)
 };
 
 // ---- kernel launchers (kernels.cu).  All asynchronous on `st`; each returns the

@@ -122,6 +122,38 @@ def test_digest_spec_and_chunk_invariance(ffm):
         assert [int(x) for x in got] == want, (chunk, small)
 
 
+@pytest.mark.parametrize("pipe", ["1", "0"])
+@pytest.mark.parametrize("small", [4096, 16384, 128])
+def test_small_pass_variants(ffm, monkeypatch, pipe, small):
+    """Small payloads through the pipelined TMA pass (k_small_fx, FFM_SMALL_PIPE=1, the
+    default) and the octet pass (k_fused_small): the same labels, benefit and digests.
+    The mix packs up to 32 records per stage (tiny ones: 8-lane teams) down to two
+    (member + leader at the threshold: whole-warp teams), with empty payloads, ragged
+    tails, members with a flipped last byte and re-uploads of several contents."""
+    from digest_spec import digest
+    monkeypatch.setenv("FFM_SMALL_PIPE", pipe)
+    rng = np.random.default_rng(17 + small)
+    bases = [rng.integers(0, 256, int(s), dtype=np.uint8).tobytes()
+             for s in list(rng.integers(0, small + 1, 40)) + [0, 1, 31, 32, 33, small - 1, small]]
+    pay = []
+    for _ in range(3000):
+        b = bases[int(rng.integers(0, len(bases)))]
+        if b and rng.random() < 0.15:
+            a = bytearray(b)
+            a[-1 if rng.random() < 0.5 else int(rng.integers(0, len(a)))] ^= 0x5A
+            b = bytes(a)
+        pay.append(b)
+    lg = loggen.from_payloads(pay, rng.integers(0, 5, len(pay)), rng.integers(0, 1 << 40, len(pay)), 5)
+    for db in (64, 0):
+        with ffm.FfmLog(lg.n_sites, small_bytes=small, chunk_bytes=max(1024, small), digest_bits=db) as log:
+            log.append_log(lg)
+            dup, ben = log.run()
+            assert_same(lg, dup, ben)
+            if db == 64:
+                got = log.digests()
+                assert all(int(got[i]) == digest(pay[i]) for i in range(0, len(pay), 7))
+
+
 def test_flip_at_boundaries(ffm):
     rng = np.random.default_rng(4)
     size = 3 * 4096 + 77
