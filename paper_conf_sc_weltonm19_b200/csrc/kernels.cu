@@ -676,6 +676,7 @@ __global__ void k_fx_fill(DevLog L, Work W, uint32_t chunk_bytes, uint32_t prefi
     })
 }
 
+template <bool kVerify>
 __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, Work W,
                                                                       const FxDesc* __restrict__ items,
                                                                       const uint32_t* __restrict__ n_items_ptr,
@@ -706,12 +707,19 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
         int stage = 0;
         uint32_t phase = 0;
         const uint4* raw = reinterpret_cast<const uint4*>(items);
+        // verify-only mode (resolve rounds, two-pass): a member's piece that starts after
+        // its already-recorded first mismatch cannot lower it -- it is not streamed (the
+        // member's mismatch word is read a batch ahead; a stale value only skips less)
+        constexpr bool vmode = kVerify;
+        const volatile unsigned long long* vmis = reinterpret_cast<const volatile unsigned long long*>(W.mis);
         // lane-parallel batch of 32 descriptors [bb, bb + 32), the next one prefetched
-        auto load = [&](uint32_t bb, uint4& a, uint4& b) {
+        auto load = [&](uint32_t bb, uint4& a, uint4& b, uint64_t& mi) {
             const uint32_t i = bb + lane;
+            mi = ~0ull;
             if (i < E) {
                 a = raw[2ull * i];
                 b = raw[2ull * i + 1];
+                if (vmode && !((a.w >> 24) & kFxLeader)) mi = vmis[a.z];
             } else {
                 a = make_uint4(0, 0, 0, 0);
                 b = make_uint4(0, 0, 0, 0);
@@ -723,8 +731,9 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
         uint32_t lo = seg * kFxSeg;
         uint32_t bb = lo;
         uint4 ca, cb, na, nb;
-        load(bb, ca, cb);
-        load(bb + 32, na, nb);
+        uint64_t cm, nm;
+        load(bb, ca, cb, cm);
+        load(bb + 32, na, nb, nm);
         uint32_t rem = 0;          // entries left in the current task
         bool started = false;      // a task starting in this segment has been seen
         while (lo < E) {
@@ -759,6 +768,7 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
                     const uint32_t w0 = __shfl_sync(0xFFFFFFFFu, cb.x, j);
                     const uint32_t slot = __shfl_sync(0xFFFFFFFFu, cb.y, j);
                     if ((lenf >> 24) & kFxSkip) continue;
+                    if (vmode && __shfl_sync(0xFFFFFFFFu, cm, j) < (uint64_t)w0) continue;
                     if (lane == 0) {
                         mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
                         FxDesc& m = meta[stage];
@@ -782,7 +792,8 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
                 bb += 32;
                 ca = na;
                 cb = nb;
-                load(bb + 32, na, nb);
+                cm = nm;
+                load(bb + 32, na, nb, nm);
             }
             // next segment
             if (lane == 0) seg = atomicAdd(&W.counters[8], 1u);
@@ -792,8 +803,8 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
             started = false;
             if (lo >= E) break;
             bb = lo;
-            load(bb, ca, cb);
-            load(bb + 32, na, nb);
+            load(bb, ca, cb, cm);
+            load(bb + 32, na, nb, nm);
         }
         if (lane == 0) {
             mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
@@ -1699,7 +1710,7 @@ int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st) {
 int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
                  cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b) {
     if (L.n == 0 || n_units == 0 || L.n_large == 0) return 0;
-    if (!smem_configured((const void*)k_fused_fx, (int)kFxSmem)) return -1;
+    if (!smem_configured((const void*)k_fused_fx<false>, (int)kFxSmem)) return -1;
     int k = 0;
     // entries per head (pieces x (members + sub-task leader copies)), their scan, the
     // stage descriptors, the pipelined pass, the per-record combine
@@ -1713,7 +1724,7 @@ int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bo
     FFM_LAUNCH_CHECK();
     k += 3;
     if (ev_a && cudaEventRecord(ev_a, st) != cudaSuccess) return -1;
-    k_fused_fx<<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
+    k_fused_fx<false><<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
         L, W, reinterpret_cast<const FxDesc*>(W.fitems), W.lstart + L.n, P.prefix_bytes >> 4, res_out);
     FFM_LAUNCH_CHECK();
     ++k;
@@ -1783,7 +1794,7 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
     if (vitem_cap && L.n_large) {
         // large members: groups per leader (scan of per-leader entry counts), then the
         // pipelined pass in verify mode (leader piece in registers, members compared)
-        if (!smem_configured((const void*)k_fused_fx, (int)kFxSmem)) return -1;
+        if (!smem_configured((const void*)k_fused_fx<true>, (int)kFxSmem)) return -1;
         k_fx_count<<<blocks_for((uint64_t)L.n + 1), 256, 0, st>>>(L, W, P.small_bytes, P.chunk_bytes, 1);
         FFM_LAUNCH_CHECK();
         size_t bytes = W.cub_tmp_bytes;
@@ -1792,7 +1803,7 @@ int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* lis
         k_fx_vfill<<<warp_grid(list ? n_list : L.n_large, P.num_sms), 256, 0, st>>>(
             L, W, list, n_list, P.small_bytes, P.chunk_bytes, reinterpret_cast<FxDesc*>(W.fitems));
         FFM_LAUNCH_CHECK();
-        k_fused_fx<<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
+        k_fused_fx<true><<<P.num_sms * FFM_FX_CTAS, kFxThreads, kFxSmem, st>>>(
             L, W, reinterpret_cast<const FxDesc*>(W.fitems), W.lstart + L.n, 0xFFFFFFFFu, res_out);
         FFM_LAUNCH_CHECK();
         k += 4;
