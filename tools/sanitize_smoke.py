@@ -1,5 +1,6 @@
-"""Small logs through every kernel (fused and two-pass round 0, pre-filter, collision
-resolve, online windows, device-payload gather), for compute-sanitizer memcheck /
+"""Small logs through every kernel (fused and two-pass round 0 incl. the TMA-pipelined k_fused_fx in
+hash and verify mode with pieces split from 64 KiB chunks and groups of > 64 members, pre-filter,
+collision resolve, online windows, device-payload gather), for compute-sanitizer memcheck /
 racecheck / synccheck."""
 import os
 import sys
@@ -12,13 +13,14 @@ import loggen  # noqa: E402
 import oracle  # noqa: E402
 import paper_conf_sc_weltonm19_b200 as ffm  # noqa: E402
 
-for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (4, 0.04, 1 / 512), (2, 0.001, 1.0)]:
+for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (3, 0.012, 1 / 128), (4, 0.04, 1 / 512), (2, 0.001, 1.0)]:
     lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
     want = oracle.dedup(lg)
     for db, rb, dev, extra in [(64, 64, False, {}), (0, 64, True, {}), (0, 0, False, {}),
                                (64, 64, False, {"two_pass": True}), (64, 64, False, {"prefilter": True}),
-                               (8, 64, True, {"fused": True})]:
-        with ffm.FfmLog(lg.n_sites, digest_bits=db, refine_bits=rb, chunk_bytes=4096, small_bytes=1024,
+                               (8, 64, True, {"fused": True}), (0, 64, False, {"chunk": 65536})]:
+        chunk = extra.pop("chunk", 4096)
+        with ffm.FfmLog(lg.n_sites, digest_bits=db, refine_bits=rb, chunk_bytes=chunk, small_bytes=1024,
                         **extra) as log:
             if dev:
                 buf = torch.from_numpy(lg.materialize()).cuda()
