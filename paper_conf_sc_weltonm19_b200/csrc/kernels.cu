@@ -1064,8 +1064,6 @@ __global__ void __launch_bounds__(256, FFM_SMALL_MINB) k_fused_small(DevLog L, W
     const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
     const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
     const unsigned omask = 0xFFu << (threadIdx.x & 24);
-    LaneKeys K0;
-    load_keys(K0, 2 * g, 0);
     // descriptors of k_leader0 at the record's position in the size-class order:
     // (own arena offset, leader's offset or ~0 when not compared, size, record)
     uint4 da = make_uint4(0, 0, 0, 0), db = make_uint4(0, 0, 0, 0);
@@ -1085,9 +1083,58 @@ __global__ void __launch_bounds__(256, FFM_SMALL_MINB) k_fused_small(DevLog L, W
         const uint8_t* base = L.arena + off;
         const uint8_t* lb = L.arena + (cmp ? loff : off);
         const uint32_t nblk = (uint32_t)((n + 31) >> 5);
-        LaneKeys K = K0;
+        const uint32_t nfull = (uint32_t)(n >> 5);   // blocks with all 32 bytes in the record
+        LaneKeys K;
+        load_keys(K, 2 * g, 0);   // (constant cache; not kept live across records: registers)
         uint64_t A = 0, B = 0, found = ~0ull;
-        for (uint32_t b0 = 0; b0 < nblk; b0 += 8 * kSmallU) {
+        bool cmp_on = cmp;                            // this lane still looking for a mismatch
+        uint32_t b0 = 0, hit = ~0u;
+        // fast path: iterations whose blocks are all full -- no tail masks, no per-block
+        // bounds, the compare an OR-reduction (the exact first mismatch only on a hit)
+#pragma unroll 1
+        for (; b0 + 8 * kSmallU <= nfull; b0 += 8 * kSmallU) {
+            Blk x[kSmallU], y[kSmallU];
+#pragma unroll
+            for (int u = 0; u < kSmallU; ++u) {
+#if FFM_SMALL_OWN_EVICT_FIRST
+                x[u] = ld_stream(base + 32ull * (b0 + 8 * u + g));
+#else
+                x[u] = ld_remote(base + 32ull * (b0 + 8 * u + g));
+#endif
+                if (cmp_on) y[u] = ld_keep(lb + 32ull * (b0 + 8 * u + g));
+            }
+#pragma unroll
+            for (int u = 0; u < kSmallU; ++u) {
+                nh_word(x[u].v[0], x[u].v[1], x[u].v[2], x[u].v[3], K.k[0], A, B);
+                nh_word(x[u].v[4], x[u].v[5], x[u].v[6], x[u].v[7], K.k[1], A, B);
+                advance<1>(K);
+            }
+            if (cmp_on) {
+                uint32_t d = 0;
+#pragma unroll
+                for (int u = 0; u < kSmallU; ++u)
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) d |= x[u].v[i] ^ y[u].v[i];
+                if (d) {          // rare: located exactly after the loop (keeps x, y short-lived)
+                    hit = b0;
+                    cmp_on = false;
+                }
+            }
+        }
+        if (hit != ~0u) {
+#pragma unroll 1
+            for (int u = 0; u < kSmallU; ++u) {   // lowest differing block of the hit iteration
+                const uint32_t b = hit + 8 * u + g;
+                const int dd = blk_diff(ld_stream(base + 32ull * b), ld_keep(lb + 32ull * b));
+                if (dd >= 0) {
+                    found = 2ull * b + dd;
+                    break;
+                }
+            }
+        }
+        // tail: the remaining (partial) iterations, masked
+#pragma unroll 1
+        for (; b0 < nblk; b0 += 8 * kSmallU) {
             Blk x[kSmallU], y[kSmallU];
 #pragma unroll
             for (int u = 0; u < kSmallU; ++u) {
@@ -1097,7 +1144,7 @@ __global__ void __launch_bounds__(256, FFM_SMALL_MINB) k_fused_small(DevLog L, W
 #else
                 x[u] = b < nblk ? ld_remote(base + 32ull * b) : zero_blk();
 #endif
-                y[u] = (cmp && b < nblk) ? ld_keep(lb + 32ull * b) : zero_blk();
+                y[u] = (cmp_on && b < nblk) ? ld_keep(lb + 32ull * b) : zero_blk();
             }
 #pragma unroll
             for (int u = 0; u < kSmallU; ++u) {
@@ -1105,7 +1152,7 @@ __global__ void __launch_bounds__(256, FFM_SMALL_MINB) k_fused_small(DevLog L, W
                 if (b < nblk) {
                     mask_tail(x[u], n, b);
                     nh_blk(x[u], K, n, b, A, B);
-                    if (cmp) {
+                    if (cmp_on) {
                         mask_tail(y[u], n, b);
                         const int d = blk_diff(x[u], y[u]);
                         if (d >= 0 && found == ~0ull) found = 2ull * b + d;
