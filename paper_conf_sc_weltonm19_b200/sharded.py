@@ -75,7 +75,14 @@ def dedup_sharded(log, device, group=None, duplicate_of=None, benefit=None, reps
     if reps_buf is None or reps_buf.shape[0] < max(n, 1):
         reps_buf = torch.empty((max(n, 1), REP_WORDS), dtype=torch.int64, device=device)
     n_reps = ffm_shard_local(log.h, reps_buf, reps_buf.shape[0])
-    all_reps, counts = allgather_reps(reps_buf[:n_reps], group)
+    # the exchange's device work (NCCL, padding, concatenation) is ordered on the
+    # library's stream, which the merge kernels then read from
+    dev = torch.device(device)
+    if dev.type == "cuda" and log.stream:
+        with torch.cuda.stream(torch.cuda.ExternalStream(log.stream, device=dev)):
+            all_reps, counts = allgather_reps(reps_buf[:n_reps], group)
+    else:
+        all_reps, counts = allgather_reps(reps_buf[:n_reps], group)
     if duplicate_of is None:
         duplicate_of = torch.empty(max(n, 1), dtype=torch.int64, device=device)
     if benefit is None:

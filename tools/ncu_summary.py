@@ -27,7 +27,7 @@ def launches(path):
         v = float(r[vi].replace(",", ""))
         u = r[ui]
         v = v / 1e3 if u in ("nsecond", "ns") else v * 1e3 if u in ("msecond", "ms") else v
-        name = r[ki].split("(")[0].replace("void ", "")
+        name = r[ki].split("(")[0].replace("void ", "").split("<")[0].split("::")[-1]
         agg[name].append(v)
     return agg
 
@@ -42,7 +42,7 @@ def full(rep):
             "smsp__inst_executed.sum", "launch__grid_size", "launch__block_size"]
     out = defaultdict(list)
     for r in rows[2:]:
-        name = r[h.index("Kernel Name")].split("(")[0].replace("void ", "")
+        name = r[h.index("Kernel Name")].split("(")[0].replace("void ", "").split("<")[0].split("::")[-1]
         d = {}
         for w in want:
             if w in h:
