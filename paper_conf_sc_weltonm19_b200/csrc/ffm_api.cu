@@ -153,10 +153,8 @@ bool is_device_ptr(const void* p) {
 // then the large ones in index order (one warp per large record in the planning
 // kernels).  Returns the number of small records.
 uint64_t build_small_order(const ffm_log* L, uint64_t begin, uint64_t end, std::vector<uint32_t>& order) {
-    // gid (= arena) order for the pipelined small pass, whose stages copy runs of
-    // consecutive records; size-class order for the octet kernels (equal lengths per warp)
     static const bool gid_order = getenv("FFM_SMALL_GID_ORDER") != nullptr;   // A/B knob (same results)
-    if (gid_order || L->params.small_pipe) {
+    if (gid_order) {
         order.clear();
         for (uint64_t i = begin; i < end; ++i)
             if (L->h_size[i] <= L->params.small_bytes) order.push_back((uint32_t)(i - begin));
@@ -726,8 +724,6 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
             const uint32_t v = (uint32_t)strtoul(e, nullptr, 10);
             if (v >= 256 && v % 256 == 0) L->params.prefix_bytes = std::min(v, chunk);
         }
-        L->params.small_pipe = 0;   // measured slower (profiles/r01c/README.md)
-        if (const char* e = getenv("FFM_SMALL_PIPE")) L->params.small_pipe = atoi(e) != 0;   // A/B knob (same results)
         L->params.chunk_bytes = chunk;
         L->params.small_bytes = small;
         L->params.digest_mask = cfg->digest_bits >= 64 ? ~0ull : ((1ull << cfg->digest_bits) - 1);

@@ -110,7 +110,6 @@ struct Params {
     int num_sms;
     int max_smem;      // opt-in dynamic shared memory per block (bytes)
     uint32_t prefix_bytes;  // fused round 0: large payloads are grouped by the NH of their first prefix_bytes
-    int small_pipe;         // fused round 0: small payloads through k_small_fx (1) or k_fused_small (0)
 };
 
 // ---- kernel launchers (kernels.cu).  All asynchronous on `st`; each returns the

@@ -1178,282 +1178,6 @@ __global__ void __launch_bounds__(256, FFM_SMALL_MINB) k_fused_small(DevLog L, W
 }
 
 // ----------------------------------------------------------------------------
-// H1 + H3 fused for small payloads, pipelined (round 0; the default).  The same work
-// as k_fused_small -- every small record hashed whole, every prefix-group member
-// byte-compared with its leader -- with the payload loads moved to the TMA engine:
-//
-//   * small records are processed in arena (gid) order, so consecutive ones are
-//     contiguous in the arena (32-byte slots, no gaps) and a stage is filled by one
-//     cp.async.bulk per *run* of consecutive records (a larger record in between
-//     starts a new run) -- a few copies of up to stage bytes, not one per record;
-//   * the producer warp takes segments of kSxSeg records (dynamic scheduling),
-//     bulk-copies their k_leader0 compare descriptors into shared memory (double-
-//     buffered, the next segment in flight), and packs records into stages: a lane per
-//     record, a warp prefix sum of the bytes each adds to the stage, the lane that
-//     starts a run issuing its copy (L2 evict_first);
-//   * the consumer warps split a stage into teams of T lanes (T = 8, 16 or 32 so that
-//     every record of the stage has a team); lane l of a team reads 32-byte blocks
-//     l, l + T, ... of its record from shared memory, adds them into its NH sums and
-//     compares them with the leader's copy;
-//   * a member's leader bytes are copied into the stage behind the runs by the
-//     producer warp with cp.async (16 B per lane, L2 evict_last: re-uploads of one
-//     content share their leader, which stays L2-resident), completing on the same
-//     mbarrier (cp.async.mbarrier.arrive.noinc) -- consumers never wait on a global
-//     load.  T is a multiple of 8, so a lane's NH positions are fixed (2 (l mod 8),
-//     +1) and its stripe advances by T / 8 per step.
-// ----------------------------------------------------------------------------
-#ifndef FFM_SX_STAGE
-#define FFM_SX_STAGE 24576
-#endif
-#ifndef FFM_SX_STAGES
-#define FFM_SX_STAGES 4
-#endif
-#ifndef FFM_SX_CTAS
-#define FFM_SX_CTAS 2
-#endif
-constexpr int kSxConsumers = 8;
-constexpr int kSxThreads = 32 * (kSxConsumers + 1);
-constexpr int kSxStages = FFM_SX_STAGES;
-constexpr uint32_t kSxSeg = 64;    // records per scheduler grab
-
-struct SxMeta {
-    uint4 r[32];       // (stage offset of the record's bytes, size, record, stage offset of its
-                       //  leader's copy or ~0u when not compared)
-    uint32_t m, T, pad0, pad1;   // records in the stage (~0u: done), team size
-};
-
-// stage bytes for a small-payload threshold (a member and its leader always fit)
-uint32_t sx_stage_bytes(uint32_t small_bytes) {
-    const uint32_t one = 2u * ((small_bytes + 31u) & ~31u);
-    return ((one > FFM_SX_STAGE ? one : FFM_SX_STAGE) + 127u) & ~127u;
-}
-static size_t sx_smem(uint32_t stage_bytes) {
-    return (size_t)kSxStages * stage_bytes + (size_t)kSxStages * sizeof(SxMeta) + 2 * kSxSeg * 32 +
-           (2 * kSxStages + 2) * sizeof(uint64_t);
-}
-
-__device__ __forceinline__ Blk lds_blk(const uint8_t* p) {
-    const uint4 a = *reinterpret_cast<const uint4*>(p), b = *reinterpret_cast<const uint4*>(p + 16);
-    Blk r;
-    r.v[0] = a.x; r.v[1] = a.y; r.v[2] = a.z; r.v[3] = a.w;
-    r.v[4] = b.x; r.v[5] = b.y; r.v[6] = b.z; r.v[7] = b.w;
-    return r;
-}
-
-__global__ void __launch_bounds__(kSxThreads, FFM_SX_CTAS) k_small_fx(DevLog L, Work W, uint32_t stage_bytes,
-                                                                      uint32_t* res_out) {
-    extern __shared__ __align__(128) uint8_t sx_smem_buf[];
-    uint8_t* bufs = sx_smem_buf;
-    SxMeta* meta = reinterpret_cast<SxMeta*>(sx_smem_buf + (size_t)kSxStages * stage_bytes);
-    uint4* dbuf = reinterpret_cast<uint4*>(meta + kSxStages);          // [2][kSxSeg][2]
-    uint64_t* full = reinterpret_cast<uint64_t*>(dbuf + 2 * 2 * kSxSeg);
-    uint64_t* empty = full + kSxStages;
-    uint64_t* dfull = empty + kSxStages;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < kSxStages; ++s) {
-            mbar_init(smem_u32(&full[s]), 33);   // expect_tx arrive + 32 cp.async arrivals
-            mbar_init(smem_u32(&empty[s]), kSxConsumers);
-        }
-        mbar_init(smem_u32(&dfull[0]), 1);
-        mbar_init(smem_u32(&dfull[1]), 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    }
-    __syncthreads();
-    const uint32_t N = L.n_small;
-
-    if (warp == kSxConsumers) {
-        // ------------------------------------------------------------ producer
-        uint64_t pol, pol_keep;
-        asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-        asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
-        auto grab = [&]() {
-            uint32_t s = 0;
-            if (lane == 0) s = atomicAdd(&W.counters[9], 1u);
-            return __shfl_sync(0xFFFFFFFFu, s, 0);
-        };
-        auto fetch = [&](uint32_t sg, int b) {   // the segment's descriptors -> dbuf[b]
-            const uint64_t lo = (uint64_t)sg * kSxSeg;
-            __syncwarp();
-            if (lo < N && lane == 0) {
-                const uint32_t cnt = (uint32_t)min((uint64_t)kSxSeg, N - lo);
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                mbar_arrive_tx(smem_u32(&dfull[b]), cnt * 32u);
-                bulk_g2s(smem_u32(dbuf + 2 * kSxSeg * b), W.sdesc + 2 * lo, cnt * 32u, smem_u32(&dfull[b]), pol);
-            }
-        };
-        int stage = 0, db = 0;
-        uint32_t phase = 0, dpar = 0;
-        uint32_t seg = grab();
-        fetch(seg, 0);
-        while ((uint64_t)seg * kSxSeg < N) {
-            const uint32_t nseg = grab();
-            fetch(nseg, db ^ 1);
-            mbar_wait(smem_u32(&dfull[db]), (dpar >> db) & 1u);
-            dpar ^= 1u << db;
-            const uint64_t lo = (uint64_t)seg * kSxSeg;
-            const uint32_t cnt = (uint32_t)min((uint64_t)kSxSeg, N - lo);
-            const uint4* D = dbuf + 2 * kSxSeg * db;
-            for (uint32_t p = 0; p < cnt;) {
-                const uint32_t j = p + lane;
-                const bool valid = j < cnt;
-                uint4 a = make_uint4(0, 0, 0, 0), b = make_uint4(0, 0, 0, 0);
-                if (valid) {
-                    a = D[2 * j];
-                    b = D[2 * j + 1];
-                }
-                const uint64_t off = (uint64_t)a.y << 32 | a.x, loff = (uint64_t)a.w << 32 | a.z;
-                const uint32_t own = valid ? ((b.x + 31u) & ~31u) : 0u;
-                const bool cmp = valid && loff != ~0ull;
-                const uint32_t lead = cmp ? own : 0u;
-                const uint64_t end = off + own;
-                // a record continues the previous lane's run when it starts where that ends
-                const uint64_t pend = (uint64_t)__shfl_up_sync(0xFFFFFFFFu, (uint32_t)(end >> 32), 1) << 32 |
-                                      __shfl_up_sync(0xFFFFFFFFu, (uint32_t)end, 1);
-                const bool start = lane == 0 || off != pend;
-                // prefix sums: own bytes (the runs) and own + leader bytes (the packing)
-                uint32_t io = own, ic = own + lead;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const uint32_t vo = __shfl_up_sync(0xFFFFFFFFu, io, o);
-                    const uint32_t vc = __shfl_up_sync(0xFFFFFFFFu, ic, o);
-                    if (lane >= o) {
-                        io += vo;
-                        ic += vc;
-                    }
-                }
-                const bool take = valid && ic <= stage_bytes;
-                const unsigned tmask = __ballot_sync(0xFFFFFFFFu, take);   // a prefix of the lanes
-                const uint32_t m = __popc(tmask);
-                const uint32_t own_total = __shfl_sync(0xFFFFFFFFu, io, m - 1);
-                // leader copies behind the runs: offset = own_total + leader bytes before
-                uint32_t il = lead;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const uint32_t v = __shfl_up_sync(0xFFFFFFFFu, il, o);
-                    if (lane >= o) il += v;
-                }
-                const uint32_t lso = own_total + il - lead;
-                // the last lane of this lane's run: before the next run start, else m - 1
-                const unsigned starts = __ballot_sync(0xFFFFFFFFu, take && start) & tmask;
-                const unsigned later = starts & ~((2u << lane) - 1u);
-                const int last = later ? __ffs(later) - 2 : (int)m - 1;
-                const uint32_t run_end = __shfl_sync(0xFFFFFFFFu, io, last < 0 ? 0 : last);
-                if (lane == 0) mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
-                __syncwarp();
-                SxMeta& M = meta[stage];
-                const uint32_t so = io - own;
-                if (take) M.r[lane] = make_uint4(so, b.x, b.y, cmp ? lso : ~0u);
-                if (lane == 0) {
-                    M.m = m;
-                    M.T = m <= 8 ? 32u : (m <= 16 ? 16u : 8u);
-                }
-                __syncwarp();
-                const uint32_t fb = smem_u32(&full[stage]);
-                const uint32_t sbase = smem_u32(bufs + (size_t)stage * stage_bytes);
-                if (lane == 0) mbar_arrive_tx(fb, own_total);
-                __syncwarp();
-                if (take && start && run_end > so) bulk_g2s(sbase + so, L.arena + off, run_end - so, fb, pol);
-                // leaders: all lanes copy one member's leader at a time, 16 B each
-                unsigned mem = __ballot_sync(0xFFFFFFFFu, take && cmp);
-                while (mem) {
-                    const int src = __ffs(mem) - 1;
-                    mem &= mem - 1;
-                    const uint64_t lsrc = (uint64_t)__shfl_sync(0xFFFFFFFFu, a.w, src) << 32 |
-                                          __shfl_sync(0xFFFFFFFFu, a.z, src);
-                    const uint32_t len = __shfl_sync(0xFFFFFFFFu, own, src);
-                    const uint32_t dst = sbase + __shfl_sync(0xFFFFFFFFu, lso, src);
-                    for (uint32_t k = 16u * lane; k < len; k += 512u)
-                        asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(dst + k),
-                                     "l"(L.arena + lsrc + k), "l"(pol_keep)
-                                     : "memory");
-                }
-                asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(fb) : "memory");
-                if (++stage == kSxStages) {
-                    stage = 0;
-                    phase ^= 1;
-                }
-                p += m;
-            }
-            seg = nseg;
-            db ^= 1;
-        }
-        if (lane == 0) {
-            mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
-            meta[stage].m = ~0u;
-            mbar_arrive(smem_u32(&full[stage]));
-        }
-        __syncwarp();
-        mbar_arrive(smem_u32(&full[stage]));   // the 32 lane arrivals of the last phase
-        return;
-    }
-
-    // ---------------------------------------------------------------- consumers
-    const uint32_t t = threadIdx.x;
-    int stage = 0;
-    uint32_t phase = 0;
-    for (;;) {
-        mbar_wait(smem_u32(&full[stage]), phase);
-        const uint32_t m = meta[stage].m;
-        if (m == ~0u) break;
-        const uint32_t T = meta[stage].T;
-        const uint32_t team = t / T, tl = t & (T - 1);
-        const bool act = team < m;
-        uint64_t A = 0, B = 0, found = ~0ull;
-        uint4 R = make_uint4(0, 0, 0, 0);
-        if (act) {
-            R = meta[stage].r[team];
-            const bool cmp = R.w != ~0u;
-            const uint8_t* sb = bufs + (size_t)stage * stage_bytes;
-            const uint8_t* own = sb + R.x;
-            const uint8_t* lb = sb + (cmp ? R.w : R.x);
-            const uint64_t n = R.y;
-            const uint32_t nblk = (R.y + 31u) >> 5;
-            const uint32_t step = T >> 3;
-            LaneKeys K;
-            load_keys(K, 2 * (tl & 7), tl >> 3);
-            uint32_t inc[6];
-#pragma unroll
-            for (int j = 0; j < 6; ++j) inc[j] = kDA(j) * step;
-            for (uint32_t b = tl; b < nblk; b += T) {
-                Blk x = lds_blk(own + 32 * b);
-                mask_tail(x, n, b);
-                nh_blk(x, K, n, b, A, B);
-                if (cmp) {
-                    Blk y = lds_blk(lb + 32 * b);
-                    mask_tail(y, n, b);
-                    const int d = blk_diff(x, y);
-                    if (d >= 0 && found == ~0ull) found = 2ull * b + d;
-                }
-#pragma unroll
-                for (int h = 0; h < 2; ++h)
-#pragma unroll
-                    for (int j = 0; j < 6; ++j) K.k[h][j] += inc[j];
-            }
-        }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(smem_u32(&empty[stage]));
-        for (uint32_t o = T >> 1; o; o >>= 1) {
-            A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
-            B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
-            const uint64_t of = __shfl_xor_sync(0xFFFFFFFFu, found, o);
-            found = of < found ? of : found;
-        }
-        if (act && tl == 0) {
-            W.accA[R.z] = A;
-            W.accB[R.z] = B;
-            W.digest[R.z] = finalize_digest(A, B, R.y);
-            if (found != ~0ull) report_mismatch(W, R.z, found, res_out, false);
-        }
-        if (++stage == kSxStages) {
-            stage = 0;
-            phase ^= 1;
-        }
-    }
-}
-
-// ----------------------------------------------------------------------------
 // H4: re-key residual members.  Round 1 refines by the full, untruncated NH sums;
 // later rounds by (first mismatching word index vs the previous leader, that word).
 // Byte-equal records always receive equal keys, so exactness never depends on the key.
@@ -1686,23 +1410,6 @@ int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st
 
 int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_out, cudaStream_t st) {
     if (L.n == 0 || L.n_small == 0) return 0;
-    if (P.small_pipe) {
-        // pipelined (TMA) small pass: persistent, one wave, segments scheduled dynamically
-        const uint32_t sb = sx_stage_bytes(P.small_bytes);
-        const size_t smem = sx_smem(sb);
-        if (!smem_configured((const void*)k_small_fx, (int)smem)) return -1;
-        int occ = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_small_fx, kSxThreads, smem) != cudaSuccess ||
-            occ < 1) {
-            cudaGetLastError();
-            occ = 1;
-        }
-        const uint64_t segs = (L.n_small + kSxSeg - 1) / kSxSeg;
-        const uint64_t cap = (uint64_t)P.num_sms * (uint64_t)occ;
-        k_small_fx<<<(uint32_t)(segs < cap ? segs : cap), kSxThreads, smem, st>>>(L, W, sb, res_out);
-        FFM_LAUNCH_CHECK();
-        return 1;
-    }
     // (measured: capping its grid so that it co-resides with the persistent large pass
     // slowed that pass more than it hid -- profiles/r01b/README.md)
     uint32_t grid = resident_grid((const void*)k_fused_small, P.num_sms);

@@ -122,16 +122,13 @@ def test_digest_spec_and_chunk_invariance(ffm):
         assert [int(x) for x in got] == want, (chunk, small)
 
 
-@pytest.mark.parametrize("pipe", ["1", "0"])
 @pytest.mark.parametrize("small", [4096, 16384, 128])
-def test_small_pass_variants(ffm, monkeypatch, pipe, small):
-    """Small payloads through the pipelined TMA pass (k_small_fx, FFM_SMALL_PIPE=1, the
-    default) and the octet pass (k_fused_small): the same labels, benefit and digests.
-    The mix packs up to 32 records per stage (tiny ones: 8-lane teams) down to two
-    (member + leader at the threshold: whole-warp teams), with empty payloads, ragged
-    tails, members with a flipped last byte and re-uploads of several contents."""
+def test_small_pass_variants(ffm, small):
+    """Small payloads through the fused small pass (k_fused_small: full-block fast path,
+    masked tail): labels, benefit and digests at three thresholds, with empty payloads,
+    ragged tails, sizes at and next to the threshold, members with a flipped last or
+    random byte and re-uploads of several contents."""
     from digest_spec import digest
-    monkeypatch.setenv("FFM_SMALL_PIPE", pipe)
     rng = np.random.default_rng(17 + small)
     bases = [rng.integers(0, 256, int(s), dtype=np.uint8).tobytes()
              for s in list(rng.integers(0, small + 1, 40)) + [0, 1, 31, 32, 33, small - 1, small]]
