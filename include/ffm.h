@@ -172,6 +172,9 @@ typedef struct ffm_run_stats {
     uint64_t prefilter_rest_bytes; /* bytes hashed beyond first chunks by the fused pass */
     double   ms_fused;          /* the fused hash + compare kernel alone (large payloads) */
     uint64_t two_pass;          /* 1 if the last run used the two-pass round 0 */
+    uint64_t n_reread;          /* residual members whose bytes were compared again; after a fused
+                                   round 0 the others are settled exactly through their difference
+                                   lists against the group head */
 } ffm_run_stats;
 
 /* Statistics of the last ffm_dedup_run. */

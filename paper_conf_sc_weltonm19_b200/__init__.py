@@ -56,7 +56,7 @@ class FfmRunStats(ctypes.Structure):
                [(k, ctypes.c_uint64) for k in ("n_records", "payload_bytes", "n_members", "n_residual",
                                                 "resolve_rounds", "kernel_launches", "hash_items",
                                                 "verify_items", "prefilter_rest_bytes")] + \
-               [("ms_fused", ctypes.c_double), ("two_pass", ctypes.c_uint64)]
+               [("ms_fused", ctypes.c_double), ("two_pass", ctypes.c_uint64), ("n_reread", ctypes.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

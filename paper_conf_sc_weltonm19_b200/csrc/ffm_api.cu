@@ -23,6 +23,8 @@ constexpr uint64_t kGatherMaxDefault = 1ull << 20;   // payloads up to this use 
 
 struct LocalRun {
     uint64_t n_members, n_res_total, rounds, prefilter_rest;
+    uint64_t n_reread;   // residual members whose bytes were compared again (not settled by difference lists)
+    uint64_t n_overflow; // round-0 residuals whose difference list against their head overflowed
     bool two_pass;
 };
 
@@ -319,6 +321,9 @@ void ensure_work(ffm_log* L, uint64_t n) {
         dev_alloc(W.gcount, c + 1);
         dev_alloc(W.pos, c);
         dev_alloc(W.fhead, c);
+        dev_alloc(W.dcnt, c);
+        dev_alloc(W.dq, (uint64_t)kDiffK * c);
+        dev_alloc(W.dv, (uint64_t)kDiffK * c);
         dev_alloc(W.sdesc, 2 * c);
         dev_alloc(W.hcount, c + 1);
         dev_alloc(W.hstart, c + 1);
@@ -530,14 +535,19 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         while (nres) {
             ++R.rounds;
             if (R.rounds > n + 2) throw CudaFail{cudaErrorUnknown, "collision resolution did not converge"};
-            ck(cudaMemsetAsync(W.counters, 0, sizeof(uint32_t), s), "memset");
+            ck(cudaMemsetAsync(W.counters, 0, 16 * sizeof(uint32_t), s), "memset");
             uint64_t capr = std::max<uint64_t>(1024, pow2_at_least(2 * nres));
-            LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)R.rounds, W.res[cur ^ 1], s));
+            // after a fused round 0 a large residual is first matched against its new
+            // leader through their difference lists (exact, no payload bytes re-read)
+            LCHK(launch_group(D, W, L->params, W.res[cur], (uint32_t)nres, capr, (int)R.rounds, W.res[cur ^ 1], s,
+                              !two_pass));
             LCHK(launch_verify(D, W, L->params, W.res[cur], (uint32_t)nres, W.res[cur ^ 1],
                                n_large ? W.vitem_cap : 0, s, nullptr, nullptr, nullptr));
-            ck(cudaMemcpyAsync(L->h_counters, W.counters, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+            ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
             ck(cudaStreamSynchronize(s), "round sync");
             nres = L->h_counters[0];
+            R.n_reread += L->h_counters[10];
+            if (R.rounds == 1) R.n_overflow = L->h_counters[11];
             R.n_res_total += nres;
             cur ^= 1;
         }
@@ -560,6 +570,7 @@ void fill_stats(ffm_log* L, const LocalRun& R, uint64_t launches, bool single) {
     S.hash_items = L->n_large_chunks;
     S.prefilter_rest_bytes = R.prefilter_rest;
     S.two_pass = R.two_pass ? 1 : 0;
+    S.n_reread = R.n_reread;
     if (timing) {
         S.ms_hash_small = ev_ms(L->ev[12], L->ev[8]);
         S.ms_hash_large = L->n_large_chunks ? ev_ms(L->ev[10], L->ev[11]) : 0.0;
@@ -885,7 +896,11 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         fill_stats(L, R, launches, true);
         // adaptive round 0: more than half of the candidates failed the fused compare
         // (near-duplicates sharing first chunks) -> hash-all-then-verify is cheaper
-        if (!R.two_pass && R.n_members >= 64 && 2 * R.n_res_total > R.n_members) L->prefer_two_pass = true;
+        // (residuals settled through difference lists cost no re-read: what counts are the
+        // members compared again, or residuals that differ from their head in many words --
+        // each of those pays the fused pass's mismatch path on every piece)
+        if (!R.two_pass && R.n_members >= 64 && 2 * std::max(R.n_reread, R.n_overflow) > R.n_members)
+            L->prefer_two_pass = true;
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
     } catch (const std::bad_alloc&) {

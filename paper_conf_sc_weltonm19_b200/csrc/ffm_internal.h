@@ -14,6 +14,7 @@ namespace ffm {
 constexpr uint32_t kArenaAlign = 32;         // record slots in the HBM arena (consecutive small records are contiguous)
 constexpr uint64_t kEmptyKey = ~0ull;         // group-by table: empty slot
 constexpr uint32_t kNoRecord = 0xFFFFFFFFu;
+constexpr uint32_t kDiffK = 4;                // difference-list entries kept per large member
 
 // Device-side views handed to the kernel launchers.
 struct DevLog {
@@ -50,6 +51,9 @@ struct Work {
     uint2* hitems = nullptr;       // large-payload hash work units (record, chunk)
     uint4* sdesc = nullptr;        // [2 * n] fused round 0: compare descriptors of small records (order position)
     uint4* fitems = nullptr;       // pipelined fused pass stage descriptors (2 x uint4 each)
+    uint32_t* dcnt = nullptr;      // [n] fused round 0: words where a large member differs from its group head
+    uint32_t* dq = nullptr;        // [n * kDiffK] their 16-B word indices (the first kDiffK recorded)
+    uint4* dv = nullptr;           // [n * kDiffK] the member's values of those words
     uint32_t* hcount = nullptr;    // [n+1] per-record hash chunk counts
     uint32_t* hstart = nullptr;    // [n+1] exclusive scan of hcount
     uint64_t* hpart = nullptr;     // [2 * hitem_cap] per-unit partial NH sums (A, B)
@@ -123,7 +127,7 @@ int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
                  cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b);
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
-                 uint64_t cap, int round, uint32_t* res_out, cudaStream_t st);
+                 uint64_t cap, int round, uint32_t* res_out, cudaStream_t st, bool use_diff = false);
 int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
                   uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st, cudaStream_t side, cudaEvent_t ev_fork,
                   cudaEvent_t ev_join);

@@ -343,14 +343,47 @@ __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ li
 // verify work of a class is laid out chunk-major: (chunk c, member p) at
 // lstart[leader] + c * gcount[leader] + p -- all members read leader chunk c back
 // to back, so the leader streams from HBM once and is re-read from L2.
+// Exact comparison of two large members of one fused round-0 group through their
+// difference lists against the group head h (k_fused_fx compared every word of both with
+// h): a == b iff D(a) == D(b) as sets of (word, value) -- at a word where one differs from
+// h the other must hold the same value, elsewhere both equal h.  Returns the first word
+// where they differ, ~0 if equal.
+__device__ __forceinline__ uint64_t diff_compare(const Work& W, uint32_t a, uint32_t b, uint32_t ca, uint32_t cb) {
+    uint64_t first = ~0ull;
+    for (uint32_t i = 0; i < ca; ++i) {
+        const uint32_t q = W.dq[(uint64_t)a * kDiffK + i];
+        const uint4 v = W.dv[(uint64_t)a * kDiffK + i];
+        bool same = false;
+        for (uint32_t j = 0; j < cb; ++j) {
+            if (W.dq[(uint64_t)b * kDiffK + j] != q) continue;
+            const uint4 u = W.dv[(uint64_t)b * kDiffK + j];
+            same = ((u.x ^ v.x) | (u.y ^ v.y) | (u.z ^ v.z) | (u.w ^ v.w)) == 0;
+        }
+        if (!same && q < first) first = q;
+    }
+    for (uint32_t j = 0; j < cb; ++j) {
+        const uint32_t q = W.dq[(uint64_t)b * kDiffK + j];
+        bool present = false;
+        for (uint32_t i = 0; i < ca; ++i) present |= W.dq[(uint64_t)a * kDiffK + i] == q;
+        if (!present && q < first) first = q;
+    }
+    return first;
+}
+
+// use_diff: resolve rounds after a fused round 0 -- a large member whose new leader
+// comes from the same round-0 group, both with complete difference lists, is settled
+// here (equal, or a residual with its exact first mismatching word) and not re-read.
 __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, uint32_t n_list, uint32_t small_bytes,
-                         uint32_t chunk_bytes, uint32_t* __restrict__ res_out) {
+                         uint32_t chunk_bytes, uint32_t* __restrict__ res_out, int use_diff) {
     uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     bool member = false;
     if (i < n_list) {
         uint32_t r = list ? list[i] : i;
         uint32_t ld = W.tval[W.slot[r]];
         W.leader[r] = ld;
+        // residuals whose difference list overflowed: heavy mismatch against their head
+        // (the adaptive round-0 choice, run_local)
+        if (use_diff && L.size[r] > small_bytes && W.dcnt[r] > kDiffK) atomicAdd(&W.counters[11], 1u);
         if (ld != r) {
             member = true;
             uint64_t n = L.size[r];
@@ -364,8 +397,25 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
                 W.mis[r] = ~0ull;
             }
             if (n > small_bytes && L.size[ld] == n && L.chan[ld] == L.chan[r]) {
-                atomicAdd(&W.lcount[ld], (uint32_t)((n + chunk_bytes - 1) / chunk_bytes));
-                W.pos[r] = atomicAdd(&W.gcount[ld], 1u);
+                bool settled = false;
+                if (use_diff && W.fhead[r] == W.fhead[ld]) {
+                    const uint32_t ca = W.dcnt[r], cb = W.dcnt[ld];
+                    if (ca <= kDiffK && cb <= kDiffK) {
+                        settled = true;
+                        W.pos[r] = 0xFFFFFFFFu;   // no verify work (k_fx_vfill skips it)
+                        const uint64_t first = diff_compare(W, r, ld, ca, cb);
+                        if (first != ~0ull) {
+                            W.eq[r] = 0;
+                            W.mis[r] = first;
+                            res_out[atomicAdd(&W.counters[0], 1u)] = r;
+                        }
+                    }
+                }
+                if (!settled) {   // compare the bytes again (k_fx_vfill + k_fused_fx verify mode)
+                    atomicAdd(&W.lcount[ld], (uint32_t)((n + chunk_bytes - 1) / chunk_bytes));
+                    W.pos[r] = atomicAdd(&W.gcount[ld], 1u);
+                    atomicAdd(&W.counters[10], 1u);
+                }
             }
         }
     }
@@ -583,7 +633,7 @@ __global__ void k_fx_vfill(DevLog L, Work W, const uint32_t* __restrict__ list, 
     const FxSplit f = fx_split(chunk_bytes);
     FFM_WARP_EACH(list ? n_list : L.n_large, list ? list[w_] : L.large_order[w_],
                   (W.leader[rec] != rec && L.size[rec] > small_bytes && L.size[W.leader[rec]] == L.size[rec] &&
-                   L.chan[W.leader[rec]] == L.chan[rec]), {
+                   L.chan[W.leader[rec]] == L.chan[rec] && W.pos[rec] != 0xFFFFFFFFu), {
         const uint32_t ld = W.leader[rec];
         const uint32_t k = W.gcount[ld] + 1, p = W.pos[rec] + 1, base = W.lstart[ld];
         const uint32_t S = fx_subtasks(k), K = k - 1 + S;
@@ -633,6 +683,7 @@ __global__ void k_fx_fill(DevLog L, Work W, uint32_t chunk_bytes, uint32_t prefi
         const uint32_t np = fx_pieces(f, n), hs = W.hstart[rec];
         const bool skip_all = prefilter && prefix_unique(W, rec);
         const uint32_t last0 = min(k - 1, kFxMaxK - 1);      // position ending sub-task 0
+        if (lane == 0) W.dcnt[rec] = 0;                       // difference list vs the head (k_fused_fx)
         for (uint32_t t = lane; t < np; t += 32) {
             const uint32_t c = t / f.ppc, j = t - c * f.ppc;
             uint64_t st = (uint64_t)c * f.chunk + (uint64_t)j * f.ps;
@@ -874,6 +925,36 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
             if (__any_sync(0xFFFFFFFFu, dmask != 0)) {
                 // rare: a near-duplicate or a collision -- first mismatching word and NH deltas
                 uint64_t found = dmask ? (uint64_t)(w0 + t + kStride * (__ffs(dmask) - 1)) : ~0ull;
+                if (!kVerify) {
+                    // the member's difference list against its head (every word of a group
+                    // member is compared in round 0): its count, and the (word, value) pairs
+                    // while they fit -- one atomic per warp, none once the list overflowed
+                    uint32_t cur = 0;
+                    if (lane == 0) cur = *reinterpret_cast<const volatile uint32_t*>(&W.dcnt[rec]);
+                    cur = __shfl_sync(0xFFFFFFFFu, cur, 0);
+                    if (cur <= kDiffK) {
+                        const uint32_t nd = __popc(dmask);
+                        uint32_t incl = nd;
+#pragma unroll
+                        for (int o = 1; o < 32; o <<= 1) {
+                            const uint32_t v = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+                            if (lane >= o) incl += v;
+                        }
+                        uint32_t base = 0;
+                        if (lane == 31) base = atomicAdd(&W.dcnt[rec], incl);
+                        base = __shfl_sync(0xFFFFFFFFu, base, 31);
+                        uint32_t sl = base + incl - nd;
+#pragma unroll
+                        for (int u = 0; u < kFxWords; ++u) {
+                            if (!(dmask & (1u << u))) continue;
+                            if (sl < kDiffK) {
+                                W.dq[(uint64_t)rec * kDiffK + sl] = w0 + t + kStride * u;
+                                W.dv[(uint64_t)rec * kDiffK + sl] = y[u];
+                            }
+                            ++sl;
+                        }
+                    }
+                }
                 uint64_t dA = 0, dB = 0;
                 if ((flags & kFxDelta) && dmask) {
                     uint64_t xA = 0, xB = 0;
@@ -1497,7 +1578,7 @@ uint64_t fx_entry_cap(uint64_t n_large_chunks, uint32_t chunk_bytes) {
 }
 
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list, uint64_t cap,
-                 int round, uint32_t* res_out, cudaStream_t st) {
+                 int round, uint32_t* res_out, cudaStream_t st, bool use_diff) {
     if (n_list == 0) return 0;
     int k = 0;
     if (round > 0) {
@@ -1515,9 +1596,10 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
     if (round == 0)
         k_leader0<<<blocks_for(n_list), 256, 0, st>>>(L, W, n_list, P.small_bytes, res_out);
     else if (round < 0)
-        k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, nullptr, n_list, P.small_bytes, P.chunk_bytes, res_out);
+        k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, nullptr, n_list, P.small_bytes, P.chunk_bytes, res_out, 0);
     else
-        k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes, res_out);
+        k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, P.small_bytes, P.chunk_bytes, res_out,
+                                                     use_diff ? 1 : 0);
     FFM_LAUNCH_CHECK();
     return k + 2;
 }

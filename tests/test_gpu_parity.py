@@ -401,9 +401,10 @@ def test_two_pass_round0(ffm, digest_bits):
         assert_same(lg, dup, ben)
 
 
-def test_adaptive_round0(ffm):
-    """Near-duplicates sharing first chunks make the fused round 0 mismatch: the log
-    switches itself to two-pass after one run; outputs never change."""
+def test_difference_lists_settle_near_duplicates(ffm):
+    """Config 3 shape: single-byte near-duplicates share their first 4 KiB with a base, so
+    they mismatch it in the fused pass; their re-uploads are then settled exactly through
+    the difference lists against the base (no bytes re-read), and the log stays fused."""
     lg = loggen.gen_config(3, n_scale=0.05, size_scale=1 / 8)
     want = oracle.dedup(lg)
     with ffm.FfmLog(lg.n_sites, timing=True) as log:
@@ -412,7 +413,46 @@ def test_adaptive_round0(ffm):
         s1 = log.stats()
         d2, b2 = [x.copy() for x in log.run()]
         s2 = log.stats()
+    assert s1["two_pass"] == 0 and s2["two_pass"] == 0
+    assert s1["n_residual"] > 0 and s1["n_reread"] * 10 <= s1["n_residual"]
+    for d, b in ((d1, b1), (d2, b2)):
+        np.testing.assert_array_equal(d, want[0])
+        np.testing.assert_array_equal(b, want[1])
+
+
+def _many_word_near_dups(seed, n_bases=6, n_var=8, reps=4, size=64 * 1024 + 48, words=9):
+    """Variants of a few bases, each differing from its base in `words` 16-byte words past
+    the first 4 KiB (more than a difference list holds), each uploaded `reps` times."""
+    rng = np.random.default_rng(seed)
+    pay = []
+    for _ in range(n_bases):
+        base = rng.integers(0, 256, size, dtype=np.uint8)
+        pay.append(base.tobytes())
+        for _ in range(n_var):
+            v = base.copy()
+            for q in rng.choice(np.arange(4096 // 16 + 1, size // 16), words, replace=False):
+                v[16 * q + int(rng.integers(0, 16))] ^= 0xA5
+            pay += [v.tobytes()] * reps
+    order = rng.permutation(len(pay))
+    order = np.concatenate([[i for i in order if i % (n_var * reps + 1) == 0],
+                            [i for i in order if i % (n_var * reps + 1) != 0]])   # bases first
+    pay = [pay[i] for i in order]
+    return loggen.from_payloads(pay, rng.integers(0, 3, len(pay)), rng.integers(0, 1 << 40, len(pay)), 3)
+
+
+def test_adaptive_round0(ffm):
+    """Near-duplicates whose difference lists overflow must be re-read in the resolve
+    rounds: the log switches itself to two-pass after one run; outputs never change."""
+    lg = _many_word_near_dups(5)
+    want = oracle.dedup(lg)
+    with ffm.FfmLog(lg.n_sites, timing=True, chunk_bytes=16384) as log:
+        log.append_log(lg)
+        d1, b1 = [x.copy() for x in log.run()]
+        s1 = log.stats()
+        d2, b2 = [x.copy() for x in log.run()]
+        s2 = log.stats()
     assert s1["two_pass"] == 0 and s2["two_pass"] == 1
+    assert 2 * s1["n_reread"] > s1["n_members"]
     for d, b in ((d1, b1), (d2, b2)):
         np.testing.assert_array_equal(d, want[0])
         np.testing.assert_array_equal(b, want[1])
@@ -421,6 +461,18 @@ def test_adaptive_round0(ffm):
         log.run()
         log.run()
         assert log.stats()["two_pass"] == 0
+
+
+@pytest.mark.parametrize("words", [1, 3, 4, 5, 9])
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_difference_list_sizes(ffm, words, digest_bits):
+    """Variants differing from their base in 1..9 words (the list holds 4): settled
+    through lists up to 4, re-read beyond; exact either way."""
+    lg = _many_word_near_dups(11 + words, n_bases=3, n_var=5, reps=3, words=words)
+    dup, ben, st = gpu_dedup(ffm, lg, digest_bits=digest_bits, chunk_bytes=16384, fused=True)
+    assert_same(lg, dup, ben)
+    if digest_bits == 64 and words <= 4:
+        assert st["n_reread"] == 0 and st["n_residual"] > 0
 
 
 def test_benefit_linear_in_durations(ffm):
