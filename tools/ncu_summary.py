@@ -75,7 +75,7 @@ def main():
              "|---|---|---|---|---|---|---|---|---|"]
     summ = {}
     for name, ds in k.items():
-        d = ds[-1]
+        d = max(ds, key=lambda x: x.get("gpu__time_duration.sum", 0))   # the kernel's dominant launch
         rb, wb = d.get("dram__bytes_read.sum", 0), d.get("dram__bytes_write.sum", 0)
         lines.append(f"| {name} | {d.get('gpu__time_duration.sum', 0) * 1e3:.3f} | {rb / 1e9:.3f} | {wb / 1e9:.3f} | "
                      f"{d.get('gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed', 0):.1f} | "
@@ -85,7 +85,7 @@ def main():
                                       "ms": d.get("gpu__time_duration.sum", 0) * 1e3,
                                       "source": os.path.basename(rep)}
     open(prefix + "_kernels.md", "w").write(
-        f"# ncu --set full ({os.path.basename(rep)}; last captured launch per kernel)\n\n" + "\n".join(lines) + "\n")
+        f"# ncu --set full ({os.path.basename(rep)}; longest captured launch per kernel)\n\n" + "\n".join(lines) + "\n")
     jpath = os.path.join(root, "profiles", "ncu_summary.json")
     try:
         doc = json.load(open(jpath))
