@@ -192,9 +192,12 @@ void upload_order(ffm_log* L, const std::vector<uint32_t>& order, uint32_t*& dpt
         if (dptr) ck(cudaFree(dptr), "cudaFree");
         dptr = nullptr;
         cap = std::max<uint64_t>(std::max<uint64_t>(ns, 2 * cap), 1024);
-        ck(cudaMalloc(&dptr, cap * sizeof(uint32_t)), "cudaMalloc(order)");
+        ck(cudaMalloc(&dptr, 2 * cap * sizeof(uint32_t)), "cudaMalloc(order)");   // order, then its inverse
     }
-    if (ns) ck(cudaMemcpyAsync(dptr, order.data(), ns * 4, cudaMemcpyHostToDevice, s), "order H2D");
+    if (ns) {
+        ck(cudaMemcpyAsync(dptr, order.data(), ns * 4, cudaMemcpyHostToDevice, s), "order H2D");
+        if (launch_invert(dptr, (uint32_t)ns, dptr + cap, s) < 0) throw CudaFail{cudaGetLastError(), "invert order"};
+    }
 }
 
 void upload_meta(ffm_log* L) {
@@ -379,6 +382,7 @@ DevLog dev_view(const ffm_log* L) {
     d.chan = L->d_chan;
     d.n = (uint32_t)L->h_size.size();
     d.small_order = L->d_small_order;
+    d.order_pos = L->d_small_order ? L->d_small_order + L->d_small_cap : nullptr;
     d.n_small = (uint32_t)L->n_small;
     d.large_order = L->d_small_order ? L->d_small_order + L->n_small : nullptr;
     d.n_large = (uint32_t)L->n_large_rec;
@@ -1151,6 +1155,7 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
             const uint64_t nsw = build_small_order(L, w0, n, order);
             upload_order(L, order, L->d_win_order, L->d_win_cap, s);
             D.small_order = L->d_win_order;
+            D.order_pos = L->d_win_order + L->d_win_cap;
             D.n_small = (uint32_t)nsw;
             D.large_order = L->d_win_order + nsw;
             D.n_large = (uint32_t)(order.size() - nsw);

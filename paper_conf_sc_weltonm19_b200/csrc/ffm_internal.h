@@ -27,6 +27,7 @@ struct DevLog {
     const uint64_t* chan;    // [n] channel (direction / destination) id, 0 = content only
     uint32_t n;
     const uint32_t* small_order;  // records <= small_bytes, sorted by block count (descending)
+    const uint32_t* order_pos;    // inverse of small_order (+ large_order): position of record r
     uint32_t n_small;
     const uint32_t* large_order;  // records > small_bytes, ascending
     uint32_t n_large;
@@ -152,6 +153,7 @@ int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, 
                        cudaStream_t st);
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
+int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t st);
 size_t cub_scan_bytes(uint64_t n);
 uint64_t fx_entry_cap(uint64_t n_large_chunks, uint32_t chunk_bytes);
 uint32_t blocks_for(uint64_t threads, uint32_t bs = 256);

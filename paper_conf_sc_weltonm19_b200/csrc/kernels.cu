@@ -429,12 +429,13 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
 // with the leader itself at p = 0 -- the leader's chunk c is read from HBM once, by
 // its own hashing unit, and re-read from L2 by every member comparing against it.
 __global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, uint32_t* __restrict__ res_out) {
-    // thread i: record order[i] (small records in size-class order, then large ones), so
-    // a small record's compare descriptor lands at its position in k_fused_small's order
-    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    // thread r: record r (gid order: its metadata loads and per-record writes coalesce);
+    // a small record's compare descriptor lands at its position i in k_fused_small's
+    // size-class order
+    const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
     bool member = false;
-    if (i < n) {
-        const uint32_t r = L.small_order[i];
+    if (r < n) {
+        const uint32_t i = L.order_pos[r];
         const uint32_t ld = W.tval[W.slot[r]];
         W.leader[r] = ld;
         const uint64_t sz = L.size[r];
@@ -1699,6 +1700,18 @@ int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream
     uint32_t grid = blocks_for((uint64_t)n * 32);
     if (grid > 148u * 16) grid = 148u * 16;
     k_gather<<<grid, 256, 0, st>>>(d_desc, n, arena);
+    FFM_LAUNCH_CHECK();
+    return 1;
+}
+
+__global__ void k_invert(const uint32_t* __restrict__ order, uint32_t n, uint32_t* __restrict__ inv) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) inv[order[i]] = i;
+}
+
+int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t st) {
+    if (n == 0) return 0;
+    k_invert<<<blocks_for(n), 256, 0, st>>>(order, n, inv);
     FFM_LAUNCH_CHECK();
     return 1;
 }
