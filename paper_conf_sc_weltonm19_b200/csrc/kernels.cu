@@ -1144,6 +1144,225 @@ __global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const
 // cross-shard / online merges need it) and, for a member of a prefix group, byte-compares
 // it with the group's leader -- re-uploads of one content share their leader, so its
 // bytes are L2-hot; the member's own bytes are read from HBM once.
+#ifndef FFM_SMALL_ASYNC   // 1: per-lane cp.async pipeline (default), 0: register octet kernel
+#define FFM_SMALL_ASYNC 1
+#endif
+#if FFM_SMALL_ASYNC
+// Per-thread cp.async pipeline: every lane is its own producer.  A lane's work is the
+// sequence of steps (record, 16*U 16-byte words of it) of its octet; it keeps S-1 steps
+// of its own and its leader's words in flight in shared memory (cp.async, no registers
+// held) while it hashes and compares the oldest, across record boundaries.  Default
+// U=2, S=2, 128 threads: 37 KB per CTA, 6 CTAs (24 warps) per SM -- occupancy beat depth
+// (S=3 / S=4 / U=1 / U=3 measured slower, profiles/r01e/README.md).
+// Lane g takes words g, g+8 of each 256-byte stripe (one warp instruction = 128
+// contiguous bytes per octet); NH is a positional sum, so the digest is unchanged.
+// Each lane reads back only what it copied itself: cp.async.wait_group is the only ordering.
+#ifndef FFM_SA_U
+#define FFM_SA_U 2
+#endif
+#ifndef FFM_SA_S
+#define FFM_SA_S 2
+#endif
+#ifndef FFM_SA_T
+#define FFM_SA_T 128
+#endif
+constexpr int kSaU = FFM_SA_U, kSaS = FFM_SA_S, kSaT = FFM_SA_T, kSaJ = 2 * kSaU;   // words per lane per step
+constexpr int kSaSmem = kSaS * kSaT * 16 * (2 * kSaJ + 1);                          // 16-B slots: data, then meta
+constexpr uint32_t kSaEnd = 1u << 31, kSaFirst = 1u << 30, kSaLast = 1u << 29, kSaCmp = 1u << 28;
+
+__device__ __forceinline__ void cp16(uint32_t dst, const uint8_t* src, uint64_t pol) {
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "l"(pol)
+                 : "memory");
+}
+
+__device__ __forceinline__ void lds16(uint32_t a, uint32_t* v) {
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(a)
+                 : "memory");
+}
+
+// zero the bytes of 16-byte word w at or beyond n
+__device__ __forceinline__ void mask_word(uint32_t* v, uint32_t n, uint32_t w) {
+    const int32_t valid = (int32_t)n - (int32_t)(16 * w);
+    if (valid >= 16) return;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int32_t vb = valid - 4 * i;
+        v[i] &= vb >= 4 ? 0xFFFFFFFFu : (vb <= 0 ? 0u : ((1u << (8 * vb)) - 1u));
+    }
+}
+
+__global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t* res_out) {
+    extern __shared__ __align__(16) uint8_t sa_smem[];
+    const int g = threadIdx.x & 7;
+    const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
+    const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
+    const unsigned omask = 0xFFu << (threadIdx.x & 24);
+    const uint32_t sbase = smem_u32(sa_smem) + threadIdx.x * 16;
+    // slot of word j of stage s (part 0 own, 1 leader); lanes interleaved so a warp's
+    // 16-B accesses to one slot are 512 contiguous bytes (conflict-free)
+    auto slot = [&](int s, int j, int part) { return sbase + (uint32_t)(((s * kSaJ + j) * 2 + part) * kSaT * 16); };
+    auto mslot = [&](int s) { return sbase + (uint32_t)((kSaS * kSaJ * 2 + s) * kSaT * 16); };
+    uint64_t pol_own, pol_keep;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_own));
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
+
+    // ---- producer state: current record (position fi, next word fw0) + next descriptor
+    uint32_t fi = oct, fw0 = 0;
+    uint64_t foff = 0, floff = 0;
+    uint32_t fn = 0, fr = 0;
+    uint4 da = make_uint4(0, 0, 0, 0), db = make_uint4(0, 0, 0, 0);
+    if (fi < L.n_small) {
+        const uint4 a = W.sdesc[2ull * fi], b = W.sdesc[2ull * fi + 1];
+        foff = (uint64_t)a.y << 32 | a.x;
+        floff = (uint64_t)a.w << 32 | a.z;
+        fn = b.x;
+        fr = b.y;
+        if (fi + noct < L.n_small) {
+            da = W.sdesc[2ull * (fi + noct)];
+            db = W.sdesc[2ull * (fi + noct) + 1];
+        }
+    }
+    auto fetch = [&](int s) {
+        uint32_t meta_z = kSaEnd;
+        uint32_t mn = 0, mr = 0;
+        if (fi < L.n_small) {
+            const uint32_t nw = (fn + 15) >> 4;
+            const bool cmp = floff != ~0ull;
+            const uint8_t* src = L.arena + foff;
+            const uint8_t* lsrc = L.arena + (cmp ? floff : foff);
+            if (fw0 + 8 * kSaJ <= nw) {   // every lane's words exist
+#pragma unroll
+                for (int j = 0; j < kSaJ; ++j) cp16(slot(s, j, 0), src + 16ull * (fw0 + 8 * j + g), pol_own);
+                if (cmp) {
+#pragma unroll
+                    for (int j = 0; j < kSaJ; ++j) cp16(slot(s, j, 1), lsrc + 16ull * (fw0 + 8 * j + g), pol_keep);
+                }
+            } else {
+#pragma unroll
+                for (int j = 0; j < kSaJ; ++j) {
+                    const uint32_t w = fw0 + 8 * j + g;
+                    if (w < nw) {
+                        cp16(slot(s, j, 0), src + 16ull * w, pol_own);
+                        if (cmp) cp16(slot(s, j, 1), lsrc + 16ull * w, pol_keep);
+                    }
+                }
+            }
+            meta_z = fw0 | (fw0 == 0 ? kSaFirst : 0u) | (cmp ? kSaCmp : 0u);
+            mn = fn;
+            mr = fr;
+            fw0 += 8 * kSaJ;
+            if (fw0 >= nw) {   // last step of this record: move to the next one
+                meta_z |= kSaLast;
+                fi += noct;
+                fw0 = 0;
+                foff = (uint64_t)da.y << 32 | da.x;
+                floff = (uint64_t)da.w << 32 | da.z;
+                fn = db.x;
+                fr = db.y;
+                if (fi + noct < L.n_small) {
+                    da = W.sdesc[2ull * (fi + noct)];
+                    db = W.sdesc[2ull * (fi + noct) + 1];
+                }
+            }
+        }
+        asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(mslot(s)), "r"(mn), "r"(mr), "r"(meta_z), "r"(0u)
+                     : "memory");
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+#pragma unroll 1
+    for (int s = 0; s < kSaS - 1; ++s) fetch(s);
+
+    // ---- consumer state
+    LaneKeys K;   // k[0]: stripe position g, k[1]: position g + 8
+    uint64_t A = 0, B = 0, found = ~0ull;
+    int sc = 0, sf = kSaS - 1;
+#pragma unroll 1
+    while (true) {
+        // refill the stage consumed last iteration (its values were used, so read), then
+        // wait for the oldest: S-1 steps stay in flight while this one is hashed
+        fetch(sf);
+        asm volatile("cp.async.wait_group %0;" ::"n"(kSaS - 1) : "memory");
+        uint32_t m[4];
+        lds16(mslot(sc), m);
+        const uint32_t n = m[0], r = m[1], z = m[2];
+        if (z & kSaEnd) break;
+        if (z & kSaFirst) {
+            A = 0;
+            B = 0;
+            found = ~0ull;
+#pragma unroll
+            for (int jj = 0; jj < 6; ++jj) {
+                K.k[0][jj] = c_nh.ka[g][jj];
+                K.k[1][jj] = c_nh.ka[g + 8][jj];
+            }
+        }
+        const uint32_t w0 = z & 0x0FFFFFFFu, nw = (n + 15) >> 4;
+        const bool cmp = z & kSaCmp;
+        if (16 * (w0 + 8 * kSaJ) <= n) {   // fast path: every word whole -- no masks, OR-reduced compare
+            uint32_t d = 0;
+#pragma unroll
+            for (int j = 0; j < kSaJ; ++j) {
+                uint32_t x[4];
+                lds16(slot(sc, j, 0), x);
+                nh_word(x[0], x[1], x[2], x[3], K.k[j & 1], A, B);
+                if (cmp) {
+                    uint32_t y[4];
+                    lds16(slot(sc, j, 1), y);
+                    d |= (x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3]);
+                }
+                if (j & 1) advance<1>(K);
+            }
+            if (d && found == ~0ull) {   // rare: the lowest differing word of this step
+#pragma unroll 1
+                for (int j = 0; j < kSaJ; ++j) {
+                    uint32_t x[4], y[4];
+                    lds16(slot(sc, j, 0), x);
+                    lds16(slot(sc, j, 1), y);
+                    if ((x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3])) {
+                        found = w0 + 8 * j + g;
+                        break;
+                    }
+                }
+            }
+        } else
+#pragma unroll
+        for (int j = 0; j < kSaJ; ++j) {
+            const uint32_t w = w0 + 8 * j + g;
+            if (w < nw) {
+                uint32_t x[4];
+                lds16(slot(sc, j, 0), x);
+                mask_word(x, n, w);
+                nh_word(x[0], x[1], x[2], x[3], K.k[j & 1], A, B);
+                if (cmp) {
+                    uint32_t y[4];
+                    lds16(slot(sc, j, 1), y);
+                    mask_word(y, n, w);
+                    if (((x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3])) && found == ~0ull) found = w;
+                }
+            }
+            if (j & 1) advance<1>(K);
+        }
+        if (z & kSaLast) {
+#pragma unroll
+            for (int o = 4; o; o >>= 1) {
+                A += __shfl_xor_sync(omask, A, o);
+                B += __shfl_xor_sync(omask, B, o);
+                const uint64_t of = __shfl_xor_sync(omask, found, o);
+                found = of < found ? of : found;
+            }
+            if (g == 0) {
+                W.accA[r] = A;
+                W.accB[r] = B;
+                W.digest[r] = finalize_digest(A, B, n);
+                if (found != ~0ull) report_mismatch(W, r, found, res_out, false);
+            }
+        }
+        sc = sc + 1 == kSaS ? 0 : sc + 1;
+        sf = sf + 1 == kSaS ? 0 : sf + 1;
+    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+}
+#else
 __global__ void __launch_bounds__(256, FFM_SMALL_MINB) k_fused_small(DevLog L, Work W, uint32_t* res_out) {
     const int g = threadIdx.x & 7;
     const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
@@ -1261,6 +1480,7 @@ __global__ void __launch_bounds__(256, FFM_SMALL_MINB) k_fused_small(DevLog L, W
         }
     }
 }
+#endif  // FFM_SMALL_ASYNC
 
 // ----------------------------------------------------------------------------
 // H4: re-key residual members.  Round 1 refines by the full, untruncated NH sums;
@@ -1497,9 +1717,20 @@ int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_
     if (L.n == 0 || L.n_small == 0) return 0;
     // (measured: capping its grid so that it co-resides with the persistent large pass
     // slowed that pass more than it hid -- profiles/r01b/README.md)
+#if FFM_SMALL_ASYNC
+    if (!smem_configured((const void*)k_fused_small, kSaSmem)) return -1;
+    static int occ = 0;   // per process: one device type
+    if (occ == 0 && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fused_small, kSaT, kSaSmem) != cudaSuccess ||
+                     occ < 1))
+        occ = 1;
+    uint32_t grid = (uint32_t)(occ * P.num_sms);
+    uint32_t need = blocks_for((uint64_t)L.n_small * 8, kSaT);
+    k_fused_small<<<need < grid ? need : grid, kSaT, kSaSmem, st>>>(L, W, res_out);
+#else
     uint32_t grid = resident_grid((const void*)k_fused_small, P.num_sms);
     uint32_t need = blocks_for((uint64_t)L.n_small * 8);
     k_fused_small<<<need < grid ? need : grid, 256, 0, st>>>(L, W, res_out);
+#endif
     FFM_LAUNCH_CHECK();
     return 1;
 }
