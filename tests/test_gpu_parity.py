@@ -539,3 +539,24 @@ def test_graph_replay_matches_direct_launches(ffm):
                 log.run(dd, bb)
                 np.testing.assert_array_equal(dd.cpu().numpy(), want[0])
                 np.testing.assert_array_equal(bb.cpu().numpy().view(np.uint64), want[1])
+
+
+def test_empty_log_and_all_empty_payloads(ffm):
+    """Degenerate logs (S8(c) edge cases): no records at all -> empty duplicate_of, zero
+    benefit; 5000 empty payloads over 7 sites (several thread blocks) -> each one after the
+    first duplicates record 0 (reading R7), benefit = the sites' duration sums
+    minus the first record's."""
+    with ffm.FfmLog(3) as log:
+        dup, ben = log.run()
+    assert dup.tolist() == [] and ben.tolist() == [0, 0, 0]
+    n = 5000
+    sites = [i % 7 for i in range(n)]
+    durs = [1000 + 3 * i for i in range(n)]
+    with ffm.FfmLog(7) as log:
+        log.append_batch(sites, [0] * n, [0] * n, durs)
+        dup, ben = log.run()
+    assert dup.tolist() == [-1] + [0] * (n - 1)
+    want = [0] * 7
+    for i in range(1, n):
+        want[sites[i]] += durs[i]
+    assert ben.tolist() == want
