@@ -3,13 +3,19 @@
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload 5] [--impl ours|reference]
 
+--gpus N > 1 without a torchrun environment re-launches itself as N ranks (one per
+GPU) under torch.distributed.run; ffm_dedup_run is then collective over the library's
+own NCCL communicator.
+
 A step = one ffm_dedup_run over the whole log (H1 hash .. H7 labels/benefit, all
 of SURVEY.md 8(a)) with the payloads already resident in HBM.  Default workload
 = BASELINE config 5 (the ~64 GB mixed application-shaped log, 2 M transfers,
 10k call sites) on one GPU; inputs (63 GB) are far larger than L2 (126 MB).
 
-  value    = sum of payload bytes / device time per step (CUDA events on the
-             library's stream), GB/s (1e9).
+  value    = sum of payload bytes / time per step (CUDA events on the library's
+             stream, max over ranks), GB/s (1e9); every run writes duplicate_of /
+             benefit_ns into pinned HOST arrays (the D2H is inside the step, SURVEY.md
+             8(d) T_run); value_device_outputs keeps them in HBM.
   e2e      = the same metric through the public C ABI from pinned HOST buffers:
              ffm_log_create + ffm_log_append_batch (H2D of every payload) +
              ffm_dedup_run + D2H of duplicate_of / benefit_ns, per step.
@@ -183,23 +189,33 @@ def ncu_traffic(kernel, capture):
         return None
 
 
+def make_ffm_log(args, lg, n_records, my_bytes, rank, world, local, **kw):
+    """This rank's log: one GPU, or a sharded world (collective: the library's NCCL
+    communicator across GPUs; the host transport when ranks share a GPU)."""
+    import paper_conf_sc_weltonm19_b200 as ffm
+    from paper_conf_sc_weltonm19_b200 import sharded
+    opts = dict(arena_bytes=my_bytes + 128 * n_records + (1 << 20), max_records=n_records, **kw)
+    if world == 1:
+        return ffm.FfmLog(lg.n_sites, device=local, **opts)
+    return sharded.create_sharded_log(lg.n_sites, local, transport="host" if args.same_device else "nccl", **opts)
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
-    import paper_conf_sc_weltonm19_b200 as ffm
-    from paper_conf_sc_weltonm19_b200 import sharded
 
     rank, world, local = dist_env()
-    if os.environ.get("FFM_BENCH_SAME_DEVICE"):      # test hook: several ranks on one GPU
+    if args.same_device:                 # test hook: several ranks on one GPU
         local = 0
+    elif world > 1 and torch.cuda.device_count() < world:
+        raise SystemExit(f"bench: {world} ranks but {torch.cuda.device_count()} visible GPUs "
+                         "(--same-device runs them on one GPU, host transport)")
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        backend = os.environ.get("FFM_BENCH_BACKEND", "nccl")   # gloo only to exercise N>1 on one GPU
-        if backend == "nccl":
-            dist.init_process_group("nccl", device_id=dev)
-        else:
-            dist.init_process_group(backend)
+        # bootstrap / host-side timing reduction only; the data plane is the library's
+        # own NCCL communicator (or its host transport under --same-device)
+        dist.init_process_group("gloo")
     lg = make_log(args.workload, args.n_scale, args.size_scale, shard=(rank, world))
     idx = lg.shard_idx
     total = lg.total_bytes                      # the whole job's payload (strong scaling)
@@ -210,58 +226,72 @@ def run_ours(args):
     t = time.time()
     content = torch.from_numpy(lg.buf).to(dev)
     ptrs = (lg.c_off[lg.content] + np.uint64(content.data_ptr())).astype(np.uint64)
-    log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * len(idx) + (1 << 20),
-                     max_records=len(idx), timing=True, rank=rank, world=world,
-                     prefilter=args.prefilter and world == 1, digest_bits=args.digest_bits,
-                     two_pass=args.two_pass)
+    import paper_conf_sc_weltonm19_b200 as ffm
+    log = make_ffm_log(args, lg, len(idx), my_bytes, rank, world, local, timing=True,
+                       prefilter=args.prefilter and world == 1, digest_bits=args.digest_bits,
+                       two_pass=args.two_pass)
     log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE,
                    gids=idx if world > 1 else None, idx=idx if world > 1 else None)
     del content
     torch.cuda.synchronize()
     torch.cuda.empty_cache()
-    if world > 1:
-        sharded.exchange_handles(log)
     log_msg(f"[bench] rank {rank}: staged {my_bytes / 1e9:.2f} GB ({len(idx)} records) into HBM "
             f"in {time.time() - t:.1f}s")
 
-    dup = torch.empty(max(len(idx), 1), dtype=torch.int64, device=dev)
-    ben = torch.empty(lg.n_sites, dtype=torch.int64, device=dev)
-    reps = torch.empty((max(len(idx), 1), ffm.REP_WORDS), dtype=torch.int64, device=dev)
+    n = len(idx)
+    # outputs: host (pinned) arrays -- the D2H of duplicate_of / benefit_ns is inside the
+    # timed run (SURVEY.md 8(d) T_run); device arrays for the kernel-side figure
+    dup_h = torch.empty(max(n, 1), dtype=torch.int64).pin_memory()
+    ben_h = torch.empty(lg.n_sites, dtype=torch.int64).pin_memory()
+    dup_hn, ben_hn = dup_h.numpy(), ben_h.numpy().view(np.uint64)
+    dup_d = torch.empty(max(n, 1), dtype=torch.int64, device=dev)
+    ben_d = torch.empty(lg.n_sites, dtype=torch.int64, device=dev)
 
-    def step():
-        if world > 1:
-            sharded.dedup_sharded(log, dev, duplicate_of=dup, benefit=ben, reps_buf=reps)
+    def step(host=True):
+        if host:
+            log.run(dup_hn, ben_hn)
         else:
-            log.run(dup, ben)
+            log.run(dup_d, ben_d)
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t_ = torch.tensor([x], dtype=torch.float64)
+        dist.all_reduce(t_, op=dist.ReduceOp.MAX)
+        return float(t_.item())
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
 
     stream = torch.cuda.ExternalStream(log.stream, device=dev)
     for _ in range(args.warmup):
         step()
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
+    barrier()
     clocks = ClockSampler(local) if rank == 0 else None
     if clocks:
         clocks.start()
         time.sleep(0.3)
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    # measured steps: production runs (CUDA-graph replay, no per-stage events)
+    # measured steps: production runs (CUDA-graph replay, no per-stage events), events on
+    # the library's stream (every kernel, collective and output copy of a run is on it)
     log.set_timing(False)
     step()
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    e0.record(stream)
-    for _ in range(args.steps):
-        step()
-    e1.record(stream)
-    torch.cuda.synchronize()
-    ms_local = e0.elapsed_time(e1) / args.steps
-    ms = ms_local
-    if world > 1:
-        t_ms = torch.tensor([ms_local], dtype=torch.float64, device=dev)
-        dist.all_reduce(t_ms, op=dist.ReduceOp.MAX)
-        ms = float(t_ms.item())
+
+    def timed(host):
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            step(host)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / args.steps
+
+    ms_local = timed(True)
+    ms = max_over_ranks(ms_local)
+    ms_dev_local = timed(False)
+    ms_dev = max_over_ranks(ms_dev_local)
     clk = clocks.stop() if clocks else None
     launches = int(log.stats()["kernel_launches"]) * args.steps
     # instrumented steps (per-stage CUDA events on the library's stream) for the kernel
@@ -270,34 +300,33 @@ def run_ours(args):
     acc = {}
     n_instr = max(3, min(args.steps, 5))
     for _ in range(n_instr):
-        step()
+        step(False)
         for k, v in log.stats().items():
             acc[k] = acc.get(k, 0) + v
     st = {k: v / n_instr for k, v in acc.items()}
     value = total / (ms * 1e-3) / 1e9
 
     # algorithmic bytes and the dominant kernel on this rank (rank 0 reports)
-    dup_h = dup[:len(idx)].cpu().numpy()
-    ab = alg_bytes(lg, idx, dup_h, 4096, two_pass=args.two_pass or st.get("two_pass", 0) >= 0.5)
+    dup_np = dup_d[:n].cpu().numpy()
+    ab = alg_bytes(lg, idx, dup_np, 4096, two_pass=args.two_pass or st.get("two_pass", 0) >= 0.5)
     if args.prefilter and world == 1:
         # only the bytes the pre-filtered path must read: the library reports the bytes it
         # hashed beyond first chunks (prefix-unique payloads skip theirs)
         sz = lg.size[idx].astype(np.int64)
         big = sz > 4096
-        mem = dup_h >= 0
+        mem = dup_np >= 0
         p0 = np.minimum(sz, 4096)
         ab["fused"] = int(st["prefilter_rest_bytes"]) + int(p0[big & mem].sum()) + 32 * int(((sz[big] + 32767) // 32768).sum())
-        ab["path"] = sum(v for k, v in ab.items() if k != "path") + 64 * len(idx)
+        ab["path"] = sum(v for k, v in ab.items() if k != "path") + 64 * n
     peak, peak_src = load_peak()
     kern_ms = {"small": st["ms_hash_small"], "prefix": st["ms_hash_large"], "fused": st["ms_fused"]}
     dom = max(kern_ms, key=lambda k: kern_ms[k])
     dom_ms = kern_ms[dom]
     achieved = ab[dom] / (dom_ms * 1e-3) / 1e9 if dom_ms > 0 else 0.0
     two_pass = args.two_pass or st.get("two_pass", 0) >= 0.5
-    fused_k = "k_fused_fx"
     kname = {"small": "k_hash_small" if two_pass else "k_fused_small",
              "prefix": "k_hash_large" if two_pass else "k_prefix_hash",
-             "fused": fused_k}[dom]
+             "fused": "k_fused_fx"}[dom]
     mode = "two-pass" if two_pass else "fused"
     capture = f"config{args.workload}/{mode}" + ("/prefilter" if args.prefilter else "") + \
         (f"/digest_bits{args.digest_bits}" if args.digest_bits < 64 else "")
@@ -306,9 +335,28 @@ def run_ours(args):
                 "frac": round(achieved / peak, 4), "traffic": traffic, "alg_bytes": ab[dom],
                 "ms": round(dom_ms, 4), "peak_source": peak_src,
                 "read_stream_ceiling_gbs": read_ceiling(),
-                "traffic_source": f"profiles/ncu_summary.json captures[{capture}] (ncu --set full, same workload and mode)"
+                "note": "peak is the driver's copy (read+write) figure; the kernel is a pure read stream, "
+                        "so frac > 1 is possible -- read_stream_ceiling_gbs is the measured 256-bit read ceiling",
+                "traffic_source": f"profiles/ncu_summary.json captures[{capture}] (ncu --set full of the same "
+                                  "workload and mode; committed capture, not measured in this run)"
                 if traffic is not None else "no committed ncu capture of this workload/mode"}
-    path_gbs = ab["path"] / (ms * 1e-3) / 1e9
+    path_gbs = ab["path"] / (ms_dev * 1e-3) / 1e9
+
+    # per-rank terms of the scaling cost model: local time, B_x, exchange
+    mine = {"rank": rank, "ms": round(ms_local, 4), "ms_device_outputs": round(ms_dev_local, 4),
+            "records": n, "payload_bytes": my_bytes,
+            "reps_local": int(st.get("n_reps_local", 0)), "reps_global": int(st.get("n_reps_global", 0)),
+            "remote_verify_bytes": int(st.get("remote_verify_bytes", 0)),
+            "exchange_bytes": int(st.get("exchange_bytes", 0)), "slow_reps": int(st.get("n_slow", 0)),
+            "host_syncs": int(st.get("host_syncs", 0)), "ms_exchange": round(st.get("ms_exchange", 0.0), 4)}
+    per_rank = [mine]
+    if world > 1:
+        per_rank = [None] * world
+        dist.all_gather_object(per_rank, mine)
+
+    parity = None
+    if args.check:
+        parity = check_parity(lg, args, idx, dup_np, ben_d.cpu().numpy().view(np.uint64), rank, world)
 
     e2e = None
     if args.e2e_steps > 0:
@@ -331,23 +379,52 @@ def run_ours(args):
                    "n_scale": args.n_scale, "size_scale": args.size_scale,
                    "l2": "inputs larger than L2 (payload %.1f GB >> 126 MB L2)" % (total / 1e9),
                    "parallelism": "single GPU" if world == 1 else
-                   f"{world} shards (site-affinity LPT); NCCL all-gather of class representatives, "
-                   "in-kernel peer byte verify over NVLink, NCCL all-reduce of benefit",
+                   f"{world} shards (site-affinity LPT), collective ffm_dedup_run: "
+                   + ("host transport, ranks sharing one GPU (test hook)" if args.same_device else
+                      "library-owned NCCL all-gather of class representatives + all-reduce of per-site sums, "
+                      "in-kernel peer byte verify over NVLink"),
+                   "outputs": "host (pinned): duplicate_of / benefit_ns D2H inside every timed run",
                    "chunk_bytes": 32768, "small_bytes": 4096, "prefilter": bool(args.prefilter and world == 1),
                    "digest_bits": args.digest_bits,
                    "round0": "two-pass (forced)" if args.two_pass else
                    ("two-pass (adaptive)" if st.get("two_pass", 0) >= 0.5 else "fused")},
+        "value_device_outputs": round(total / (ms_dev * 1e-3) / 1e9, 2),
+        "ms_per_step_device_outputs": round(ms_dev, 4),
         "pct_hbm_roofline_path": round(path_gbs / peak, 4),
         "path_alg_gbs": round(path_gbs, 1),
         "stage_ms": {k: round(st[k], 4) for k in ("ms_hash_small", "ms_hash_large", "ms_group", "ms_verify",
-                                                  "ms_fused", "ms_resolve", "ms_label", "ms_output", "ms_total")},
+                                                  "ms_fused", "ms_resolve", "ms_label", "ms_output", "ms_total",
+                                                  "ms_exchange")},
         "clocks": clk, "gpu_launches": launches, "roofline": roofline, "e2e": e2e, "cpu_baseline": cpu,
-        "duplicates_rank0": int((dup_h >= 0).sum()),
+        "per_rank": per_rank, "parity": parity,
+        "duplicates_rank0": int((dup_np >= 0).sum()),
         "collisions": {"residual_members": int(round(st["n_residual"])), "resolve_rounds": int(round(st["resolve_rounds"]))},
     }
     print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def check_parity(lg, args, idx, dup, ben, rank, world):
+    """Every rank's duplicate_of (global gids) and the global benefit against the CPU
+    oracle on the whole log (rank 0; small logs)."""
+    import oracle
+    import loggen
+    import torch.distributed as dist
+    parts = [(idx, dup)]
+    if world > 1:
+        parts = [None] * world
+        dist.all_gather_object(parts, (idx, dup))
+    if rank != 0:
+        return None
+    full = loggen.gen_config(args.workload, n_scale=args.n_scale, size_scale=args.size_scale)
+    want_d, want_b = oracle.dedup(full)
+    got = np.full(full.n, -7, np.int64)
+    for i, d in parts:
+        got[i] = d
+    ok = bool(np.array_equal(got, want_d) and np.array_equal(ben, want_b))
+    return {"oracle": "ok" if ok else "MISMATCH", "records": int(full.n),
+            "mismatched_records": int((got != want_d).sum())}
 
 
 def read_ceiling():
@@ -361,69 +438,73 @@ def read_ceiling():
 
 
 def run_e2e(args, lg, local, rank=0, world=1):
+    """The metric end to end through the public C ABI, per step: ffm_log_reset +
+    ffm_log_append_batch of every payload from HOST memory (H2D inside the step) +
+    ffm_dedup_run with host output arrays (D2H inside).  Pinned source buffers (the
+    copy engines / k_gather read them in place) and pageable ones (staged through the
+    library's pinned ring), each over args.e2e_steps steps after one warm-up step."""
     import torch
     import torch.distributed as dist
     import paper_conf_sc_weltonm19_b200 as ffm
-    from paper_conf_sc_weltonm19_b200 import sharded
     buf = lg.buf
-    cudart = torch.cuda.cudart()
-    try:
-        reg = int(cudart.cudaHostRegister(buf.ctypes.data, buf.nbytes, 0))
-    except Exception:
-        reg = -1
     idx = lg.shard_idx
     ptrs = lg.payload_ptrs()[idx]
     n = len(idx)
     my_bytes = int(lg.size[idx].sum())
-    dev = torch.device("cuda", local)
     dup_pin = torch.empty(max(n, 1), dtype=torch.int64).pin_memory()
     ben_pin = torch.empty(lg.n_sites, dtype=torch.int64).pin_memory()
-    times, phases = [], []
     # one long-lived log (allocated once, like any buffer); every step empties it
-    # (ffm_log_reset keeps the HBM allocations), appends every payload from pinned
-    # host memory (H2D inside the step), runs, and reads the results back (D2H).
-    log = ffm.FfmLog(lg.n_sites, device=local, arena_bytes=my_bytes + 128 * n + (1 << 20),
-                     max_records=n, rank=rank, world=world)
-    for step in range(args.e2e_steps + 1):
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
-        t0 = time.perf_counter()
-        log.reset()
-        t1 = time.perf_counter()
-        log.append_batch(lg.site[idx], lg.size[idx], ptrs, lg.dur[idx],
-                         gids=idx if world > 1 else None,
-                         payload_kind=ffm.FFM_PAYLOAD_HOST_PINNED if reg == 0 else ffm.FFM_PAYLOAD_HOST)
-        t2 = time.perf_counter()
-        if world > 1:
-            sharded.exchange_handles(log)
-            d, b = sharded.dedup_sharded(log, dev)
-            dup_pin[:n].copy_(d[:n])
-            ben_pin.copy_(b)
-            dist.barrier()           # peers stop reading this arena before it is reused
-        else:
+    # (ffm_log_reset keeps the HBM allocations)
+    log = make_ffm_log(args, lg, n, my_bytes, rank, world, local)
+    cudart = torch.cuda.cudart()
+
+    def measure(kind, steps):
+        times, phases = [], []
+        for step in range(steps + 1):
+            torch.cuda.synchronize()
+            if world > 1:
+                dist.barrier()
+            t0 = time.perf_counter()
+            log.reset()
+            t1 = time.perf_counter()
+            log.append_batch(lg.site[idx], lg.size[idx], ptrs, lg.dur[idx], gids=idx if world > 1 else None,
+                             payload_kind=kind)
+            t2 = time.perf_counter()
             log.run(dup_pin.numpy(), ben_pin.numpy().view(np.uint64))
-        t3 = time.perf_counter()
-        sec_step = t3 - t0
-        if world > 1:
-            tt = torch.tensor([sec_step], dtype=torch.float64, device=dev)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            sec_step = float(tt.item())
-        if step > 0:                     # first step warms up
-            times.append(sec_step)
-            phases.append((t1 - t0, t2 - t1, t3 - t2))
-    log.close()
+            t3 = time.perf_counter()
+            sec = t3 - t0
+            if world > 1:
+                tt = torch.tensor([sec], dtype=torch.float64)
+                dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+                sec = float(tt.item())
+            if step > 0:                     # the first step warms up
+                times.append(sec)
+                phases.append((t1 - t0, t2 - t1, t3 - t2))
+        sec = statistics.median(times)
+        return {"value": round(lg.total_bytes / sec / 1e9, 3), "steps": len(times), "s_per_step": round(sec, 4),
+                "phases_s": dict(zip(("reset", "append_h2d", "run_d2h"),
+                                     [round(statistics.median(p), 4) for p in zip(*phases)]))}
+
+    reg = -1
+    try:
+        reg = int(cudart.cudaHostRegister(buf.ctypes.data, buf.nbytes, 0))
+    except Exception:
+        pass
+    pinned = measure(ffm.FFM_PAYLOAD_HOST_PINNED if reg == 0 else ffm.FFM_PAYLOAD_HOST, args.e2e_steps)
     if reg == 0:
         cudart.cudaHostUnregister(buf.ctypes.data)
-    sec = statistics.median(times)
-    meta = lg.n * (4 + 8 + 8) // max(world, 1)
-    return {"value": round(lg.total_bytes / sec / 1e9, 3), "unit": UNIT,
-            "h2d_bytes_per_step": int(lg.total_bytes + meta * world), "d2h_bytes_per_step": int(8 * lg.n + 8 * lg.n_sites * world),
-            "steps": len(times), "s_per_step": round(sec, 4),
-            "phases_s": dict(zip(("reset", "append_h2d", "run_d2h"),
-                                 [round(statistics.median(p), 4) for p in zip(*phases)])),
-            "note": "wall clock per step on a reused log: ffm_log_reset + append (pinned host -> HBM) + "
-                    "run + D2H of duplicate_of/benefit, median"}
+    pageable = measure(ffm.FFM_PAYLOAD_HOST, args.e2e_steps) if args.e2e_pageable else None
+    log.close()
+    meta = lg.n * (4 + 8 + 8 + 8)
+    out = {"value": pinned["value"], "unit": UNIT,
+           "h2d_bytes_per_step": int(lg.total_bytes + meta), "d2h_bytes_per_step": int(8 * lg.n + 8 * lg.n_sites * world),
+           "steps": pinned["steps"], "s_per_step": pinned["s_per_step"], "phases_s": pinned["phases_s"],
+           "source": "pinned host buffers (cudaHostRegister)" if reg == 0 else "pageable host buffers",
+           "note": "wall clock per step, max over ranks, median: ffm_log_reset + append (host -> HBM) + "
+                   "ffm_dedup_run with host output arrays (D2H of duplicate_of / benefit_ns)"}
+    if pageable:
+        out["pageable"] = dict(pageable, unit=UNIT, source="pageable host buffers (library's pinned staging ring)")
+    return out
 
 
 def oracle_sample(lg, seconds_budget):
@@ -462,17 +543,27 @@ def cpu_baseline(lg, seconds):
 
 
 def run_reference(args):
+    """The reference arm of this tier: the CPU oracle as it stands, 1 core, on this arm's
+    workload -- the whole log per timed step when K of them fit args.ref_budget seconds
+    (else the largest gid prefix that does, said in `sample`).  Warm-up steps run the
+    oracle on a small prefix (it keeps no state between calls)."""
     rank, world, _ = dist_env()
     if rank != 0:
         return
     import oracle
     lg = make_log(args.workload, args.n_scale, args.size_scale)
     os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
-    k, _ = oracle_sample(lg, args.ref_step_seconds)
+    k_cal, rate = oracle_sample(lg, 1.0)
+    t_full = lg.total_bytes / rate
+    if args.steps * t_full <= args.ref_budget:
+        k = lg.n
+    else:
+        k, _ = oracle_sample(lg, args.ref_budget / args.steps)
     sub = lg.subset(np.arange(k))
+    warm = lg.subset(np.arange(k_cal))
     b = int(lg.size[:k].sum())
     for _ in range(args.warmup):
-        oracle.dedup(sub)
+        oracle.dedup(warm)
     ts = []
     for _ in range(args.steps):
         t = time.perf_counter()
@@ -480,16 +571,38 @@ def run_reference(args):
         ts.append(time.perf_counter() - t)
     sec = sum(ts) / len(ts)
     v = round(b / sec / 1e9, 3)
-    sample = f"gid prefix of {k} of {lg.n} records ({b / 1e9:.2f} GB) per step"
+    sample = (f"the whole log ({lg.n} records, {b / 1e9:.2f} GB) per step" if k == lg.n else
+              f"gid prefix of {k} of {lg.n} records ({b / 1e9:.2f} GB) per step") + \
+        f"; warm-up steps on a {k_cal}-record prefix; 1 of {os.cpu_count()} host cores"
     out = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(sec * 1e3, 3),
            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
            "data": "synthetic",
            "config": {"workload": WORKLOADS[args.workload], "records": lg.n, "payload_bytes": lg.total_bytes,
-                      "n_sites": lg.n_sites, "n_scale": args.n_scale, "size_scale": args.size_scale},
+                      "n_sites": lg.n_sites, "n_scale": args.n_scale, "size_scale": args.size_scale,
+                      "whole_log_per_step": k == lg.n},
            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
+
+
+def spawn_ranks(args):
+    """--gpus N without a torchrun environment: launch N ranks of this script (one per
+    GPU) under torch.distributed.run and return its exit code."""
+    import socket
+    import torch
+    if not args.same_device and torch.cuda.device_count() < args.gpus:
+        log_msg(f"[bench] --gpus {args.gpus} but {torch.cuda.device_count()} GPUs are visible "
+                "(--same-device runs the ranks on one GPU over the host transport)")
+        return 2
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    log_msg("[bench] " + " ".join(cmd))
+    return subprocess.run(cmd).returncode
 
 
 def main():
@@ -501,9 +614,15 @@ def main():
     ap.add_argument("--workload", type=int, default=5, choices=[1, 2, 3, 4, 5])
     ap.add_argument("--n-scale", type=float, default=1.0)
     ap.add_argument("--size-scale", type=float, default=1.0)
-    ap.add_argument("--e2e-steps", type=int, default=2)
-    ap.add_argument("--cpu-seconds", type=float, default=15.0)
-    ap.add_argument("--ref-step-seconds", type=float, default=6.0)
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--e2e-pageable", type=int, default=1, help="also measure e2e from pageable host memory")
+    ap.add_argument("--cpu-seconds", type=float, default=30.0)
+    ap.add_argument("--ref-budget", type=float, default=400.0,
+                    help="reference arm: seconds of timed oracle steps; the whole log per step if it fits")
+    ap.add_argument("--same-device", action="store_true",
+                    help="test hook: run the N ranks on one GPU (host exchange transport instead of NCCL)")
+    ap.add_argument("--check", action="store_true", help="check the result against the CPU oracle (small logs)")
+    ap.add_argument("--lib", default=None, help="load another build of libffm.so (tools/build_variants.sh)")
     ap.add_argument("--digest-bits", type=int, default=64,
                     help="< 64 truncates the group-by digest (forced collisions, verify stress; config 3)")
     ap.add_argument("--two-pass", action="store_true",
@@ -514,9 +633,16 @@ def main():
     if args.warmup < 3:
         log_msg("[bench] warmup raised to 3 (timing rules)")
         args.warmup = 3
+    if args.lib:
+        import paper_conf_sc_weltonm19_b200 as ffm
+        ffm.set_library_path(args.lib)
     if args.impl == "reference":
         run_reference(args)
+    elif args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(args))
     else:
+        if int(os.environ.get("WORLD_SIZE", 1)) != args.gpus:
+            raise SystemExit(f"bench: --gpus {args.gpus} but WORLD_SIZE={os.environ.get('WORLD_SIZE')}")
         run_ours(args)
 
 

@@ -70,11 +70,26 @@ enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_s
        FFM_FLAG_NO_GRAPH = 16u   /* launch every kernel directly instead of replaying the captured
                                     CUDA graph of a run (default: graph while the log is unchanged) */ };
 
+/* Caller-provided exchange transport of a sharded log (world > 1), used instead of the
+   library's own NCCL communicator when NCCL cannot connect the ranks (e.g. several ranks
+   sharing one GPU in tests).  Both functions are collective over the world, take HOST
+   buffers and return 0 on success (anything else fails the run with FFM_E_COMM).
+     allgather:     recv[world * bytes] = every rank's send[bytes], rank-major
+     allreduce_u64: buf[n] = elementwise sum over ranks, mod 2^64, in place
+   The struct is copied at ffm_log_create; ctx and the functions must stay valid until
+   ffm_log_destroy. */
+typedef struct ffm_comm_ops {
+    void* ctx;
+    int (*allgather)(void* ctx, const void* send, void* recv, uint64_t bytes);
+    int (*allreduce_u64)(void* ctx, uint64_t* buf, uint64_t n);
+} ffm_comm_ops;
+
 typedef struct ffm_config {
     uint32_t n_sites;      /* call_site must be < n_sites.  Sites are caller-interned stack
                               traces, matched by instruction address. */
     int32_t  device;       /* CUDA ordinal this log lives on */
-    int32_t  rank, world;  /* shard id / count (P > 1: see ffm_shard_* below); 0, 1 for one GPU */
+    int32_t  rank, world;  /* shard id / count; 0, 1 for one GPU.  world > 1 makes ffm_log_create
+                              and ffm_dedup_run collective (see "Sharded logs" below) */
     uint64_t arena_bytes;  /* initial HBM payload arena capacity (bytes); grows x2 on demand */
     uint64_t max_records;  /* initial record capacity hint; grows on demand */
     uint32_t digest_bits;  /* 64 normally.  < 64 truncates the group-by digest to FORCE
@@ -89,6 +104,9 @@ typedef struct ffm_config {
     uint32_t flags;        /* FFM_FLAG_* */
     uint32_t reserved0;
     void*    stream;       /* cudaStream_t to run on, or NULL: the log creates its own */
+    const void* nccl_id;   /* world > 1: the 128-byte ncclUniqueId of the world (ffm_nccl_unique_id on
+                              one rank, broadcast by the caller); the log owns the communicator */
+    const ffm_comm_ops* comm;  /* world > 1, instead of nccl_id: caller transport (copied) */
 } ffm_config;
 
 /* Fill *cfg with defaults: n_sites 1, device 0, rank 0, world 1, digest_bits 64,
@@ -96,8 +114,11 @@ typedef struct ffm_config {
 void ffm_config_init(ffm_config* cfg);
 
 /* Create a log on cfg->device.  *out is owned by the library until ffm_log_destroy.
-   Errors: FFM_E_INVAL (NULL, n_sites == 0, bad chunk/small bytes, digest_bits > 64),
-   FFM_E_NODEV, FFM_E_NOMEM, FFM_E_CUDA. */
+   With world > 1 this is collective: every rank calls it with the same nccl_id (the
+   library's NCCL communicator is created here) or with its comm transport.
+   Errors: FFM_E_INVAL (NULL, n_sites == 0, bad chunk/small bytes, digest_bits > 64,
+   world > 1 without exactly one of nccl_id / comm), FFM_E_NODEV, FFM_E_NOMEM, FFM_E_CUDA,
+   FFM_E_COMM (NCCL unavailable or its init failed). */
 int ffm_log_create(const ffm_config* cfg, ffm_log** out);
 
 /* Append one transfer record (the intercepted call's payload location
@@ -116,9 +137,15 @@ int ffm_log_append(ffm_log* log, uint32_t call_site, uint64_t size,
 /* Append n records at once (host arrays of length n).  payloads[i] follows the
    rules of ffm_log_append; payload_kind says whether they are all HOST, all DEVICE,
    or AUTO (detected per pointer).  gids may be NULL (local append order) or give
-   each record's GLOBAL gid, strictly increasing across all appends to this log
-   (sharded logs: records of one global program order split over ranks).
-   All-or-nothing: on error the log is unchanged. */
+   each record's GLOBAL gid, strictly increasing across all appends to this log and
+   < 2^63 (sharded logs: records of one global program order split over ranks; there
+   gids are REQUIRED -- every rank numbering from 0 would repeat gids across ranks).
+   A device payload on another GPU is copied by the copy engines (cudaMemcpyDefault).
+   Device payloads are read on the library's staging stream after it waits on the log's
+   stream (cfg->stream) and on the legacy default stream; a producer on any other stream
+   must synchronize before the append.
+   All-or-nothing: on error the log is unchanged.  Errors as ffm_log_append, plus
+   FFM_E_RANGE (gids not increasing, or >= 2^63), FFM_E_INVAL (world > 1 and gids NULL). */
 int ffm_log_append_batch(ffm_log* log, uint64_t n, const uint32_t* call_sites,
                          const uint64_t* sizes, const void* const* payloads,
                          const uint64_t* durations_ns, const uint64_t* gids,
@@ -141,7 +168,10 @@ int ffm_log_append_batch_ex(ffm_log* log, uint64_t n, const uint32_t* call_sites
    Either array may be host or device memory (caller-owned; device arrays must be
    on cfg->device).  benefit_ns may be NULL.  Idempotent: re-running over an
    unchanged log gives identical outputs; appends after a run are allowed.
-   Synchronous: returns when the outputs are written. */
+   Synchronous: returns when the outputs are written.
+   world > 1: COLLECTIVE -- every rank calls it; duplicate_of[n_local] receives GLOBAL
+   gids (the earliest byte-identical record on any rank) and benefit_ns the global
+   per-site sums, identical on every rank (see "Sharded logs"). */
 int ffm_dedup_run(ffm_log* log, int64_t* duplicate_of, uint64_t* benefit_ns);
 
 /* Number of records appended (local) / payload bytes appended. */
@@ -175,6 +205,15 @@ typedef struct ffm_run_stats {
     uint64_t n_reread;          /* residual members whose bytes were compared again; after a fused
                                    round 0 the others are settled exactly through their difference
                                    lists against the group head */
+    /* sharded runs (world > 1); 0 otherwise */
+    uint64_t n_reps_local;      /* exact local classes exported by this rank */
+    uint64_t n_reps_global;     /* representatives of all ranks */
+    uint64_t exchange_bytes;    /* bytes this rank received through the collectives of the run */
+    uint64_t remote_verify_bytes; /* B_x: payload bytes this rank compared against peer arenas over
+                                   NVLink */
+    uint64_t n_slow;            /* representatives resolved by the same-key segment scan */
+    uint64_t host_syncs;        /* host synchronisations of the run's stream */
+    double   ms_exchange;       /* CUDA-event time from the end of the local pass to the outputs */
 } ffm_run_stats;
 
 /* Statistics of the last ffm_dedup_run. */
@@ -182,7 +221,7 @@ int ffm_last_run_stats(const ffm_log* log, ffm_run_stats* out);
 
 /* Number of duplicates per call site in the last run ("Number of Transfer Issues",
    Fig. 6), [n_sites] uint64, host or device.  For a sharded log these are
-   this rank's partial counts (all-reduce them like the benefit). */
+   the global counts (all-reduced with the benefit). */
 int ffm_site_duplicate_counts(ffm_log* log, uint64_t* counts_out);
 
 /* Folded grouping: group_values_out[g] = sum of site_values[s] over the
@@ -218,29 +257,28 @@ uint64_t ffm_online_done(const ffm_log* log);
 int ffm_debug_digests(ffm_log* log, uint64_t* digests_out);
 
 /* ---------------------------------------------------------------------------
- * Sharded logs (world > 1).  One process per GPU.
- * Exact byte equality is transitive, so the per-rank results merge through one
- * exchange of class-representative tuples.  Per run, on every rank:
- *   1. ffm_shard_local   -- H1..H4 on this rank's records; export one ffm_rep per
- *                           exact local class into caller DEVICE memory.
- *   2. caller all-gathers the reps of all ranks, in rank order, into one device array
- *      (e.g. torch.distributed all_gather over NCCL / NVLink), with the counts.
- *   3. ffm_shard_merge   -- global group-by over all reps; a remote candidate is
- *                           byte-verified by loading its bytes straight from the peer
- *                           GPU's arena (IPC-mapped, over NVLink) inside the kernel;
- *                           writes duplicate_of for this rank's records (global gids)
- *                           and this rank's PARTIAL benefit.
- *   4. caller all-reduces the partial benefits (uint64 sum).
- * Peer arenas are mapped once per arena allocation: exchange ffm_shard_ipc_handle
- * outputs (after the last append) and call ffm_shard_open_peer for every other rank.
+ * Sharded logs (world > 1).  One process per GPU; the
+ * caller assigns records to ranks (ffm_shard_plan) and appends each rank's records with
+ * their GLOBAL gids.  Exact byte equality is transitive, so per-rank results merge
+ * through one exchange of class representatives.  ffm_dedup_run on every rank:
+ *   1. H1..H4 on this rank's records -> exact local classes, one representative each
+ *      (key of the full digest, size, gid, arena offset, channel);
+ *   2. all-gather of the representatives (NCCL over NVLink / NVSwitch on the log's
+ *      stream, or the caller's ffm_comm_ops);
+ *   3. every rank builds the same global group-by over all representatives; a rank's
+ *      representative whose candidate lives on another rank is byte-verified by a
+ *      kernel that loads the candidate's bytes straight from the peer GPU's arena
+ *      (CUDA-IPC mapping, exchanged by the library whenever an arena was reallocated);
+ *      digest collisions take a scan of the key's segment;
+ *   4. labels (global gids), per-site partial sums, and an all-reduce of the sums.
+ * Two host synchronisations per run when no rank has digest collisions.  When the run
+ * returns, no peer reads this rank's arena any more (the all-reduce orders every rank's
+ * compare kernels before it), so appends / reset may follow.
  * ------------------------------------------------------------------------- */
-typedef struct ffm_rep {
-    uint64_t key;    /* group key of (digest, size, channel) (identical function on every rank) */
-    uint64_t size;   /* payload bytes */
-    uint64_t gid;    /* global gid of the class's first record on the owning rank */
-    uint64_t off;    /* arena offset on the owning rank */
-    uint64_t chan;   /* channel id (0 unless ffm_log_append_batch_ex gave one) */
-} ffm_rep;
+
+/* The 128-byte ncclUniqueId for a new world (call on one rank, broadcast it).
+   Errors: FFM_E_INVAL (NULL), FFM_E_COMM (libnccl.so.2 unavailable). */
+int ffm_nccl_unique_id(void* id_out);
 
 enum { FFM_SHARD_SITE_LPT = 0,     /* whole call sites, bin-packed by bytes (largest first) */
        FFM_SHARD_CONTIGUOUS = 1 }; /* contiguous gid ranges of ~equal bytes */
@@ -251,32 +289,12 @@ enum { FFM_SHARD_SITE_LPT = 0,     /* whole call sites, bin-packed by bytes (lar
 int ffm_shard_plan(uint64_t n, const uint32_t* call_sites, const uint64_t* sizes, uint32_t n_sites,
                    int32_t world, int policy, int32_t* rank_out);
 
-/* 64-byte CUDA IPC handle of this log's HBM arena (valid until the arena grows:
-   exchange after the last append). */
-int ffm_shard_ipc_handle(ffm_log* log, void* handle_out);
-
-/* Map peer `rank`'s arena from its ffm_shard_ipc_handle bytes (no-op for own rank;
-   re-mapping the same handle is free). */
-int ffm_shard_open_peer(ffm_log* log, int32_t rank, const void* handle);
-
-/* Step 1.  reps_out: device array of at least ffm_log_count(log) entries.
-   *n_reps_out = number written (in local gid order). */
-int ffm_shard_local(ffm_log* log, ffm_rep* reps_out, uint64_t cap, uint64_t* n_reps_out);
-
-/* Step 3.  all_reps: device array of all ranks' reps, rank-major; counts: host array
-   [world].  counts[rank] must equal this rank's last n_reps (else FFM_E_COMM).
-   duplicate_of [n_local] (host or device) receives global gids; benefit_partial
-   [n_sites] receives this rank's partial sums (all-reduce them). */
-int ffm_shard_merge(ffm_log* log, const ffm_rep* all_reps, const uint64_t* counts, int64_t* duplicate_of,
-                    uint64_t* benefit_partial);
-
 /* Replace cfg.flags of a live log (e.g. toggle FFM_FLAG_TIMING between measured and
    instrumented runs).  Takes effect at the next run. */
 int ffm_log_set_flags(ffm_log* log, uint32_t flags);
 
 /* Empty the log (records, online state) but keep every allocation (HBM arena, work
-   buffers, staging ring): the next batch of transfers reuses them.  Peer mappings of
-   a sharded log stay valid while the arena is not reallocated. */
+   buffers, staging ring): the next batch of transfers reuses them. */
 int ffm_log_reset(ffm_log* log);
 
 /* Destroy the log and release its memory.  NULL is a no-op (returns FFM_OK). */

@@ -18,8 +18,17 @@ import numpy as np
 
 from ._build import LIB as _LIB_DEFAULT
 
-# FFM_LIB: a tuning-variant build of the same sources (tools/build_variants.sh)
-_LIB_PATH = os.environ.get("FFM_LIB") or _LIB_DEFAULT
+_LIB_PATH = _LIB_DEFAULT
+
+
+def set_library_path(path: str) -> None:
+    """Load another build of the same sources (a tuning variant from
+    tools/build_variants.sh) instead of the in-tree libffm.so; call before the first
+    use of the library."""
+    global _LIB_PATH
+    if _lib is not None:
+        raise RuntimeError("libffm.so is already loaded")
+    _LIB_PATH = path
 
 FFM_OK, FFM_E_INVAL, FFM_E_RANGE, FFM_E_NOMEM, FFM_E_CUDA, FFM_E_COMM, FFM_E_STATE, FFM_E_NODEV = \
     0, -1, -2, -3, -4, -5, -6, -7
@@ -34,11 +43,18 @@ FFM_FLAG_NO_GRAPH = 16
 EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_append_batch", "ffm_log_append_batch_ex",
            "ffm_dedup_run", "ffm_log_count", "ffm_log_payload_bytes", "ffm_log_stream",
            "ffm_last_run_stats", "ffm_debug_digests", "ffm_log_destroy", "ffm_strerror",
-           "ffm_last_error", "ffm_version", "ffm_shard_plan", "ffm_shard_ipc_handle", "ffm_shard_open_peer",
-           "ffm_shard_local", "ffm_shard_merge", "ffm_site_duplicate_counts", "ffm_fold_sites",
+           "ffm_last_error", "ffm_version", "ffm_shard_plan", "ffm_nccl_unique_id",
+           "ffm_site_duplicate_counts", "ffm_fold_sites",
            "ffm_online_step", "ffm_online_done", "ffm_log_reset", "ffm_log_set_flags"]
 FFM_SHARD_SITE_LPT, FFM_SHARD_CONTIGUOUS = 0, 1
-REP_WORDS = 5        # ffm_rep = {key, size, gid, off, chan}, 5 x u64
+
+# ffm_comm_ops callbacks (host buffers)
+ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64)
+ALLREDUCE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64)
+
+
+class FfmCommOps(ctypes.Structure):
+    _fields_ = [("ctx", ctypes.c_void_p), ("allgather", ALLGATHER_FN), ("allreduce_u64", ALLREDUCE_FN)]
 
 
 class FfmConfig(ctypes.Structure):
@@ -47,7 +63,8 @@ class FfmConfig(ctypes.Structure):
                 ("max_records", ctypes.c_uint64), ("digest_bits", ctypes.c_uint32),
                 ("refine_bits", ctypes.c_uint32), ("chunk_bytes", ctypes.c_uint32),
                 ("small_bytes", ctypes.c_uint32), ("flags", ctypes.c_uint32),
-                ("reserved0", ctypes.c_uint32), ("stream", ctypes.c_void_p)]
+                ("reserved0", ctypes.c_uint32), ("stream", ctypes.c_void_p),
+                ("nccl_id", ctypes.c_void_p), ("comm", ctypes.POINTER(FfmCommOps))]
 
 
 class FfmRunStats(ctypes.Structure):
@@ -56,7 +73,10 @@ class FfmRunStats(ctypes.Structure):
                [(k, ctypes.c_uint64) for k in ("n_records", "payload_bytes", "n_members", "n_residual",
                                                 "resolve_rounds", "kernel_launches", "hash_items",
                                                 "verify_items", "prefilter_rest_bytes")] + \
-               [("ms_fused", ctypes.c_double), ("two_pass", ctypes.c_uint64), ("n_reread", ctypes.c_uint64)]
+               [("ms_fused", ctypes.c_double), ("two_pass", ctypes.c_uint64), ("n_reread", ctypes.c_uint64)] + \
+               [(k, ctypes.c_uint64) for k in ("n_reps_local", "n_reps_global", "exchange_bytes",
+                                                "remote_verify_bytes", "n_slow", "host_syncs")] + \
+               [("ms_exchange", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -116,14 +136,8 @@ def lib() -> ctypes.CDLL:
         L.ffm_version.restype = ctypes.c_char_p
         L.ffm_shard_plan.argtypes = [u64, vp, vp, u32, ctypes.c_int32, i32, vp]
         L.ffm_shard_plan.restype = i32
-        L.ffm_shard_ipc_handle.argtypes = [vp, vp]
-        L.ffm_shard_ipc_handle.restype = i32
-        L.ffm_shard_open_peer.argtypes = [vp, ctypes.c_int32, vp]
-        L.ffm_shard_open_peer.restype = i32
-        L.ffm_shard_local.argtypes = [vp, vp, u64, ctypes.POINTER(u64)]
-        L.ffm_shard_local.restype = i32
-        L.ffm_shard_merge.argtypes = [vp, vp, vp, vp, vp]
-        L.ffm_shard_merge.restype = i32
+        L.ffm_nccl_unique_id.argtypes = [vp]
+        L.ffm_nccl_unique_id.restype = i32
         L.ffm_site_duplicate_counts.argtypes = [vp, vp]
         L.ffm_site_duplicate_counts.restype = i32
         L.ffm_fold_sites.argtypes = [vp, vp, vp, u32, vp]
@@ -256,27 +270,13 @@ def ffm_shard_plan(call_sites, sizes, n_sites: int, world: int, policy: int = FF
     return out[:len(sites)]
 
 
-def ffm_shard_ipc_handle(h) -> bytes:
-    buf = ctypes.create_string_buffer(64)
-    _check(h, lib().ffm_shard_ipc_handle(h, buf))
+def ffm_nccl_unique_id() -> bytes:
+    """128-byte ncclUniqueId for a new sharded world (call on one rank, broadcast it)."""
+    buf = ctypes.create_string_buffer(128)
+    rc = lib().ffm_nccl_unique_id(buf)
+    if rc != FFM_OK:
+        raise FfmError(rc, "libnccl.so.2 unavailable")
     return buf.raw
-
-
-def ffm_shard_open_peer(h, rank: int, handle: bytes):
-    buf = ctypes.create_string_buffer(bytes(handle), 64)
-    _check(h, lib().ffm_shard_open_peer(h, rank, buf))
-
-
-def ffm_shard_local(h, reps_out, cap: int) -> int:
-    """reps_out: device buffer (torch CUDA tensor) of >= ffm_log_count ffm_rep entries."""
-    n = ctypes.c_uint64()
-    _check(h, lib().ffm_shard_local(h, _addr(reps_out), cap, ctypes.byref(n)))
-    return int(n.value)
-
-
-def ffm_shard_merge(h, all_reps, counts, duplicate_of, benefit_partial):
-    c = np.ascontiguousarray(counts, dtype=np.uint64)
-    _check(h, lib().ffm_shard_merge(h, _addr(all_reps), _addr(c), _addr(duplicate_of), _addr(benefit_partial)))
 
 
 def ffm_site_duplicate_counts(h, n_sites: int, out=None):
@@ -315,7 +315,10 @@ class FfmLog:
                  digest_bits: int = 64, refine_bits: int = 64, chunk_bytes: int = 0, small_bytes: int = 0,
                  timing: bool = False, stream: int = 0, rank: int = 0, world: int = 1,
                  prefilter: bool = False, two_pass: bool = False, fused: bool = False,
-                 graph: bool = True):
+                 graph: bool = True, nccl_id: bytes | None = None, comm: FfmCommOps | None = None):
+        """world > 1 (collective): pass the world's nccl_id (ffm_nccl_unique_id) or a comm
+        transport (FfmCommOps, e.g. sharded.HostComm)."""
+        self.h = None
         cfg = ffm_config_init()
         cfg.n_sites, cfg.device, cfg.rank, cfg.world = n_sites, device, rank, world
         cfg.arena_bytes, cfg.max_records = arena_bytes, max_records
@@ -325,7 +328,14 @@ class FfmLog:
             (FFM_FLAG_TWO_PASS if two_pass else 0) | (FFM_FLAG_FUSED if fused else 0) | \
             (0 if graph else FFM_FLAG_NO_GRAPH)
         cfg.stream = stream or None
+        self._keep = (nccl_id, comm)     # alive while the library may use them
+        if nccl_id is not None:
+            self._id_buf = ctypes.create_string_buffer(bytes(nccl_id), 128)
+            cfg.nccl_id = ctypes.cast(self._id_buf, ctypes.c_void_p)
+        if comm is not None:
+            cfg.comm = ctypes.pointer(comm)
         self.n_sites = n_sites
+        self.rank, self.world = rank, world
         self.flags = cfg.flags
         self.h = ffm_log_create(cfg)
 

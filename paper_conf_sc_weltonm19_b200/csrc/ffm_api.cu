@@ -7,6 +7,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <functional>
 #include <new>
 #include <string>
 #include <vector>
@@ -19,7 +20,7 @@ namespace {
 
 constexpr uint64_t kRingBytes = 16ull << 20;      // per half of the pinned staging ring
 constexpr uint64_t kDirectCopy = 4ull << 20;      // host payloads above this bypass the ring
-constexpr uint64_t kGatherMaxDefault = 1ull << 20;   // payloads up to this use k_gather (not DMA)
+constexpr uint64_t kGatherMax = 1ull << 20;   // device / pinned payloads up to this use k_gather (not DMA)
 
 struct LocalRun {
     uint64_t n_members, n_res_total, rounds, prefilter_rest;
@@ -31,6 +32,11 @@ struct LocalRun {
 struct CudaFail {
     cudaError_t e;
     const char* what;
+};
+
+struct CommFail {   // an exchange error of a sharded run (FFM_E_COMM), or a range error
+    int code;
+    std::string what;
 };
 
 inline void ck(cudaError_t e, const char* what) {
@@ -112,6 +118,7 @@ void ensure_arena(ffm_log* L, uint64_t need) {
     L->arena = na;
     L->arena_cap = nc;
     ++L->epoch;
+    ++L->arena_gen;   // peers of a sharded log re-map it at their next run
 }
 
 void stage_host(ffm_log* L, const void* src, uint64_t size, uint64_t off) {
@@ -129,14 +136,19 @@ void stage_host(ffm_log* L, const void* src, uint64_t size, uint64_t off) {
     L->ring_fill = off + size - L->ring_arena_start;
 }
 
-// FFM_PAYLOAD_DEVICE / _HOST_PINNED / _HOST (pageable) of one pointer.
-int pointer_kind(const void* p) {
+// FFM_PAYLOAD_DEVICE / _HOST_PINNED / _HOST (pageable) of one pointer; *dev = the
+// device a device pointer lives on (-1 for host memory).
+int pointer_kind(const void* p, int* dev) {
+    *dev = -1;
     cudaPointerAttributes a;
     if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
         cudaGetLastError();
         return FFM_PAYLOAD_HOST;
     }
-    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return FFM_PAYLOAD_DEVICE;
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
+        *dev = a.device;
+        return FFM_PAYLOAD_DEVICE;
+    }
     if (a.type == cudaMemoryTypeHost) return FFM_PAYLOAD_HOST_PINNED;
     return FFM_PAYLOAD_HOST;
 }
@@ -155,16 +167,6 @@ bool is_device_ptr(const void* p) {
 // then the large ones in index order (one warp per large record in the planning
 // kernels).  Returns the number of small records.
 uint64_t build_small_order(const ffm_log* L, uint64_t begin, uint64_t end, std::vector<uint32_t>& order) {
-    static const bool gid_order = getenv("FFM_SMALL_GID_ORDER") != nullptr;   // A/B knob (same results)
-    if (gid_order) {
-        order.clear();
-        for (uint64_t i = begin; i < end; ++i)
-            if (L->h_size[i] <= L->params.small_bytes) order.push_back((uint32_t)(i - begin));
-        const uint64_t ns = order.size();
-        for (uint64_t i = begin; i < end; ++i)
-            if (L->h_size[i] > L->params.small_bytes) order.push_back((uint32_t)(i - begin));
-        return ns;
-    }
     const uint32_t nb = (L->params.small_bytes + 31) / 32 + 1;
     std::vector<uint32_t> start(nb + 1, 0);
     uint64_t ns = 0;
@@ -257,12 +259,15 @@ int plan_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* si
     bool any = L->any_gid || !L->h_gid.empty();
     uint64_t base_n = L->h_size.size();
     if (base_n + n >= 0xFFFFFFFFull) return set_err(L, FFM_E_RANGE, "too many records for one log (2^32-1)");
+    if (L->cfg.world > 1 && !gids)
+        return set_err(L, FFM_E_INVAL, "a sharded log needs the records' global gids (gids == NULL)");
     offs.resize(n);
     for (uint64_t i = 0; i < n; ++i) {
         if (sites[i] >= L->cfg.n_sites) return set_err(L, FFM_E_RANGE, "call_site >= n_sites");
         if (sizes[i] > 0 && payloads[i] == nullptr) return set_err(L, FFM_E_INVAL, "NULL payload with size > 0");
         uint64_t g = gids ? gids[i] : (any ? last + 1 : 0);
         if (gids && any && g <= last) return set_err(L, FFM_E_RANGE, "gids must be strictly increasing");
+        if (g >> 63) return set_err(L, FFM_E_RANGE, "gid >= 2^63 (duplicate_of is int64)");
         last = g;
         any = true;
         cur = align_up(cur, kArenaAlign);
@@ -361,8 +366,8 @@ void ensure_work(ffm_log* L, uint64_t n) {
     }
     if (L->cfg.n_sites > W.site_cap) {
         ++L->epoch;
-        dev_alloc(W.ben, L->cfg.n_sites);
-        dev_alloc(W.cnt, L->cfg.n_sites);
+        dev_alloc(W.ben, 2 * (uint64_t)L->cfg.n_sites);   // [benefit | duplicate counts]: one all-reduce
+        W.cnt = W.ben + L->cfg.n_sites;
         if (label_smem_bytes(L->cfg.n_sites) <= (uint64_t)L->params.max_smem) {
             dev_alloc(W.label_part, (uint64_t)label_hist_rows(L->params.num_sms) * L->cfg.n_sites);
             dev_alloc(W.label_cpart, (uint64_t)label_hist_rows(L->params.num_sms) * L->cfg.n_sites);
@@ -407,10 +412,17 @@ float ev_ms(cudaEvent_t a, cudaEvent_t b) {
 
 
 // ---------------------------------------------------------------- run pipeline
+// A host synchronisation of the run's stream (counted: ffm_run_stats.host_syncs).
+void sync_run(ffm_log* L, const char* what) {
+    ++L->n_syncs;
+    ck(cudaStreamSynchronize(L->stream), what);
+}
+
 void run_prologue(ffm_log* L) {
     ck(cudaSetDevice(L->device), "cudaSetDevice");
     // H0 tail: flush staged payloads and metadata, order the run after them
     ring_flush(L);
+    if (L->cfg.world > 1) ensure_arena(L, 1);   // peers map it: it exists before the header exchange
     upload_meta(L);
     ck(cudaEventRecord(L->ring_ev[L->ring_cur], L->stage_stream), "event");
     ck(cudaStreamWaitEvent(L->stream, L->ring_ev[L->ring_cur], 0), "wait staging");
@@ -421,8 +433,10 @@ void run_prologue(ffm_log* L) {
 // leader (the min local index of its exact byte class).  With `label` the H5/H6
 // kernels are queued before the first sync (single-GPU fast path: one sync when
 // there are no digest collisions) and re-run after collision resolution.
+// pre_sync: more stream work queued after segment A, before its host sync (a sharded
+// run's representative export and header exchange).
 LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& launches, bool label, int64_t* d_dup,
-                   bool prefilter = false) {
+                   bool prefilter = false, const std::function<void()>* pre_sync = nullptr) {
     const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
     const uint64_t n = D.n;
     Work& W = L->work;
@@ -526,7 +540,8 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     } else {
         segment_a();
     }
-    ck(cudaStreamSynchronize(s), "run sync");
+    if (pre_sync) (*pre_sync)();
+    sync_run(L, "run sync");
     R.n_members = L->h_counters[1];
     R.two_pass = two_pass;
     R.prefilter_rest = (uint64_t)L->h_counters[4] | ((uint64_t)L->h_counters[5] << 32);
@@ -548,7 +563,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
             LCHK(launch_verify(D, W, L->params, W.res[cur], (uint32_t)nres, W.res[cur ^ 1],
                                n_large ? W.vitem_cap : 0, s, nullptr, nullptr, nullptr));
             ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
-            ck(cudaStreamSynchronize(s), "round sync");
+            sync_run(L, "round sync");
             nres = L->h_counters[0];
             R.n_reread += L->h_counters[10];
             if (R.rounds == 1) R.n_overflow = L->h_counters[11];
@@ -594,6 +609,24 @@ void fill_stats(ffm_log* L, const LocalRun& R, uint64_t launches, bool single) {
 
 
 // ---------------------------------------------------------------- sharded runs
+template <class T>
+void dev_alloc_zero(T*& p, uint64_t count) {
+    dev_alloc(p, count);
+    ck(cudaMemset(p, 0, std::max<uint64_t>(count, 1) * sizeof(T)), "memset");
+}
+
+void ensure_cub(ffm_log* L, uint64_t n) {
+    size_t cb = cub_scan_bytes(n);
+    if (cb > L->work.cub_tmp_bytes) {
+        if (L->work.cub_tmp) cudaFree(L->work.cub_tmp);
+        L->work.cub_tmp = nullptr;
+        ck(cudaMalloc(&L->work.cub_tmp, cb), "cudaMalloc(cub)");
+        L->work.cub_tmp_bytes = cb;
+    }
+}
+
+// Buffers of the merge: n local records, M representatives of all ranks, nloc of them
+// this rank's, vcap verify work units.
 void ensure_shard(ffm_log* L, uint64_t n, uint64_t M, uint64_t nloc, uint64_t vcap, int world) {
     ShardWork& S = L->shard;
     if (n + 1 > S.n_cap || !S.flag) {
@@ -601,33 +634,23 @@ void ensure_shard(ffm_log* L, uint64_t n, uint64_t M, uint64_t nloc, uint64_t vc
         dev_alloc(S.flag, c);
         dev_alloc(S.rep_idx, c);
         S.n_cap = c;
-        size_t cb = cub_scan_bytes(c);
-        if (cb > L->work.cub_tmp_bytes) {
-            if (L->work.cub_tmp) cudaFree(L->work.cub_tmp);
-            L->work.cub_tmp = nullptr;
-            ck(cudaMalloc(&L->work.cub_tmp, cb), "cudaMalloc(cub)");
-            L->work.cub_tmp_bytes = cb;
-        }
+        ensure_cub(L, c);
     }
     uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(M, 1)));
     if (cap > S.t_cap) {
         dev_alloc(S.tkey, cap);
         dev_alloc(S.tgid, cap);
         dev_alloc(S.tidx, cap);
+        dev_alloc_zero(S.need, cap);   // zero between runs (k_seg_clear)
+        dev_alloc_zero(S.scnt, cap);
+        dev_alloc(S.sbase, cap);
+        dev_alloc(S.sfill, cap);
         S.t_cap = cap;
     }
     if (M > S.m_cap || !S.tslot) {
         uint64_t c = std::max<uint64_t>(M, 1024);
         dev_alloc(S.tslot, c);
-        dev_alloc(S.sort_keys_in, c);
-        dev_alloc(S.sort_keys_out, c);
-        dev_alloc(S.sort_vals_in, c);
-        dev_alloc(S.order, c);
-        size_t sb = sort_tmp_bytes((uint32_t)c);
-        if (S.sort_tmp) cudaFree(S.sort_tmp);
-        S.sort_tmp = nullptr;
-        ck(cudaMalloc(&S.sort_tmp, std::max<size_t>(sb, 256)), "cudaMalloc(sort)");
-        S.sort_tmp_bytes = std::max<size_t>(sb, 256);
+        dev_alloc(S.seg, c);
         S.m_cap = c;
     }
     if (nloc + 1 > S.l_cap || !S.state) {
@@ -639,13 +662,7 @@ void ensure_shard(ffm_log* L, uint64_t n, uint64_t M, uint64_t nloc, uint64_t vc
         dev_alloc(S.G, c);
         dev_alloc(S.slow_list, c);
         S.l_cap = c;
-        size_t cb = cub_scan_bytes(c);
-        if (cb > L->work.cub_tmp_bytes) {
-            if (L->work.cub_tmp) cudaFree(L->work.cub_tmp);
-            L->work.cub_tmp = nullptr;
-            ck(cudaMalloc(&L->work.cub_tmp, cb), "cudaMalloc(cub)");
-            L->work.cub_tmp_bytes = cb;
-        }
+        ensure_cub(L, c);
     }
     if (vcap > S.v_cap || !S.vitems) {
         uint64_t c = std::max<uint64_t>(vcap, 1024);
@@ -655,17 +672,166 @@ void ensure_shard(ffm_log* L, uint64_t n, uint64_t M, uint64_t nloc, uint64_t vc
     if ((uint64_t)world > S.w_cap || !S.rank_lo) {
         dev_alloc(S.rank_lo, world);
         dev_alloc(S.bases, world);
-        if (!S.n_slow) dev_alloc(S.n_slow, 1);
+        if (!S.sctr) dev_alloc(S.sctr, 4);
         S.w_cap = world;
     }
 }
 
 void free_shard(ShardWork& S) {
-    void* ptrs[] = {S.flag, S.rep_idx, S.tkey, S.tgid, S.tidx, S.tslot, S.state, S.cand, S.vcount, S.vstart,
-                    S.G, S.slow_list, S.vitems, S.rank_lo, (void*)S.bases, S.n_slow, S.sort_keys_in,
-                    S.sort_keys_out, S.sort_vals_in, S.order, S.sort_tmp};
+    void* ptrs[] = {S.flag, S.rep_idx, S.tkey, S.tgid, S.tidx, S.need, S.scnt, S.sbase, S.sfill, S.tslot, S.seg,
+                    S.state, S.cand, S.vcount, S.vstart, S.G, S.slow_list, S.vitems, S.rank_lo, (void*)S.bases, S.sctr};
     for (void* p : ptrs)
         if (p) cudaFree(p);
+}
+
+void comm_ck(ffm_log* L, int rc) {
+    if (rc == FFM_OK) return;
+    if (rc == FFM_E_CUDA) throw CudaFail{cudaErrorUnknown, L->comm.err.c_str()};
+    throw CommFail{rc, L->comm.err};
+}
+
+// grow a tuple buffer keeping its first `keep` entries (stream-ordered copy)
+void grow_tuples(ffm_log* L, RepTuple*& p, uint64_t& cap, uint64_t need, uint64_t keep) {
+    if (need <= cap && p) return;
+    RepTuple* np = nullptr;
+    const uint64_t c = std::max<uint64_t>(std::max<uint64_t>(need, 1024), cap + cap / 2);
+    ck(cudaMalloc(&np, c * sizeof(RepTuple)), "cudaMalloc(reps)");
+    if (p && keep) ck(cudaMemcpyAsync(np, p, keep * sizeof(RepTuple), cudaMemcpyDeviceToDevice, L->stream), "copy");
+    ck(cudaStreamSynchronize(L->stream), "grow sync");
+    if (p) ck(cudaFree(p), "cudaFree");
+    p = np;
+    cap = c;
+}
+
+// Peer arenas (CUDA IPC).  The handles travel through the exchange transport whenever
+// some rank's arena generation changed since the last exchange -- a decision every rank
+// takes identically from the all-gathered headers (collective).  A peer's arena is
+// mapped only while it has representatives (a rank with none is never read).
+void map_peers(ffm_log* L, const std::vector<uint64_t>& gens, const std::vector<uint64_t>& counts) {
+    const int world = L->cfg.world, rank = L->cfg.rank;
+    if (L->xgen != gens) {
+        cudaIpcMemHandle_t h;
+        static_assert(sizeof(h) == 64, "IPC handle size");
+        ck(cudaIpcGetMemHandle(&h, L->arena), "cudaIpcGetMemHandle");
+        uint8_t* hh = reinterpret_cast<uint8_t*>(L->h_hdr + 8 + 4 * (uint64_t)world);   // pinned scratch
+        memcpy(hh, &h, 64);
+        ck(cudaMemcpyAsync(L->d_ipc, hh, 64, cudaMemcpyHostToDevice, L->stream), "H2D");
+        comm_ck(L, comm_allgather(L->comm, L->d_ipc, L->d_ipc + 64, 64, L->stream));
+        ck(cudaMemcpyAsync(hh, L->d_ipc + 64, 64 * (uint64_t)world, cudaMemcpyDeviceToHost, L->stream), "D2H");
+        sync_run(L, "handle exchange sync");
+        L->xhandles.assign(hh, hh + 64 * (size_t)world);
+        L->xgen = gens;
+    }
+    L->peer_ptr.resize(world, nullptr);
+    L->peer_gen.resize(world, ~0ull);
+    for (int r = 0; r < world; ++r) {
+        if (r == rank || counts[r] == 0 || (L->peer_ptr[r] && L->peer_gen[r] == gens[r])) continue;
+        if (L->peer_ptr[r]) ck(cudaIpcCloseMemHandle(L->peer_ptr[r]), "cudaIpcCloseMemHandle");
+        L->peer_ptr[r] = nullptr;
+        cudaIpcMemHandle_t ph;
+        memcpy(&ph, L->xhandles.data() + 64ull * r, 64);
+        void* p = nullptr;
+        ck(cudaIpcOpenMemHandle(&p, ph, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+        L->peer_ptr[r] = p;
+        L->peer_gen[r] = gens[r];
+    }
+}
+
+// One collective run of a sharded log (include/ffm.h "Sharded logs"): local H1..H4 with
+// the representative export and the header exchange queued before the first sync; then
+// the representative all-gather, the merge (global group-by, peer-memory verify, slow
+// segments decided on the device), labels, the all-reduce of the per-site sums and the
+// outputs before the second.
+void run_sharded(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, bool dup_dev, bool ben_dev, LocalRun& R,
+                 uint64_t& launches) {
+    const int world = L->cfg.world, rank = L->cfg.rank;
+    const uint64_t n = L->h_size.size();
+    const uint32_t ns = L->cfg.n_sites;
+    Work& W = L->work;
+    ShardWork& S = L->shard;
+    cudaStream_t s = L->stream;
+    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
+    ensure_shard(L, n, 1, 1, 1, world);
+    grow_tuples(L, L->d_send, L->send_cap, std::max<uint64_t>(n, 1), 0);
+    const DevLog D = dev_view(L);
+    const std::function<void()> exchange_header = [&]() {
+        LCHK(launch_rep_export(D, W, S, L->params, L->d_send, s));
+        LCHK(launch_shard_header(S.rep_idx + n, W.counters, L->arena_gen, n, L->d_hdr, s));
+        comm_ck(L, comm_allgather(L->comm, L->d_hdr, L->d_hdr + 4, 4 * sizeof(uint64_t), s));
+        ck(cudaMemcpyAsync(L->h_hdr, L->d_hdr + 4, 32 * (uint64_t)world, cudaMemcpyDeviceToHost, s), "D2H");
+    };
+    // sync 1: local classes (speculative export: valid unless some rank had residuals)
+    R = run_local(L, D, L->n_large_chunks, launches, false, nullptr, false, &exchange_header);
+    bool any_res = false;
+    for (int r = 0; r < world; ++r) any_res |= L->h_hdr[4 * r + 1] != 0;
+    if (any_res) {   // every rank re-exports its final classes (collective)
+        exchange_header();
+        sync_run(L, "header sync");
+    }
+    if (timing) ck(cudaEventRecord(L->ev[13], s), "event");
+    std::vector<uint64_t> counts(world), gens(world);
+    std::vector<uint32_t> rank_lo(world);
+    uint64_t M = 0, maxc = 0;
+    for (int r = 0; r < world; ++r) {
+        counts[r] = L->h_hdr[4 * r];
+        gens[r] = L->h_hdr[4 * r + 2];
+        rank_lo[r] = (uint32_t)M;
+        M += counts[r];
+        maxc = std::max(maxc, counts[r]);
+    }
+    if (M >= 0xFFFFFFFFull) throw CommFail{FFM_E_RANGE, "too many representatives"};
+    map_peers(L, gens, counts);
+    const uint64_t nloc = counts[rank], lo = rank_lo[rank];
+    ensure_shard(L, n, M, nloc, nloc + L->n_large_chunks + 64, world);
+    // all-gather of the representatives (padded to the largest count), compacted rank-major
+    grow_tuples(L, L->d_send, L->send_cap, std::max<uint64_t>(maxc, 1), nloc);
+    grow_tuples(L, L->d_recv, L->recv_cap, std::max<uint64_t>(maxc * world, 1), 0);
+    grow_tuples(L, L->d_T, L->T_cap, std::max<uint64_t>(M, 1), 0);
+    if (maxc) comm_ck(L, comm_allgather(L->comm, L->d_send, L->d_recv, maxc * sizeof(RepTuple), s));
+    for (int r = 0; r < world; ++r)
+        if (counts[r])
+            ck(cudaMemcpyAsync(L->d_T + rank_lo[r], L->d_recv + maxc * r, counts[r] * sizeof(RepTuple),
+                               cudaMemcpyDeviceToDevice, s),
+               "compact reps");
+    // rank tables (pinned staging: the copies stay asynchronous)
+    uint32_t* h_lo = reinterpret_cast<uint32_t*>(L->h_hdr + 8 + 4 * (uint64_t)world + 8 * (uint64_t)world);
+    const uint8_t** h_bases = reinterpret_cast<const uint8_t**>(h_lo + world + (world & 1));
+    for (int r = 0; r < world; ++r) {
+        h_lo[r] = rank_lo[r];
+        h_bases[r] = r == rank ? L->arena : (const uint8_t*)L->peer_ptr[r];
+    }
+    ck(cudaMemcpyAsync(S.rank_lo, h_lo, world * sizeof(uint32_t), cudaMemcpyHostToDevice, s), "H2D");
+    ck(cudaMemcpyAsync((void*)S.bases, h_bases, world * sizeof(void*), cudaMemcpyHostToDevice, s), "H2D");
+    const uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(M, 1)));
+    LCHK(launch_merge(D, W, S, L->params, L->d_T, (uint32_t)M, (uint32_t)lo, (uint32_t)nloc, world, rank, cap, s));
+    int64_t* d_dup = dup_dev ? dup_out : W.dup;
+    LCHK(launch_merge_label(D, W, S, L->params, ns, d_dup, s));
+    // per-site benefit and duplicate counts ([ben | cnt], contiguous) summed over ranks
+    comm_ck(L, comm_allreduce_u64(L->comm, W.ben, 2 * (uint64_t)ns, s));
+    if (!dup_dev && n)
+        ck(cudaMemcpyAsync(dup_out, d_dup, n * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
+    if (ben_out)
+        ck(cudaMemcpyAsync(ben_out, W.ben, ns * sizeof(uint64_t),
+                           ben_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s),
+           "copy ben");
+    ck(cudaMemcpyAsync(L->h_hdr + 4 * (uint64_t)world, S.sctr, 4 * sizeof(uint64_t), cudaMemcpyDeviceToHost, s),
+       "D2H");
+    if (timing) ck(cudaEventRecord(L->ev[14], s), "event");
+    // sync 2: outputs written; every peer finished reading this rank's arena (its
+    // compare kernels precede its part of the all-reduce)
+    sync_run(L, "sharded output sync");
+    ck(cudaGetLastError(), "sharded run");
+    fill_stats(L, R, launches, false);
+    L->stats.n_reps_local = nloc;
+    L->stats.n_reps_global = M;
+    L->stats.n_slow = L->h_hdr[4 * world];
+    L->stats.remote_verify_bytes = L->h_hdr[4 * world + 2];
+    L->stats.n_residual += L->stats.n_slow;
+    L->stats.exchange_bytes = L->comm.bytes_moved;
+    if (timing) {
+        L->stats.ms_exchange = ev_ms(L->ev[13], L->ev[14]);
+        L->stats.ms_total = ev_ms(L->ev[0], L->ev[14]);
+    }
 }
 
 }  // namespace
@@ -706,6 +872,8 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
     if (cfg->n_sites == 0 || cfg->digest_bits > 64 || cfg->refine_bits > 64 || cfg->world < 1 ||
         cfg->rank < 0 || cfg->rank >= cfg->world)
         return FFM_E_INVAL;
+    if (cfg->world > 1 && (cfg->nccl_id == nullptr) == (cfg->comm == nullptr))
+        return FFM_E_INVAL;   // a sharded log needs exactly one exchange transport
     uint32_t chunk = cfg->chunk_bytes ? cfg->chunk_bytes : 32768;
     uint32_t small = cfg->small_bytes ? cfg->small_bytes : 4096;
     if (chunk % 1024 || small % 128 || chunk == 0) return FFM_E_INVAL;
@@ -732,13 +900,8 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
         int hp = 0;
         ck(cudaDeviceGetAttribute(&hp, cudaDevAttrCanUseHostPointerForRegisteredMem, L->device), "attr");
         L->host_ptr_ok = hp != 0;
-        L->gather_max = kGatherMaxDefault;
-        if (const char* e = getenv("FFM_GATHER_MAX")) L->gather_max = strtoull(e, nullptr, 10);   // tuning knob
+        L->gather_max = kGatherMax;
         L->params.prefix_bytes = std::min<uint32_t>(4096, chunk);   // a multiple of 256 (chunk: of 1024)
-        if (const char* e = getenv("FFM_PREFIX_BYTES")) {                // tuning knob (same results)
-            const uint32_t v = (uint32_t)strtoul(e, nullptr, 10);
-            if (v >= 256 && v % 256 == 0) L->params.prefix_bytes = std::min(v, chunk);
-        }
         L->params.chunk_bytes = chunk;
         L->params.small_bytes = small;
         L->params.digest_mask = cfg->digest_bits >= 64 ? ~0ull : ((1ull << cfg->digest_bits) - 1);
@@ -760,6 +923,19 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
         }
         for (auto& e : L->ev) ck(cudaEventCreate(&e), "event");
         ck(cudaHostAlloc((void**)&L->h_counters, 16 * sizeof(uint32_t), cudaHostAllocDefault), "cudaHostAlloc");
+        if (cfg->world > 1) {
+            const uint64_t w = (uint64_t)cfg->world;
+            ck(cudaMalloc(&L->d_hdr, (4 + 4 * w) * sizeof(uint64_t)), "cudaMalloc(hdr)");
+            ck(cudaMalloc(&L->d_ipc, 64 * (w + 1)), "cudaMalloc(ipc)");
+            // headers [4w] | run counters [8] | IPC handles [8w] | rank table [w u32] | bases [w]
+            ck(cudaHostAlloc((void**)&L->h_hdr, (16 + 16 * w) * sizeof(uint64_t), cudaHostAllocDefault),
+               "cudaHostAlloc(hdr)");
+            const int rc = comm_init(L->comm, cfg->world, cfg->rank, cfg->nccl_id, cfg->comm);
+            if (rc != FFM_OK) {
+                ffm_log_destroy(L);
+                return rc;
+            }
+        }
         if (cfg->arena_bytes) ensure_arena(L, cfg->arena_bytes);
         if (cfg->max_records) {
             L->h_site.reserve(cfg->max_records);
@@ -804,18 +980,36 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
         ensure_arena(L, end);
         std::vector<uint64_t> desc;
         if (kind == FFM_PAYLOAD_DEVICE || kind == FFM_PAYLOAD_HOST_PINNED) desc.reserve(3 * n);
-        bool need_sync = false;
+        bool need_sync = false, ordered = false;
         for (uint64_t i = 0; i < n; ++i) {
             if (sizes[i] == 0) continue;
-            int src = kind;
-            if (kind == FFM_PAYLOAD_AUTO) src = pointer_kind(payloads[i]);
+            int src = kind, pdev = L->device;
+            if (kind == FFM_PAYLOAD_AUTO) {
+                src = pointer_kind(payloads[i], &pdev);
+            } else if (kind == FFM_PAYLOAD_DEVICE) {
+                int d = -1;   // which GPU (a peer GPU's memory is never dereferenced by k_gather)
+                if (pointer_kind(payloads[i], &d) == FFM_PAYLOAD_DEVICE) pdev = d;
+            }
             const bool ring = src == FFM_PAYLOAD_HOST;        // pageable host: via the pinned ring
+            if (src == FFM_PAYLOAD_DEVICE && !ordered) {
+                // device payloads may still be being produced: the staging stream waits for
+                // the log's stream and the legacy default stream first (ffm.h)
+                ordered = true;
+                ck(cudaEventRecord(L->fork_ev[0], cudaStreamLegacy), "event");
+                ck(cudaStreamWaitEvent(L->stage_stream, L->fork_ev[0], 0), "wait producer");
+                if (L->stream != cudaStreamLegacy) {
+                    ck(cudaEventRecord(L->fork_ev[1], L->stream), "event");
+                    ck(cudaStreamWaitEvent(L->stage_stream, L->fork_ev[1], 0), "wait producer");
+                }
+            }
             // the ring uploads one contiguous arena range: close it before a record that
             // is written into the arena by another path
             if (!ring && L->ring_fill) ring_flush(L);
             if (ring) {
                 stage_host(L, payloads[i], sizes[i], offs[i]);
-            } else if (sizes[i] > L->gather_max || (src == FFM_PAYLOAD_HOST_PINNED && !L->host_ptr_ok)) {
+            } else if (sizes[i] > L->gather_max || (src == FFM_PAYLOAD_HOST_PINNED && !L->host_ptr_ok) ||
+                       (src == FFM_PAYLOAD_DEVICE && pdev != L->device)) {
+                // (a payload on another GPU: the copy engines, never a kernel dereference)
                 need_sync = true;     // async copy engine from caller memory: sync before return
                 ck(cudaMemcpyAsync(L->arena + offs[i], payloads[i], sizes[i], cudaMemcpyDefault, L->stage_stream),
                    "copy");
@@ -844,7 +1038,6 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
         if (need_sync) ck(cudaStreamSynchronize(L->stage_stream), "append sync");   // snapshot before return
         push_meta(L, n, sites, sizes, durs, gids, channels, offs, end);
         L->digests_valid = false;
-        if (n > 1) upload_meta(L);
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
     } catch (const std::bad_alloc&) {
@@ -873,8 +1066,9 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
     if (st) return st;
     uint64_t n = L->h_size.size();
     if (n > 0 && !dup_out) return set_err(L, FFM_E_INVAL, "duplicate_of is NULL");
-    if (L->cfg.world > 1) return set_err(L, FFM_E_STATE, "sharded log: use ffm_shard_local / ffm_shard_merge");
     try {
+        L->n_syncs = 0;
+        L->comm.bytes_moved = 0;
         run_prologue(L);
         Work& W = L->work;
         cudaStream_t s = L->stream;
@@ -883,6 +1077,12 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         bool ben_dev = ben_out && is_device_ptr(ben_out);
         int64_t* d_dup = dup_dev ? dup_out : W.dup;
         uint64_t launches = 0;
+        if (L->cfg.world > 1) {
+            LocalRun R{};
+            run_sharded(L, dup_out, ben_out, dup_dev, ben_dev, R, launches);
+            L->stats.host_syncs = L->n_syncs;
+            return FFM_OK;
+        }
         const bool prefilter = (L->cfg.flags & FFM_FLAG_PREFILTER) != 0;
         LocalRun R = run_local(L, dev_view(L), L->n_large_chunks, launches, true, d_dup, prefilter);
         // H7 return
@@ -895,9 +1095,10 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
                                ben_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s),
                "copy ben");
         if (timing) ck(cudaEventRecord(L->ev[5], s), "event");
-        ck(cudaStreamSynchronize(s), "output sync");
+        sync_run(L, "output sync");
         ck(cudaGetLastError(), "run");
         fill_stats(L, R, launches, true);
+        L->stats.host_syncs = L->n_syncs;
         // adaptive round 0: more than half of the candidates failed the fused compare
         // (near-duplicates sharing first chunks) -> hash-all-then-verify is cheaper
         // (residuals settled through difference lists cost no re-read: what counts are the
@@ -907,161 +1108,19 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
             L->prefer_two_pass = true;
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
+    } catch (const CommFail& f) {
+        // an exchange failed part-way through a collective: the ranks are out of step
+        L->poisoned = true;
+        return set_err(L, f.code, f.what);
     } catch (const std::bad_alloc&) {
         return set_err(L, FFM_E_NOMEM, "host allocation failed");
     }
     return FFM_OK;
 }
 
-int ffm_shard_ipc_handle(ffm_log* L, void* out) {
-    int st = check_state(L);
-    if (st) return st;
-    if (!out) return FFM_E_INVAL;
-    try {
-        ck(cudaSetDevice(L->device), "cudaSetDevice");
-        ensure_arena(L, 1);
-        cudaIpcMemHandle_t h;
-        ck(cudaIpcGetMemHandle(&h, L->arena), "cudaIpcGetMemHandle");
-        static_assert(sizeof(h) == 64, "IPC handle size");
-        memcpy(out, &h, 64);
-    } catch (const CudaFail& f) {
-        return fail_cuda(L, f);
-    }
-    return FFM_OK;
-}
-
-int ffm_shard_open_peer(ffm_log* L, int32_t peer, const void* handle) {
-    int st = check_state(L);
-    if (st) return st;
-    if (!handle || peer < 0 || peer >= L->cfg.world) return set_err(L, FFM_E_INVAL, "bad peer rank / handle");
-    if (peer == L->cfg.rank) return FFM_OK;
-    try {
-        ck(cudaSetDevice(L->device), "cudaSetDevice");
-        if (L->peer_ptr.size() < (size_t)L->cfg.world) {
-            L->peer_ptr.resize(L->cfg.world, nullptr);
-            L->peer_handle.resize(L->cfg.world);
-        }
-        std::string hb((const char*)handle, 64);
-        if (L->peer_ptr[peer] && L->peer_handle[peer] == hb) return FFM_OK;
-        if (L->peer_ptr[peer]) ck(cudaIpcCloseMemHandle(L->peer_ptr[peer]), "cudaIpcCloseMemHandle");
-        L->peer_ptr[peer] = nullptr;
-        cudaIpcMemHandle_t h;
-        memcpy(&h, handle, 64);
-        void* p = nullptr;
-        ck(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
-        L->peer_ptr[peer] = p;
-        L->peer_handle[peer] = hb;
-    } catch (const CudaFail& f) {
-        return fail_cuda(L, f);
-    }
-    return FFM_OK;
-}
-
-int ffm_shard_local(ffm_log* L, ffm_rep* reps_out, uint64_t cap, uint64_t* n_reps_out) {
-    int st = check_state(L);
-    if (st) return st;
-    uint64_t n = L->h_size.size();
-    if (!n_reps_out || (n && !reps_out)) return set_err(L, FFM_E_INVAL, "NULL argument");
-    if (cap < n) return set_err(L, FFM_E_RANGE, "reps_out capacity < ffm_log_count");
-    try {
-        run_prologue(L);
-        uint64_t launches = 0;
-        LocalRun R = run_local(L, dev_view(L), L->n_large_chunks, launches, false, nullptr);
-        ensure_shard(L, n, 1, 1, 1, std::max(L->cfg.world, 1));
-        DevLog D = dev_view(L);
-        cudaStream_t s = L->stream;
-        LCHK(launch_rep_export(D, L->work, L->shard, L->params, (RepTuple*)reps_out, s));
-        ck(cudaMemcpyAsync(L->h_counters, L->shard.rep_idx + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
-        ck(cudaStreamSynchronize(s), "shard local sync");
-        L->n_reps = L->h_counters[0];
-        L->reps_valid = true;
-        *n_reps_out = L->n_reps;
-        fill_stats(L, R, launches, false);
-    } catch (const CudaFail& f) {
-        return fail_cuda(L, f);
-    } catch (const std::bad_alloc&) {
-        return set_err(L, FFM_E_NOMEM, "host allocation failed");
-    }
-    return FFM_OK;
-}
-
-int ffm_shard_merge(ffm_log* L, const ffm_rep* all_reps, const uint64_t* counts, int64_t* dup_out,
-                    uint64_t* ben_out) {
-    int st = check_state(L);
-    if (st) return st;
-    const int world = L->cfg.world, rank = L->cfg.rank;
-    uint64_t n = L->h_size.size();
-    if (!counts || (n && !dup_out) || !ben_out) return set_err(L, FFM_E_INVAL, "NULL argument");
-    if (!L->reps_valid) return set_err(L, FFM_E_STATE, "ffm_shard_local must run first");
-    uint64_t M = 0, lo = 0;
-    std::vector<uint32_t> rank_lo(world);
-    for (int r = 0; r < world; ++r) {
-        rank_lo[r] = (uint32_t)M;
-        if (r == rank) lo = M;
-        M += counts[r];
-    }
-    if (counts[rank] != L->n_reps) return set_err(L, FFM_E_COMM, "counts[rank] != this rank's n_reps");
-    if (M >= 0xFFFFFFFFull) return set_err(L, FFM_E_RANGE, "too many representatives");
-    if (M && !all_reps) return set_err(L, FFM_E_INVAL, "NULL all_reps");
-    std::vector<const uint8_t*> bases(world, nullptr);
-    for (int r = 0; r < world; ++r) {
-        if (r == rank) {
-            bases[r] = L->arena;
-        } else if (counts[r]) {
-            if ((size_t)r >= L->peer_ptr.size() || !L->peer_ptr[r])
-                return set_err(L, FFM_E_STATE, "peer arena not mapped (ffm_shard_open_peer)");
-            bases[r] = (const uint8_t*)L->peer_ptr[r];
-        }
-    }
-    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
-    try {
-        ck(cudaSetDevice(L->device), "cudaSetDevice");
-        const uint64_t nloc = L->n_reps;
-        uint64_t vcap = nloc + L->n_large_chunks + 64;
-        ensure_shard(L, n, M, nloc, vcap, world);
-        ShardWork& S = L->shard;
-        Work& W = L->work;
-        cudaStream_t s = L->stream;
-        DevLog D = dev_view(L);
-        uint64_t launches = 0;
-        if (timing) ck(cudaEventRecord(L->ev[13], s), "event");
-        ck(cudaMemcpyAsync(S.rank_lo, rank_lo.data(), world * sizeof(uint32_t), cudaMemcpyHostToDevice, s), "H2D");
-        ck(cudaMemcpyAsync((void*)S.bases, bases.data(), world * sizeof(void*), cudaMemcpyHostToDevice, s), "H2D");
-        uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(M, 1)));
-        LCHK(launch_merge(D, W, S, L->params, (const RepTuple*)all_reps, (uint32_t)M, (uint32_t)lo, (uint32_t)nloc,
-                          world, rank, cap, s));
-        ck(cudaMemcpyAsync(L->h_counters, S.n_slow, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
-        ck(cudaStreamSynchronize(s), "merge sync");
-        uint32_t n_slow = L->h_counters[0];
-        if (n_slow) {
-            LCHK(launch_sort_prep(S, (const RepTuple*)all_reps, (uint32_t)M, s));
-            LCHK(launch_merge_slow(D, W, S, L->params, (const RepTuple*)all_reps, (uint32_t)M, (uint32_t)lo, world,
-                                   rank, n_slow, s));
-        }
-        bool dup_dev = dup_out && is_device_ptr(dup_out);
-        bool ben_dev = is_device_ptr(ben_out);
-        int64_t* d_dup = dup_dev ? dup_out : W.dup;
-        LCHK(launch_merge_label(D, W, S, L->params, L->cfg.n_sites, d_dup, s));
-        if (!dup_dev && n)
-            ck(cudaMemcpyAsync(dup_out, d_dup, n * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
-        ck(cudaMemcpyAsync(ben_out, W.ben, L->cfg.n_sites * sizeof(uint64_t),
-                           ben_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s),
-           "copy ben");
-        if (timing) ck(cudaEventRecord(L->ev[14], s), "event");
-        ck(cudaStreamSynchronize(s), "merge output sync");
-        ck(cudaGetLastError(), "merge");
-        L->stats.kernel_launches += launches;
-        L->stats.n_residual += n_slow;
-        if (timing) {
-            L->stats.ms_output = ev_ms(L->ev[13], L->ev[14]);
-            L->stats.ms_total = ev_ms(L->ev[0], L->ev[14]);
-        }
-    } catch (const CudaFail& f) {
-        return fail_cuda(L, f);
-    } catch (const std::bad_alloc&) {
-        return set_err(L, FFM_E_NOMEM, "host allocation failed");
-    }
-    return FFM_OK;
+int ffm_nccl_unique_id(void* id_out) {
+    if (!id_out) return FFM_E_INVAL;
+    return comm_unique_id(id_out);
 }
 
 int ffm_site_duplicate_counts(ffm_log* L, uint64_t* counts_out) {
@@ -1191,14 +1250,6 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
             ck(cudaMemcpyAsync((void*)S.bases, bases, sizeof(bases), cudaMemcpyHostToDevice, s), "H2D");
             uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(M, 1)));
             LCHK(launch_merge(D, W, S, L->params, L->online_T, (uint32_t)M, (uint32_t)np, (uint32_t)nloc, 2, 1, cap, s));
-            ck(cudaMemcpyAsync(L->h_counters, S.n_slow, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
-            ck(cudaStreamSynchronize(s), "online merge sync");
-            n_slow = L->h_counters[0];
-            if (n_slow) {
-                LCHK(launch_sort_prep(S, L->online_T, (uint32_t)M, s));
-                LCHK(launch_merge_slow(D, W, S, L->params, L->online_T, (uint32_t)M, (uint32_t)np, 2, 1,
-                                       (uint32_t)n_slow, s));
-            }
             const bool dup_dev = is_device_ptr(dup_out);
             int64_t* d_dup = dup_dev ? dup_out : W.dup;
             LCHK(launch_merge_label(D, W, S, L->params, ns, d_dup, s));
@@ -1207,10 +1258,12 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
             // new classes join the stored representatives
             LCHK(launch_online_newreps(W, S, L->online_T + np, (uint32_t)nloc, L->online_tmp, s));
             ck(cudaMemcpyAsync(L->h_counters, S.vstart + nloc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+            ck(cudaMemcpyAsync(L->h_counters + 2, S.sctr, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
             if (!dup_dev)
                 ck(cudaMemcpyAsync(dup_out, d_dup, nw * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
             ck(cudaStreamSynchronize(s), "online new reps sync");
             const uint64_t n_new = L->h_counters[0];
+            n_slow = L->h_counters[2];
             if (n_new)
                 ck(cudaMemcpyAsync(L->online_T + np, L->online_tmp, n_new * sizeof(ffm::RepTuple),
                                    cudaMemcpyDeviceToDevice, s),
@@ -1281,8 +1334,6 @@ int ffm_log_reset(ffm_log* L) {
     L->n_large_rec = 0;
     L->arena_used = 0;
     L->ring_fill = 0;
-    L->n_reps = 0;
-    L->reps_valid = false;
     L->online_done = L->online_np = 0;
     if (L->online_ben) {
         cudaMemset(L->online_ben, 0, L->cfg.n_sites * sizeof(uint64_t));
@@ -1303,7 +1354,7 @@ int ffm_log_destroy(ffm_log* L) {
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
                     W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.fitems, W.sdesc, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
-                    W.dup, W.ben, W.cnt, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
+                    W.dup, W.ben, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
                     L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)
         if (p) cudaFree(p);
@@ -1314,6 +1365,11 @@ int ffm_log_destroy(ffm_log* L) {
         if (p) cudaFree(p);
     for (void* p : L->peer_ptr)
         if (p) cudaIpcCloseMemHandle(p);
+    void* sp[] = {L->d_send, L->d_recv, L->d_T, L->d_hdr, L->d_ipc};
+    for (void* p : sp)
+        if (p) cudaFree(p);
+    if (L->h_hdr) cudaFreeHost(L->h_hdr);
+    comm_destroy(L->comm);
     for (int i = 0; i < 2; ++i) {
         if (L->ring[i]) cudaFreeHost(L->ring[i]);
         if (L->ring_ev[i]) cudaEventDestroy(L->ring_ev[i]);

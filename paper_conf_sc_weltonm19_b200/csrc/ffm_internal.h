@@ -8,6 +8,7 @@
 #include <vector>
 
 #include "../../include/ffm.h"
+#include "ffm_comm.h"
 
 namespace ffm {
 
@@ -72,22 +73,27 @@ struct Work {
 };
 
 // One representative per exact local class, exported for the cross-shard merge.
-// Layout identical to ffm_rep (include/ffm.h).
 struct RepTuple {
     uint64_t key;    // group key of the full digest (same function on every rank)
     uint64_t size;
     uint64_t gid;    // global gid of the class's first local record
     uint64_t off;    // arena offset on the owning rank
     uint64_t chan;   // channel id (destination-aware variant), 0 = content only
+    uint64_t dig;    // full 64-bit digest (prunes the slow path; a function of the bytes)
 };
 
 struct ShardWork {
     uint32_t* flag = nullptr;        // [n+1]
     uint32_t* rep_idx = nullptr;     // [n+1] exclusive scan of flag: tuple index of each local rep
-    uint64_t* tkey = nullptr;        // [cap]
+    uint64_t* tkey = nullptr;        // [cap] global table over all representatives
     uint64_t* tgid = nullptr;        // [cap]
     uint32_t* tidx = nullptr;        // [cap]
+    uint32_t* need = nullptr;        // [cap] slow path: key has a slow representative (zero between runs)
+    uint32_t* scnt = nullptr;        // [cap] its segment length (zero between runs)
+    uint32_t* sbase = nullptr;       // [cap] its segment start
+    uint32_t* sfill = nullptr;       // [cap]
     uint32_t* tslot = nullptr;       // [M]
+    uint32_t* seg = nullptr;         // [M] tuple indices, grouped by key segment
     uint32_t* state = nullptr;       // [nloc]
     uint32_t* cand = nullptr;        // [nloc]
     uint32_t* vcount = nullptr;      // [nloc+1]
@@ -97,13 +103,7 @@ struct ShardWork {
     uint2* vitems = nullptr;         // merge verify work units
     uint32_t* rank_lo = nullptr;     // [world] first tuple index of each rank
     const uint8_t** bases = nullptr; // [world] arena base of each rank (peer ones IPC-mapped)
-    uint32_t* n_slow = nullptr;
-    uint64_t* sort_keys_in = nullptr;
-    uint64_t* sort_keys_out = nullptr;
-    uint32_t* sort_vals_in = nullptr;
-    uint32_t* order = nullptr;       // [M] tuple indices sorted by gid (slow path)
-    void* sort_tmp = nullptr;
-    size_t sort_tmp_bytes = 0;
+    unsigned long long* sctr = nullptr;  // [4] n_slow, segment cursor, remote verify bytes (B_x)
     uint64_t n_cap = 0, m_cap = 0, t_cap = 0, l_cap = 0, v_cap = 0, w_cap = 0;
 };
 
@@ -143,14 +143,12 @@ int launch_site_reduce(const uint64_t* part, const uint32_t* cpart, uint32_t row
 int launch_rep_export(const DevLog& L, Work& W, ShardWork& S, const Params& P, RepTuple* out, cudaStream_t st);
 int launch_merge(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
                  uint32_t lo, uint32_t nloc, int world, int rank, uint64_t cap, cudaStream_t st);
-int launch_sort_prep(ShardWork& S, const RepTuple* T, uint32_t M, cudaStream_t st);
-size_t sort_tmp_bytes(uint32_t M);
-int launch_merge_slow(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
-                      uint32_t lo, int world, int rank, uint32_t n_slow, cudaStream_t st);
 int launch_online_newreps(Work& W, ShardWork& S, RepTuple* Tw, uint32_t nloc, RepTuple* tmp, cudaStream_t st);
 int launch_vec_add(uint64_t* a, const uint64_t* b, uint32_t n, cudaStream_t st);
 int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
                        cudaStream_t st);
+int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uint64_t gen, uint64_t n,
+                        uint64_t* hdr, cudaStream_t st);
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t st);
@@ -225,12 +223,21 @@ struct ffm_log {
     uint64_t ring_fill = 0;         // bytes used in ring[cur]
     bool ring_pending = false;
 
-    // sharded runs
+    // sharded runs (world > 1)
+    ffm::Comm comm;
     ffm::ShardWork shard;
-    uint64_t n_reps = 0;            // representatives exported by the last ffm_shard_local
-    bool reps_valid = false;
+    uint64_t arena_gen = 0;         // bumped whenever the arena is reallocated (peers re-map it)
+    std::vector<uint64_t> xgen;     // every rank's arena generation at the last handle exchange
+    std::vector<uint8_t> xhandles;  // the IPC handles of that exchange (64 B per rank)
+    std::vector<uint64_t> peer_gen; // generation of each mapped peer arena
     std::vector<void*> peer_ptr;    // IPC-mapped peer arenas (index = rank)
-    std::vector<std::string> peer_handle;
+    ffm::RepTuple* d_send = nullptr;   // this rank's representatives (padded to the max count)
+    ffm::RepTuple* d_recv = nullptr;   // all-gathered, world x max count
+    ffm::RepTuple* d_T = nullptr;      // compacted, rank-major
+    uint64_t send_cap = 0, recv_cap = 0, T_cap = 0;
+    uint64_t* d_hdr = nullptr;         // [4] this rank's header; [4 + 4 * world] all headers
+    uint8_t* d_ipc = nullptr;          // [64 * (world + 1)] IPC handle exchange
+    uint64_t* h_hdr = nullptr;         // pinned mirror of all headers (+ run counters)
 
     // online (streaming) mode: representatives of every class seen so far
     uint64_t online_done = 0;        // records already labelled online
@@ -256,5 +263,6 @@ struct ffm_log {
     uint32_t* h_counters = nullptr;   // pinned mirror
     cudaEvent_t ev[20] = {};
     ffm_run_stats stats{};
+    uint64_t n_syncs = 0;             // host synchronisations of the run stream (this run)
     bool digests_valid = false;
 };

@@ -122,9 +122,6 @@ constexpr int kVerifyU = 2;
 #ifndef FFM_SMALL_U
 #define FFM_SMALL_U 2
 #endif
-#ifndef FFM_SMALL_MINB
-#define FFM_SMALL_MINB 3
-#endif
 constexpr int kSmallU = FFM_SMALL_U;
 
 __global__ void __launch_bounds__(256, 4) k_hash_small(DevLog L, uint32_t small_bytes, uint64_t* __restrict__ accA,
@@ -515,9 +512,6 @@ __device__ __forceinline__ bool prefix_unique(const Work& W, uint32_t r) {
 #endif
 #ifndef FFM_FX_MINB          // __launch_bounds__ min blocks (register budget)
 #define FFM_FX_MINB FFM_FX_CTAS
-#endif
-#ifndef FFM_SMALL_OWN_EVICT_FIRST  // k_fused_small: own bytes evict_first (1) or normal L2 policy (0)
-#define FFM_SMALL_OWN_EVICT_FIRST 1
 #endif
 constexpr int kFxConsumers = 8;                       // consumer warps
 constexpr int kFxThreads = 32 * (kFxConsumers + 1);   // + one producer warp
@@ -1144,10 +1138,6 @@ __global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const
 // cross-shard / online merges need it) and, for a member of a prefix group, byte-compares
 // it with the group's leader -- re-uploads of one content share their leader, so its
 // bytes are L2-hot; the member's own bytes are read from HBM once.
-#ifndef FFM_SMALL_ASYNC   // 1: per-lane cp.async pipeline (default), 0: register octet kernel
-#define FFM_SMALL_ASYNC 1
-#endif
-#if FFM_SMALL_ASYNC
 // Per-thread cp.async pipeline: every lane is its own producer.  A lane's work is the
 // sequence of steps (record, 16*U 16-byte words of it) of its octet; it keeps S-1 steps
 // of its own and its leader's words in flight in shared memory (cp.async, no registers
@@ -1362,125 +1352,6 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
 }
-#else
-__global__ void __launch_bounds__(256, FFM_SMALL_MINB) k_fused_small(DevLog L, Work W, uint32_t* res_out) {
-    const int g = threadIdx.x & 7;
-    const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
-    const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
-    const unsigned omask = 0xFFu << (threadIdx.x & 24);
-    // descriptors of k_leader0 at the record's position in the size-class order:
-    // (own arena offset, leader's offset or ~0 when not compared, size, record)
-    uint4 da = make_uint4(0, 0, 0, 0), db = make_uint4(0, 0, 0, 0);
-    if (oct < L.n_small) {
-        da = W.sdesc[2ull * oct];
-        db = W.sdesc[2ull * oct + 1];
-    }
-    for (uint32_t i = oct; i < L.n_small; i += noct) {
-        const uint64_t off = (uint64_t)da.y << 32 | da.x, loff = (uint64_t)da.w << 32 | da.z;
-        const uint64_t n = db.x;
-        const uint32_t r = db.y;
-        if (i + noct < L.n_small) {   // the next record's descriptor, in flight meanwhile
-            da = W.sdesc[2ull * (i + noct)];
-            db = W.sdesc[2ull * (i + noct) + 1];
-        }
-        const bool cmp = loff != ~0ull;
-        const uint8_t* base = L.arena + off;
-        const uint8_t* lb = L.arena + (cmp ? loff : off);
-        const uint32_t nblk = (uint32_t)((n + 31) >> 5);
-        const uint32_t nfull = (uint32_t)(n >> 5);   // blocks with all 32 bytes in the record
-        LaneKeys K;
-        load_keys(K, 2 * g, 0);   // (constant cache; not kept live across records: registers)
-        uint64_t A = 0, B = 0, found = ~0ull;
-        bool cmp_on = cmp;                            // this lane still looking for a mismatch
-        uint32_t b0 = 0, hit = ~0u;
-        // fast path: iterations whose blocks are all full -- no tail masks, no per-block
-        // bounds, the compare an OR-reduction (the exact first mismatch only on a hit)
-#pragma unroll 1
-        for (; b0 + 8 * kSmallU <= nfull; b0 += 8 * kSmallU) {
-            Blk x[kSmallU], y[kSmallU];
-#pragma unroll
-            for (int u = 0; u < kSmallU; ++u) {
-#if FFM_SMALL_OWN_EVICT_FIRST
-                x[u] = ld_stream(base + 32ull * (b0 + 8 * u + g));
-#else
-                x[u] = ld_remote(base + 32ull * (b0 + 8 * u + g));
-#endif
-                if (cmp_on) y[u] = ld_keep(lb + 32ull * (b0 + 8 * u + g));
-            }
-#pragma unroll
-            for (int u = 0; u < kSmallU; ++u) {
-                nh_word(x[u].v[0], x[u].v[1], x[u].v[2], x[u].v[3], K.k[0], A, B);
-                nh_word(x[u].v[4], x[u].v[5], x[u].v[6], x[u].v[7], K.k[1], A, B);
-                advance<1>(K);
-            }
-            if (cmp_on) {
-                uint32_t d = 0;
-#pragma unroll
-                for (int u = 0; u < kSmallU; ++u)
-#pragma unroll
-                    for (int i = 0; i < 8; ++i) d |= x[u].v[i] ^ y[u].v[i];
-                if (d) {          // rare: located exactly after the loop (keeps x, y short-lived)
-                    hit = b0;
-                    cmp_on = false;
-                }
-            }
-        }
-        if (hit != ~0u) {
-#pragma unroll 1
-            for (int u = 0; u < kSmallU; ++u) {   // lowest differing block of the hit iteration
-                const uint32_t b = hit + 8 * u + g;
-                const int dd = blk_diff(ld_stream(base + 32ull * b), ld_keep(lb + 32ull * b));
-                if (dd >= 0) {
-                    found = 2ull * b + dd;
-                    break;
-                }
-            }
-        }
-        // tail: the remaining (partial) iterations, masked
-#pragma unroll 1
-        for (; b0 < nblk; b0 += 8 * kSmallU) {
-            Blk x[kSmallU], y[kSmallU];
-#pragma unroll
-            for (int u = 0; u < kSmallU; ++u) {
-                const uint32_t b = b0 + 8 * u + g;
-#if FFM_SMALL_OWN_EVICT_FIRST
-                x[u] = b < nblk ? ld_stream(base + 32ull * b) : zero_blk();
-#else
-                x[u] = b < nblk ? ld_remote(base + 32ull * b) : zero_blk();
-#endif
-                y[u] = (cmp_on && b < nblk) ? ld_keep(lb + 32ull * b) : zero_blk();
-            }
-#pragma unroll
-            for (int u = 0; u < kSmallU; ++u) {
-                const uint32_t b = b0 + 8 * u + g;
-                if (b < nblk) {
-                    mask_tail(x[u], n, b);
-                    nh_blk(x[u], K, n, b, A, B);
-                    if (cmp_on) {
-                        mask_tail(y[u], n, b);
-                        const int d = blk_diff(x[u], y[u]);
-                        if (d >= 0 && found == ~0ull) found = 2ull * b + d;
-                    }
-                }
-                advance<1>(K);
-            }
-        }
-#pragma unroll
-        for (int o = 4; o; o >>= 1) {
-            A += __shfl_xor_sync(omask, A, o);
-            B += __shfl_xor_sync(omask, B, o);
-            const uint64_t of = __shfl_xor_sync(omask, found, o);
-            found = of < found ? of : found;
-        }
-        if (g == 0) {
-            W.accA[r] = A;
-            W.accB[r] = B;
-            W.digest[r] = finalize_digest(A, B, n);
-            if (found != ~0ull) report_mismatch(W, r, found, res_out, false);
-        }
-    }
-}
-#endif  // FFM_SMALL_ASYNC
 
 // ----------------------------------------------------------------------------
 // H4: re-key residual members.  Round 1 refines by the full, untruncated NH sums;
@@ -1717,7 +1588,6 @@ int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_
     if (L.n == 0 || L.n_small == 0) return 0;
     // (measured: capping its grid so that it co-resides with the persistent large pass
     // slowed that pass more than it hid -- profiles/r01b/README.md)
-#if FFM_SMALL_ASYNC
     if (!smem_configured((const void*)k_fused_small, kSaSmem)) return -1;
     static int occ = 0;   // per process: one device type
     if (occ == 0 && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fused_small, kSaT, kSaSmem) != cudaSuccess ||
@@ -1726,11 +1596,6 @@ int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_
     uint32_t grid = (uint32_t)(occ * P.num_sms);
     uint32_t need = blocks_for((uint64_t)L.n_small * 8, kSaT);
     k_fused_small<<<need < grid ? need : grid, kSaT, kSaSmem, st>>>(L, W, res_out);
-#else
-    uint32_t grid = resident_grid((const void*)k_fused_small, P.num_sms);
-    uint32_t need = blocks_for((uint64_t)L.n_small * 8);
-    k_fused_small<<<need < grid ? need : grid, 256, 0, st>>>(L, W, res_out);
-#endif
     FFM_LAUNCH_CHECK();
     return 1;
 }

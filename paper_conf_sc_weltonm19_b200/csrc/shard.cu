@@ -2,16 +2,18 @@
 //
 // Exact byte equality is transitive, so after H1-H4 on its own records each rank
 // holds exact local classes.  One representative per local class (its min local
-// gid) is exported as a tuple; ranks all-gather the tuples (NCCL over NVLink, done
-// by the caller), then every rank resolves ITS OWN representatives:
+// gid) is exported as a tuple; ranks all-gather the tuples (comm.cu: NCCL over
+// NVLink), then every rank resolves ITS OWN representatives:
 //   global leader G(x) = min gid over representatives with bytes equal to x's.
 // The global group-by gives the min-gid representative with x's key; a remote
 // candidate is confirmed by a byte compare that loads the candidate's bytes straight
 // from the owning GPU's arena (CUDA-IPC-mapped peer memory over NVLink) -- the
 // transfer is fused into the verify kernel, there is no staging copy.  A
 // representative whose candidate is local (same key, different exact local class)
-// or fails the compare takes the slow path: scan same-key representatives in gid
-// order and byte-compare the remote ones until the first equal one.
+// or fails the compare takes the slow path: the tuples of its key are gathered into
+// a segment (only for keys that have such a representative) and scanned; the minimum
+// gid among the remote ones with equal bytes wins.  Every step is stream-ordered and
+// decided on the device (no host round trip when nothing is slow).
 #include <cub/cub.cuh>
 
 #include "digest.cuh"
@@ -45,6 +47,7 @@ __global__ void k_rep_export(DevLog L, Work W, const uint32_t* __restrict__ rep_
     t.gid = L.gid[r];
     t.off = L.off[r];
     t.chan = L.chan[r];
+    t.dig = W.digest[r];
     out[rep_idx[r]] = t;
 }
 
@@ -97,6 +100,7 @@ __global__ void k_merge_classify(const RepTuple* __restrict__ T, uint32_t lo, ui
         S.cand[j] = c;
         uint64_t n = T[t].size;
         cnt = n == 0 ? 1u : (uint32_t)((n + chunk_bytes - 1) / chunk_bytes);
+        if (n) atomicAdd(&S.sctr[2], (unsigned long long)n);   // B_x: bytes read from the peer
     }
     S.state[j] = st;
     S.vcount[j] = cnt;
@@ -142,66 +146,119 @@ __global__ void __launch_bounds__(256) k_merge_verify(const RepTuple* __restrict
     }
 }
 
-__global__ void k_merge_finish(const RepTuple* __restrict__ T, uint32_t nloc, ShardWork S, uint32_t* n_slow) {
+__global__ void k_merge_finish(const RepTuple* __restrict__ T, uint32_t lo, uint32_t nloc,
+                               const uint32_t* __restrict__ tslot, ShardWork S) {
     uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
-    bool slow = false;
     if (j < nloc) {
         uint32_t st = S.state[j];
         if (st == kVerify) S.G[j] = T[S.cand[j]].gid;
-        slow = st == kSlow;
-        if (slow) S.slow_list[atomicAdd(n_slow, 1u)] = j;
+        if (st == kSlow) {
+            S.slow_list[atomicAdd(&S.sctr[0], 1ull)] = j;
+            S.need[tslot[lo + j]] = 1u;   // this key's tuples are gathered into a segment
+        }
     }
 }
 
-// Slow path (digest collisions only): scan all representatives in gid order; the first
-// remote one with the same key and equal bytes is the global leader.  One warp per
-// slow representative; 32 candidates tested per step, lowest gid first.
-__global__ void __launch_bounds__(256) k_merge_slow(const RepTuple* __restrict__ T, uint32_t M, uint32_t lo,
-                                                    const uint32_t* __restrict__ order,
+// Slow path (digest collisions, or a candidate from this rank's own other class):
+// segments of the keys that have a slow representative -- count, allocate, fill.  Each
+// kernel returns at once when no representative is slow (decided on the device).
+__global__ void k_seg_count(uint32_t M, const uint32_t* __restrict__ tslot, ShardWork S) {
+    if (S.sctr[0] == 0) return;
+    for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < M; t += gridDim.x * blockDim.x) {
+        const uint32_t h = tslot[t];
+        if (S.need[h]) atomicAdd(&S.scnt[h], 1u);
+    }
+}
+
+__global__ void k_seg_alloc(uint32_t M, const uint32_t* __restrict__ tslot, const uint32_t* __restrict__ tidx,
+                            ShardWork S) {
+    if (S.sctr[0] == 0) return;
+    for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < M; t += gridDim.x * blockDim.x) {
+        const uint32_t h = tslot[t];
+        if (S.need[h] && tidx[h] == t) {   // one owner per key: its min-gid tuple
+            S.sbase[h] = (uint32_t)atomicAdd(&S.sctr[1], (unsigned long long)S.scnt[h]);
+            S.sfill[h] = 0;
+        }
+    }
+}
+
+__global__ void k_seg_fill(uint32_t M, const uint32_t* __restrict__ tslot, ShardWork S) {
+    if (S.sctr[0] == 0) return;
+    for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < M; t += gridDim.x * blockDim.x) {
+        const uint32_t h = tslot[t];
+        if (S.need[h]) S.seg[S.sbase[h] + atomicAdd(&S.sfill[h], 1u)] = t;
+    }
+}
+
+// One warp per slow representative x: scan its key's segment, 32 tuples per step; a
+// candidate y is an earlier representative (gid below the best so far) on another rank
+// with x's size and channel (and, unless refine_bits weakens it, x's full digest -- a
+// function of the bytes, so a different digest cannot be equal bytes).  Candidates are
+// byte-compared against x (peer bytes over NVLink), stopping at the first differing
+// 1 KiB step; the least gid among equal ones is x's global leader.
+__global__ void __launch_bounds__(256) k_merge_slow(const RepTuple* __restrict__ T, uint32_t lo,
+                                                    const uint32_t* __restrict__ tslot,
                                                     const uint32_t* __restrict__ rank_lo, int world, int rank,
-                                                    const uint8_t* const* __restrict__ bases, uint32_t n_slow,
+                                                    const uint8_t* const* __restrict__ bases, uint64_t refine_mask,
                                                     ShardWork S) {
+    const uint32_t n_slow = (uint32_t)S.sctr[0];
+    if (n_slow == 0) return;
     const int lane = threadIdx.x & 31;
     const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+    unsigned long long bx = 0;
     for (uint32_t q = warp; q < n_slow; q += nwarps) {
         const uint32_t j = S.slow_list[q];
         const uint32_t x = lo + j;
         const RepTuple tx = T[x];
         const uint64_t nblk = (tx.size + 31) >> 5;
         const uint8_t* px = bases[rank] + tx.off;
-        uint64_t G = tx.gid;
-        bool found = false;
-        for (uint32_t s0 = 0; s0 < M && !found; s0 += 32) {
-            uint32_t s = s0 + lane;
-            uint32_t y = s < M ? order[s] : 0;
-            bool earlier = s < M && T[y].gid < tx.gid;
-            bool cand = earlier && T[y].key == tx.key && T[y].size == tx.size && T[y].chan == tx.chan &&
-                        owner_of(y, rank_lo, world) != rank;
-            unsigned any_earlier = __ballot_sync(0xFFFFFFFFu, earlier);
+        const uint32_t h = tslot[x];
+        const uint32_t s0 = S.sbase[h], sn = S.scnt[h];
+        uint64_t best = tx.gid;
+        for (uint32_t i0 = 0; i0 < sn; i0 += 32) {
+            const uint32_t y = i0 + lane < sn ? S.seg[s0 + i0 + lane] : x;
+            const RepTuple ty = T[y];
+            const bool cand = ty.gid < best && ty.key == tx.key && ty.size == tx.size && ty.chan == tx.chan &&
+                              ((ty.dig ^ tx.dig) & refine_mask) == 0 && owner_of(y, rank_lo, world) != rank;
             unsigned cm = __ballot_sync(0xFFFFFFFFu, cand);
             while (cm) {
                 const int src = __ffs(cm) - 1;
                 cm &= cm - 1;
+                const uint64_t gy = __shfl_sync(0xFFFFFFFFu, ty.gid, src);
+                const uint64_t oy = __shfl_sync(0xFFFFFFFFu, ty.off, src);
                 const uint32_t yy = __shfl_sync(0xFFFFFFFFu, y, src);
-                const uint8_t* py = bases[owner_of(yy, rank_lo, world)] + T[yy].off;
+                if (gy >= best) continue;   // an equal earlier one is already known
+                const uint8_t* py = bases[owner_of(yy, rank_lo, world)] + oy;
                 bool diff = false;
-                for (uint64_t b = lane; b < nblk; b += 32) {
-                    Blk a = ld_stream(px + 32 * b);
-                    Blk r = ld_remote(py + 32 * b);
-                    mask_tail(a, tx.size, b);
-                    mask_tail(r, tx.size, b);
-                    diff |= !blk_equal(a, r);
+                for (uint64_t b0 = 0; b0 < nblk && !diff; b0 += 32) {
+                    const uint64_t b = b0 + lane;
+                    bool d = false;
+                    if (b < nblk) {
+                        Blk a = ld_stream(px + 32 * b);
+                        Blk r = ld_remote(py + 32 * b);
+                        mask_tail(a, tx.size, b);
+                        mask_tail(r, tx.size, b);
+                        d = !blk_equal(a, r);
+                        bx += 32;
+                    }
+                    diff = __any_sync(0xFFFFFFFFu, d);
                 }
-                if (!__any_sync(0xFFFFFFFFu, diff)) {
-                    G = T[yy].gid;
-                    found = true;
-                    break;
-                }
+                if (!diff) best = gy;
             }
-            if (any_earlier != 0xFFFFFFFFu) break;    // sorted by gid: nothing earlier beyond here
         }
-        if (lane == 0) S.G[j] = G;
+        if (lane == 0) S.G[j] = best;
+    }
+    if (bx) atomicAdd(&S.sctr[2], bx);
+}
+
+// Segments are cleared where they were used (the arrays stay zero between runs).
+__global__ void k_seg_clear(uint32_t lo, const uint32_t* __restrict__ tslot, ShardWork S) {
+    const uint32_t n_slow = (uint32_t)S.sctr[0];
+    for (uint32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < n_slow; q += gridDim.x * blockDim.x) {
+        const uint32_t h = tslot[lo + S.slow_list[q]];
+        S.need[h] = 0;
+        S.scnt[h] = 0;
     }
 }
 
@@ -273,6 +330,7 @@ int launch_merge(const DevLog& L, Work& W, ShardWork& S, const Params& P, const 
     int k = 0;
     if (cudaMemsetAsync(S.tkey, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
     if (cudaMemsetAsync(S.tgid, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(S.sctr, 0, 4 * sizeof(unsigned long long), st) != cudaSuccess) return -1;
     if (M) {
         k_merge_insert<<<blocks_for(M), 256, 0, st>>>(T, M, cap - 1, S.tkey, S.tgid, S.tslot);
         SHARD_CHECK();
@@ -294,49 +352,25 @@ int launch_merge(const DevLog& L, Work& W, ShardWork& S, const Params& P, const 
         k_merge_verify<<<grid, 256, 0, st>>>(T, lo, S.rank_lo, world, rank, S.bases, P.chunk_bytes, S.vstart + nloc,
                                              S);
         SHARD_CHECK();
-        k += 2;
-    }
-    if (cudaMemsetAsync(S.n_slow, 0, sizeof(uint32_t), st) != cudaSuccess) return -1;
-    if (nloc) {
-        k_merge_finish<<<blocks_for(nloc), 256, 0, st>>>(T, nloc, S, S.n_slow);
+        k_merge_finish<<<blocks_for(nloc), 256, 0, st>>>(T, lo, nloc, S.tslot, S);
         SHARD_CHECK();
-        ++k;
+        k += 3;
+        // slow path, decided on the device (each kernel exits when nothing is slow)
+        const uint32_t gm = std::min<uint32_t>(blocks_for(M), (uint32_t)P.num_sms * 4);
+        k_seg_count<<<gm, 256, 0, st>>>(M, S.tslot, S);
+        SHARD_CHECK();
+        k_seg_alloc<<<gm, 256, 0, st>>>(M, S.tslot, S.tidx, S);
+        SHARD_CHECK();
+        k_seg_fill<<<gm, 256, 0, st>>>(M, S.tslot, S);
+        SHARD_CHECK();
+        k_merge_slow<<<resident_grid((const void*)k_merge_slow, P.num_sms), 256, 0, st>>>(
+            T, lo, S.tslot, S.rank_lo, world, rank, S.bases, P.refine_mask, S);
+        SHARD_CHECK();
+        k_seg_clear<<<std::min<uint32_t>(blocks_for(nloc), (uint32_t)P.num_sms), 256, 0, st>>>(lo, S.tslot, S);
+        SHARD_CHECK();
+        k += 5;
     }
     return k;
-}
-
-int launch_merge_slow(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
-                      uint32_t lo, int world, int rank, uint32_t n_slow, cudaStream_t st) {
-    // order[] = representatives sorted by gid
-    size_t bytes = S.sort_tmp_bytes;
-    if (cub::DeviceRadixSort::SortPairs(S.sort_tmp, bytes, S.sort_keys_in, S.sort_keys_out, S.sort_vals_in,
-                                        S.order, (int)M, 0, 64, st) != cudaSuccess)
-        return -1;
-    uint32_t grid = resident_grid((const void*)k_merge_slow, P.num_sms);
-    k_merge_slow<<<grid, 256, 0, st>>>(T, M, lo, S.order, S.rank_lo, world, rank, S.bases, n_slow, S);
-    SHARD_CHECK();
-    return 2;
-}
-
-__global__ void k_sort_prep(const RepTuple* __restrict__ T, uint32_t M, uint64_t* keys, uint32_t* vals) {
-    uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= M) return;
-    keys[t] = T[t].gid;
-    vals[t] = t;
-}
-
-int launch_sort_prep(ShardWork& S, const RepTuple* T, uint32_t M, cudaStream_t st) {
-    if (!M) return 0;
-    k_sort_prep<<<blocks_for(M), 256, 0, st>>>(T, M, S.sort_keys_in, S.sort_vals_in);
-    SHARD_CHECK();
-    return 1;
-}
-
-size_t sort_tmp_bytes(uint32_t M) {
-    size_t bytes = 0;
-    cub::DeviceRadixSort::SortPairs(nullptr, bytes, (const uint64_t*)nullptr, (uint64_t*)nullptr,
-                                    (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)M, 0, 64);
-    return bytes;
 }
 
 int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
@@ -358,6 +392,26 @@ int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, 
     if (cudaMemsetAsync(W.cnt, 0, (uint64_t)n_sites * 8, st) != cudaSuccess) return -1;
     k_merge_label<<<(uint32_t)P.num_sms * 4, 512, 0, st>>>(L, W.leader, S.rep_idx, S.G, n_sites, dup_out, nullptr,
                                                            nullptr, W.ben, W.cnt);
+    SHARD_CHECK();
+    return 1;
+}
+
+// The per-rank header exchanged after the local pass: representatives exported, residual
+// members (a rank with residuals re-exports after resolving them), arena generation (peers
+// re-map a reallocated arena), record count.
+__global__ void k_shard_header(const uint32_t* __restrict__ rep_count, const uint32_t* __restrict__ counters,
+                               uint64_t gen, uint64_t n, uint64_t* __restrict__ hdr) {
+    if (threadIdx.x == 0) {
+        hdr[0] = *rep_count;
+        hdr[1] = counters[0];
+        hdr[2] = gen;
+        hdr[3] = n;
+    }
+}
+
+int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uint64_t gen, uint64_t n,
+                        uint64_t* hdr, cudaStream_t st) {
+    k_shard_header<<<1, 32, 0, st>>>(rep_count, counters, gen, n, hdr);
     SHARD_CHECK();
     return 1;
 }

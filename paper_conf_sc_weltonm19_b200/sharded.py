@@ -1,94 +1,83 @@
-"""Multi-GPU orchestration of a sharded log (include/ffm.h "Sharded logs").
+"""Bootstrap of a sharded log (include/ffm.h "Sharded logs").
 
-Plumbing only: torch.distributed moves the representative tuples and the benefit
-partials (NCCL over NVLink / NVSwitch on GPUs; gloo with host staging when NCCL is
-unavailable, e.g. several ranks sharing one GPU in tests).  Every step of the hot
-path -- H1..H4, the global group-by, the peer-memory byte verify and the labels --
-runs in libffm's kernels.
+Plumbing only.  The library runs the whole sharded step inside the collective
+``ffm_dedup_run`` -- H1..H4 per rank, the all-gather of class representatives, the
+peer-memory byte verify over NVLink, the labels and the all-reduce of the per-site
+sums -- on the log's stream, over its own NCCL communicator.  This module only hands
+it the world: rank 0's ``ncclUniqueId`` broadcast through a torch.distributed group,
+or, where NCCL cannot connect the ranks (several ranks sharing one GPU in tests), a
+host transport built from that group's gloo collectives (``HostComm``).
 """
 from __future__ import annotations
+
+import ctypes
 
 import numpy as np
 import torch
 import torch.distributed as dist
 
-from . import (REP_WORDS, ffm_log_count, ffm_shard_ipc_handle, ffm_shard_local, ffm_shard_merge,
-               ffm_shard_open_peer, ffm_site_duplicate_counts)
+from . import ALLGATHER_FN, ALLREDUCE_FN, FfmCommOps, FfmLog, ffm_nccl_unique_id
 
 
-def _on_nccl(group=None) -> bool:
-    return dist.get_backend(group) == "nccl"
+class HostComm:
+    """ffm_comm_ops over a torch.distributed group (host buffers; gloo).  Collective
+    callbacks the library invokes from inside ffm_log_create / ffm_dedup_run."""
+
+    def __init__(self, group=None):
+        self.group = group
+        self.world = dist.get_world_size(group)
+        self.error = None
+        self._ag = ALLGATHER_FN(self._allgather)
+        self._ar = ALLREDUCE_FN(self._allreduce)
+        self.ops = FfmCommOps(None, self._ag, self._ar)
+
+    def allgather(self, send: np.ndarray) -> np.ndarray:
+        """recv[world * bytes] = every rank's send (uint8), rank-major."""
+        t = torch.from_numpy(np.ascontiguousarray(send, np.uint8))
+        parts = [torch.empty_like(t) for _ in range(self.world)]
+        dist.all_gather(parts, t, group=self.group)
+        return torch.cat(parts).numpy()
+
+    def allreduce_u64(self, buf: np.ndarray) -> np.ndarray:
+        """Elementwise sum mod 2^64 (int64 two's complement sums wrap identically)."""
+        t = torch.from_numpy(np.ascontiguousarray(buf, np.uint64).view(np.int64).copy())
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=self.group)
+        return t.numpy().view(np.uint64)
+
+    def _allgather(self, ctx, send, recv, nbytes):
+        try:
+            src = np.ctypeslib.as_array((ctypes.c_uint8 * max(nbytes, 1)).from_address(send))[:nbytes] \
+                if nbytes else np.empty(0, np.uint8)
+            out = self.allgather(src)
+            if out.size:
+                ctypes.memmove(recv, out.ctypes.data, out.size)
+            return 0
+        except Exception as e:          # never raise through the C ABI
+            self.error = e
+            return -1
+
+    def _allreduce(self, ctx, buf, n):
+        try:
+            a = np.ctypeslib.as_array((ctypes.c_uint64 * n).from_address(buf))
+            a[:] = self.allreduce_u64(a)
+            return 0
+        except Exception as e:
+            self.error = e
+            return -1
 
 
-def exchange_handles(log, group=None):
-    """Map every peer's HBM arena (CUDA IPC).  Call after the last append."""
-    world = dist.get_world_size(group)
-    mine = ffm_shard_ipc_handle(log.h)
-    allh = [None] * world
-    dist.all_gather_object(allh, mine, group=group)
-    for r, hb in enumerate(allh):
-        ffm_shard_open_peer(log.h, r, hb)
-
-
-def allgather_reps(local: torch.Tensor, group=None):
-    """local: int64 [n, REP_WORDS] (any device).  Returns (all reps rank-major on
-    local.device, counts list)."""
-    world = dist.get_world_size(group)
-    comm_dev = local.device if _on_nccl(group) else torch.device("cpu")
-    n = torch.tensor([local.shape[0]], dtype=torch.int64, device=comm_dev)
-    counts_t = [torch.zeros_like(n) for _ in range(world)]
-    dist.all_gather(counts_t, n, group=group)
-    counts = [int(c.item()) for c in counts_t]
-    mx = max(counts) if counts else 0
-    if mx == 0:
-        return local.new_empty((0, REP_WORDS)), counts
-    pad = torch.zeros((mx, REP_WORDS), dtype=torch.int64, device=comm_dev)
-    pad[: local.shape[0]] = local.to(comm_dev)
-    out = torch.empty((world * mx, REP_WORDS), dtype=torch.int64, device=comm_dev)
-    dist.all_gather_into_tensor(out, pad, group=group)
-    parts = [out[r * mx: r * mx + counts[r]] for r in range(world)]
-    return torch.cat(parts).to(local.device).contiguous(), counts
-
-
-def allreduce_benefit(ben: torch.Tensor, group=None) -> torch.Tensor:
-    """Sum int64 (two's complement == uint64 mod 2^64) partial benefits over ranks."""
-    if _on_nccl(group) or ben.device.type == "cpu":
-        dist.all_reduce(ben, op=dist.ReduceOp.SUM, group=group)
-        return ben
-    h = ben.cpu()
-    dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
-    ben.copy_(h)
-    return ben
-
-
-def site_counts_sharded(log, device, group=None) -> torch.Tensor:
-    """All-reduced duplicates per call site of the last sharded run (int64 [n_sites])."""
-    c = torch.empty(log.n_sites, dtype=torch.int64, device=device)
-    ffm_site_duplicate_counts(log.h, log.n_sites, c)
-    return allreduce_benefit(c, group)
-
-
-def dedup_sharded(log, device, group=None, duplicate_of=None, benefit=None, reps_buf=None):
-    """One sharded run.  Returns (duplicate_of for this rank's records [global gids],
-    global benefit_ns as int64 [n_sites]); both on `device` unless given."""
-    n = ffm_log_count(log.h)
-    if reps_buf is None or reps_buf.shape[0] < max(n, 1):
-        reps_buf = torch.empty((max(n, 1), REP_WORDS), dtype=torch.int64, device=device)
-    n_reps = ffm_shard_local(log.h, reps_buf, reps_buf.shape[0])
-    # the exchange's device work (NCCL, padding, concatenation) is ordered on the
-    # library's stream, which the merge kernels then read from
-    dev = torch.device(device)
-    if dev.type == "cuda" and log.stream:
-        with torch.cuda.stream(torch.cuda.ExternalStream(log.stream, device=dev)):
-            all_reps, counts = allgather_reps(reps_buf[:n_reps], group)
-    else:
-        all_reps, counts = allgather_reps(reps_buf[:n_reps], group)
-    if duplicate_of is None:
-        duplicate_of = torch.empty(max(n, 1), dtype=torch.int64, device=device)
-    if benefit is None:
-        benefit = torch.empty(log.n_sites, dtype=torch.int64, device=device)
-    if all_reps.shape[0] == 0:
-        all_reps = torch.empty((1, REP_WORDS), dtype=torch.int64, device=device)
-    ffm_shard_merge(log.h, all_reps, np.asarray(counts, np.uint64), duplicate_of, benefit)
-    allreduce_benefit(benefit, group)
-    return duplicate_of[:n], benefit
+def create_sharded_log(n_sites: int, device: int, *, group=None, transport: str = "nccl", **kw) -> FfmLog:
+    """A log for this rank of a sharded world (collective over `group`).
+    transport "nccl": the library's own NCCL communicator (one GPU per rank);
+    "host": HostComm over the group (gloo; ranks may share a GPU)."""
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    if transport == "nccl":
+        uid = [ffm_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=dist.get_global_rank(group, 0) if group else 0, group=group)
+        return FfmLog(n_sites, device, rank=rank, world=world, nccl_id=uid[0], **kw)
+    if transport == "host":
+        hc = HostComm(group)
+        log = FfmLog(n_sites, device, rank=rank, world=world, comm=hc.ops, **kw)
+        log.host_comm = hc
+        return log
+    raise ValueError(f"transport {transport!r}: 'nccl' or 'host'")

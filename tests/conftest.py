@@ -11,3 +11,15 @@ if ROOT not in sys.path:
 def pytest_configure(config):
     config.addinivalue_line("markers", "gpu: needs a CUDA device (B200); runs the CUDA path")
     config.addinivalue_line("markers", "slow: long-running (full-size configs)")
+
+
+def pytest_addoption(parser):
+    parser.addoption("--ffm-lib", default=None,
+                     help="run the tests against another build of libffm.so (tools/build_variants.sh)")
+
+
+def pytest_sessionstart(session):
+    path = session.config.getoption("--ffm-lib")
+    if path:
+        import paper_conf_sc_weltonm19_b200 as ffm
+        ffm.set_library_path(path)

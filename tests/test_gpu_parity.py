@@ -484,34 +484,68 @@ def test_benefit_linear_in_durations(ffm):
     np.testing.assert_array_equal(b7, b1 * np.uint64(7))
 
 
-def test_sharded_api_errors(ffm):
-    """Call-order and consistency errors of the sharded / online API (one process)."""
-    import torch
+class _LonelyWorld:
+    """An ffm_comm_ops transport for a world of 2 in which rank 1 never has records: the
+    collective run can be driven from one process (peer blocks are zeros)."""
+
+    def __init__(self, ffm, fail=False):
+        self.fail, self.calls = fail, 0
+        self._ag = ffm.ALLGATHER_FN(self._allgather)
+        self._ar = ffm.ALLREDUCE_FN(lambda ctx, buf, n: 0)      # sum with an all-zero peer
+        self.ops = ffm.FfmCommOps(None, self._ag, self._ar)
+
+    def _allgather(self, ctx, send, recv, nbytes):
+        import ctypes
+        self.calls += 1
+        if self.fail:
+            return -1
+        if nbytes:
+            ctypes.memmove(recv, send, nbytes)
+            ctypes.memset(recv + nbytes, 0, nbytes)
+        return 0
+
+
+def test_sharded_api_errors_and_lonely_world(ffm):
+    """Sharded-log rules (include/ffm.h): gids are required and < 2^63; online mode is
+    single-log; a failing exchange poisons the handle; a world whose other rank is empty
+    gives the single-log result through the whole collective path (header, export,
+    all-gather, merge, all-reduce)."""
     x = np.frombuffer(b"abcdefgh" * 8, np.uint8).copy()
-    with ffm.FfmLog(2, rank=0, world=2) as log:
-        log.append_batch([0, 1], [64, 64], [x.ctypes.data] * 2, [1, 2], gids=[0, 3])
+    w = _LonelyWorld(ffm)
+    with ffm.FfmLog(2, rank=0, world=2, comm=w.ops) as log:
         with pytest.raises(ffm.FfmError) as e:
-            log.run()                                   # a sharded log has no single-log run
-        assert e.value.code == ffm.FFM_E_STATE
+            log.append_batch([0, 1], [64, 64], [x.ctypes.data] * 2, [1, 2])      # no gids
+        assert e.value.code == ffm.FFM_E_INVAL
+        with pytest.raises(ffm.FfmError) as e:
+            log.append_batch([0], [64], [x.ctypes.data], [1], gids=[1 << 63])
+        assert e.value.code == ffm.FFM_E_RANGE
+        log.append_batch([0, 1], [64, 64], [x.ctypes.data] * 2, [1, 2], gids=[0, 3])
         with pytest.raises(ffm.FfmError) as e:
             log.online_step()
         assert e.value.code == ffm.FFM_E_STATE
-        reps = torch.empty((4, ffm.REP_WORDS), dtype=torch.int64, device="cuda")
-        dup = torch.empty(2, dtype=torch.int64, device="cuda")
-        ben = torch.empty(2, dtype=torch.int64, device="cuda")
-        with pytest.raises(ffm.FfmError) as e:          # merge before local
-            ffm.ffm_shard_merge(log.h, reps, [1, 0], dup, ben)
-        assert e.value.code == ffm.FFM_E_STATE
-        n = ffm.ffm_shard_local(log.h, reps, 4)
-        assert n == 1                                   # two equal payloads: one class
-        with pytest.raises(ffm.FfmError) as e:          # counts disagree with this rank
-            ffm.ffm_shard_merge(log.h, reps, [2, 0], dup, ben)
+        for _ in range(2):
+            dup, ben = log.run()
+            assert dup.tolist() == [-1, 0] and ben.tolist() == [0, 2]
+        assert log.site_counts().tolist() == [0, 1]
+        st = log.stats()
+        assert st["n_reps_local"] == 1 and st["n_reps_global"] == 1 and st["host_syncs"] == 2
+    lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 32)
+    want = oracle.dedup(lg)
+    w = _LonelyWorld(ffm)
+    with ffm.FfmLog(lg.n_sites, rank=0, world=2, comm=w.ops, chunk_bytes=4096) as log:
+        log.append_log(lg, gids=np.arange(lg.n) * 3 + 5)
+        dup, ben = log.run()
+        np.testing.assert_array_equal(np.where(want[0] >= 0, want[0] * 3 + 5, -1), dup)
+        np.testing.assert_array_equal(ben, want[1])
+    bad = _LonelyWorld(ffm, fail=True)
+    with ffm.FfmLog(2, rank=0, world=2, comm=bad.ops) as log:
+        log.append_batch([0, 1], [64, 64], [x.ctypes.data] * 2, [1, 2], gids=[0, 3])
+        with pytest.raises(ffm.FfmError) as e:
+            log.run()
         assert e.value.code == ffm.FFM_E_COMM
-        with pytest.raises(ffm.FfmError) as e:          # a peer with reps but no mapping
-            ffm.ffm_shard_merge(log.h, reps, [1, 1], dup, ben)
-        assert e.value.code == ffm.FFM_E_STATE
-        ffm.ffm_shard_merge(log.h, reps, [1, 0], dup, ben)   # alone: duplicates stay local
-        assert dup.cpu().tolist() == [-1, 0] and ben.cpu().tolist() == [0, 2]
+        with pytest.raises(ffm.FfmError) as e:
+            log.run()
+        assert e.value.code == ffm.FFM_E_STATE                 # poisoned
 
 
 def test_graph_replay_matches_direct_launches(ffm):

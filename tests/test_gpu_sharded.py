@@ -1,8 +1,9 @@
-"""Sharded (multi-rank) parity on the GPU: P processes share cuda:0 (NCCL refuses two
-ranks on one device, so the tuple exchange uses gloo with host staging; peer arenas
-are CUDA-IPC mapped exactly as across NVLink).  Every rank's duplicate_of (global
-gids) and the all-reduced benefit must equal the single-log oracle bit-exactly, for
-both shard planners and with forced digest collisions (slow merge path)."""
+"""Sharded (multi-rank) parity on the GPU through the collective ffm_dedup_run: P
+processes share cuda:0 (NCCL refuses two ranks on one device, so the library's exchange
+runs over the host transport -- sharded.HostComm on gloo; peer arenas are CUDA-IPC
+mapped exactly as across NVLink).  Every rank's duplicate_of (global gids), the global
+benefit and the duplicate counts must equal the single-log oracle bit-exactly, for both
+shard planners, P in {2, 3, 4, 8} and with forced digest collisions (slow segments)."""
 import os
 import socket
 
@@ -39,7 +40,7 @@ def _make(case):
     return lg
 
 
-def _worker(rank, world, port, out_dir, case, policy, digest_bits, device_payloads):
+def _worker(rank, world, port, out_dir, case, policy, digest_bits, device_payloads, refine_bits=64):
     import torch
     import torch.distributed as dist
     import paper_conf_sc_weltonm19_b200 as ffm
@@ -52,33 +53,32 @@ def _worker(rank, world, port, out_dir, case, policy, digest_bits, device_payloa
         lg = _make(case)
         ranks = ffm.ffm_shard_plan(lg.site, lg.size, lg.n_sites, world, policy)
         idx = np.nonzero(ranks == rank)[0]
-        log = ffm.FfmLog(lg.n_sites, device=0, rank=rank, world=world, digest_bits=digest_bits,
-                         chunk_bytes=4096, timing=True)
+        log = sharded.create_sharded_log(lg.n_sites, 0, transport="host", digest_bits=digest_bits,
+                                         refine_bits=refine_bits, chunk_bytes=4096, timing=True)
         if device_payloads:
             buf = torch.from_numpy(lg.materialize()).cuda()
             ptrs = (lg.c_off[lg.content] + np.uint64(buf.data_ptr())).astype(np.uint64)
             log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE, gids=idx, idx=idx)
         else:
             log.append_log(lg, gids=idx, idx=idx)
-        sharded.exchange_handles(log)
         outs = []
         for _ in range(2):                                   # re-runnable
-            dup, ben = sharded.dedup_sharded(log, torch.device("cuda", 0))
-            outs.append((dup.cpu().numpy().copy(), ben.cpu().numpy().view(np.uint64).copy()))
-        cnt = sharded.site_counts_sharded(log, torch.device("cuda", 0)).cpu().numpy()
-        dist.barrier()            # peers must not unmap while others still read their arenas
+            dup, ben = log.run()
+            outs.append((dup.copy(), ben.copy()))
+        st = log.stats()
+        cnt = log.site_counts()
         np.savez(os.path.join(out_dir, f"r{rank}.npz"), idx=idx, dup=outs[0][0], ben=outs[0][1],
-                 dup2=outs[1][0], ben2=outs[1][1], cnt=cnt)
-        dist.barrier()
+                 dup2=outs[1][0], ben2=outs[1][1], cnt=cnt, n_slow=st["n_slow"], syncs=st["host_syncs"],
+                 bx=st["remote_verify_bytes"], reps=st["n_reps_global"])
         log.close()
     finally:
         dist.destroy_process_group()
 
 
-def _run(tmp_path, world, case, policy, digest_bits=64, device_payloads=False):
+def _run(tmp_path, world, case, policy, digest_bits=64, device_payloads=False, refine_bits=64):
     import torch.multiprocessing as mp
-    mp.spawn(_worker, args=(world, _free_port(), str(tmp_path), case, policy, digest_bits, device_payloads),
-             nprocs=world, join=True)
+    mp.spawn(_worker, args=(world, _free_port(), str(tmp_path), case, policy, digest_bits, device_payloads,
+                            refine_bits), nprocs=world, join=True)
     lg = _make(case)
     want_dup, want_ben = oracle.dedup(lg)
     got = np.full(lg.n, -7, np.int64)
@@ -122,3 +122,28 @@ def test_four_ranks_device_payloads(tmp_path):
 @pytest.mark.parametrize("digest_bits", [64, 0])
 def test_sharded_with_channels(tmp_path, digest_bits):
     _run(tmp_path, 3, "c5+ch", 1, digest_bits=digest_bits)
+
+
+@pytest.mark.parametrize("case,policy", [("c5", 0), ("c5", 1), ("c4", 1)])
+def test_eight_ranks(tmp_path, case, policy):
+    """P = 8 through the collective run."""
+    lg, got = _run(tmp_path, 8, case, policy)
+    assert (got >= 0).any()
+    z = [np.load(tmp_path / f"r{r}.npz") for r in range(8)]
+    assert len({int(x["reps"]) for x in z}) == 1                 # one global table on every rank
+
+
+def test_eight_ranks_forced_collisions(tmp_path):
+    """Every representative of a size in one key (digest_bits 0) and no digest pruning
+    (refine_bits 0): the same-key segment scan resolves every cross-rank class."""
+    _run(tmp_path, 8, "c3", 1, digest_bits=0, refine_bits=0)
+    assert sum(int(np.load(tmp_path / f"r{r}.npz")["n_slow"]) for r in range(8)) > 0
+
+
+def test_two_host_syncs_without_collisions(tmp_path):
+    """The collective run synchronises the host twice when no rank has digest collisions
+    (the host transport's own staging copies aside, which NCCL does not need)."""
+    lg, got = _run(tmp_path, 2, "c5", 0)
+    for r in range(2):
+        z = np.load(tmp_path / f"r{r}.npz")
+        assert int(z["syncs"]) == 2, int(z["syncs"])

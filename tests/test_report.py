@@ -2,6 +2,7 @@
 import json
 
 import numpy as np
+import pytest
 
 from paper_conf_sc_weltonm19_b200 import report
 
@@ -29,7 +30,15 @@ def test_ranked_report_orders_and_totals():
     ben = np.array([5, 0, 30, 10], np.uint64)
     cnt = np.array([1, 0, 3, 2], np.uint64)
     names = ["als.cpp:738", "als.cpp:739", "als.cpp:760", "x.cu:1"]
-    rep = report.ranked_report(ben, names, cnt, ["f<int>()", "g()", "f<long>()", "h()"], exec_time_ns=100)
+    funcs = ["f<int>()", "g()", "f<long>()", "h()"]
+    with pytest.raises(ValueError):          # the group sums are the device's (ffm_fold_sites)
+        report.ranked_report(ben, names, cnt, funcs)
+
+    def fold(v, g, n):                       # stands in for FfmLog.fold on a CPU-only box
+        out = np.zeros(n, np.uint64)
+        np.add.at(out, np.asarray(g, np.int64), np.asarray(v, np.uint64))
+        return out
+    rep = report.ranked_report(ben, names, cnt, funcs, fold=fold, exec_time_ns=100)
     assert [r["name"] for r in rep["single_point"]] == ["als.cpp:760", "x.cu:1", "als.cpp:738"]
     assert rep["total"] == {"benefit_ns": 45, "benefit_s": 45e-9, "transfer_issues": 3, "pct_exec": 45.0,
                             "duplicates": 6}

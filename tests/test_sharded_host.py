@@ -1,5 +1,5 @@
-"""Host-side logic of the multi-GPU path, on CPU: the shard planner (C ABI, host only)
-and the torch.distributed exchange steps at world_size 2 over gloo."""
+"""Host-side logic of the multi-GPU path, on CPU: the shard planner (C ABI, host only),
+the host exchange transport of a sharded log at world_size 2 / 3 over gloo, config checks."""
 import os
 import socket
 
@@ -52,31 +52,43 @@ def _free_port():
 
 
 def _worker(rank, world, port, out_dir):
+    import ctypes
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        # ragged counts, one rank empty when world > 2
-        n = [3, 0, 5][rank] if world == 3 else [3, 5][rank]
-        local = torch.arange(n * ffm.REP_WORDS, dtype=torch.int64).reshape(n, ffm.REP_WORDS) + 1000 * rank
-        allr, counts = sharded.allgather_reps(local)
-        ben = torch.tensor([rank + 1, -1, (1 << 62)], dtype=torch.int64)   # -1 == 2^64-1 as u64
-        sharded.allreduce_benefit(ben)
-        torch.save({"all": allr, "counts": counts, "ben": ben}, os.path.join(out_dir, f"r{rank}.pt"))
+        hc = sharded.HostComm()
+        # the library's calls, through the same C function pointers it receives
+        send = (np.arange(40, dtype=np.uint8) + 50 * rank).astype(np.uint8)
+        recv = np.zeros(40 * world, np.uint8)
+        rc1 = hc.ops.allgather(None, send.ctypes.data, recv.ctypes.data, 40)
+        rc0 = hc.ops.allgather(None, None, None, 0)                  # an empty block
+        ben = np.array([rank + 1, 2**64 - 1, 1 << 62], np.uint64)    # wraps mod 2^64
+        rc2 = hc.ops.allreduce_u64(None, ben.ctypes.data, 3)
+        np.savez(os.path.join(out_dir, f"r{rank}.npz"), recv=recv, ben=ben, rc=[rc0, rc1, rc2])
+        del ctypes
     finally:
         dist.destroy_process_group()
 
 
 @pytest.mark.parametrize("world", [2, 3])
-def test_exchange_steps_gloo(tmp_path, world):
+def test_host_transport_gloo(tmp_path, world):
+    """The ffm_comm_ops transport of a sharded log (sharded.HostComm) over gloo, world 2/3."""
     mp.spawn(_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
-    res = [torch.load(tmp_path / f"r{r}.pt") for r in range(world)]
-    ns = [3, 0, 5] if world == 3 else [3, 5]
-    want = torch.cat([torch.arange(n * ffm.REP_WORDS, dtype=torch.int64).reshape(n, ffm.REP_WORDS) + 1000 * r
-                      for r, n in enumerate(ns)])
-    for r in res:
-        assert r["counts"] == ns
-        assert torch.equal(r["all"], want)                 # rank-major, padding stripped
-        u = r["ben"].numpy().view(np.uint64)
-        assert u[0] == sum(range(1, world + 1))
-        assert u[1] == (world * ((1 << 64) - 1)) % (1 << 64)   # wraps mod 2^64 like the u64 sums
-        assert u[2] == (world * (1 << 62)) % (1 << 64)
+    want = np.concatenate([(np.arange(40, dtype=np.uint8) + 50 * r).astype(np.uint8) for r in range(world)])
+    for r in range(world):
+        z = np.load(tmp_path / f"r{r}.npz")
+        assert z["rc"].tolist() == [0, 0, 0]
+        np.testing.assert_array_equal(z["recv"], want)               # rank-major blocks
+        u = z["ben"]
+        assert int(u[0]) == sum(range(1, world + 1))
+        assert int(u[1]) == (world * (2**64 - 1)) % 2**64
+        assert int(u[2]) == (world * (1 << 62)) % 2**64
+
+
+def test_sharded_config_validation():
+    """world > 1 needs exactly one exchange transport (checked before any device work)."""
+    c = ffm.ffm_config_init()
+    c.world, c.rank, c.n_sites = 2, 0, 4
+    with pytest.raises(ffm.FfmError) as e:
+        ffm.ffm_log_create(c)
+    assert e.value.code == ffm.FFM_E_INVAL

@@ -5,12 +5,13 @@ set -u
 T=$1; CFGS=$2; KX=$3; shift 3
 mkdir -p gpurun_out
 for v in "$@"; do
-  if [ "$v" = default ]; then e=(); else e=(FFM_LIB=build/variants/$v/libffm.so); fi
-  env "${e[@]}" timeout 600 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "$KX" > gpurun_out/${T}_${v}_parity.log 2>&1
+  if [ "$v" = default ]; then e=(); else e=(--ffm-lib build/variants/$v/libffm.so); fi
+  timeout 600 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "$KX" "${e[@]}" > gpurun_out/${T}_${v}_parity.log 2>&1
   echo "$v parity rc=$? $(tail -1 gpurun_out/${T}_${v}_parity.log)"
   for k in $CFGS; do
     out=gpurun_out/${T}_c${k}_${v}.json
-    env "${e[@]}" timeout 600 python bench.py --workload $k --steps 10 --e2e-steps 0 --cpu-seconds 0 > $out 2> ${out%.json}.err
+    if [ "$v" = default ]; then b=(); else b=(--lib build/variants/$v/libffm.so); fi
+    timeout 600 python bench.py "${b[@]}" --workload $k --steps 10 --e2e-steps 0 --cpu-seconds 0 > $out 2> ${out%.json}.err
     python - "$out" "$k" "$v" <<'PY'
 import json, sys
 out, k, v = sys.argv[1:]

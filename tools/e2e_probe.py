@@ -32,5 +32,5 @@ for it in range(3):
     log.close()
     t4 = time.perf_counter()
     print(f"it{it}: create {t1-t0:.3f}s append {t2-t1:.3f}s ({lg.total_bytes/(t2-t1)/1e9:.1f} GB/s) "
-          f"run {t3-t2:.3f}s destroy {t4-t3:.3f}s total {t4-t0:.3f}s  gather_max={os.environ.get('FFM_GATHER_MAX')}",
+          f"run {t3-t2:.3f}s destroy {t4-t3:.3f}s total {t4-t0:.3f}s",
           flush=True)
