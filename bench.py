@@ -405,6 +405,85 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
+def run_online(args):
+    """S8(f) #2 measurement: the log streamed through ffm_online_step in fixed windows
+    (FFM_FLAG_ONLINE: each append hashes its records on the hashing stream), against the
+    batch run of the same log.  Per window size: median step latency (host wall clock of
+    the synchronous ffm_online_step) and streamed throughput = payload / (sum of append +
+    step times); appends snapshot device-resident payloads (D2D)."""
+    import torch
+    import paper_conf_sc_weltonm19_b200 as ffm
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    lg = make_log(args.workload, args.n_scale, args.size_scale)
+    content = torch.from_numpy(lg.buf).to(dev)
+    ptrs = (lg.c_off[lg.content] + np.uint64(content.data_ptr())).astype(np.uint64)
+    want = None
+    if args.check:
+        import oracle
+        want = oracle.dedup(lg)
+    opts = dict(arena_bytes=lg.total_bytes + 128 * lg.n + (1 << 20), max_records=lg.n)
+    # batch reference: the same log in one ffm_dedup_run (device outputs)
+    with ffm.FfmLog(lg.n_sites, **opts) as log:
+        log.append_log(lg, ptrs=ptrs, payload_kind=ffm.FFM_PAYLOAD_DEVICE)
+        d = torch.empty(lg.n, dtype=torch.int64, device=dev)
+        b = torch.empty(lg.n_sites, dtype=torch.int64, device=dev)
+        for _ in range(args.warmup):
+            log.run(d, b)
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        for _ in range(args.steps):
+            log.run(d, b)
+        torch.cuda.synchronize()
+        batch_s = (time.perf_counter() - t) / args.steps
+    rows = []
+    for w in [int(x) for x in args.online.split(",")]:
+        n_win = (lg.n + w - 1) // w
+        if n_win > args.online_max_windows:          # latency only, over a bounded prefix
+            n_win = args.online_max_windows
+        end = min(lg.n, n_win * w)
+        dup = torch.empty(max(w, 1), dtype=torch.int64, device=dev)
+        ben = torch.empty(lg.n_sites, dtype=torch.int64, device=dev)
+        got = np.empty(end, np.int64) if want is not None else None
+        t_app, t_step = [], []
+        with ffm.FfmLog(lg.n_sites, online=True, **opts) as log:
+            for rep in range(2):                     # rep 0 warms up (allocations), rep 1 is measured
+                log.reset()
+                t_app.clear()
+                t_step.clear()
+                torch.cuda.synchronize()
+                for a in range(0, end, w):
+                    e = min(end, a + w)
+                    t0 = time.perf_counter()
+                    log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e],
+                                     payload_kind=ffm.FFM_PAYLOAD_DEVICE)
+                    t1 = time.perf_counter()
+                    log.online_step(dup, ben)
+                    t2 = time.perf_counter()
+                    t_app.append(t1 - t0)
+                    t_step.append(t2 - t1)
+                    if got is not None and rep == 1:
+                        got[a:e] = dup[:e - a].cpu().numpy()
+        byts = int(lg.size[:end].sum())
+        row = {"window": w, "windows": len(t_step), "records": end, "payload_bytes": byts,
+               "step_ms_median": round(statistics.median(t_step) * 1e3, 4),
+               "step_ms_p90": round(float(np.percentile(t_step, 90)) * 1e3, 4),
+               "append_ms_median": round(statistics.median(t_app) * 1e3, 4),
+               "streamed_gbs": round(byts / (sum(t_app) + sum(t_step)) / 1e9, 2),
+               "steps_only_gbs": round(byts / sum(t_step) / 1e9, 2)}
+        if got is not None:
+            row["parity"] = "ok" if np.array_equal(got, want[0][:end]) else "MISMATCH"
+        rows.append(row)
+        log_msg(f"[bench] online window {w}: {row}")
+    out = {"metric": METRIC, "mode": "online (S8(f) #2)", "workload": WORKLOADS[args.workload],
+           "records": lg.n, "payload_bytes": lg.total_bytes, "n_scale": args.n_scale,
+           "batch_ms": round(batch_s * 1e3, 4), "batch_gbs": round(lg.total_bytes / batch_s / 1e9, 2),
+           "windows": rows,
+           "note": "host wall clock; appends snapshot device-resident payloads and queue their hashing "
+                   "(FFM_FLAG_ONLINE); each step is synchronous (labels in device memory)"}
+    print(json.dumps(out), flush=True)
+
+
 def check_parity(lg, args, idx, dup, ben, rank, world):
     """Every rank's duplicate_of (global gids) and the global benefit against the CPU
     oracle on the whole log (rank 0; small logs)."""
@@ -623,6 +702,10 @@ def main():
                     help="test hook: run the N ranks on one GPU (host exchange transport instead of NCCL)")
     ap.add_argument("--check", action="store_true", help="check the result against the CPU oracle (small logs)")
     ap.add_argument("--lib", default=None, help="load another build of libffm.so (tools/build_variants.sh)")
+    ap.add_argument("--online", default=None,
+                    help="comma-separated window sizes: measure online mode (ffm_online_step) instead")
+    ap.add_argument("--online-max-windows", type=int, default=3000,
+                    help="online: at most this many windows per size (small windows: latency over a prefix)")
     ap.add_argument("--digest-bits", type=int, default=64,
                     help="< 64 truncates the group-by digest (forced collisions, verify stress; config 3)")
     ap.add_argument("--two-pass", action="store_true",
@@ -638,6 +721,8 @@ def main():
         ffm.set_library_path(args.lib)
     if args.impl == "reference":
         run_reference(args)
+    elif args.online:
+        run_online(args)
     elif args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         sys.exit(spawn_ranks(args))
     else:

@@ -27,6 +27,7 @@ struct LocalRun {
     uint64_t n_reread;   // residual members whose bytes were compared again (not settled by difference lists)
     uint64_t n_overflow; // round-0 residuals whose difference list against their head overflowed
     bool two_pass;
+    bool spec_stale;     // the speculative host labels need the final copy (residuals)
 };
 
 struct CudaFail {
@@ -153,6 +154,15 @@ int pointer_kind(const void* p, int* dev) {
     return FFM_PAYLOAD_HOST;
 }
 
+bool is_pinned_host(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeHost;
+}
+
 bool is_device_ptr(const void* p) {
     cudaPointerAttributes a;
     if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
@@ -202,7 +212,9 @@ void upload_order(ffm_log* L, const std::vector<uint32_t>& order, uint32_t*& dpt
     }
 }
 
-void upload_meta(ffm_log* L) {
+// H0 tail: the metadata SoA of records appended since the last upload (incremental;
+// pageable-source copies are staged before the call returns, no sync needed).
+void upload_meta_arrays(ffm_log* L) {
     uint64_t n = L->h_size.size();
     if (L->d_meta_n == n) return;
     uint64_t c0 = L->d_meta_cap, keep = L->d_meta_n;
@@ -227,16 +239,21 @@ void upload_meta(ffm_log* L) {
     ck(cudaMemcpyAsync(L->d_dur + a, L->h_dur.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
     ck(cudaMemcpyAsync(L->d_gid + a, L->h_gid.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
     ck(cudaMemcpyAsync(L->d_chan + a, L->h_chan.data() + a, k * 8, cudaMemcpyHostToDevice, s), "meta H2D");
-    // small records ordered by block count, largest first (counting sort): the four
-    // 8-lane groups of a warp then get payloads of near-equal length (no idle lanes)
-    {
-        std::vector<uint32_t> order;
-        L->n_small = build_small_order(L, 0, n, order);
-        L->n_large_rec = order.size() - L->n_small;
-        upload_order(L, order, L->d_small_order, L->d_small_cap, s);
-    }
-    ck(cudaStreamSynchronize(s), "meta sync");
     L->d_meta_n = n;
+}
+
+// The whole log's record order of the batch passes: small records by size class
+// (largest first: the four 8-lane groups of a warp then get payloads of near-equal
+// length), then the large ones.  Rebuilt only when records were appended since.
+void upload_meta(ffm_log* L) {
+    upload_meta_arrays(L);
+    const uint64_t n = L->h_size.size();
+    if (L->d_order_n == n && L->d_small_order) return;
+    std::vector<uint32_t> order;
+    L->n_small = build_small_order(L, 0, n, order);
+    L->n_large_rec = order.size() - L->n_small;
+    upload_order(L, order, L->d_small_order, L->d_small_cap, L->stage_stream);
+    L->d_order_n = n;
 }
 
 uint64_t large_chunks(const ffm_log* L, uint64_t size) {
@@ -311,6 +328,14 @@ void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* si
 void ensure_work(ffm_log* L, uint64_t n) {
     Work& W = L->work;
     uint64_t tcap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
+    const uint64_t fcap0 = fx_entry_cap(L->n_large_chunks, L->params.chunk_bytes);
+    if (n > W.n_cap || W.accA == nullptr || tcap > W.t_cap || L->n_large_chunks > W.hitem_cap ||
+        fcap0 > W.fitem_cap || L->cfg.n_sites > W.site_cap) {
+        // growing frees buffers that append-time hashing (staging stream) may still read
+        ck(cudaStreamSynchronize(L->stage_stream), "work sync");
+        ck(cudaStreamSynchronize(L->hash_stream), "work sync");
+        ck(cudaStreamSynchronize(L->stream), "work sync");
+    }
     if (n > W.n_cap || W.accA == nullptr) {
         ++L->epoch;
         uint64_t c = std::max<uint64_t>(n, 1024);
@@ -333,6 +358,12 @@ void ensure_work(ffm_log* L, uint64_t n) {
         dev_alloc(W.dq, (uint64_t)kDiffK * c);
         dev_alloc(W.dv, (uint64_t)kDiffK * c);
         dev_alloc(W.sdesc, 2 * c);
+        dev_alloc(W.sflag, c);
+        dev_alloc(W.sitems, 2 * c);
+        if (W.part_tmp) cudaFree(W.part_tmp);
+        W.part_tmp = nullptr;
+        W.part_tmp_bytes = std::max<size_t>(small_partition_bytes(c), 256);
+        ck(cudaMalloc(&W.part_tmp, W.part_tmp_bytes), "cudaMalloc(partition)");
         dev_alloc(W.hcount, c + 1);
         dev_alloc(W.hstart, c + 1);
         dev_alloc(W.dup, c);
@@ -426,7 +457,98 @@ void run_prologue(ffm_log* L) {
     upload_meta(L);
     ck(cudaEventRecord(L->ring_ev[L->ring_cur], L->stage_stream), "event");
     ck(cudaStreamWaitEvent(L->stream, L->ring_ev[L->ring_cur], 0), "wait staging");
+    ck(cudaStreamWaitEvent(L->stream, L->hash_ev, 0), "wait append-time hashing");
     ensure_work(L, L->h_size.size());
+}
+
+// A window [a, b) of the log as a log of its own (indices relative to a), with its
+// record order in `order` (capacity ocap: the inverse follows at order + ocap).
+DevLog window_view(const ffm_log* L, uint64_t a, uint64_t b, const uint32_t* order, uint64_t ocap, uint64_t ns,
+                   uint64_t nl) {
+    DevLog D = dev_view(L);
+    D.off += a;
+    D.size += a;
+    D.site += a;
+    D.dur += a;
+    D.gid += a;
+    D.chan += a;
+    D.n = (uint32_t)(b - a);
+    D.small_order = order;
+    D.order_pos = order + ocap;
+    D.n_small = (uint32_t)ns;
+    D.large_order = order + ns;
+    D.n_large = (uint32_t)nl;
+    return D;
+}
+
+// Online mode (S8(f) #2): the NH sums of records [a, b) into on_A / on_B (global record
+// index), on stream st -- at append time on the hashing stream (FFM_FLAG_ONLINE), else
+// at the start of a step.
+void online_hash(ffm_log* L, uint64_t a, uint64_t b, cudaStream_t st, uint64_t& launches) {
+    if (a >= b) return;
+    if (b > L->on_cap) {
+        uint64_t c0 = L->on_cap, cap = c0;
+        const uint64_t need = std::max<uint64_t>(b, 2 * c0);
+        dev_grow(L->on_A, cap, need, a, st);
+        cap = c0;
+        dev_grow(L->on_B, cap, need, a, st);
+        L->on_cap = cap;
+    }
+    std::vector<uint32_t> order;
+    const uint64_t ns = build_small_order(L, a, b, order);
+    upload_order(L, order, L->d_hash_order, L->d_hash_cap, st);
+    const DevLog D = window_view(L, a, b, L->d_hash_order, L->d_hash_cap, ns, order.size() - ns);
+    Work W2 = L->work;
+    W2.accA = L->on_A + a;
+    W2.accB = L->on_B + a;
+    uint64_t n_large = 0;
+    for (uint64_t i = a; i < b; ++i) n_large += large_chunks(L, L->h_size[i]);
+    LCHK(launch_hash_small(D, W2, L->params, st));
+    if (n_large) {
+        LCHK(launch_hash_plan(D, W2, L->params, true, st));
+        LCHK(launch_hash_large(D, W2, L->params, n_large, st));
+        LCHK(launch_combine(D, W2, L->params, st));
+    }
+}
+
+// Capacity of the persistent online table for nw more representatives (the table is
+// rehashed only when it has to grow: never by a step that fits).
+void ensure_online(ffm_log* L, uint64_t nw) {
+    OnlineTable& T = L->otab;
+    cudaStream_t s = L->stream;
+    if (!T.count) {
+        ck(cudaMalloc(&T.count, sizeof(uint32_t)), "cudaMalloc(online)");
+        ck(cudaMemsetAsync(T.count, 0, sizeof(uint32_t), s), "memset");
+    }
+    const uint64_t need = L->online_np + nw;
+    if (need > L->pool_cap) {
+        const uint64_t c = std::max<uint64_t>(std::max<uint64_t>(need, 1024), 2 * L->pool_cap);
+        OnlineRep* np = nullptr;
+        ck(cudaMalloc(&np, c * sizeof(OnlineRep)), "cudaMalloc(online pool)");
+        if (L->online_np)
+            ck(cudaMemcpyAsync(np, T.pool, L->online_np * sizeof(OnlineRep), cudaMemcpyDeviceToDevice, s), "copy");
+        ck(cudaStreamSynchronize(s), "pool sync");
+        if (T.pool) ck(cudaFree(T.pool), "cudaFree");
+        T.pool = np;
+        L->pool_cap = c;
+    }
+    if (2 * need > T.mask + 1 || !T.key) {
+        const uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(4 * need));
+        ck(cudaStreamSynchronize(s), "table sync");
+        if (T.key) ck(cudaFree(T.key), "cudaFree");
+        if (T.head) ck(cudaFree(T.head), "cudaFree");
+        T.key = nullptr;
+        T.head = nullptr;
+        ck(cudaMalloc(&T.key, cap * sizeof(uint64_t)), "cudaMalloc(online table)");
+        ck(cudaMalloc(&T.head, cap * sizeof(uint32_t)), "cudaMalloc(online table)");
+        T.mask = cap - 1;
+        if (launch_online_rehash(T, (uint32_t)L->online_np, L->params.digest_mask, s) < 0)
+            throw CudaFail{cudaGetLastError(), "online rehash"};
+    }
+    if (nw > L->on_G_cap) {
+        dev_alloc(L->on_G, nw);
+        L->on_G_cap = nw;
+    }
 }
 
 // H1..H4 over the local log: on return W.leader holds every record's final local
@@ -435,8 +557,14 @@ void run_prologue(ffm_log* L) {
 // there are no digest collisions) and re-run after collision resolution.
 // pre_sync: more stream work queued after segment A, before its host sync (a sharded
 // run's representative export and header exchange).
+// prehashed: the NH sums are already in W.accA / W.accB (online windows): two-pass
+// round 0 without H1.
+// h_spec: pinned host duplicate_of: the labels are written speculatively after the
+// round-0 group-by and copied there while H3 runs (R.spec_stale: residuals changed some;
+// the caller copies again).
 LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& launches, bool label, int64_t* d_dup,
-                   bool prefilter = false, const std::function<void()>* pre_sync = nullptr) {
+                   bool prefilter = false, const std::function<void()>* pre_sync = nullptr, bool prehashed = false,
+                   int64_t* h_spec = nullptr) {
     const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
     const uint64_t n = D.n;
     Work& W = L->work;
@@ -446,7 +574,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     cudaStream_t side = L->side_stream;
     // round-0 mode: forced by a flag, else adaptive -- a log whose fused run found most
     // large candidates to be near-duplicate mismatches uses the two-pass round 0 next time
-    const bool two_pass = (L->cfg.flags & FFM_FLAG_TWO_PASS) != 0 ||
+    const bool two_pass = prehashed || (L->cfg.flags & FFM_FLAG_TWO_PASS) != 0 ||
                           (!(L->cfg.flags & FFM_FLAG_FUSED) && L->prefer_two_pass);
     // segment A: everything up to the first host sync (H1, H2, H3, speculative H5/H6 and
     // the counters read-back) -- ~30 launches on two streams, no host dependency
@@ -455,7 +583,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         if (launch_zero_counters(W, s) < 0) throw CudaFail{cudaGetLastError(), "zero counters"};
         // two-pass H1 of small payloads on the side stream, concurrently with the large path
         // (fused: small payloads are grouped by their first 32 bytes, hashed after H2)
-        if (two_pass) {
+        if (two_pass && !prehashed) {
             ck(cudaEventRecord(L->fork_ev[0], s), "event");
             ck(cudaStreamWaitEvent(side, L->fork_ev[0], 0), "fork");
             if (timing) ck(cudaEventRecord(L->ev[12], side), "event");
@@ -463,7 +591,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
             if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
             ck(cudaEventRecord(L->fork_ev[1], side), "event");
         }
-        if (n_large) {
+        if (n_large && !prehashed) {
             LCHK(launch_hash_plan(D, W, L->params, two_pass, s));
             if (timing) ck(cudaEventRecord(L->ev[10], s), "event");
             // fused: the prefix pass (first prefix_bytes); two-pass: every chunk, then the combine
@@ -472,12 +600,22 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
             if (timing) ck(cudaEventRecord(L->ev[11], s), "event");
             if (two_pass) LCHK(launch_combine(D, W, L->params, s));
         }
-        if (two_pass) ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
+        if (two_pass && !prehashed) ck(cudaStreamWaitEvent(s, L->fork_ev[1], 0), "join");
         if (timing) ck(cudaEventRecord(L->ev[1], s), "event");
         // H2 group-by (round 0): two-pass -- every payload by its full digest; fused -- small
         // payloads by their first 32 bytes, large ones by their first-chunk digest
         uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
         LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, two_pass ? -1 : 0, W.res[0], s));
+        if (h_spec) {
+            // speculative labels, copied to the host on the copy stream during H3
+            LCHK(launch_spec_label(D, W, d_dup, s));
+            ck(cudaEventRecord(L->copy_ev[0], s), "event");
+            ck(cudaStreamWaitEvent(L->copy_stream, L->copy_ev[0], 0), "fork copy");
+            ck(cudaMemcpyAsync(h_spec, d_dup, (uint64_t)D.n * sizeof(int64_t), cudaMemcpyDeviceToHost,
+                               L->copy_stream),
+               "D2H dup (speculative)");
+            ck(cudaEventRecord(L->copy_ev[1], L->copy_stream), "event");
+        }
         if (timing) ck(cudaEventRecord(L->ev[2], s), "event");
         if (two_pass) {
             // H3 (two-pass): every member byte-verified against its full-digest candidate
@@ -502,7 +640,8 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         }
         if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
         // H5 + H6 (speculative: valid unless H3 found residuals)
-        if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, s));
+        if (label) LCHK(launch_label(D, W, L->params, ns, h_spec ? nullptr : d_dup, s));
+        if (h_spec) ck(cudaStreamWaitEvent(s, L->copy_ev[1], 0), "join copy");
         if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
         ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
     };
@@ -511,7 +650,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     if (graph) {
         // replay a CUDA graph of segment A while the log, its buffers and the run mode are
         // unchanged: one launch instead of ~30 (launch-bound small logs)
-        const GraphKey key{L->epoch, d_dup, two_pass, prefilter, timing};
+        const GraphKey key{L->epoch, d_dup, h_spec, two_pass, prefilter, timing};
         if (!L->graph_exec || !(key == L->graph_key)) {
             if (L->graph_exec) cudaGraphExecDestroy(L->graph_exec);
             L->graph_exec = nullptr;
@@ -550,6 +689,8 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     if (nres) {
         // H4 collision resolution: exact classes among the residual members
         if (timing) ck(cudaEventRecord(L->ev[6], s), "event");
+        // a fused round 0 hashed no small member: the residual ones are hashed now
+        if (!two_pass && D.n_small) LCHK(launch_hash_small_list(D, W, L->params, W.res[0], (uint32_t)nres, s));
         int cur = 0;
         while (nres) {
             ++R.rounds;
@@ -572,6 +713,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         }
         if (label) LCHK(launch_label(D, W, L->params, ns, d_dup, s));
         if (timing) ck(cudaEventRecord(L->ev[7], s), "event");
+        R.spec_stale = h_spec != nullptr;
     }
     return R;
 }
@@ -609,10 +751,12 @@ void fill_stats(ffm_log* L, const LocalRun& R, uint64_t launches, bool single) {
 
 
 // ---------------------------------------------------------------- sharded runs
+// (zeroed on the run stream: the legacy-stream cudaMemset does not order before kernels
+// on the library's non-blocking streams)
 template <class T>
-void dev_alloc_zero(T*& p, uint64_t count) {
+void dev_alloc_zero(T*& p, uint64_t count, cudaStream_t st) {
     dev_alloc(p, count);
-    ck(cudaMemset(p, 0, std::max<uint64_t>(count, 1) * sizeof(T)), "memset");
+    ck(cudaMemsetAsync(p, 0, std::max<uint64_t>(count, 1) * sizeof(T), st), "memset");
 }
 
 void ensure_cub(ffm_log* L, uint64_t n) {
@@ -641,8 +785,8 @@ void ensure_shard(ffm_log* L, uint64_t n, uint64_t M, uint64_t nloc, uint64_t vc
         dev_alloc(S.tkey, cap);
         dev_alloc(S.tgid, cap);
         dev_alloc(S.tidx, cap);
-        dev_alloc_zero(S.need, cap);   // zero between runs (k_seg_clear)
-        dev_alloc_zero(S.scnt, cap);
+        dev_alloc_zero(S.need, cap, L->stream);   // zero between runs (k_seg_clear)
+        dev_alloc_zero(S.scnt, cap, L->stream);
         dev_alloc(S.sbase, cap);
         dev_alloc(S.sfill, cap);
         S.t_cap = cap;
@@ -914,6 +1058,11 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
         }
         ck(cudaStreamCreateWithFlags(&L->stage_stream, cudaStreamNonBlocking), "stream");
         ck(cudaStreamCreateWithFlags(&L->side_stream, cudaStreamNonBlocking), "stream");
+        ck(cudaStreamCreateWithFlags(&L->hash_stream, cudaStreamNonBlocking), "stream");
+        ck(cudaStreamCreateWithFlags(&L->copy_stream, cudaStreamNonBlocking), "stream");
+        for (auto& e : L->copy_ev) ck(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
+        ck(cudaEventCreateWithFlags(&L->hash_ev, cudaEventDisableTiming), "event");
+        ck(cudaEventRecord(L->hash_ev, L->hash_stream), "event");
         for (auto& e : L->fork_ev) ck(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
         L->ring_bytes = kRingBytes;
         for (int i = 0; i < 2; ++i) {
@@ -1038,6 +1187,20 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
         if (need_sync) ck(cudaStreamSynchronize(L->stage_stream), "append sync");   // snapshot before return
         push_meta(L, n, sites, sizes, durs, gids, channels, offs, end);
         L->digests_valid = false;
+        if (L->cfg.flags & FFM_FLAG_ONLINE) {
+            // online mode: hash the new records now, on the hashing stream after their
+            // staging copies -- the next append's staging overlaps this hashing
+            ring_flush(L);
+            upload_meta_arrays(L);
+            ensure_work(L, L->h_size.size());
+            ck(cudaEventRecord(L->fork_ev[2], L->stage_stream), "event");
+            ck(cudaStreamWaitEvent(L->hash_stream, L->fork_ev[2], 0), "wait staging");
+            uint64_t launches = 0;
+            const uint64_t a = std::max(L->online_hashed, L->online_done), b = L->h_size.size();
+            online_hash(L, a, b, L->hash_stream, launches);
+            ck(cudaEventRecord(L->hash_ev, L->hash_stream), "event");
+            L->online_hashed = b;
+        }
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
     } catch (const std::bad_alloc&) {
@@ -1084,11 +1247,14 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
             return FFM_OK;
         }
         const bool prefilter = (L->cfg.flags & FFM_FLAG_PREFILTER) != 0;
-        LocalRun R = run_local(L, dev_view(L), L->n_large_chunks, launches, true, d_dup, prefilter);
+        // pinned host output: the labels travel over PCIe while H3 streams HBM
+        const bool spec = !dup_dev && n && is_pinned_host(dup_out);
+        LocalRun R = run_local(L, dev_view(L), L->n_large_chunks, launches, true, d_dup, prefilter, nullptr, false,
+                               spec ? dup_out : nullptr);
         // H7 return
         const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
         if (timing) ck(cudaEventRecord(L->ev[9], s), "event");
-        if (!dup_dev && n)
+        if (!dup_dev && n && (!spec || R.spec_stale))
             ck(cudaMemcpyAsync(dup_out, d_dup, n * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
         if (ben_out)
             ck(cudaMemcpyAsync(ben_out, W.ben, ns * sizeof(uint64_t),
@@ -1185,101 +1351,75 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
     const uint64_t n = L->h_size.size(), w0 = L->online_done, nw = n - w0;
     if (nw && !dup_out) return set_err(L, FFM_E_INVAL, "duplicate_of is NULL");
     const uint32_t ns = L->cfg.n_sites;
-    const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
     try {
-        run_prologue(L);
+        L->n_syncs = 0;
+        ck(cudaSetDevice(L->device), "cudaSetDevice");
         Work& W = L->work;
-        ShardWork& S = L->shard;
         cudaStream_t s = L->stream;
+        // H0 tail for the window only (no whole-log order: O(window) host work per step)
+        ring_flush(L);
+        upload_meta_arrays(L);
+        ck(cudaEventRecord(L->ring_ev[L->ring_cur], L->stage_stream), "event");
+        ck(cudaStreamWaitEvent(s, L->ring_ev[L->ring_cur], 0), "wait staging");
+        ck(cudaStreamWaitEvent(s, L->hash_ev, 0), "wait append-time hashing");
+        ensure_work(L, n);
         if (!L->online_ben) {
-            ck(cudaMalloc(&L->online_ben, ns * sizeof(uint64_t)), "cudaMalloc(online)");
-            ck(cudaMalloc(&L->online_cnt, ns * sizeof(uint64_t)), "cudaMalloc(online)");
-            ck(cudaMemsetAsync(L->online_ben, 0, ns * sizeof(uint64_t), s), "memset");
-            ck(cudaMemsetAsync(L->online_cnt, 0, ns * sizeof(uint64_t), s), "memset");
+            ck(cudaMalloc(&L->online_ben, 2 * (uint64_t)ns * sizeof(uint64_t)), "cudaMalloc(online)");
+            ck(cudaMemsetAsync(L->online_ben, 0, 2 * (uint64_t)ns * sizeof(uint64_t), s), "memset");
+            L->online_cnt = L->online_ben + ns;
         }
         uint64_t launches = 0;
         LocalRun R{};
-        uint64_t n_slow = 0;
         if (nw) {
-            // the window view: records [w0, n) as a log of their own (indices relative to w0)
-            DevLog D = dev_view(L);
-            D.off += w0;
-            D.size += w0;
-            D.site += w0;
-            D.dur += w0;
-            D.gid += w0;
-            D.chan += w0;
-            D.n = (uint32_t)nw;
+            // H1 (unless the appends hashed already, FFM_FLAG_ONLINE)
+            const uint64_t h0 = std::max(L->online_hashed, w0);
+            if (h0 < n) online_hash(L, h0, n, s, launches);
+            L->online_hashed = n;
             std::vector<uint32_t> order;
             const uint64_t nsw = build_small_order(L, w0, n, order);
             upload_order(L, order, L->d_win_order, L->d_win_cap, s);
-            D.small_order = L->d_win_order;
-            D.order_pos = L->d_win_order + L->d_win_cap;
-            D.n_small = (uint32_t)nsw;
-            D.large_order = L->d_win_order + nsw;
-            D.n_large = (uint32_t)(order.size() - nsw);
+            const DevLog D = window_view(L, w0, n, L->d_win_order, L->d_win_cap, nsw, order.size() - nsw);
             uint64_t n_large = 0;
             for (uint64_t i = w0; i < n; ++i) n_large += large_chunks(L, L->h_size[i]);
-            // H1..H4 on the window: exact window-local classes
-            R = run_local(L, D, n_large, launches, false, nullptr);
-            // window representatives appended after the prior ones
-            const uint64_t np = L->online_np;
-            if (np + nw > L->online_cap) {
-                uint64_t c = std::max<uint64_t>(np + nw, 2 * L->online_cap);
-                ffm::RepTuple* t = nullptr;
-                ck(cudaMalloc(&t, c * sizeof(ffm::RepTuple)), "cudaMalloc(online)");
-                if (np) ck(cudaMemcpyAsync(t, L->online_T, np * sizeof(ffm::RepTuple), cudaMemcpyDeviceToDevice, s),
-                           "copy");
-                ck(cudaStreamSynchronize(s), "sync");
-                if (L->online_T) ck(cudaFree(L->online_T), "cudaFree");
-                if (L->online_tmp) ck(cudaFree(L->online_tmp), "cudaFree");
-                L->online_T = t;
-                ck(cudaMalloc(&L->online_tmp, c * sizeof(ffm::RepTuple)), "cudaMalloc(online)");
-                L->online_cap = c;
+            // H2..H4 on the window: exact window classes (the NH sums are the window's slice
+            // of on_A / on_B)
+            {
+                uint64_t* keepA = W.accA;
+                uint64_t* keepB = W.accB;
+                W.accA = L->on_A + w0;
+                W.accB = L->on_B + w0;
+                try {
+                    R = run_local(L, D, n_large, launches, false, nullptr, false, nullptr, true);
+                } catch (...) {
+                    W.accA = keepA;
+                    W.accB = keepB;
+                    throw;
+                }
+                W.accA = keepA;
+                W.accB = keepB;
             }
-            ensure_shard(L, nw, np + nw, nw, nw + n_large + 64, 2);
-            LCHK(launch_rep_export(D, W, S, L->params, L->online_T + np, s));
-            ck(cudaMemcpyAsync(L->h_counters, S.rep_idx + nw, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
-            ck(cudaStreamSynchronize(s), "online sync");
-            const uint64_t nloc = L->h_counters[0], M = np + nloc;
-            // "compared to the stored hashes from prior transfers": the prior
-            // classes play the part of a peer shard living in the same arena
-            const uint32_t rank_lo[2] = {0u, (uint32_t)np};
-            const uint8_t* bases[2] = {L->arena, L->arena};
-            ck(cudaMemcpyAsync(S.rank_lo, rank_lo, sizeof(rank_lo), cudaMemcpyHostToDevice, s), "H2D");
-            ck(cudaMemcpyAsync((void*)S.bases, bases, sizeof(bases), cudaMemcpyHostToDevice, s), "H2D");
-            uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(M, 1)));
-            LCHK(launch_merge(D, W, S, L->params, L->online_T, (uint32_t)M, (uint32_t)np, (uint32_t)nloc, 2, 1, cap, s));
+            // each window class against the stored classes of all earlier windows ("compared
+            // to the stored hashes from prior transfers"); new classes are stored
+            ensure_online(L, nw);
             const bool dup_dev = is_device_ptr(dup_out);
             int64_t* d_dup = dup_dev ? dup_out : W.dup;
-            LCHK(launch_merge_label(D, W, S, L->params, ns, d_dup, s));
-            LCHK(launch_vec_add(L->online_ben, W.ben, ns, s));
-            LCHK(launch_vec_add(L->online_cnt, W.cnt, ns, s));
-            // new classes join the stored representatives
-            LCHK(launch_online_newreps(W, S, L->online_T + np, (uint32_t)nloc, L->online_tmp, s));
-            ck(cudaMemcpyAsync(L->h_counters, S.vstart + nloc, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
-            ck(cudaMemcpyAsync(L->h_counters + 2, S.sctr, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+            LCHK(launch_online_window(D, W, L->on_A + w0, L->on_B + w0, L->otab, L->params, ns, L->on_G, d_dup,
+                                      L->online_ben, L->online_cnt, s));
             if (!dup_dev)
                 ck(cudaMemcpyAsync(dup_out, d_dup, nw * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
-            ck(cudaStreamSynchronize(s), "online new reps sync");
-            const uint64_t n_new = L->h_counters[0];
-            n_slow = L->h_counters[2];
-            if (n_new)
-                ck(cudaMemcpyAsync(L->online_T + np, L->online_tmp, n_new * sizeof(ffm::RepTuple),
-                                   cudaMemcpyDeviceToDevice, s),
-                   "copy reps");
-            L->online_np = np + n_new;
+            ck(cudaMemcpyAsync(L->h_counters + 2, L->otab.count, sizeof(uint32_t), cudaMemcpyDeviceToHost, s),
+               "D2H");
         }
         if (ben_out)
             ck(cudaMemcpyAsync(ben_out, L->online_ben, ns * sizeof(uint64_t), cudaMemcpyDefault, s), "copy ben");
-        ck(cudaStreamSynchronize(s), "online sync");
+        sync_run(L, "online sync");
         ck(cudaGetLastError(), "online step");
+        if (nw) L->online_np = L->h_counters[2];
         L->online_done = n;
         fill_stats(L, R, launches, false);
-        L->stats.n_residual += n_slow;
         L->stats.n_records = nw;
+        L->stats.host_syncs = L->n_syncs;
         L->digests_valid = false;
-        (void)timing;
         if (n_out) *n_out = nw;
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
@@ -1297,7 +1437,10 @@ int ffm_debug_digests(ffm_log* L, uint64_t* out) {
     try {
         ck(cudaSetDevice(L->device), "cudaSetDevice");
         uint64_t n = L->h_size.size();
-        if (n) ck(cudaMemcpy(out, L->work.digest, n * 8, cudaMemcpyDeviceToHost), "D2H digests");
+        if (n && launch_digest_fill(dev_view(L), L->work, L->params, L->stream) < 0)
+            throw CudaFail{cudaGetLastError(), "digest fill"};
+        if (n) ck(cudaMemcpyAsync(out, L->work.digest, n * 8, cudaMemcpyDeviceToHost, L->stream), "D2H digests");
+        ck(cudaStreamSynchronize(L->stream), "digests sync");
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
     }
@@ -1317,6 +1460,7 @@ int ffm_log_reset(ffm_log* L) {
     try {
         ck(cudaSetDevice(L->device), "cudaSetDevice");
         ck(cudaStreamSynchronize(L->stage_stream), "reset sync");
+        ck(cudaStreamSynchronize(L->hash_stream), "reset sync");
         ck(cudaStreamSynchronize(L->stream), "reset sync");
     } catch (const CudaFail& f) {
         return fail_cuda(L, f);
@@ -1330,14 +1474,22 @@ int ffm_log_reset(ffm_log* L) {
     L->payload_bytes = L->n_large_chunks = L->last_gid = 0;
     L->any_gid = false;
     L->d_meta_n = 0;
+    L->d_order_n = 0;
     L->n_small = 0;
     L->n_large_rec = 0;
     L->arena_used = 0;
     L->ring_fill = 0;
-    L->online_done = L->online_np = 0;
-    if (L->online_ben) {
-        cudaMemset(L->online_ben, 0, L->cfg.n_sites * sizeof(uint64_t));
-        cudaMemset(L->online_cnt, 0, L->cfg.n_sites * sizeof(uint64_t));
+    L->online_done = L->online_np = L->online_hashed = 0;
+    if (L->online_ben) cudaMemsetAsync(L->online_ben, 0, 2 * (uint64_t)L->cfg.n_sites * sizeof(uint64_t), L->stream);
+    if (L->otab.count) {   // an empty table (keeps its capacity)
+        cudaMemsetAsync(L->otab.count, 0, sizeof(uint32_t), L->stream);
+        cudaMemsetAsync(L->otab.key, 0xFF, (L->otab.mask + 1) * sizeof(uint64_t), L->stream);
+        cudaMemsetAsync(L->otab.head, 0xFF, (L->otab.mask + 1) * sizeof(uint32_t), L->stream);
+    }
+    if (cudaStreamSynchronize(L->stream) != cudaSuccess) {
+        L->poisoned = true;
+        L->last_error = "reset sync failed";
+        return FFM_E_CUDA;
     }
     L->digests_valid = false;
     L->prefer_two_pass = false;
@@ -1353,14 +1505,15 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->stage_stream) cudaStreamSynchronize(L->stage_stream);
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
-                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.fitems, W.sdesc, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
+                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.fitems, W.sdesc, W.sflag, W.sitems, W.part_tmp, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
                     W.dup, W.ben, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
                     L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     free_shard(L->shard);
     if (L->fold_buf) cudaFree(L->fold_buf);
-    void* op[] = {L->online_T, L->online_tmp, L->online_ben, L->online_cnt, L->d_win_order};
+    void* op[] = {L->otab.key, L->otab.head, L->otab.pool, L->otab.count, L->on_A, L->on_B, L->on_G,
+                  L->online_ben, L->d_win_order, L->d_hash_order};
     for (void* p : op)
         if (p) cudaFree(p);
     for (void* p : L->peer_ptr)
@@ -1379,6 +1532,14 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->h_counters) cudaFreeHost(L->h_counters);
     if (L->stage_stream) cudaStreamDestroy(L->stage_stream);
     if (L->side_stream) cudaStreamDestroy(L->side_stream);
+    if (L->hash_stream) {
+        cudaStreamSynchronize(L->hash_stream);
+        cudaStreamDestroy(L->hash_stream);
+    }
+    if (L->hash_ev) cudaEventDestroy(L->hash_ev);
+    if (L->copy_stream) cudaStreamDestroy(L->copy_stream);
+    for (auto e : L->copy_ev)
+        if (e) cudaEventDestroy(e);
     for (auto e : L->fork_ev)
         if (e) cudaEventDestroy(e);
     if (L->graph_exec) cudaGraphExecDestroy(L->graph_exec);

@@ -52,6 +52,10 @@ struct Work {
     uint32_t* fhead = nullptr;     // [n] round 0: head (leader) of a large record's fused group
     uint2* hitems = nullptr;       // large-payload hash work units (record, chunk)
     uint4* sdesc = nullptr;        // [2 * n] fused round 0: compare descriptors of small records (order position)
+    uint8_t* sflag = nullptr;      // [n] 1: that small record is a member (compared), 0: hashed
+    uint4* sitems = nullptr;       // [2 * n] sdesc partitioned: members, then the others (reversed)
+    void* part_tmp = nullptr;      // cub partition scratch
+    size_t part_tmp_bytes = 0;
     uint4* fitems = nullptr;       // pipelined fused pass stage descriptors (2 x uint4 each)
     uint32_t* dcnt = nullptr;      // [n] fused round 0: words where a large member differs from its group head
     uint32_t* dq = nullptr;        // [n * kDiffK] their 16-B word indices (the first kDiffK recorded)
@@ -107,6 +111,20 @@ struct ShardWork {
     uint64_t n_cap = 0, m_cap = 0, t_cap = 0, l_cap = 0, v_cap = 0, w_cap = 0;
 };
 
+// Online mode: stored class representatives (insert-only pool) and the table over them.
+struct OnlineRep {
+    uint64_t gid, off, size, chan, dig;   // dig: full 64-bit digest
+    uint32_t next, pad;                   // chain of the key (kNoRep-terminated)
+};
+
+struct OnlineTable {
+    uint64_t* key = nullptr;     // [mask + 1] group key, kEmptyKey = free
+    uint32_t* head = nullptr;    // [mask + 1] first pool entry of the key's chain
+    OnlineRep* pool = nullptr;   // [pool_cap]
+    uint32_t* count = nullptr;   // device: pool entries used
+    uint64_t mask = 0;
+};
+
 struct Params {
     uint64_t digest_mask;
     uint64_t refine_mask;
@@ -143,8 +161,11 @@ int launch_site_reduce(const uint64_t* part, const uint32_t* cpart, uint32_t row
 int launch_rep_export(const DevLog& L, Work& W, ShardWork& S, const Params& P, RepTuple* out, cudaStream_t st);
 int launch_merge(const DevLog& L, Work& W, ShardWork& S, const Params& P, const RepTuple* T, uint32_t M,
                  uint32_t lo, uint32_t nloc, int world, int rank, uint64_t cap, cudaStream_t st);
-int launch_online_newreps(Work& W, ShardWork& S, RepTuple* Tw, uint32_t nloc, RepTuple* tmp, cudaStream_t st);
-int launch_vec_add(uint64_t* a, const uint64_t* b, uint32_t n, cudaStream_t st);
+// online.cu
+int launch_online_rehash(OnlineTable& T, uint32_t np, uint64_t digest_mask, cudaStream_t st);
+int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, const uint64_t* accB,
+                         OnlineTable& T, const Params& P, uint32_t n_sites, uint64_t* G, int64_t* dup_out,
+                         uint64_t* ben, uint64_t* cnt, cudaStream_t st);
 int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
                        cudaStream_t st);
 int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uint64_t gen, uint64_t n,
@@ -152,7 +173,12 @@ int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uin
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t st);
+int launch_spec_label(const DevLog& L, Work& W, int64_t* dup_out, cudaStream_t st);
+int launch_digest_fill(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
+int launch_hash_small_list(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
+                           cudaStream_t st);
 size_t cub_scan_bytes(uint64_t n);
+size_t small_partition_bytes(uint64_t n);
 uint64_t fx_entry_cap(uint64_t n_large_chunks, uint32_t chunk_bytes);
 uint32_t blocks_for(uint64_t threads, uint32_t bs = 256);
 uint32_t resident_grid(const void* kernel, int num_sms, int block = 256);
@@ -164,10 +190,11 @@ bool smem_configured(const void* kernel, int bytes);
 struct GraphKey {
     uint64_t epoch = ~0ull;
     const void* dup = nullptr;
+    const void* hdup = nullptr;   // pinned host duplicate_of of the speculative D2H (or null)
     bool two_pass = false, prefilter = false, timing = false;
     bool operator==(const GraphKey& o) const {
-        return epoch == o.epoch && dup == o.dup && two_pass == o.two_pass && prefilter == o.prefilter &&
-               timing == o.timing;
+        return epoch == o.epoch && dup == o.dup && hdup == o.hdup && two_pass == o.two_pass &&
+               prefilter == o.prefilter && timing == o.timing;
     }
 };
 
@@ -178,6 +205,10 @@ struct ffm_log {
     cudaStream_t stream = nullptr;
     cudaStream_t stage_stream = nullptr;
     cudaStream_t side_stream = nullptr;   // small-payload kernels run concurrently here
+    cudaStream_t hash_stream = nullptr;   // append-time hashing (online mode)
+    cudaStream_t copy_stream = nullptr;   // speculative D2H of duplicate_of during H3
+    cudaEvent_t copy_ev[2] = {};
+    cudaEvent_t hash_ev = nullptr;        // the last append-time hashing
     cudaEvent_t fork_ev[4] = {};
     bool own_stream = false;
     bool poisoned = false;
@@ -207,6 +238,7 @@ struct ffm_log {
     uint64_t* d_chan = nullptr;
     uint64_t d_meta_cap = 0;       // records
     uint64_t d_meta_n = 0;         // records uploaded
+    uint64_t d_order_n = 0;        // records covered by d_small_order
     uint32_t* d_small_order = nullptr;   // small records by size class (built at upload)
     uint64_t d_small_cap = 0, n_small = 0, n_large_rec = 0;
 
@@ -239,15 +271,23 @@ struct ffm_log {
     uint8_t* d_ipc = nullptr;          // [64 * (world + 1)] IPC handle exchange
     uint64_t* h_hdr = nullptr;         // pinned mirror of all headers (+ run counters)
 
-    // online (streaming) mode: representatives of every class seen so far
+    // online (streaming) mode: the persistent table of every class seen so far
     uint64_t online_done = 0;        // records already labelled online
-    ffm::RepTuple* online_T = nullptr;   // [online_np prior reps | window reps]
-    ffm::RepTuple* online_tmp = nullptr;
-    uint64_t online_np = 0, online_cap = 0;
-    uint64_t* online_ben = nullptr;  // cumulative per-site benefit / duplicate counts
-    uint64_t* online_cnt = nullptr;
-    uint32_t* d_win_order = nullptr;
+    uint64_t online_hashed = 0;      // records whose NH sums are in on_A / on_B
+    ffm::OnlineTable otab;
+    uint64_t online_np = 0;          // stored representatives (read back after each step)
+    uint64_t pool_cap = 0;
+    uint64_t* on_A = nullptr;        // [records] NH sums (global record index)
+    uint64_t* on_B = nullptr;
+    uint64_t on_cap = 0;
+    uint64_t* on_G = nullptr;        // [window] global leader gid of each window class
+    uint64_t on_G_cap = 0;
+    uint64_t* online_ben = nullptr;  // [2 * n_sites] cumulative per-site benefit | duplicate counts
+    uint64_t* online_cnt = nullptr;  //   (= online_ben + n_sites)
+    uint32_t* d_win_order = nullptr; // the step's window order
     uint64_t d_win_cap = 0;
+    uint32_t* d_hash_order = nullptr;   // the append-time hashing's window order
+    uint64_t d_hash_cap = 0;
 
     // folded grouping scratch
     void* fold_buf = nullptr;

@@ -1,0 +1,195 @@
+// online.cu -- online (streaming) mode, SURVEY.md 8(f) #2 / DESIGN.md §10: the paper's
+// per-call semantics (Sec. 3.3.2): "The data being transferred is hashed and
+// then compared to the stored hashes from prior transfers."
+//
+// The stored hashes are a persistent device table of every exact class seen so far:
+// open addressing on the group key of (full digest, size, channel) -> a chain of class
+// representatives in an insert-only pool (gid, arena offset, size, channel, digest).
+// A step labels one window of new records:
+//   1. the window's NH sums were computed at append time on the staging stream
+//      (FFM_FLAG_ONLINE), else at the start of the step;
+//   2. H2-H4 on the window alone -> exact window classes (two-pass round 0 without H1);
+//   3. k_online_match: each window class representative looks its key up in the table
+//      and byte-compares the chained prior representatives of its size / channel /
+//      digest (their bytes stay resident in the HBM arena) -- at most one prior class
+//      can be equal, so the chain order does not matter;
+//   4. k_online_insert: classes with no equal prior class join the table;
+//   5. k_online_label: labels (gids) and the cumulative per-site benefit / counts.
+// The table is never rebuilt by a step; it is rehashed only when its capacity doubles.
+#include "digest.cuh"
+#include "ffm_internal.h"
+
+namespace ffm {
+
+constexpr uint32_t kNoRep = 0xFFFFFFFFu;
+
+// slot of `key` in the table (probing), or the empty slot where it would go
+__device__ __forceinline__ uint64_t online_probe(const OnlineTable& T, uint64_t key) {
+    uint64_t h = key & T.mask;
+    while (true) {
+        const uint64_t k = T.key[h];
+        if (k == key || k == kEmptyKey) return h;
+        h = (h + 1) & T.mask;
+    }
+}
+
+__device__ __forceinline__ void online_link(OnlineTable& T, uint64_t key, uint32_t idx) {
+    uint64_t h = key & T.mask;
+    while (true) {
+        unsigned long long prev =
+            atomicCAS((unsigned long long*)&T.key[h], (unsigned long long)kEmptyKey, (unsigned long long)key);
+        if (prev == kEmptyKey || prev == key) break;
+        h = (h + 1) & T.mask;
+    }
+    T.pool[idx].next = atomicExch(&T.head[h], idx);
+}
+
+// One warp per window class representative r (leader[r] == r).
+__global__ void __launch_bounds__(256) k_online_match(DevLog L, const uint32_t* __restrict__ leader,
+                                                      const uint64_t* __restrict__ accA,
+                                                      const uint64_t* __restrict__ accB, OnlineTable T,
+                                                      uint64_t digest_mask, uint64_t refine_mask,
+                                                      uint64_t* __restrict__ G) {
+    const uint32_t* nolist = nullptr;
+    FFM_WARP_COMPACT(L.n, nolist, (leader[r_] == r_), {
+        const uint64_t n = L.size[rec], chan = L.chan[rec];
+        const uint64_t dig = finalize_digest(accA[rec], accB[rec], n);
+        const uint64_t key = group_key(dig, n, digest_mask, chan);
+        const uint64_t h = online_probe(T, key);
+        uint32_t idx = T.key[h] == key ? T.head[h] : kNoRep;
+        uint64_t g = L.gid[rec];
+        const uint8_t* px = L.arena + L.off[rec];
+        const uint64_t nblk = (n + 31) >> 5;
+        while (idx != kNoRep) {
+            const OnlineRep e = T.pool[idx];
+            if (e.size == n && e.chan == chan && ((e.dig ^ dig) & refine_mask) == 0) {
+                const uint8_t* py = L.arena + e.off;
+                bool diff = false;
+                for (uint64_t b0 = 0; b0 < nblk && !diff; b0 += 32) {
+                    const uint64_t b = b0 + lane;
+                    bool d = false;
+                    if (b < nblk) {
+                        Blk a = ld_stream(px + 32 * b);
+                        Blk y = ld_keep(py + 32 * b);
+                        mask_tail(a, n, b);
+                        mask_tail(y, n, b);
+                        d = !blk_equal(a, y);
+                    }
+                    diff = __any_sync(0xFFFFFFFFu, d);
+                }
+                if (!diff) {   // the (only) equal prior class
+                    g = e.gid;
+                    break;
+                }
+            }
+            idx = e.next;
+        }
+        if (lane == 0) G[rec] = g;
+    })
+}
+
+// Window classes without an equal prior class become stored representatives.
+__global__ void k_online_insert(DevLog L, const uint32_t* __restrict__ leader, const uint64_t* __restrict__ accA,
+                                const uint64_t* __restrict__ accB, const uint64_t* __restrict__ G, OnlineTable T,
+                                uint64_t digest_mask) {
+    const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= L.n || leader[r] != r || G[r] != L.gid[r]) return;
+    const uint64_t n = L.size[r];
+    const uint64_t dig = finalize_digest(accA[r], accB[r], n);
+    const uint32_t idx = atomicAdd(T.count, 1u);
+    OnlineRep e;
+    e.gid = L.gid[r];
+    e.off = L.off[r];
+    e.size = n;
+    e.chan = L.chan[r];
+    e.dig = dig;
+    e.next = kNoRep;
+    e.pad = 0;
+    T.pool[idx] = e;
+    online_link(T, group_key(dig, n, digest_mask, e.chan), idx);
+}
+
+// Capacity growth: re-link every stored representative into a fresh (larger) table.
+__global__ void k_online_rehash(OnlineTable T, uint32_t np, uint64_t digest_mask) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= np) return;
+    const OnlineRep e = T.pool[i];
+    online_link(T, group_key(e.dig, e.size, digest_mask, e.chan), i);
+}
+
+// Labels of the window and the cumulative per-site sums (block histograms in shared
+// memory when the sites fit, then one atomic per (block, site)).
+template <bool kHist>
+__global__ void __launch_bounds__(1024) k_online_label(DevLog L, const uint32_t* __restrict__ leader,
+                                                       const uint64_t* __restrict__ G, uint32_t n_sites,
+                                                       int64_t* __restrict__ dup_out, uint64_t* __restrict__ ben,
+                                                       uint64_t* __restrict__ cnt) {
+    extern __shared__ unsigned long long sben[];
+    uint32_t* scnt = (uint32_t*)(sben + n_sites);
+    if (kHist) {
+        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) {
+            sben[s] = 0;
+            scnt[s] = 0;
+        }
+        __syncthreads();
+    }
+    for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < L.n; r += gridDim.x * blockDim.x) {
+        const uint64_t g = G[leader[r]];
+        const int64_t d = g == L.gid[r] ? -1 : (int64_t)g;
+        dup_out[r] = d;
+        if (d >= 0) {
+            const uint32_t s = L.site[r];
+            if (kHist) {
+                atomicAdd(&sben[s], (unsigned long long)L.dur[r]);
+                atomicAdd(&scnt[s], 1u);
+            } else {
+                atomicAdd((unsigned long long*)&ben[s], (unsigned long long)L.dur[r]);
+                atomicAdd((unsigned long long*)&cnt[s], 1ull);
+            }
+        }
+    }
+    if (kHist) {
+        __syncthreads();
+        for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) {
+            if (sben[s]) atomicAdd((unsigned long long*)&ben[s], sben[s]);
+            if (scnt[s]) atomicAdd((unsigned long long*)&cnt[s], (unsigned long long)scnt[s]);
+        }
+    }
+}
+
+#define ONLINE_CHECK()                                    \
+    do {                                                  \
+        if (cudaGetLastError() != cudaSuccess) return -1; \
+    } while (0)
+
+int launch_online_rehash(OnlineTable& T, uint32_t np, uint64_t digest_mask, cudaStream_t st) {
+    if (cudaMemsetAsync(T.key, 0xFF, (T.mask + 1) * sizeof(uint64_t), st) != cudaSuccess) return -1;
+    if (cudaMemsetAsync(T.head, 0xFF, (T.mask + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
+    if (!np) return 0;
+    k_online_rehash<<<blocks_for(np), 256, 0, st>>>(T, np, digest_mask);
+    ONLINE_CHECK();
+    return 1;
+}
+
+int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, const uint64_t* accB,
+                         OnlineTable& T, const Params& P, uint32_t n_sites, uint64_t* G, int64_t* dup_out,
+                         uint64_t* ben, uint64_t* cnt, cudaStream_t st) {
+    if (L.n == 0) return 0;
+    k_online_match<<<blocks_for(L.n), 256, 0, st>>>(
+        L, W.leader, accA, accB, T, P.digest_mask, P.refine_mask, G);
+    ONLINE_CHECK();
+    k_online_insert<<<blocks_for(L.n), 256, 0, st>>>(L, W.leader, accA, accB, G, T, P.digest_mask);
+    ONLINE_CHECK();
+    const size_t smem = label_smem_bytes(n_sites);
+    const uint32_t grid = std::min<uint32_t>(blocks_for(L.n, 1024), (uint32_t)P.num_sms);
+    if (smem <= (size_t)P.max_smem) {
+        if (!smem_configured((const void*)k_online_label<true>, P.max_smem)) return -1;
+        k_online_label<true><<<grid, 1024, smem, st>>>(L, W.leader, G, n_sites, dup_out, ben, cnt);
+    } else {
+        k_online_label<false><<<grid, 1024, 0, st>>>(L, W.leader, G, n_sites, dup_out, ben, cnt);
+    }
+    ONLINE_CHECK();
+    return 3;
+}
+
+}  // namespace ffm

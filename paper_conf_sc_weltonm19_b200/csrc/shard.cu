@@ -416,45 +416,4 @@ int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uin
     return 1;
 }
 
-// ---- online (streaming) mode helpers ---------------------------------------------
-// New classes of a window (G == own gid) are appended to the persistent list of prior
-// representatives, in gid order (flag -> scan -> scatter through a temporary).
-__global__ void k_online_flag(const RepTuple* __restrict__ Tw, uint32_t nloc, const uint64_t* __restrict__ G,
-                              uint32_t* __restrict__ flag) {
-    uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
-    if (j > nloc) return;
-    flag[j] = (j < nloc && G[j] == Tw[j].gid) ? 1u : 0u;
-}
-
-__global__ void k_online_scatter(const RepTuple* __restrict__ Tw, uint32_t nloc, const uint32_t* __restrict__ flag,
-                                 const uint32_t* __restrict__ pos, RepTuple* __restrict__ out) {
-    uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
-    if (j < nloc && flag[j]) out[pos[j]] = Tw[j];
-}
-
-__global__ void k_vec_add(uint64_t* __restrict__ a, const uint64_t* __restrict__ b, uint32_t n) {
-    uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i < n) a[i] += b[i];
-}
-
-int launch_online_newreps(Work& W, ShardWork& S, RepTuple* Tw, uint32_t nloc, RepTuple* tmp, cudaStream_t st) {
-    k_online_flag<<<blocks_for((uint64_t)nloc + 1), 256, 0, st>>>(Tw, nloc, S.G, S.vcount);
-    SHARD_CHECK();
-    size_t bytes = W.cub_tmp_bytes;
-    if (cub::DeviceScan::ExclusiveSum(W.cub_tmp, bytes, S.vcount, S.vstart, (int)(nloc + 1), st) != cudaSuccess)
-        return -1;
-    if (nloc) {
-        k_online_scatter<<<blocks_for(nloc), 256, 0, st>>>(Tw, nloc, S.vcount, S.vstart, tmp);
-        SHARD_CHECK();
-    }
-    return 3;
-}
-
-int launch_vec_add(uint64_t* a, const uint64_t* b, uint32_t n, cudaStream_t st) {
-    if (!n) return 0;
-    k_vec_add<<<blocks_for(n), 256, 0, st>>>(a, b, n);
-    SHARD_CHECK();
-    return 1;
-}
-
 }  // namespace ffm

@@ -40,12 +40,14 @@ def _online(ffm, lg, cuts, **kw):
 @pytest.mark.parametrize("k,ns,ss", [(1, 0.5, 0.25), (2, 0.01, 1.0), (3, 0.03, 1 / 32), (4, 0.1, 1 / 64),
                                      (5, 0.003, 1 / 32)])
 @pytest.mark.parametrize("digest_bits", [64, 0])
-def test_online_equals_batch_and_oracle(ffm, k, ns, ss, digest_bits):
+@pytest.mark.parametrize("online", [True, False])
+def test_online_equals_batch_and_oracle(ffm, k, ns, ss, digest_bits, online):
+    """online=True hashes at append time (FFM_FLAG_ONLINE); False hashes in the step."""
     lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
     rng = np.random.default_rng(k)
     cuts = sorted(set(rng.integers(1, lg.n, 6).tolist()))
     want_d, want_b = oracle.dedup(lg)
-    got_d, bens, bd, bb = _online(ffm, lg, cuts, digest_bits=digest_bits, chunk_bytes=4096)
+    got_d, bens, bd, bb = _online(ffm, lg, cuts, digest_bits=digest_bits, chunk_bytes=4096, online=online)
     np.testing.assert_array_equal(got_d, want_d)
     np.testing.assert_array_equal(bd, want_d)
     np.testing.assert_array_equal(bb, want_b)
@@ -73,3 +75,35 @@ def test_online_with_channels(ffm):
     np.testing.assert_array_equal(got_d, want_d)
     np.testing.assert_array_equal(bd, want_d)
     np.testing.assert_array_equal(bb, want_b)
+
+
+@pytest.mark.parametrize("window", [1, 64, 4096])
+def test_online_fixed_windows_grow_the_table(ffm, window):
+    """Fixed-size windows over a config-2-shaped log (many small transfers):
+    the persistent table grows (rehash on doubling) across steps; the result never changes."""
+    lg = loggen.gen_config(2, n_scale=0.004 if window == 1 else 0.02)
+    cuts = list(range(window, lg.n, window))
+    want_d, want_b = oracle.dedup(lg)
+    got_d, bens, bd, bb = _online(ffm, lg, cuts, online=True)
+    np.testing.assert_array_equal(got_d, want_d)
+    np.testing.assert_array_equal(bens[-1][1], want_b)
+    np.testing.assert_array_equal(bd, want_d)
+
+
+def test_online_after_reset_and_forced_collisions_across_windows(ffm):
+    """ffm_log_reset empties the stored classes too; with digest_bits = refine_bits = 0
+    every stored class of a size shares one chain (byte compares decide)."""
+    lg = loggen.gen_config(3, n_scale=0.02, size_scale=1 / 64)
+    want_d, want_b = oracle.dedup(lg)
+    ptrs = lg.payload_ptrs()
+    with ffm.FfmLog(lg.n_sites, digest_bits=0, refine_bits=0, online=True) as log:
+        for rep in range(2):
+            dups = []
+            for a in range(0, lg.n, 37):
+                b = min(lg.n, a + 37)
+                log.append_batch(lg.site[a:b], lg.size[a:b], ptrs[a:b], lg.dur[a:b])
+                d, ben = log.online_step()
+                dups.append(d.copy())
+            np.testing.assert_array_equal(np.concatenate(dups), want_d)
+            np.testing.assert_array_equal(ben, want_b)
+            log.reset()
