@@ -154,6 +154,43 @@ int pointer_kind(const void* p, int* dev) {
     return FFM_PAYLOAD_HOST;
 }
 
+// Kind / device of many payload pointers: one attribute query per allocation (the
+// driver's address range of a device or pinned allocation is cached), not per record.
+struct PtrCache {
+    uintptr_t lo = 0, hi = 0;
+    int kind = FFM_PAYLOAD_HOST, dev = -1;
+    int (*get_attr)(void*, int, uintptr_t) = nullptr;   // cuPointerGetAttribute
+    bool tried = false;
+
+    int classify(const void* p, int* dev_out) {
+        const uintptr_t a = (uintptr_t)p;
+        if (a >= lo && a < hi) {
+            *dev_out = dev;
+            return kind;
+        }
+        const int k = pointer_kind(p, dev_out);
+        if (k == FFM_PAYLOAD_HOST) return k;   // pageable: no range to cache
+        if (!tried) {
+            tried = true;
+            void* fn = nullptr;
+            if (cudaGetDriverEntryPoint("cuPointerGetAttribute", &fn, cudaEnableDefault, nullptr) == cudaSuccess)
+                get_attr = (int (*)(void*, int, uintptr_t))fn;
+            else
+                cudaGetLastError();
+        }
+        uintptr_t start = 0;
+        size_t size = 0;
+        if (get_attr && get_attr(&start, 11 /* RANGE_START_ADDR */, a) == 0 &&
+            get_attr(&size, 12 /* RANGE_SIZE */, a) == 0 && size) {
+            lo = start;
+            hi = start + size;
+            kind = k;
+            dev = *dev_out;
+        }
+        return k;
+    }
+};
+
 bool is_pinned_host(const void* p) {
     cudaPointerAttributes a;
     if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
@@ -358,12 +395,6 @@ void ensure_work(ffm_log* L, uint64_t n) {
         dev_alloc(W.dq, (uint64_t)kDiffK * c);
         dev_alloc(W.dv, (uint64_t)kDiffK * c);
         dev_alloc(W.sdesc, 2 * c);
-        dev_alloc(W.sflag, c);
-        dev_alloc(W.sitems, 2 * c);
-        if (W.part_tmp) cudaFree(W.part_tmp);
-        W.part_tmp = nullptr;
-        W.part_tmp_bytes = std::max<size_t>(small_partition_bytes(c), 256);
-        ck(cudaMalloc(&W.part_tmp, W.part_tmp_bytes), "cudaMalloc(partition)");
         dev_alloc(W.hcount, c + 1);
         dev_alloc(W.hstart, c + 1);
         dev_alloc(W.dup, c);
@@ -461,10 +492,19 @@ void run_prologue(ffm_log* L) {
     ensure_work(L, L->h_size.size());
 }
 
-// A window [a, b) of the log as a log of its own (indices relative to a), with its
-// record order in `order` (capacity ocap: the inverse follows at order + ocap).
-DevLog window_view(const ffm_log* L, uint64_t a, uint64_t b, const uint32_t* order, uint64_t ocap, uint64_t ns,
-                   uint64_t nl) {
+// An online window [a, b) of the log as a log of its own (indices relative to a) in the
+// identity record order: no host-side order build per window -- the small / large
+// kernels skip records of the other kind by size (two-pass round 0, hashing).
+DevLog window_view(ffm_log* L, uint64_t a, uint64_t b, cudaStream_t st) {
+    const uint64_t nw = b - a;
+    if (nw > L->iota_cap) {
+        if (L->d_iota) ck(cudaFree(L->d_iota), "cudaFree");
+        L->d_iota = nullptr;
+        const uint64_t c = std::max<uint64_t>(std::max<uint64_t>(nw, 2 * L->iota_cap), 4096);
+        ck(cudaMalloc(&L->d_iota, c * sizeof(uint32_t)), "cudaMalloc(iota)");
+        if (launch_iota(L->d_iota, (uint32_t)c, st) < 0) throw CudaFail{cudaGetLastError(), "iota"};
+        L->iota_cap = c;
+    }
     DevLog D = dev_view(L);
     D.off += a;
     D.size += a;
@@ -472,12 +512,12 @@ DevLog window_view(const ffm_log* L, uint64_t a, uint64_t b, const uint32_t* ord
     D.dur += a;
     D.gid += a;
     D.chan += a;
-    D.n = (uint32_t)(b - a);
-    D.small_order = order;
-    D.order_pos = order + ocap;
-    D.n_small = (uint32_t)ns;
-    D.large_order = order + ns;
-    D.n_large = (uint32_t)nl;
+    D.n = (uint32_t)nw;
+    D.small_order = L->d_iota;
+    D.order_pos = L->d_iota;
+    D.n_small = (uint32_t)nw;
+    D.large_order = L->d_iota;
+    D.n_large = (uint32_t)nw;
     return D;
 }
 
@@ -494,10 +534,7 @@ void online_hash(ffm_log* L, uint64_t a, uint64_t b, cudaStream_t st, uint64_t& 
         dev_grow(L->on_B, cap, need, a, st);
         L->on_cap = cap;
     }
-    std::vector<uint32_t> order;
-    const uint64_t ns = build_small_order(L, a, b, order);
-    upload_order(L, order, L->d_hash_order, L->d_hash_cap, st);
-    const DevLog D = window_view(L, a, b, L->d_hash_order, L->d_hash_cap, ns, order.size() - ns);
+    const DevLog D = window_view(L, a, b, st);
     Work W2 = L->work;
     W2.accA = L->on_A + a;
     W2.accB = L->on_B + a;
@@ -1130,14 +1167,15 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
         std::vector<uint64_t> desc;
         if (kind == FFM_PAYLOAD_DEVICE || kind == FFM_PAYLOAD_HOST_PINNED) desc.reserve(3 * n);
         bool need_sync = false, ordered = false;
+        PtrCache pc;
         for (uint64_t i = 0; i < n; ++i) {
             if (sizes[i] == 0) continue;
             int src = kind, pdev = L->device;
             if (kind == FFM_PAYLOAD_AUTO) {
-                src = pointer_kind(payloads[i], &pdev);
+                src = pc.classify(payloads[i], &pdev);
             } else if (kind == FFM_PAYLOAD_DEVICE) {
                 int d = -1;   // which GPU (a peer GPU's memory is never dereferenced by k_gather)
-                if (pointer_kind(payloads[i], &d) == FFM_PAYLOAD_DEVICE) pdev = d;
+                if (pc.classify(payloads[i], &d) == FFM_PAYLOAD_DEVICE) pdev = d;
             }
             const bool ring = src == FFM_PAYLOAD_HOST;        // pageable host: via the pinned ring
             if (src == FFM_PAYLOAD_DEVICE && !ordered) {
@@ -1375,10 +1413,7 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
             const uint64_t h0 = std::max(L->online_hashed, w0);
             if (h0 < n) online_hash(L, h0, n, s, launches);
             L->online_hashed = n;
-            std::vector<uint32_t> order;
-            const uint64_t nsw = build_small_order(L, w0, n, order);
-            upload_order(L, order, L->d_win_order, L->d_win_cap, s);
-            const DevLog D = window_view(L, w0, n, L->d_win_order, L->d_win_cap, nsw, order.size() - nsw);
+            const DevLog D = window_view(L, w0, n, s);
             uint64_t n_large = 0;
             for (uint64_t i = w0; i < n; ++i) n_large += large_chunks(L, L->h_size[i]);
             // H2..H4 on the window: exact window classes (the NH sums are the window's slice
@@ -1505,7 +1540,7 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->stage_stream) cudaStreamSynchronize(L->stage_stream);
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
-                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.fitems, W.sdesc, W.sflag, W.sitems, W.part_tmp, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
+                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.fitems, W.sdesc, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
                     W.dup, W.ben, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
                     L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)
@@ -1513,7 +1548,7 @@ int ffm_log_destroy(ffm_log* L) {
     free_shard(L->shard);
     if (L->fold_buf) cudaFree(L->fold_buf);
     void* op[] = {L->otab.key, L->otab.head, L->otab.pool, L->otab.count, L->on_A, L->on_B, L->on_G,
-                  L->online_ben, L->d_win_order, L->d_hash_order};
+                  L->online_ben, L->d_iota};
     for (void* p : op)
         if (p) cudaFree(p);
     for (void* p : L->peer_ptr)

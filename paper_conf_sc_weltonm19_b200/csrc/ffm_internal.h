@@ -52,10 +52,6 @@ struct Work {
     uint32_t* fhead = nullptr;     // [n] round 0: head (leader) of a large record's fused group
     uint2* hitems = nullptr;       // large-payload hash work units (record, chunk)
     uint4* sdesc = nullptr;        // [2 * n] fused round 0: compare descriptors of small records (order position)
-    uint8_t* sflag = nullptr;      // [n] 1: that small record is a member (compared), 0: hashed
-    uint4* sitems = nullptr;       // [2 * n] sdesc partitioned: members, then the others (reversed)
-    void* part_tmp = nullptr;      // cub partition scratch
-    size_t part_tmp_bytes = 0;
     uint4* fitems = nullptr;       // pipelined fused pass stage descriptors (2 x uint4 each)
     uint32_t* dcnt = nullptr;      // [n] fused round 0: words where a large member differs from its group head
     uint32_t* dq = nullptr;        // [n * kDiffK] their 16-B word indices (the first kDiffK recorded)
@@ -173,12 +169,12 @@ int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uin
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t st);
+int launch_iota(uint32_t* a, uint32_t n, cudaStream_t st);
 int launch_spec_label(const DevLog& L, Work& W, int64_t* dup_out, cudaStream_t st);
 int launch_digest_fill(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_hash_small_list(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
                            cudaStream_t st);
 size_t cub_scan_bytes(uint64_t n);
-size_t small_partition_bytes(uint64_t n);
 uint64_t fx_entry_cap(uint64_t n_large_chunks, uint32_t chunk_bytes);
 uint32_t blocks_for(uint64_t threads, uint32_t bs = 256);
 uint32_t resident_grid(const void* kernel, int num_sms, int block = 256);
@@ -284,10 +280,8 @@ struct ffm_log {
     uint64_t on_G_cap = 0;
     uint64_t* online_ben = nullptr;  // [2 * n_sites] cumulative per-site benefit | duplicate counts
     uint64_t* online_cnt = nullptr;  //   (= online_ben + n_sites)
-    uint32_t* d_win_order = nullptr; // the step's window order
-    uint64_t d_win_cap = 0;
-    uint32_t* d_hash_order = nullptr;   // the append-time hashing's window order
-    uint64_t d_hash_cap = 0;
+    uint32_t* d_iota = nullptr;      // identity record order of online windows (0, 1, 2, ...)
+    uint64_t iota_cap = 0;
 
     // folded grouping scratch
     void* fold_buf = nullptr;

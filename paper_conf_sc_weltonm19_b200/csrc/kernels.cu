@@ -465,7 +465,6 @@ __global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, ui
             const uint64_t off = L.off[r], loff = (ld != r && same) ? L.off[ld] : ~0ull;
             W.sdesc[2ull * i] = make_uint4((uint32_t)off, (uint32_t)(off >> 32), (uint32_t)loff, (uint32_t)(loff >> 32));
             W.sdesc[2ull * i + 1] = make_uint4((uint32_t)sz, r, 0, 0);
-            W.sflag[i] = (ld != r && same) ? 1 : 0;   // compared (member) or hashed
         }
     }
     unsigned b = __ballot_sync(0xFFFFFFFFu, member);
@@ -1029,7 +1028,8 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
 __global__ void __launch_bounds__(256) k_hash_combine(DevLog L, Work W, uint32_t chunk_bytes, uint32_t prefix_bytes,
                                                       int prefilter, int fx) {
     unsigned long long rest = 0;
-    FFM_WARP_EACH(L.n_large, L.large_order[w_], true, {
+    // (an identity order -- online windows -- lists small records too: no chunk slots)
+    FFM_WARP_EACH(L.n_large, L.large_order[w_], (W.hstart[rec + 1] != W.hstart[rec]), {
         const uint32_t s0 = W.hstart[rec];
         const bool skip = fx && prefilter && prefix_unique(W, rec);
         const uint32_t e0 = skip ? s0 : W.hstart[rec + 1];
@@ -1153,9 +1153,6 @@ __global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const
 // Lane g takes words g, g+8 of each 256-byte stripe (one warp instruction = 128
 // contiguous bytes per octet); NH is a positional sum, so the digest is unchanged.
 // Each lane reads back only what it copied itself: cp.async.wait_group is the only ordering.
-#ifndef FFM_SMALL_SPLIT
-#define FFM_SMALL_SPLIT 1   // 1: role-split pass (k_small_role), 0: mixed octet kernel (k_fused_small)
-#endif
 #ifndef FFM_SA_U
 #define FFM_SA_U 2
 #endif
@@ -1273,7 +1270,7 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
 
     // ---- consumer state
     LaneKeys K;   // k[0]: stripe position g, k[1]: position g + 8
-    uint64_t A = 0, B = 0, found = ~0ull;
+    uint64_t A = 0, B = 0, A2 = 0, B2 = 0, found = ~0ull;
     int sc = 0, sf = kSaS - 1;
 #pragma unroll 1
     while (true) {
@@ -1286,8 +1283,7 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
         const uint32_t n = m[0], r = m[1], z = m[2];
         if (z & kSaEnd) break;
         if (z & kSaFirst) {
-            A = 0;
-            B = 0;
+            A = B = A2 = B2 = 0;
             found = ~0ull;
 #pragma unroll
             for (int jj = 0; jj < 6; ++jj) {
@@ -1350,13 +1346,14 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
                 if (g == 0 && found != ~0ull) report_mismatch(W, r, found, res_out, false);
             }
         } else {
-            // leader / singleton: hash
+            // leader / singleton: hash (two accumulator chains: even / odd words)
             if (full) {
 #pragma unroll
                 for (int j = 0; j < kSaJ; ++j) {
                     uint32_t x[4];
                     lds16(slot(sc, j, 0), x);
-                    nh_word(x[0], x[1], x[2], x[3], K.k[j & 1], A, B);
+                    if (j & 1) nh_word(x[0], x[1], x[2], x[3], K.k[1], A2, B2);
+                    else nh_word(x[0], x[1], x[2], x[3], K.k[0], A, B);
                     if (j & 1) advance<1>(K);
                 }
             } else {
@@ -1367,12 +1364,15 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
                         uint32_t x[4];
                         lds16(slot(sc, j, 0), x);
                         mask_word(x, n, w);
-                        nh_word(x[0], x[1], x[2], x[3], K.k[j & 1], A, B);
+                        if (j & 1) nh_word(x[0], x[1], x[2], x[3], K.k[1], A2, B2);
+                        else nh_word(x[0], x[1], x[2], x[3], K.k[0], A, B);
                     }
                     if (j & 1) advance<1>(K);
                 }
             }
             if (z & kSaLast) {
+                A += A2;
+                B += B2;
 #pragma unroll
                 for (int o = 4; o; o >>= 1) {
                     A += __shfl_xor_sync(omask, A, o);
@@ -1387,225 +1387,6 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
         }
         sc = sc + 1 == kSaS ? 0 : sc + 1;
         sf = sf + 1 == kSaS ? 0 : sf + 1;
-    }
-    asm volatile("cp.async.wait_group 0;" ::: "memory");
-}
-
-// ----------------------------------------------------------------------------
-// The small-payload pass split by role (default).  After the round-0 group-by the small
-// records' descriptors are partitioned (stable, cub) into members -- compared with their
-// group leader, never hashed (an equal member has its leader's digest) -- and records
-// that lead their group -- hashed, nothing to compare.  One specialised kernel per part:
-// no per-octet role divergence inside a warp (the mixed kernel ran both paths in every
-// warp holding both roles), no leader staging in the hashing kernel, and each kernel's
-// shared-memory ring sized for its own role (higher occupancy).  Same per-lane cp.async
-// pipeline as k_fused_small: lane g of an octet takes words g, g+8 of each 256-byte
-// stripe; S - 1 steps stay in flight while the oldest is consumed.
-// ----------------------------------------------------------------------------
-struct SDesc {
-    uint4 a, b;   // a = (off lo, off hi, leader off lo, hi); b = (size, record, 0, 0)
-};
-
-#ifndef FFM_SPC_J
-#define FFM_SPC_J 2    // compare kernel: 16-B words per lane per step (own + leader staged)
-#endif
-#ifndef FFM_SPH_J
-#define FFM_SPH_J 4    // hash kernel: 16-B words per lane per step
-#endif
-#ifndef FFM_SP_S
-#define FFM_SP_S 2     // stages
-#endif
-#ifndef FFM_SP_T
-#define FFM_SP_T 128
-#endif
-constexpr int kSpS = FFM_SP_S, kSpT = FFM_SP_T;
-template <bool kCmp>
-__host__ __device__ constexpr int sp_j() {
-    return kCmp ? FFM_SPC_J : FFM_SPH_J;
-}
-template <bool kCmp>
-__host__ __device__ constexpr int sp_smem() {
-    return kSpS * kSpT * 16 * ((kCmp ? 2 : 1) * sp_j<kCmp>() + 1);
-}
-
-template <bool kCmp>
-__global__ void __launch_bounds__(kSpT) k_small_role(DevLog L, Work W, const SDesc* __restrict__ items,
-                                                     const uint32_t* __restrict__ nsel_ptr, uint32_t* res_out) {
-    constexpr int kSpJ = sp_j<kCmp>();
-    extern __shared__ __align__(16) uint8_t sp_smem_buf[];
-    constexpr int P = kCmp ? 2 : 1;   // staged parts per word: own (+ leader)
-    const int g = threadIdx.x & 7;
-    const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
-    const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
-    const unsigned omask = 0xFFu << (threadIdx.x & 24);
-    // members: items [0, nsel); leaders: [nsel, n_small) (cub places them reversed: ascending
-    // size -- neighbouring octets still get near-equal lengths)
-    const uint32_t nsel = *nsel_ptr;
-    const uint32_t lo = kCmp ? 0u : nsel, hi = kCmp ? nsel : L.n_small;
-    const uint32_t sbase = smem_u32(sp_smem_buf) + threadIdx.x * 16;
-    auto slot = [&](int s, int j, int part) { return sbase + (uint32_t)(((s * kSpJ + j) * P + part) * kSpT * 16); };
-    auto mslot = [&](int s) { return sbase + (uint32_t)((kSpS * kSpJ * P + s) * kSpT * 16); };
-    uint64_t pol_own, pol_keep;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_own));
-    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
-
-    // ---- producer: current record (item fi, next word fw0) + the next item's descriptor
-    uint32_t fi = lo + oct, fw0 = 0;
-    uint64_t foff = 0, floff = 0;
-    uint32_t fn = 0, fr = 0;
-    uint4 da = make_uint4(0, 0, 0, 0), db = make_uint4(0, 0, 0, 0);
-    if (fi < hi) {
-        const SDesc d = items[fi];
-        foff = (uint64_t)d.a.y << 32 | d.a.x;
-        floff = (uint64_t)d.a.w << 32 | d.a.z;
-        fn = d.b.x;
-        fr = d.b.y;
-        if (fi + noct < hi) {
-            da = items[fi + noct].a;
-            db = items[fi + noct].b;
-        }
-    }
-    auto fetch = [&](int s) {
-        uint32_t meta_z = kSaEnd;
-        uint32_t mn = 0, mr = 0;
-        if (fi < hi) {
-            const uint32_t nw = (fn + 15) >> 4;
-            const uint8_t* src = L.arena + foff + 16ull * (fw0 + g);
-            const uint8_t* lsrc = L.arena + floff + 16ull * (fw0 + g);
-            if (fw0 + 8 * kSpJ <= nw) {   // every lane's words exist
-#pragma unroll
-                for (int j = 0; j < kSpJ; ++j) {
-                    cp16(slot(s, j, 0), src + 128 * j, pol_own);
-                    if (kCmp) cp16(slot(s, j, 1), lsrc + 128 * j, pol_keep);
-                }
-            } else {
-#pragma unroll
-                for (int j = 0; j < kSpJ; ++j) {
-                    if (fw0 + 8 * j + g < nw) {
-                        cp16(slot(s, j, 0), src + 128 * j, pol_own);
-                        if (kCmp) cp16(slot(s, j, 1), lsrc + 128 * j, pol_keep);
-                    }
-                }
-            }
-            meta_z = fw0 | (fw0 == 0 ? kSaFirst : 0u);
-            mn = fn;
-            mr = fr;
-            fw0 += 8 * kSpJ;
-            if (fw0 >= nw) {   // last step of this record: move to the next one
-                meta_z |= kSaLast;
-                fi += noct;
-                fw0 = 0;
-                foff = (uint64_t)da.y << 32 | da.x;
-                floff = (uint64_t)da.w << 32 | da.z;
-                fn = db.x;
-                fr = db.y;
-                if (fi + noct < hi) {
-                    da = items[fi + noct].a;
-                    db = items[fi + noct].b;
-                }
-            }
-        }
-        asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(mslot(s)), "r"(mn), "r"(mr), "r"(meta_z), "r"(0u)
-                     : "memory");
-        asm volatile("cp.async.commit_group;" ::: "memory");
-    };
-#pragma unroll 1
-    for (int s = 0; s < kSpS - 1; ++s) fetch(s);
-
-    LaneKeys K;                      // (hashing) k[0]: position g, k[1]: position g + 8
-    uint64_t A0 = 0, A1 = 0, B0 = 0, B1 = 0;   // two chains each: even / odd words
-    uint64_t found = ~0ull;          // (compare) lowest differing word
-    int sc = 0, sf = kSpS - 1;
-#pragma unroll 1
-    while (true) {
-        fetch(sf);
-        asm volatile("cp.async.wait_group %0;" ::"n"(kSpS - 1) : "memory");
-        uint32_t m[4];
-        lds16(mslot(sc), m);
-        const uint32_t n = m[0], r = m[1], z = m[2];
-        if (z & kSaEnd) break;
-        const uint32_t w0 = z & 0x0FFFFFFFu, nw = (n + 15) >> 4;
-        const bool full = 16 * (w0 + 8 * kSpJ) <= n;
-        if (kCmp) {
-            if (z & kSaFirst) found = ~0ull;
-            if (found == ~0ull) {
-                uint32_t d = 0;
-#pragma unroll
-                for (int j = 0; j < kSpJ; ++j) {
-                    const uint32_t w = w0 + 8 * j + g;
-                    if (full || w < nw) {
-                        uint32_t x[4], y[4];
-                        lds16(slot(sc, j, 0), x);
-                        lds16(slot(sc, j, 1), y);
-                        if (!full) {
-                            mask_word(x, n, w);
-                            mask_word(y, n, w);
-                        }
-                        d |= (x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3]);
-                    }
-                }
-                if (d) {   // rare: the lowest differing word of this step
-#pragma unroll 1
-                    for (int j = 0; j < kSpJ; ++j) {
-                        const uint32_t w = w0 + 8 * j + g;
-                        if (w >= nw) break;
-                        uint32_t x[4], y[4];
-                        lds16(slot(sc, j, 0), x);
-                        lds16(slot(sc, j, 1), y);
-                        mask_word(x, n, w);
-                        mask_word(y, n, w);
-                        if ((x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3])) {
-                            found = w;
-                            break;
-                        }
-                    }
-                }
-            }
-            if (z & kSaLast) {
-#pragma unroll
-                for (int o = 4; o; o >>= 1) {
-                    const uint64_t of = __shfl_xor_sync(omask, found, o);
-                    found = of < found ? of : found;
-                }
-                if (g == 0 && found != ~0ull) report_mismatch(W, r, found, res_out, false);
-            }
-        } else {
-            if (z & kSaFirst) {
-                A0 = A1 = B0 = B1 = 0;
-#pragma unroll
-                for (int jj = 0; jj < 6; ++jj) {
-                    K.k[0][jj] = c_nh.ka[g][jj];
-                    K.k[1][jj] = c_nh.ka[g + 8][jj];
-                }
-            }
-#pragma unroll
-            for (int j = 0; j < kSpJ; ++j) {
-                const uint32_t w = w0 + 8 * j + g;
-                if (full || w < nw) {
-                    uint32_t x[4];
-                    lds16(slot(sc, j, 0), x);
-                    if (!full) mask_word(x, n, w);
-                    if (j & 1) nh_word(x[0], x[1], x[2], x[3], K.k[1], A1, B1);
-                    else nh_word(x[0], x[1], x[2], x[3], K.k[0], A0, B0);
-                }
-                if (j & 1) advance<1>(K);
-            }
-            if (z & kSaLast) {
-                uint64_t A = A0 + A1, B = B0 + B1;
-#pragma unroll
-                for (int o = 4; o; o >>= 1) {
-                    A += __shfl_xor_sync(omask, A, o);
-                    B += __shfl_xor_sync(omask, B, o);
-                }
-                if (g == 0) {
-                    W.accA[r] = A;
-                    W.accB[r] = B;
-                    W.digest[r] = finalize_digest(A, B, n);
-                }
-            }
-        }
-        sc = sc + 1 == kSpS ? 0 : sc + 1;
-        sf = sf + 1 == kSpS ? 0 : sf + 1;
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
 }
@@ -1851,45 +1632,9 @@ int launch_hash_small(const DevLog& L, Work& W, const Params& P, cudaStream_t st
     return 1;
 }
 
-size_t small_partition_bytes(uint64_t n) {
-    size_t bytes = 0;
-    cub::DevicePartition::Flagged(nullptr, bytes, (const SDesc*)nullptr, (const uint8_t*)nullptr, (SDesc*)nullptr,
-                                  (uint32_t*)nullptr, (int)n);
-    return bytes;
-}
-
 int launch_fused_small(const DevLog& L, Work& W, const Params& P, uint32_t* res_out, cudaStream_t st) {
     if (L.n == 0 || L.n_small == 0) return 0;
-#if FFM_SMALL_SPLIT
-    {
-        // members | leaders (stable partition of the size-class-ordered descriptors)
-        size_t bytes = W.part_tmp_bytes;
-        if (cub::DevicePartition::Flagged(W.part_tmp, bytes, reinterpret_cast<const SDesc*>(W.sdesc), W.sflag,
-                                          reinterpret_cast<SDesc*>(W.sitems), W.counters + 12, (int)L.n_small,
-                                          st) != cudaSuccess)
-            return -1;
-        static int occ[2] = {0, 0};   // per process: one device type
-        const void* kern[2] = {(const void*)k_small_role<true>, (const void*)k_small_role<false>};
-        const int smem[2] = {sp_smem<true>(), sp_smem<false>()};
-        for (int k = 0; k < 2; ++k) {
-            if (!smem_configured(kern[k], smem[k])) return -1;
-            if (occ[k] == 0 &&
-                (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ[k], kern[k], kSpT, smem[k]) != cudaSuccess ||
-                 occ[k] < 1))
-                occ[k] = 1;
-        }
-        const uint32_t need = blocks_for((uint64_t)L.n_small * 8, kSpT);
-        const uint32_t g0 = std::min<uint32_t>(need, (uint32_t)(occ[0] * P.num_sms));
-        const uint32_t g1 = std::min<uint32_t>(need, (uint32_t)(occ[1] * P.num_sms));
-        k_small_role<true><<<g0, kSpT, smem[0], st>>>(L, W, reinterpret_cast<const SDesc*>(W.sitems), W.counters + 12,
-                                                      res_out);
-        FFM_LAUNCH_CHECK();
-        k_small_role<false><<<g1, kSpT, smem[1], st>>>(L, W, reinterpret_cast<const SDesc*>(W.sitems),
-                                                       W.counters + 12, res_out);
-        FFM_LAUNCH_CHECK();
-        return 3;
-    }
-#endif
+
     // (measured: capping its grid so that it co-resides with the persistent large pass
     // slowed that pass more than it hid -- profiles/r01b/README.md)
     if (!smem_configured((const void*)k_fused_small, kSaSmem)) return -1;
@@ -2148,6 +1893,18 @@ int launch_hash_small_list(const DevLog& L, Work& W, const Params& P, const uint
     D.small_order = list;
     D.n_small = n_list;
     return launch_hash_small(D, W, P, st);
+}
+
+__global__ void k_iota(uint32_t* __restrict__ a, uint32_t n) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) a[i] = i;
+}
+
+int launch_iota(uint32_t* a, uint32_t n, cudaStream_t st) {
+    if (n == 0) return 0;
+    k_iota<<<blocks_for(n), 256, 0, st>>>(a, n);
+    FFM_LAUNCH_CHECK();
+    return 1;
 }
 
 __global__ void k_invert(const uint32_t* __restrict__ order, uint32_t n, uint32_t* __restrict__ inv) {

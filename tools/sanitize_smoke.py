@@ -1,6 +1,7 @@
 """Small logs through every kernel (fused and two-pass round 0 incl. the TMA-pipelined k_fused_fx in
 hash and verify mode with pieces split from 64 KiB chunks and groups of > 64 members, pre-filter,
-collision resolve, online windows, device-payload gather), for compute-sanitizer memcheck /
+collision resolve, online windows, the collective sharded merge, device-payload gather), for
+compute-sanitizer memcheck /
 racecheck / synccheck."""
 import os
 import sys
@@ -12,6 +13,23 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import loggen  # noqa: E402
 import oracle  # noqa: E402
 import paper_conf_sc_weltonm19_b200 as ffm  # noqa: E402
+
+class LonelyWorld:
+    """ffm_comm_ops of a world of 2 whose rank 1 has no records (peer blocks are zeros)."""
+
+    def __init__(self):
+        import ctypes
+        self._ag = ffm.ALLGATHER_FN(self._allgather)
+        self._ar = ffm.ALLREDUCE_FN(lambda ctx, buf, n: 0)
+        self.ops = ffm.FfmCommOps(None, self._ag, self._ar)
+        self._ct = ctypes
+
+    def _allgather(self, ctx, send, recv, nbytes):
+        if nbytes:
+            self._ct.memmove(recv, send, nbytes)
+            self._ct.memset(recv + nbytes, 0, nbytes)
+        return 0
+
 
 for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (3, 0.012, 1 / 128), (4, 0.04, 1 / 512), (2, 0.001, 1.0)]:
     lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
@@ -30,12 +48,21 @@ for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (3, 0.012, 1 / 128), (
                 log.append_log(lg)
             d, b = log.run()
             assert np.array_equal(d, want[0]) and np.array_equal(b, want[1]), (k, db, rb, extra)
-    # online windows
-    with ffm.FfmLog(lg.n_sites, digest_bits=8, chunk_bytes=4096) as log:
-        ptrs = lg.payload_ptrs()
-        got = []
-        for a, e in ((0, lg.n // 3), (lg.n // 3, lg.n)):
-            log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e])
-            got.append(log.online_step()[0].copy())
-        assert np.array_equal(np.concatenate(got), want[0]), ("online", k)
+    # online windows (append-time hashing and in-step hashing)
+    for online in (True, False):
+        with ffm.FfmLog(lg.n_sites, digest_bits=8, chunk_bytes=4096, online=online) as log:
+            ptrs = lg.payload_ptrs()
+            got = []
+            for a, e in ((0, lg.n // 3), (lg.n // 3, lg.n)):
+                log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e])
+                got.append(log.online_step()[0].copy())
+            assert np.array_equal(np.concatenate(got), want[0]), ("online", k)
+    # the collective sharded run in one process: a world of 2 whose other rank is empty
+    # (header, export, all-gather, merge incl. the same-key segment scan, all-reduce)
+    for db in (64, 0):
+        w = LonelyWorld()
+        with ffm.FfmLog(lg.n_sites, rank=0, world=2, comm=w.ops, digest_bits=db, chunk_bytes=4096) as log:
+            log.append_log(lg, gids=np.arange(lg.n))
+            d, b = log.run()
+            assert np.array_equal(d, want[0]) and np.array_equal(b, want[1]), ("sharded", k, db)
 print("sanitize smoke ok")
