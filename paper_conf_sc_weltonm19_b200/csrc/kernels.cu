@@ -509,6 +509,9 @@ __device__ __forceinline__ bool prefix_unique(const Work& W, uint32_t r) {
 #ifndef FFM_FX_STAGES
 #define FFM_FX_STAGES 3
 #endif
+#ifndef FFM_FX_PROXY_FENCE
+#define FFM_FX_PROXY_FENCE 0
+#endif
 #ifndef FFM_FX_CTAS
 #define FFM_FX_CTAS 2
 #endif
@@ -581,6 +584,14 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
         "l"(src), "r"(bytes), "r"(bar), "l"(pol)
         : "memory");
 }
+
+// A consumer releases a stage with one arrive per LANE on the stage's empty barrier, after
+// that lane's own last read of it: each read is ordered before the producer's next bulk
+// write by the reading thread's own release (compute-sanitizer racecheck follows this
+// chain; it does not follow __syncwarp + one arrive per warp, which it flagged as 4.9 M
+// hazards in round 1 -- profiles/sanitizer/README.md).  Measured no slower (r02i).
+constexpr uint32_t kFxEmptyArrivals = 32u * kFxConsumers;
+__device__ __forceinline__ void fx_release(uint32_t bar) { mbar_arrive(bar); }
 
 // keep the first `valid` bytes of a 16-B word, zero the rest
 __device__ __forceinline__ void mask_word(uint4& w, int32_t valid) {
@@ -743,7 +754,7 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
     if (threadIdx.x == 0) {
         for (int s = 0; s < kFxStages; ++s) {
             mbar_init(smem_u32(&full[s]), 1);
-            mbar_init(smem_u32(&empty[s]), kFxConsumers);
+            mbar_init(smem_u32(&empty[s]), kFxEmptyArrivals);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -822,6 +833,11 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
                     if (vmode && __shfl_sync(0xFFFFFFFFu, cm, j) < (uint64_t)w0) continue;
                     if (lane == 0) {
                         mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+#if FFM_FX_PROXY_FENCE
+                        // the consumers' generic-proxy reads of this stage (released through the
+                        // empty barrier) before the async-proxy write of the next bulk copy
+                        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+#endif
                         FxDesc& m = meta[stage];
                         m.rec = rec;
                         m.lenf = lenf;
@@ -891,8 +907,7 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
                 const int32_t vb = len - 16 * (int32_t)(t + kStride * u);
                 x[u] = vb > 0 ? *reinterpret_cast<const uint4*>(buf + 16 * (t + kStride * u)) : make_uint4(0, 0, 0, 0);
             }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(smem_u32(&empty[stage]));
+            fx_release(smem_u32(&empty[stage]));
 #pragma unroll
             for (int u = 0; u < kFxWords; ++u) mask_word(x[u], len - 16 * (int32_t)(t + kStride * u));
             if (flags & kFxHash) {
@@ -914,8 +929,7 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
                 const int32_t vb = len - 16 * (int32_t)(t + kStride * u);
                 y[u] = vb > 0 ? *reinterpret_cast<const uint4*>(buf + 16 * (t + kStride * u)) : make_uint4(0, 0, 0, 0);
             }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(smem_u32(&empty[stage]));
+            fx_release(smem_u32(&empty[stage]));
             uint32_t dmask = 0;
 #pragma unroll
             for (int u = 0; u < kFxWords; ++u) {
