@@ -495,7 +495,7 @@ void run_prologue(ffm_log* L) {
 // An online window [a, b) of the log as a log of its own (indices relative to a) in the
 // identity record order: no host-side order build per window -- the small / large
 // kernels skip records of the other kind by size (two-pass round 0, hashing).
-DevLog window_view(ffm_log* L, uint64_t a, uint64_t b, cudaStream_t st) {
+DevLog window_view(ffm_log* L, uint64_t a, uint64_t b, bool has_large, cudaStream_t st) {
     const uint64_t nw = b - a;
     if (nw > L->iota_cap) {
         if (L->d_iota) ck(cudaFree(L->d_iota), "cudaFree");
@@ -517,7 +517,7 @@ DevLog window_view(ffm_log* L, uint64_t a, uint64_t b, cudaStream_t st) {
     D.order_pos = L->d_iota;
     D.n_small = (uint32_t)nw;
     D.large_order = L->d_iota;
-    D.n_large = (uint32_t)nw;
+    D.n_large = has_large ? (uint32_t)nw : 0u;   // (no large-record kernels for a window without any)
     return D;
 }
 
@@ -534,12 +534,12 @@ void online_hash(ffm_log* L, uint64_t a, uint64_t b, cudaStream_t st, uint64_t& 
         dev_grow(L->on_B, cap, need, a, st);
         L->on_cap = cap;
     }
-    const DevLog D = window_view(L, a, b, st);
+    uint64_t n_large = 0;
+    for (uint64_t i = a; i < b; ++i) n_large += large_chunks(L, L->h_size[i]);
+    const DevLog D = window_view(L, a, b, n_large != 0, st);
     Work W2 = L->work;
     W2.accA = L->on_A + a;
     W2.accB = L->on_B + a;
-    uint64_t n_large = 0;
-    for (uint64_t i = a; i < b; ++i) n_large += large_chunks(L, L->h_size[i]);
     LCHK(launch_hash_small(D, W2, L->params, st));
     if (n_large) {
         LCHK(launch_hash_plan(D, W2, L->params, true, st));
@@ -1413,9 +1413,9 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
             const uint64_t h0 = std::max(L->online_hashed, w0);
             if (h0 < n) online_hash(L, h0, n, s, launches);
             L->online_hashed = n;
-            const DevLog D = window_view(L, w0, n, s);
             uint64_t n_large = 0;
             for (uint64_t i = w0; i < n; ++i) n_large += large_chunks(L, L->h_size[i]);
+            const DevLog D = window_view(L, w0, n, n_large != 0, s);
             // H2..H4 on the window: exact window classes (the NH sums are the window's slice
             // of on_A / on_B)
             {

@@ -509,9 +509,6 @@ __device__ __forceinline__ bool prefix_unique(const Work& W, uint32_t r) {
 #ifndef FFM_FX_STAGES
 #define FFM_FX_STAGES 3
 #endif
-#ifndef FFM_FX_PROXY_FENCE
-#define FFM_FX_PROXY_FENCE 0
-#endif
 #ifndef FFM_FX_CTAS
 #define FFM_FX_CTAS 2
 #endif
@@ -833,11 +830,6 @@ __global__ void __launch_bounds__(kFxThreads, FFM_FX_MINB) k_fused_fx(DevLog L, 
                     if (vmode && __shfl_sync(0xFFFFFFFFu, cm, j) < (uint64_t)w0) continue;
                     if (lane == 0) {
                         mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
-#if FFM_FX_PROXY_FENCE
-                        // the consumers' generic-proxy reads of this stage (released through the
-                        // empty barrier) before the async-proxy write of the next bulk copy
-                        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-#endif
                         FxDesc& m = meta[stage];
                         m.rec = rec;
                         m.lenf = lenf;

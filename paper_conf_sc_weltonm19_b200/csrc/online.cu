@@ -12,9 +12,9 @@
 //   3. k_online_match: each window class representative looks its key up in the table
 //      and byte-compares the chained prior representatives of its size / channel /
 //      digest (their bytes stay resident in the HBM arena) -- at most one prior class
-//      can be equal, so the chain order does not matter;
-//   4. k_online_insert: classes with no equal prior class join the table;
-//   5. k_online_label: labels (gids) and the cumulative per-site benefit / counts.
+//      can be equal, so the chain order does not matter; a class with no equal stored
+//      class is inserted by the same kernel;
+//   4. k_online_label: labels (gids) and the cumulative per-site benefit / counts.
 // The table is never rebuilt by a step; it is rehashed only when its capacity doubles.
 #include "digest.cuh"
 #include "ffm_internal.h"
@@ -44,29 +44,40 @@ __device__ __forceinline__ void online_link(OnlineTable& T, uint64_t key, uint32
     T.pool[idx].next = atomicExch(&T.head[h], idx);
 }
 
-// One warp per window class representative r (leader[r] == r).
+// One 8-lane group per window class representative r (leader[r] == r), grid-stride:
+// look its key up, byte-compare the chained stored classes of its size / channel /
+// digest (32-byte blocks per lane, stopping at the first differing step); with no equal
+// stored class, r's class is stored right away.  Concurrent inserts are safe: a window's
+// classes are pairwise distinct, so a walker that misses (or meets) a class being
+// inserted by another window representative loses nothing, and an entry is complete
+// before the CAS that publishes it.
 __global__ void __launch_bounds__(256) k_online_match(DevLog L, const uint32_t* __restrict__ leader,
                                                       const uint64_t* __restrict__ accA,
                                                       const uint64_t* __restrict__ accB, OnlineTable T,
                                                       uint64_t digest_mask, uint64_t refine_mask,
                                                       uint64_t* __restrict__ G) {
-    const uint32_t* nolist = nullptr;
-    FFM_WARP_COMPACT(L.n, nolist, (leader[r_] == r_), {
-        const uint64_t n = L.size[rec], chan = L.chan[rec];
-        const uint64_t dig = finalize_digest(accA[rec], accB[rec], n);
+    const int g = threadIdx.x & 7;
+    const unsigned omask = 0xFFu << (threadIdx.x & 24);
+    const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
+    for (uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 3; r < L.n; r += noct) {
+        if (leader[r] != r) continue;   // (uniform per octet)
+        const uint64_t n = L.size[r], chan = L.chan[r];
+        const uint64_t dig = finalize_digest(accA[r], accB[r], n);
         const uint64_t key = group_key(dig, n, digest_mask, chan);
         const uint64_t h = online_probe(T, key);
-        uint32_t idx = T.key[h] == key ? T.head[h] : kNoRep;
-        uint64_t g = L.gid[rec];
-        const uint8_t* px = L.arena + L.off[rec];
+        uint32_t idx = kNoRep;
+        if (T.key[h] == key) idx = *reinterpret_cast<volatile uint32_t*>(&T.head[h]);
+        uint64_t gl = L.gid[r];
+        bool found = false;
+        const uint8_t* px = L.arena + L.off[r];
         const uint64_t nblk = (n + 31) >> 5;
         while (idx != kNoRep) {
             const OnlineRep e = T.pool[idx];
             if (e.size == n && e.chan == chan && ((e.dig ^ dig) & refine_mask) == 0) {
                 const uint8_t* py = L.arena + e.off;
                 bool diff = false;
-                for (uint64_t b0 = 0; b0 < nblk && !diff; b0 += 32) {
-                    const uint64_t b = b0 + lane;
+                for (uint64_t b0 = 0; b0 < nblk && !diff; b0 += 8) {
+                    const uint64_t b = b0 + g;
                     bool d = false;
                     if (b < nblk) {
                         Blk a = ld_stream(px + 32 * b);
@@ -75,38 +86,46 @@ __global__ void __launch_bounds__(256) k_online_match(DevLog L, const uint32_t* 
                         mask_tail(y, n, b);
                         d = !blk_equal(a, y);
                     }
-                    diff = __any_sync(0xFFFFFFFFu, d);
+                    diff = __ballot_sync(omask, d) != 0;
                 }
-                if (!diff) {   // the (only) equal prior class
-                    g = e.gid;
+                if (!diff) {   // the (only) equal stored class
+                    gl = e.gid;
+                    found = true;
                     break;
                 }
             }
             idx = e.next;
         }
-        if (lane == 0) G[rec] = g;
-    })
-}
-
-// Window classes without an equal prior class become stored representatives.
-__global__ void k_online_insert(DevLog L, const uint32_t* __restrict__ leader, const uint64_t* __restrict__ accA,
-                                const uint64_t* __restrict__ accB, const uint64_t* __restrict__ G, OnlineTable T,
-                                uint64_t digest_mask) {
-    const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-    if (r >= L.n || leader[r] != r || G[r] != L.gid[r]) return;
-    const uint64_t n = L.size[r];
-    const uint64_t dig = finalize_digest(accA[r], accB[r], n);
-    const uint32_t idx = atomicAdd(T.count, 1u);
-    OnlineRep e;
-    e.gid = L.gid[r];
-    e.off = L.off[r];
-    e.size = n;
-    e.chan = L.chan[r];
-    e.dig = dig;
-    e.next = kNoRep;
-    e.pad = 0;
-    T.pool[idx] = e;
-    online_link(T, group_key(dig, n, digest_mask, e.chan), idx);
+        if (g == 0) {
+            G[r] = gl;
+            if (!found) {   // a new class: stored now
+                const uint32_t ni = atomicAdd(T.count, 1u);
+                OnlineRep e;
+                e.gid = gl;
+                e.off = L.off[r];
+                e.size = n;
+                e.chan = chan;
+                e.dig = dig;
+                e.pad = 0;
+                uint64_t hh = key & T.mask;
+                while (true) {
+                    unsigned long long prev = atomicCAS((unsigned long long*)&T.key[hh], (unsigned long long)kEmptyKey,
+                                                        (unsigned long long)key);
+                    if (prev == kEmptyKey || prev == key) break;
+                    hh = (hh + 1) & T.mask;
+                }
+                uint32_t old = *reinterpret_cast<volatile uint32_t*>(&T.head[hh]);
+                while (true) {
+                    e.next = old;
+                    T.pool[ni] = e;
+                    __threadfence();
+                    const uint32_t seen = atomicCAS(&T.head[hh], old, ni);
+                    if (seen == old) break;
+                    old = seen;
+                }
+            }
+        }
+    }
 }
 
 // Capacity growth: re-link every stored representative into a fresh (larger) table.
@@ -175,10 +194,8 @@ int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, c
                          OnlineTable& T, const Params& P, uint32_t n_sites, uint64_t* G, int64_t* dup_out,
                          uint64_t* ben, uint64_t* cnt, cudaStream_t st) {
     if (L.n == 0) return 0;
-    k_online_match<<<blocks_for(L.n), 256, 0, st>>>(
+    k_online_match<<<std::min<uint32_t>(blocks_for((uint64_t)L.n * 8), (uint32_t)P.num_sms * 8), 256, 0, st>>>(
         L, W.leader, accA, accB, T, P.digest_mask, P.refine_mask, G);
-    ONLINE_CHECK();
-    k_online_insert<<<blocks_for(L.n), 256, 0, st>>>(L, W.leader, accA, accB, G, T, P.digest_mask);
     ONLINE_CHECK();
     const size_t smem = label_smem_bytes(n_sites);
     const uint32_t grid = std::min<uint32_t>(blocks_for(L.n, 1024), (uint32_t)P.num_sms);
@@ -189,7 +206,7 @@ int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, c
         k_online_label<false><<<grid, 1024, 0, st>>>(L, W.leader, G, n_sites, dup_out, ben, cnt);
     }
     ONLINE_CHECK();
-    return 3;
+    return 2;
 }
 
 }  // namespace ffm
