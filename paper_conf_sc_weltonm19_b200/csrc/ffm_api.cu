@@ -409,7 +409,6 @@ void ensure_work(ffm_log* L, uint64_t n) {
     if (tcap > W.t_cap) {
         ++L->epoch;
         dev_alloc(W.tkey, tcap);
-        dev_alloc(W.tval, tcap);
         W.t_cap = tcap;
     }
     if (L->n_large_chunks > W.hitem_cap) {
@@ -1540,7 +1539,7 @@ int ffm_log_destroy(ffm_log* L) {
     if (L->stage_stream) cudaStreamSynchronize(L->stage_stream);
     Work& W = L->work;
     void* ptrs[] = {W.accA, W.accB, W.key, W.digest, W.slot, W.leader, W.eq, W.mis, W.res[0], W.res[1],
-                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.fitems, W.sdesc, W.hcount, W.hstart, W.hpart, W.tkey, W.tval,
+                    W.lcount, W.lstart, W.gcount, W.pos, W.fhead, W.hitems, W.fitems, W.sdesc, W.hcount, W.hstart, W.hpart, W.tkey,
                     W.dup, W.ben, W.label_part, W.label_cpart, W.counters, W.cub_tmp, L->d_off, L->d_size, L->d_site, L->d_dur, L->d_gid, L->d_chan,
                     L->arena, L->d_desc, L->d_small_order};
     for (void* p : ptrs)

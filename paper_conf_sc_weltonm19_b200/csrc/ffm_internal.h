@@ -59,8 +59,7 @@ struct Work {
     uint32_t* hcount = nullptr;    // [n+1] per-record hash chunk counts
     uint32_t* hstart = nullptr;    // [n+1] exclusive scan of hcount
     uint64_t* hpart = nullptr;     // [2 * hitem_cap] per-unit partial NH sums (A, B)
-    uint64_t* tkey = nullptr;      // [cap] table keys
-    uint32_t* tval = nullptr;      // [cap] table min local index
+    uint64_t* tkey = nullptr;      // [cap] group-by table: (32-bit key fingerprint << 32 | min local index)
     int64_t* dup = nullptr;        // [n] output staging
     uint64_t* ben = nullptr;       // [n_sites]
     uint64_t* label_part = nullptr; // [label_hist_rows * n_sites] per-block benefit partials

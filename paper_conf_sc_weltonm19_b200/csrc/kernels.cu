@@ -330,15 +330,26 @@ __global__ void k_group_insert(DevLog L, Work W, const uint32_t* __restrict__ li
         key = W.key[r];
     }
     uint64_t h = key & cap_mask;
+    // one 64-bit slot per group: (32-bit key fingerprint << 32 | min local index) -- one
+    // random access per insert and per lookup.  Two keys with the same slot chain and
+    // fingerprint merge their groups; every member is byte-verified, so that only costs
+    // a residual, never a wrong result.
+    const unsigned long long packed = ((unsigned long long)(uint32_t)(key >> 32) << 32) | r;
     while (true) {
-        unsigned long long prev =
-            atomicCAS((unsigned long long*)&W.tkey[h], (unsigned long long)kEmptyKey, (unsigned long long)key);
-        if (prev == kEmptyKey || prev == key) break;
+        const unsigned long long prev =
+            atomicCAS((unsigned long long*)&W.tkey[h], (unsigned long long)kEmptyKey, packed);
+        if (prev == kEmptyKey) break;
+        if ((prev >> 32) == (packed >> 32)) {
+            if (packed < prev) atomicMin((unsigned long long*)&W.tkey[h], packed);
+            break;
+        }
         h = (h + 1) & cap_mask;
     }
-    atomicMin(&W.tval[h], r);
     W.slot[r] = (uint32_t)h;
 }
+
+// min local index of the group at table slot h
+__device__ __forceinline__ uint32_t table_leader(const Work& W, uint32_t h) { return (uint32_t)W.tkey[h]; }
 
 // Leader lookup.  Members (leader != self) are reset for verification; a large
 // member of its leader's size gets a position in its leader's group so that the
@@ -381,7 +392,7 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
     bool member = false;
     if (i < n_list) {
         uint32_t r = list ? list[i] : i;
-        uint32_t ld = W.tval[W.slot[r]];
+        uint32_t ld = table_leader(W, W.slot[r]);
         W.leader[r] = ld;
         // residuals whose difference list overflowed: heavy mismatch against their head
         // (the adaptive round-0 choice, run_local)
@@ -438,7 +449,7 @@ __global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, ui
     bool member = false;
     if (r < n) {
         const uint32_t i = L.order_pos[r];
-        const uint32_t ld = W.tval[W.slot[r]];
+        const uint32_t ld = table_leader(W, W.slot[r]);
         W.leader[r] = ld;
         const uint64_t sz = L.size[r];
         const bool same = L.size[ld] == sz && L.chan[ld] == L.chan[r];
@@ -1742,7 +1753,6 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
         ++k;
     }
     if (cudaMemsetAsync(W.tkey, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
-    if (cudaMemsetAsync(W.tval, 0xFF, cap * sizeof(uint32_t), st) != cudaSuccess) return -1;
     if (cudaMemsetAsync(W.lcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
     if (cudaMemsetAsync(W.gcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
     k_group_insert<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, cap - 1, P.digest_mask, round,
