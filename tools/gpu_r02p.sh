@@ -1,11 +1,11 @@
 set -x
-T=r02p
+T=r02r
 mkdir -p gpurun_out/$T
 timeout 600 python -m pytest tests/test_gpu_parity.py tests/test_gpu_online.py -m gpu -x -q -p no:cacheprovider > gpurun_out/$T/parity.log 2>&1; echo parity rc=$?; tail -2 gpurun_out/$T/parity.log
 for rep in 1 2; do
-for v in default unpacked; do
+for v in default prev; do
   if [ $v = default ]; then b=(); else b=(--lib build/variants/$v/libffm.so); fi
-  for k in 2 5; do
+  for k in 5 4 3; do
     timeout 200 python bench.py "${b[@]}" --workload $k --steps 20 --e2e-steps 0 --cpu-seconds 0 > gpurun_out/$T/c${k}_${v}_$rep.json 2>/dev/null
     python -c "
 import json
