@@ -195,6 +195,8 @@ def make_ffm_log(args, lg, n_records, my_bytes, rank, world, local, **kw):
     import paper_conf_sc_weltonm19_b200 as ffm
     from paper_conf_sc_weltonm19_b200 import sharded
     opts = dict(arena_bytes=my_bytes + 128 * n_records + (1 << 20), max_records=n_records, **kw)
+    if world == 1 and args.collective:     # the collective path (library NCCL) in a world of one
+        return ffm.FfmLog(lg.n_sites, device=local, nccl_id=ffm.ffm_nccl_unique_id(), **opts)
     if world == 1:
         return ffm.FfmLog(lg.n_sites, device=local, **opts)
     return sharded.create_sharded_log(lg.n_sites, local, transport="host" if args.same_device else "nccl", **opts)
@@ -378,7 +380,8 @@ def run_ours(args):
                    "n_sites": lg.n_sites, "seed": "0x5C19D1000%d" % args.workload,
                    "n_scale": args.n_scale, "size_scale": args.size_scale,
                    "l2": "inputs larger than L2 (payload %.1f GB >> 126 MB L2)" % (total / 1e9),
-                   "parallelism": "single GPU" if world == 1 else
+                   "parallelism": ("single GPU, collective path (library NCCL communicator, world of one)"
+                                   if args.collective else "single GPU") if world == 1 else
                    f"{world} shards (site-affinity LPT), collective ffm_dedup_run: "
                    + ("host transport, ranks sharing one GPU (test hook)" if args.same_device else
                       "library-owned NCCL all-gather of class representatives + all-reduce of per-site sums, "
@@ -685,6 +688,8 @@ def spawn_ranks(args):
 
 
 def main():
+    import faulthandler
+    faulthandler.enable()          # a native crash prints a stack instead of dying silently
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
@@ -701,6 +706,8 @@ def main():
     ap.add_argument("--same-device", action="store_true",
                     help="test hook: run the N ranks on one GPU (host exchange transport instead of NCCL)")
     ap.add_argument("--check", action="store_true", help="check the result against the CPU oracle (small logs)")
+    ap.add_argument("--collective", action="store_true",
+                    help="--gpus 1: run the collective (sharded) path over the library's NCCL in a world of one")
     ap.add_argument("--lib", default=None, help="load another build of libffm.so (tools/build_variants.sh)")
     ap.add_argument("--online", default=None,
                     help="comma-separated window sizes: measure online mode (ffm_online_step) instead")

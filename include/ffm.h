@@ -109,8 +109,10 @@ typedef struct ffm_config {
     uint32_t reserved0;
     void*    stream;       /* cudaStream_t to run on, or NULL: the log creates its own */
     const void* nccl_id;   /* world > 1: the 128-byte ncclUniqueId of the world (ffm_nccl_unique_id on
-                              one rank, broadcast by the caller); the log owns the communicator */
-    const ffm_comm_ops* comm;  /* world > 1, instead of nccl_id: caller transport (copied) */
+                              one rank, broadcast by the caller); the log owns the communicator.
+                              Also allowed with world == 1: a world of one runs the collective
+                              path (NCCL included) on its own */
+    const ffm_comm_ops* comm;  /* instead of nccl_id: caller transport (copied) */
 } ffm_config;
 
 /* Fill *cfg with defaults: n_sites 1, device 0, rank 0, world 1, digest_bits 64,

@@ -106,7 +106,7 @@ int comm_unique_id(void* out) {
 int comm_init(Comm& c, int world, int rank, const void* nccl_id, const ffm_comm_ops* ops) {
     c.world = world;
     c.rank = rank;
-    if (world <= 1) return FFM_OK;
+    if (!nccl_id && !ops) return FFM_OK;   // a single log: no transport
     if (ops) {
         if (!ops->allgather || !ops->allreduce_u64) {
             c.err = "ffm_comm_ops with a NULL function";
@@ -140,7 +140,7 @@ void comm_destroy(Comm& c) {
 }
 
 int comm_allgather(Comm& c, const void* send, void* recv, size_t bytes, cudaStream_t st) {
-    if (c.world <= 1) {
+    if (!c.nccl && !c.has_ops) {   // no transport: a world of one, local copy
         if (bytes && send != recv) {
             cudaError_t e = cudaMemcpyAsync(recv, send, bytes, cudaMemcpyDeviceToDevice, st);
             if (e != cudaSuccess) return cuda_fail(c, "allgather copy", e);
@@ -172,7 +172,7 @@ int comm_allgather(Comm& c, const void* send, void* recv, size_t bytes, cudaStre
 }
 
 int comm_allreduce_u64(Comm& c, uint64_t* buf, size_t n, cudaStream_t st) {
-    if (c.world <= 1 || n == 0) return FFM_OK;
+    if ((!c.nccl && !c.has_ops) || n == 0) return FFM_OK;
     c.bytes_moved += 8 * (uint64_t)n;
     if (!c.has_ops) {
         int r = nccl().AllReduce(buf, buf, n, kNcclUint64, kNcclSum, c.nccl, st);

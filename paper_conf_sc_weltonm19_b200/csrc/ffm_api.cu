@@ -483,7 +483,7 @@ void run_prologue(ffm_log* L) {
     ck(cudaSetDevice(L->device), "cudaSetDevice");
     // H0 tail: flush staged payloads and metadata, order the run after them
     ring_flush(L);
-    if (L->cfg.world > 1) ensure_arena(L, 1);   // peers map it: it exists before the header exchange
+    if (L->collective) ensure_arena(L, 1);   // peers map it: it exists before the header exchange
     upload_meta(L);
     ck(cudaEventRecord(L->ring_ev[L->ring_cur], L->stage_stream), "event");
     ck(cudaStreamWaitEvent(L->stream, L->ring_ev[L->ring_cur], 0), "wait staging");
@@ -1052,7 +1052,7 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
     if (cfg->n_sites == 0 || cfg->digest_bits > 64 || cfg->refine_bits > 64 || cfg->world < 1 ||
         cfg->rank < 0 || cfg->rank >= cfg->world)
         return FFM_E_INVAL;
-    if (cfg->world > 1 && (cfg->nccl_id == nullptr) == (cfg->comm == nullptr))
+    if ((cfg->world > 1 && (cfg->nccl_id == nullptr) == (cfg->comm == nullptr)) || (cfg->nccl_id && cfg->comm))
         return FFM_E_INVAL;   // a sharded log needs exactly one exchange transport
     uint32_t chunk = cfg->chunk_bytes ? cfg->chunk_bytes : 32768;
     uint32_t small = cfg->small_bytes ? cfg->small_bytes : 4096;
@@ -1108,7 +1108,10 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
         }
         for (auto& e : L->ev) ck(cudaEventCreate(&e), "event");
         ck(cudaHostAlloc((void**)&L->h_counters, 16 * sizeof(uint32_t), cudaHostAllocDefault), "cudaHostAlloc");
-        if (cfg->world > 1) {
+        // a transport makes the log collective -- also a world of one (the whole collective
+        // path, NCCL included, then runs on a single GPU)
+        L->collective = cfg->world > 1 || cfg->nccl_id || cfg->comm;
+        if (L->collective) {
             const uint64_t w = (uint64_t)cfg->world;
             ck(cudaMalloc(&L->d_hdr, (4 + 4 * w) * sizeof(uint64_t)), "cudaMalloc(hdr)");
             ck(cudaMalloc(&L->d_ipc, 64 * (w + 1)), "cudaMalloc(ipc)");
@@ -1277,7 +1280,7 @@ int ffm_dedup_run(ffm_log* L, int64_t* dup_out, uint64_t* ben_out) {
         bool ben_dev = ben_out && is_device_ptr(ben_out);
         int64_t* d_dup = dup_dev ? dup_out : W.dup;
         uint64_t launches = 0;
-        if (L->cfg.world > 1) {
+        if (L->collective) {
             LocalRun R{};
             run_sharded(L, dup_out, ben_out, dup_dev, ben_dev, R, launches);
             L->stats.host_syncs = L->n_syncs;
@@ -1384,7 +1387,7 @@ uint64_t ffm_online_done(const ffm_log* L) { return L ? L->online_done : 0; }
 int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n_out) {
     int st = check_state(L);
     if (st) return st;
-    if (L->cfg.world > 1) return set_err(L, FFM_E_STATE, "online mode is single-log (world == 1)");
+    if (L->collective) return set_err(L, FFM_E_STATE, "online mode is single-log (no exchange transport)");
     const uint64_t n = L->h_size.size(), w0 = L->online_done, nw = n - w0;
     if (nw && !dup_out) return set_err(L, FFM_E_INVAL, "duplicate_of is NULL");
     const uint32_t ns = L->cfg.n_sites;

@@ -22,7 +22,8 @@ struct Comm {
 };
 
 int comm_unique_id(void* out128);
-// world <= 1: no-op.  Else exactly one of nccl_id (128-byte ncclUniqueId) / ops.
+// Neither nccl_id (128-byte ncclUniqueId) nor ops: no transport (a single log).  Else the
+// given transport, for any world size (a world of one runs the collective path alone).
 int comm_init(Comm& c, int world, int rank, const void* nccl_id, const ffm_comm_ops* ops);
 void comm_destroy(Comm& c);
 // recv[world * bytes] = every rank's send[bytes], rank-major (device buffers, on st).

@@ -250,7 +250,8 @@ struct ffm_log {
     uint64_t ring_fill = 0;         // bytes used in ring[cur]
     bool ring_pending = false;
 
-    // sharded runs (world > 1)
+    // sharded runs (world > 1, or a transport given: collective ffm_dedup_run)
+    bool collective = false;
     ffm::Comm comm;
     ffm::ShardWork shard;
     uint64_t arena_gen = 0;         // bumped whenever the arena is reallocated (peers re-map it)

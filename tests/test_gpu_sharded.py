@@ -147,3 +147,24 @@ def test_two_host_syncs_without_collisions(tmp_path):
     for r in range(2):
         z = np.load(tmp_path / f"r{r}.npz")
         assert int(z["syncs"]) == 2, int(z["syncs"])
+
+
+def test_nccl_world_of_one():
+    """The collective run over the library's own NCCL communicator (ncclCommInitRank,
+    ncclAllGather of the headers and representatives, ncclAllReduce of the per-site sums,
+    all on the log's stream) in a world of one: the NCCL data plane on a single GPU."""
+    import torch  # noqa: F401  (the process's NCCL is torch's)
+    import paper_conf_sc_weltonm19_b200 as ffm
+    lg = loggen.gen_config(5, n_scale=0.004, size_scale=1 / 32)
+    want_dup, want_ben = oracle.dedup(lg)
+    with ffm.FfmLog(lg.n_sites, rank=0, world=1, nccl_id=ffm.ffm_nccl_unique_id(), chunk_bytes=4096) as log:
+        log.append_log(lg)
+        for _ in range(2):
+            dup, ben = log.run()
+            np.testing.assert_array_equal(dup, want_dup)
+            np.testing.assert_array_equal(ben, want_ben)
+        st = log.stats()
+        assert st["exchange_bytes"] > 0 and st["host_syncs"] == 2
+        assert st["n_reps_local"] == st["n_reps_global"] > 0
+        np.testing.assert_array_equal(log.site_counts(),
+                                      np.bincount(lg.site[want_dup >= 0].astype(np.int64), minlength=lg.n_sites))

@@ -92,3 +92,11 @@ def test_sharded_config_validation():
     with pytest.raises(ffm.FfmError) as e:
         ffm.ffm_log_create(c)
     assert e.value.code == ffm.FFM_E_INVAL
+
+
+def test_nccl_unique_id_host_only():
+    """ffm_nccl_unique_id opens the process's libnccl.so.2 (torch's) and returns a 128-byte
+    ncclUniqueId without any GPU work."""
+    import torch  # noqa: F401  (loads torch's NCCL)
+    a, b = ffm.ffm_nccl_unique_id(), ffm.ffm_nccl_unique_id()
+    assert len(a) == 128 and len(b) == 128 and a != b
