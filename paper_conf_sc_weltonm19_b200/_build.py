@@ -7,8 +7,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB = os.path.join(HERE, "libffm.so")
 SOURCES = [os.path.join(HERE, "csrc", f) for f in ("kernels.cu", "shard.cu", "online.cu", "comm.cu", "ffm_api.cu", "shard_plan.cpp")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-FLAGS = ["-shared", "-Xcompiler", "-fPIC", "-O3", "-lineinfo", "-std=c++17",
-         "-gencode", "arch=compute_100a,code=sm_100a", "-ldl"]
+FLAGS = ["-shared", "-Xcompiler", "-fPIC,-fopenmp", "-O3", "-lineinfo", "-std=c++17",
+         "-gencode", "arch=compute_100a,code=sm_100a", "-ldl", "-lgomp"]
 
 
 def _stale() -> bool:

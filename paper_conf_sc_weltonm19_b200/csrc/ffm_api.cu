@@ -2,6 +2,7 @@
 // run pipeline (H1..H7).  No C++ exception crosses the boundary; every CUDA error
 // poisons the handle.  There is no CPU fallback: without a device, create fails.
 #include <cuda_runtime.h>
+#include <omp.h>
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
@@ -18,7 +19,7 @@ using namespace ffm;
 
 namespace {
 
-constexpr uint64_t kRingBytes = 16ull << 20;      // per half of the pinned staging ring
+constexpr uint64_t kRingBytes = 32ull << 20;      // per half of the pinned staging ring
 constexpr uint64_t kDirectCopy = 4ull << 20;      // host payloads above this bypass the ring
 constexpr uint64_t kGatherMax = 1ull << 20;   // device / pinned payloads up to this use k_gather (not DMA)
 
@@ -135,6 +136,50 @@ void stage_host(ffm_log* L, const void* src, uint64_t size, uint64_t off) {
     if (!L->ring_fill) L->ring_arena_start = off;
     memcpy(L->ring[L->ring_cur] + (off - L->ring_arena_start), src, size);
     L->ring_fill = off + size - L->ring_arena_start;
+}
+
+// Pageable payloads of one batch, staged in parallel: the arena range they cover is cut
+// into ring-sized windows; for each window the host threads copy every record piece that
+// falls in it into one half of the pinned ring (OpenMP), then that half goes to HBM
+// asynchronously while the next window fills the other half.  The bytes are snapshotted
+// (in the ring, or already in HBM) before the append returns (reading R11).
+// host threads of the pageable staging copies (at most 8: several ranks may share a node)
+int stage_threads() {
+    static const int t = std::max(1, std::min(8, omp_get_max_threads()));
+    return t;
+}
+
+void stage_pageable(ffm_log* L, const std::vector<PageablePiece>& recs) {
+    if (recs.empty()) return;
+    ring_flush(L);
+    const uint64_t R = L->ring_bytes;
+    const uint64_t a0 = recs.front().off, a1 = recs.back().off + recs.back().size;
+    size_t first = 0;   // first record that may reach into the current window
+    for (uint64_t w0 = a0; w0 < a1; w0 += R) {
+        const uint64_t w1 = std::min(a1, w0 + R);
+        while (first < recs.size() && recs[first].off + recs[first].size <= w0) ++first;
+        size_t last = first;
+        while (last < recs.size() && recs[last].off < w1) ++last;
+        const int c = L->ring_cur;
+        uint8_t* ring = L->ring[c];
+        // copy jobs of at most 1 MiB (a large record is split across the threads)
+        std::vector<PageablePiece>& jobs = L->stage_jobs;
+        jobs.clear();
+        for (size_t k = first; k < last; ++k) {
+            const PageablePiece& p = recs[k];
+            for (uint64_t lo = std::max(p.off, w0), hi = std::min(p.off + p.size, w1); lo < hi; lo += (1ull << 20))
+                jobs.push_back({p.src + (lo - p.off), lo - w0, std::min<uint64_t>(hi - lo, 1ull << 20)});
+        }
+        const long nj = (long)jobs.size();
+        uint64_t bytes = 0;
+        for (const PageablePiece& j : jobs) bytes += j.size;
+#pragma omp parallel for schedule(dynamic, 1) num_threads(stage_threads()) if (bytes > (1ull << 20))
+        for (long k = 0; k < nj; ++k) memcpy(ring + jobs[(size_t)k].off, jobs[(size_t)k].src, jobs[(size_t)k].size);
+        ck(cudaMemcpyAsync(L->arena + w0, ring, w1 - w0, cudaMemcpyHostToDevice, L->stage_stream), "ring H2D");
+        ck(cudaEventRecord(L->ring_ev[c], L->stage_stream), "ring event");
+        L->ring_cur = c ^ 1;
+        ck(cudaEventSynchronize(L->ring_ev[L->ring_cur]), "ring wait");   // the other half is free again
+    }
 }
 
 // FFM_PAYLOAD_DEVICE / _HOST_PINNED / _HOST (pageable) of one pointer; *dev = the
@@ -1170,6 +1215,7 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
         if (kind == FFM_PAYLOAD_DEVICE || kind == FFM_PAYLOAD_HOST_PINNED) desc.reserve(3 * n);
         bool need_sync = false, ordered = false;
         PtrCache pc;
+        std::vector<PageablePiece> pageable;   // consecutive pageable records, staged together
         for (uint64_t i = 0; i < n; ++i) {
             if (sizes[i] == 0) continue;
             int src = kind, pdev = L->device;
@@ -1193,9 +1239,14 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
             }
             // the ring uploads one contiguous arena range: close it before a record that
             // is written into the arena by another path
-            if (!ring && L->ring_fill) ring_flush(L);
+            if (!ring) {
+                stage_pageable(L, pageable);
+                pageable.clear();
+                if (L->ring_fill) ring_flush(L);
+            }
             if (ring) {
-                stage_host(L, payloads[i], sizes[i], offs[i]);
+                if (n == 1) stage_host(L, payloads[i], sizes[i], offs[i]);   // single appends: the ring
+                else pageable.push_back({(const uint8_t*)payloads[i], offs[i], sizes[i]});
             } else if (sizes[i] > L->gather_max || (src == FFM_PAYLOAD_HOST_PINNED && !L->host_ptr_ok) ||
                        (src == FFM_PAYLOAD_DEVICE && pdev != L->device)) {
                 // (a payload on another GPU: the copy engines, never a kernel dereference)
@@ -1209,6 +1260,7 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
                 desc.push_back(sizes[i]);
             }
         }
+        stage_pageable(L, pageable);
         if (!desc.empty()) {
             uint64_t nd = desc.size() / 3;
             uint64_t cap = L->desc_cap;

@@ -71,6 +71,13 @@ struct Work {
     uint64_t n_cap = 0, t_cap = 0, hitem_cap = 0, vitem_cap = 0, site_cap = 0, fitem_cap = 0;
 };
 
+// A pageable payload (or a piece of one) to stage: source, arena offset (or offset in a
+// ring half), bytes.
+struct PageablePiece {
+    const uint8_t* src;
+    uint64_t off, size;
+};
+
 // One representative per exact local class, exported for the cross-shard merge.
 struct RepTuple {
     uint64_t key;    // group key of the full digest (same function on every rank)
@@ -249,6 +256,7 @@ struct ffm_log {
     uint64_t ring_arena_start = 0;  // arena offset corresponding to ring[cur][0]
     uint64_t ring_fill = 0;         // bytes used in ring[cur]
     bool ring_pending = false;
+    std::vector<ffm::PageablePiece> stage_jobs;   // copy jobs of one ring window (reused)
 
     // sharded runs (world > 1, or a transport given: collective ffm_dedup_run)
     bool collective = false;
