@@ -1464,7 +1464,8 @@ __global__ void __launch_bounds__(1024) k_label_hist(DevLog L, const uint32_t* _
 #pragma unroll
         for (int u = 0; u < kLabelU; ++u) {
             const uint32_t r = r0 + u * stride;
-            d[u] = (r >= L.n || ld[u] == r) ? -1 : (int64_t)L.gid[ld[u]];
+            // (no labels to write -- they went out speculatively: membership suffices)
+            d[u] = (r >= L.n || ld[u] == r) ? -1 : (dup_out ? (int64_t)L.gid[ld[u]] : 0);
         }
 #pragma unroll
         for (int u = 0; u < kLabelU; ++u) {
