@@ -727,7 +727,8 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
     };
     // (per-stage timing needs directly recorded events: FFM_FLAG_TIMING runs launch directly)
-    const bool graph = label && !(L->cfg.flags & FFM_FLAG_NO_GRAPH) && !timing;
+    // (online windows move their view every step: recapturing would cost more than it saves)
+    const bool graph = !prehashed && !(L->cfg.flags & FFM_FLAG_NO_GRAPH) && !timing;
     if (graph) {
         // replay a CUDA graph of segment A while the log, its buffers and the run mode are
         // unchanged: one launch instead of ~30 (launch-bound small logs)
