@@ -1289,6 +1289,9 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
     LaneKeys K;   // k[0]: stripe position g, k[1]: position g + 8
     uint64_t A = 0, B = 0, A2 = 0, B2 = 0, found = ~0ull;
     int sc = 0, sf = kSaS - 1;
+    // The warp stays converged across the loop (an octet whose records are done idles
+    // until all four are), so the octet reductions at record ends use full-mask shuffles
+    // (xor 4 / 2 / 1 stay inside an octet) executed warp-uniformly -- no per-octet masks.
 #pragma unroll 1
     while (true) {
         // refill the stage consumed last iteration (its values were used, so read), then
@@ -1298,107 +1301,108 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
         uint32_t m[4];
         lds16(mslot(sc), m);
         const uint32_t n = m[0], r = m[1], z = m[2];
-        if (z & kSaEnd) break;
-        if (z & kSaFirst) {
-            A = B = A2 = B2 = 0;
-            found = ~0ull;
+        const bool done = (z & kSaEnd) != 0;
+        if (__all_sync(0xFFFFFFFFu, done)) break;
+        if (!done) {
+            if (z & kSaFirst) {
+                A = B = A2 = B2 = 0;
+                found = ~0ull;
 #pragma unroll
-            for (int jj = 0; jj < 6; ++jj) {
-                K.k[0][jj] = c_nh.ka[g][jj];
-                K.k[1][jj] = c_nh.ka[g + 8][jj];
+                for (int jj = 0; jj < 6; ++jj) {
+                    K.k[0][jj] = c_nh.ka[g][jj];
+                    K.k[1][jj] = c_nh.ka[g + 8][jj];
+                }
             }
-        }
-        const uint32_t w0 = z & 0x0FFFFFFFu, nw = (n + 15) >> 4;
-        const bool cmp = z & kSaCmp;
-        const bool full = 16 * (w0 + 8 * kSaJ) <= n;   // every word of the step whole
-        if (cmp) {
-            // member: compare only, until its first differing word
-            if (found == ~0ull) {
-                uint32_t d = 0;
+            const uint32_t w0 = z & 0x0FFFFFFFu, nw = (n + 15) >> 4;
+            const bool full = 16 * (w0 + 8 * kSaJ) <= n;   // every word of the step whole
+            if (z & kSaCmp) {
+                // member: compare only, until its first differing word
+                if (found == ~0ull) {
+                    uint32_t d = 0;
+                    if (full) {
+#pragma unroll
+                        for (int j = 0; j < kSaJ; ++j) {
+                            uint32_t x[4], y[4];
+                            lds16(slot(sc, j, 0), x);
+                            lds16(slot(sc, j, 1), y);
+                            d |= (x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3]);
+                        }
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < kSaJ; ++j) {
+                            const uint32_t w = w0 + 8 * j + g;
+                            if (w < nw) {
+                                uint32_t x[4], y[4];
+                                lds16(slot(sc, j, 0), x);
+                                lds16(slot(sc, j, 1), y);
+                                mask_word(x, n, w);
+                                mask_word(y, n, w);
+                                d |= (x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3]);
+                            }
+                        }
+                    }
+                    if (d) {   // rare: the lowest differing word of this step
+#pragma unroll 1
+                        for (int j = 0; j < kSaJ; ++j) {
+                            const uint32_t w = w0 + 8 * j + g;
+                            if (w >= nw) break;
+                            uint32_t x[4], y[4];
+                            lds16(slot(sc, j, 0), x);
+                            lds16(slot(sc, j, 1), y);
+                            mask_word(x, n, w);
+                            mask_word(y, n, w);
+                            if ((x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3])) {
+                                found = w;
+                                break;
+                            }
+                        }
+                    }
+                }
+            } else {
+                // leader / singleton: hash (two accumulator chains: even / odd words)
                 if (full) {
 #pragma unroll
                     for (int j = 0; j < kSaJ; ++j) {
-                        uint32_t x[4], y[4];
+                        uint32_t x[4];
                         lds16(slot(sc, j, 0), x);
-                        lds16(slot(sc, j, 1), y);
-                        d |= (x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3]);
+                        if (j & 1) nh_word(x[0], x[1], x[2], x[3], K.k[1], A2, B2);
+                        else nh_word(x[0], x[1], x[2], x[3], K.k[0], A, B);
+                        if (j & 1) advance<1>(K);
                     }
                 } else {
 #pragma unroll
                     for (int j = 0; j < kSaJ; ++j) {
                         const uint32_t w = w0 + 8 * j + g;
                         if (w < nw) {
-                            uint32_t x[4], y[4];
+                            uint32_t x[4];
                             lds16(slot(sc, j, 0), x);
-                            lds16(slot(sc, j, 1), y);
                             mask_word(x, n, w);
-                            mask_word(y, n, w);
-                            d |= (x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3]);
+                            if (j & 1) nh_word(x[0], x[1], x[2], x[3], K.k[1], A2, B2);
+                            else nh_word(x[0], x[1], x[2], x[3], K.k[0], A, B);
                         }
-                    }
-                }
-                if (d) {   // rare: the lowest differing word of this step
-#pragma unroll 1
-                    for (int j = 0; j < kSaJ; ++j) {
-                        const uint32_t w = w0 + 8 * j + g;
-                        if (w >= nw) break;
-                        uint32_t x[4], y[4];
-                        lds16(slot(sc, j, 0), x);
-                        lds16(slot(sc, j, 1), y);
-                        mask_word(x, n, w);
-                        mask_word(y, n, w);
-                        if ((x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3])) {
-                            found = w;
-                            break;
-                        }
+                        if (j & 1) advance<1>(K);
                     }
                 }
             }
-            if (z & kSaLast) {
+        }
+        // record ends (warp-uniform: any octet finishing one reduces with all four)
+        const bool last = !done && (z & kSaLast) != 0;
+        if (__any_sync(0xFFFFFFFFu, last)) {
+            uint64_t a = A + A2, b = B + B2, f = found;
 #pragma unroll
-                for (int o = 4; o; o >>= 1) {
-                    const uint64_t of = __shfl_xor_sync(omask, found, o);
-                    found = of < found ? of : found;
-                }
-                if (g == 0 && found != ~0ull) report_mismatch(W, r, found, res_out, false);
+            for (int o = 4; o; o >>= 1) {
+                a += __shfl_xor_sync(0xFFFFFFFFu, a, o);
+                b += __shfl_xor_sync(0xFFFFFFFFu, b, o);
+                const uint64_t of = __shfl_xor_sync(0xFFFFFFFFu, f, o);
+                f = of < f ? of : f;
             }
-        } else {
-            // leader / singleton: hash (two accumulator chains: even / odd words)
-            if (full) {
-#pragma unroll
-                for (int j = 0; j < kSaJ; ++j) {
-                    uint32_t x[4];
-                    lds16(slot(sc, j, 0), x);
-                    if (j & 1) nh_word(x[0], x[1], x[2], x[3], K.k[1], A2, B2);
-                    else nh_word(x[0], x[1], x[2], x[3], K.k[0], A, B);
-                    if (j & 1) advance<1>(K);
-                }
-            } else {
-#pragma unroll
-                for (int j = 0; j < kSaJ; ++j) {
-                    const uint32_t w = w0 + 8 * j + g;
-                    if (w < nw) {
-                        uint32_t x[4];
-                        lds16(slot(sc, j, 0), x);
-                        mask_word(x, n, w);
-                        if (j & 1) nh_word(x[0], x[1], x[2], x[3], K.k[1], A2, B2);
-                        else nh_word(x[0], x[1], x[2], x[3], K.k[0], A, B);
-                    }
-                    if (j & 1) advance<1>(K);
-                }
-            }
-            if (z & kSaLast) {
-                A += A2;
-                B += B2;
-#pragma unroll
-                for (int o = 4; o; o >>= 1) {
-                    A += __shfl_xor_sync(omask, A, o);
-                    B += __shfl_xor_sync(omask, B, o);
-                }
-                if (g == 0) {
-                    W.accA[r] = A;
-                    W.accB[r] = B;
-                    W.digest[r] = finalize_digest(A, B, n);
+            if (last && g == 0) {
+                if (z & kSaCmp) {
+                    if (f != ~0ull) report_mismatch(W, r, f, res_out, false);
+                } else {
+                    W.accA[r] = a;
+                    W.accB[r] = b;
+                    W.digest[r] = finalize_digest(a, b, n);
                 }
             }
         }
