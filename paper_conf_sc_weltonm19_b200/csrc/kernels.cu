@@ -1241,22 +1241,25 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
         if (fi < L.n_small) {
             const uint32_t nw = (fn + 15) >> 4;
             const bool cmp = floff != ~0ull;
-            const uint8_t* src = L.arena + foff;
-            const uint8_t* lsrc = L.arena + (cmp ? floff : foff);
+            // this lane's first word of the step; word j is 128 * j bytes further (immediate
+            // offsets), shared-memory slot j of part p is (2 j + p) * kSaT * 16 further
+            const uint8_t* src = L.arena + foff + 16ull * (fw0 + g);
+            const uint8_t* lsrc = L.arena + (cmp ? floff : foff) + 16ull * (fw0 + g);
+            const uint32_t s0 = slot(s, 0, 0);
             if (fw0 + 8 * kSaJ <= nw) {   // every lane's words exist
 #pragma unroll
-                for (int j = 0; j < kSaJ; ++j) cp16(slot(s, j, 0), src + 16ull * (fw0 + 8 * j + g), pol_own);
+                for (int j = 0; j < kSaJ; ++j) cp16(s0 + (uint32_t)(2 * j * kSaT * 16), src + 128 * j, pol_own);
                 if (cmp) {
 #pragma unroll
-                    for (int j = 0; j < kSaJ; ++j) cp16(slot(s, j, 1), lsrc + 16ull * (fw0 + 8 * j + g), pol_keep);
+                    for (int j = 0; j < kSaJ; ++j)
+                        cp16(s0 + (uint32_t)((2 * j + 1) * kSaT * 16), lsrc + 128 * j, pol_keep);
                 }
             } else {
 #pragma unroll
                 for (int j = 0; j < kSaJ; ++j) {
-                    const uint32_t w = fw0 + 8 * j + g;
-                    if (w < nw) {
-                        cp16(slot(s, j, 0), src + 16ull * w, pol_own);
-                        if (cmp) cp16(slot(s, j, 1), lsrc + 16ull * w, pol_keep);
+                    if (fw0 + 8 * j + g < nw) {
+                        cp16(s0 + (uint32_t)(2 * j * kSaT * 16), src + 128 * j, pol_own);
+                        if (cmp) cp16(s0 + (uint32_t)((2 * j + 1) * kSaT * 16), lsrc + 128 * j, pol_keep);
                     }
                 }
             }
