@@ -107,3 +107,24 @@ def test_online_after_reset_and_forced_collisions_across_windows(ffm):
             np.testing.assert_array_equal(np.concatenate(dups), want_d)
             np.testing.assert_array_equal(ben, want_b)
             log.reset()
+
+
+def test_online_device_payloads_and_outputs(ffm):
+    """Appends of device-resident payloads hashed at append time, labels written to
+    device memory (the streaming shape of bench.py --online)."""
+    import torch
+    lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 32)
+    want_d, want_b = oracle.dedup(lg)
+    buf = torch.from_numpy(lg.materialize()).cuda()
+    ptrs = (lg.c_off[lg.content] + np.uint64(buf.data_ptr())).astype(np.uint64)
+    dup = torch.empty(lg.n, dtype=torch.int64, device="cuda")
+    ben = torch.empty(lg.n_sites, dtype=torch.int64, device="cuda")
+    got = []
+    with ffm.FfmLog(lg.n_sites, online=True, chunk_bytes=4096) as log:
+        for a in range(0, lg.n, 777):
+            e = min(lg.n, a + 777)
+            log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e], payload_kind=ffm.FFM_PAYLOAD_DEVICE)
+            log.online_step(dup, ben)
+            got.append(dup[:e - a].cpu().numpy().copy())
+    np.testing.assert_array_equal(np.concatenate(got), want_d)
+    np.testing.assert_array_equal(ben.cpu().numpy().view(np.uint64), want_b)

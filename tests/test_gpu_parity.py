@@ -198,6 +198,31 @@ def test_single_appends_mixed_host_device(ffm):
     assert_same(lg, dup, ben)
 
 
+def test_batch_mixed_pageable_pinned_device(ffm):
+    """One AUTO batch interleaving pageable, pinned and device payloads (runs of each, runs
+    spanning several ring windows): the parallel pageable staging closes its run
+    before every record written by another path; pageable bytes are snapshotted."""
+    import torch
+    lg = loggen.gen_config(5, n_scale=0.003, size_scale=1 / 8)
+    host = lg.materialize()
+    pageable = host.copy()
+    pinned = torch.from_numpy(host.copy()).pin_memory()
+    dev = torch.from_numpy(host).cuda()
+    bases = [pageable.ctypes.data, pinned.data_ptr(), dev.data_ptr()]
+    rng = np.random.default_rng(7)
+    kind = np.repeat(rng.integers(0, 3, lg.n // 40 + 1), 40)[:lg.n]   # runs of 40 records
+    ptrs = np.array([lg.c_off[lg.content[i]] + np.uint64(bases[kind[i]]) for i in range(lg.n)], np.uint64)
+    with ffm.FfmLog(lg.n_sites) as log:
+        log.append_batch(lg.site, lg.size, ptrs, lg.dur, payload_kind=ffm.FFM_PAYLOAD_AUTO)
+        pageable[:] = 0                      # snapshot taken: later writes are invisible
+        pinned.zero_()
+        dup, ben = log.run()
+    assert_same(lg, dup, ben)
+    # (ring windows are 32 MiB: some pageable run spans several, so records straddle windows)
+    spans = [int(lg.size[i:i + 40].sum()) for i in range(0, lg.n, 40) if kind[i] == 0]
+    assert max(spans) > (32 << 20)
+
+
 @pytest.mark.parametrize("kind", ["pinned", "auto_pinned", "pageable"])
 def test_host_payload_kinds(ffm, kind):
     import torch
