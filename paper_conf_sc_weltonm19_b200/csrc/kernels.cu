@@ -1209,7 +1209,6 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
     const int g = threadIdx.x & 7;
     const uint32_t oct = (blockIdx.x * blockDim.x + threadIdx.x) >> 3;
     const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
-    const unsigned omask = 0xFFu << (threadIdx.x & 24);
     const uint32_t sbase = smem_u32(sa_smem) + threadIdx.x * 16;
     // slot of word j of stage s (part 0 own, 1 leader); lanes interleaved so a warp's
     // 16-B accesses to one slot are 512 contiguous bytes (conflict-free)
@@ -1219,22 +1218,24 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_own));
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
 
-    // ---- producer state: current record (position fi, next word fw0) + next descriptor
+    // ---- producer state: current record (position fi, next word fw0).  The descriptor
+    // of the octet's next record is held spread over its 8 lanes (lane g: 32-bit word g
+    // of the 32-byte descriptor, one coalesced load per octet), loaded a whole record
+    // ahead and gathered by shuffles when the record changes -- the load's destination is
+    // read only then, so no step waits on it.
+    const uint32_t* sd32 = reinterpret_cast<const uint32_t*>(W.sdesc);
     uint32_t fi = oct, fw0 = 0;
     uint64_t foff = 0, floff = 0;
-    uint32_t fn = 0, fr = 0;
-    uint4 da = make_uint4(0, 0, 0, 0), db = make_uint4(0, 0, 0, 0);
+    uint32_t fn = 0, fr = 0, nd = 0;
     if (fi < L.n_small) {
         const uint4 a = W.sdesc[2ull * fi], b = W.sdesc[2ull * fi + 1];
         foff = (uint64_t)a.y << 32 | a.x;
         floff = (uint64_t)a.w << 32 | a.z;
         fn = b.x;
         fr = b.y;
-        if (fi + noct < L.n_small) {
-            da = W.sdesc[2ull * (fi + noct)];
-            db = W.sdesc[2ull * (fi + noct) + 1];
-        }
+        if (fi + noct < L.n_small) nd = sd32[8ull * (fi + noct) + g];
     }
+    const int obase = threadIdx.x & 24;
     auto fetch = [&](int s) {
         uint32_t meta_z = kSaEnd;
         uint32_t mn = 0, mr = 0;
@@ -1267,18 +1268,23 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
             mn = fn;
             mr = fr;
             fw0 += 8 * kSaJ;
-            if (fw0 >= nw) {   // last step of this record: move to the next one
-                meta_z |= kSaLast;
+            if (fw0 >= nw) meta_z |= kSaLast;
+        }
+        // last step of the octet's record: move to the next one (shuffles executed by the
+        // whole warp; an octet that is not changing ignores them)
+        const bool change = (meta_z & (kSaLast | kSaEnd)) == kSaLast;
+        if (__any_sync(0xFFFFFFFFu, change)) {
+            const uint32_t d0 = __shfl_sync(0xFFFFFFFFu, nd, obase + 0), d1 = __shfl_sync(0xFFFFFFFFu, nd, obase + 1);
+            const uint32_t d2 = __shfl_sync(0xFFFFFFFFu, nd, obase + 2), d3 = __shfl_sync(0xFFFFFFFFu, nd, obase + 3);
+            const uint32_t d4 = __shfl_sync(0xFFFFFFFFu, nd, obase + 4), d5 = __shfl_sync(0xFFFFFFFFu, nd, obase + 5);
+            if (change) {
                 fi += noct;
                 fw0 = 0;
-                foff = (uint64_t)da.y << 32 | da.x;
-                floff = (uint64_t)da.w << 32 | da.z;
-                fn = db.x;
-                fr = db.y;
-                if (fi + noct < L.n_small) {
-                    da = W.sdesc[2ull * (fi + noct)];
-                    db = W.sdesc[2ull * (fi + noct) + 1];
-                }
+                foff = (uint64_t)d1 << 32 | d0;
+                floff = (uint64_t)d3 << 32 | d2;
+                fn = d4;
+                fr = d5;
+                if (fi + noct < L.n_small) nd = sd32[8ull * (fi + noct) + g];
             }
         }
         asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(mslot(s)), "r"(mn), "r"(mr), "r"(meta_z), "r"(0u)
@@ -1290,6 +1296,12 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
 
     // ---- consumer state
     LaneKeys K;   // k[0]: stripe position g, k[1]: position g + 8
+    uint32_t ka0[6], ka1[6];   // their stripe-0 keys (fixed per lane: no constant-bank loads per record)
+#pragma unroll
+    for (int jj = 0; jj < 6; ++jj) {
+        ka0[jj] = c_nh.ka[g][jj];
+        ka1[jj] = c_nh.ka[g + 8][jj];
+    }
     uint64_t A = 0, B = 0, A2 = 0, B2 = 0, found = ~0ull;
     int sc = 0, sf = kSaS - 1;
     // The warp stays converged across the loop (an octet whose records are done idles
@@ -1312,8 +1324,8 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
                 found = ~0ull;
 #pragma unroll
                 for (int jj = 0; jj < 6; ++jj) {
-                    K.k[0][jj] = c_nh.ka[g][jj];
-                    K.k[1][jj] = c_nh.ka[g + 8][jj];
+                    K.k[0][jj] = ka0[jj];
+                    K.k[1][jj] = ka1[jj];
                 }
             }
             const uint32_t w0 = z & 0x0FFFFFFFu, nw = (n + 15) >> 4;
