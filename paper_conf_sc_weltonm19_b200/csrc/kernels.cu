@@ -1180,7 +1180,8 @@ __global__ void __launch_bounds__(256, 4) k_verify_small(DevLog L, Work W, const
 #define FFM_SA_T 128
 #endif
 constexpr int kSaU = FFM_SA_U, kSaS = FFM_SA_S, kSaT = FFM_SA_T, kSaJ = 2 * kSaU;   // words per lane per step
-constexpr int kSaSmem = kSaS * kSaT * 16 * (2 * kSaJ + 1);                          // 16-B slots: data, then meta
+constexpr int kSaSmem = kSaS * kSaT * 16 * (2 * kSaJ);                               // 16-B data slots (own, leader)
+static_assert(kSaS == 2, "k_fused_small carries the in-flight step's meta in registers (one step ahead)");
 constexpr uint32_t kSaEnd = 1u << 31, kSaFirst = 1u << 30, kSaLast = 1u << 29, kSaCmp = 1u << 28;
 
 __device__ __forceinline__ void cp16(uint32_t dst, const uint8_t* src, uint64_t pol) {
@@ -1213,7 +1214,6 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
     // slot of word j of stage s (part 0 own, 1 leader); lanes interleaved so a warp's
     // 16-B accesses to one slot are 512 contiguous bytes (conflict-free)
     auto slot = [&](int s, int j, int part) { return sbase + (uint32_t)(((s * kSaJ + j) * 2 + part) * kSaT * 16); };
-    auto mslot = [&](int s) { return sbase + (uint32_t)((kSaS * kSaJ * 2 + s) * kSaT * 16); };
     uint64_t pol_own, pol_keep;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_own));
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
@@ -1236,9 +1236,12 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
         if (fi + noct < L.n_small) nd = sd32[8ull * (fi + noct) + g];
     }
     const int obase = threadIdx.x & 24;
+    // meta of the step a fetch issued: (bytes, record, word | flags), consumed one iteration later
+    uint32_t mn = 0, mr = 0, meta_z = kSaEnd;
     auto fetch = [&](int s) {
-        uint32_t meta_z = kSaEnd;
-        uint32_t mn = 0, mr = 0;
+        meta_z = kSaEnd;
+        mn = 0;
+        mr = 0;
         if (fi < L.n_small) {
             const uint32_t nw = (fn + 15) >> 4;
             const bool cmp = floff != ~0ull;
@@ -1287,8 +1290,6 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
                 if (fi + noct < L.n_small) nd = sd32[8ull * (fi + noct) + g];
             }
         }
-        asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(mslot(s)), "r"(mn), "r"(mr), "r"(meta_z), "r"(0u)
-                     : "memory");
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
 #pragma unroll 1
@@ -1311,11 +1312,9 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
     while (true) {
         // refill the stage consumed last iteration (its values were used, so read), then
         // wait for the oldest: S-1 steps stay in flight while this one is hashed
+        const uint32_t n = mn, r = mr, z = meta_z;   // the step fetched last iteration
         fetch(sf);
         asm volatile("cp.async.wait_group %0;" ::"n"(kSaS - 1) : "memory");
-        uint32_t m[4];
-        lds16(mslot(sc), m);
-        const uint32_t n = m[0], r = m[1], z = m[2];
         const bool done = (z & kSaEnd) != 0;
         if (__all_sync(0xFFFFFFFFu, done)) break;
         if (!done) {
