@@ -410,7 +410,7 @@ def run_ours(args):
 
 def run_online(args):
     """S8(f) #2 measurement: the log streamed through ffm_online_step in fixed windows
-    (FFM_FLAG_ONLINE: each append hashes its records on the hashing stream), against the
+    (FFM_FLAG_ONLINE; FFM_FLAG_APPEND_HASH: each append hashes its records on the hashing stream), against the
     batch run of the same log.  Per window size: median step latency (host wall clock of
     the synchronous ffm_online_step) and streamed throughput = payload / (sum of append +
     step times); appends snapshot device-resident payloads (D2D)."""
@@ -440,7 +440,10 @@ def run_online(args):
         torch.cuda.synchronize()
         batch_s = (time.perf_counter() - t) / args.steps
     rows = []
-    for w in [int(x) for x in args.online.split(",")]:
+    for (mode, append_hash), w in [(m, int(x)) for m in (("fused", False), ("append_hash", True))
+                                   for x in args.online.split(",")]:
+        # both modes are online logs (FFM_FLAG_ONLINE: appends upload their metadata);
+        # append_hash also hashes at append time (FFM_FLAG_APPEND_HASH)
         n_win = (lg.n + w - 1) // w
         if n_win > args.online_max_windows:          # latency only, over a bounded prefix
             n_win = args.online_max_windows
@@ -449,7 +452,7 @@ def run_online(args):
         ben = torch.empty(lg.n_sites, dtype=torch.int64, device=dev)
         got = np.empty(end, np.int64) if want is not None else None
         t_app, t_step = [], []
-        with ffm.FfmLog(lg.n_sites, online=True, **opts) as log:
+        with ffm.FfmLog(lg.n_sites, online=True, append_hash=append_hash, **opts) as log:
             for rep in range(2):                     # rep 0 warms up (allocations), rep 1 is measured
                 log.reset()
                 t_app.clear()
@@ -468,7 +471,7 @@ def run_online(args):
                     if got is not None and rep == 1:
                         got[a:e] = dup[:e - a].cpu().numpy()
         byts = int(lg.size[:end].sum())
-        row = {"window": w, "windows": len(t_step), "records": end, "payload_bytes": byts,
+        row = {"mode": mode, "window": w, "windows": len(t_step), "records": end, "payload_bytes": byts,
                "step_ms_median": round(statistics.median(t_step) * 1e3, 4),
                "step_ms_p90": round(float(np.percentile(t_step, 90)) * 1e3, 4),
                "append_ms_median": round(statistics.median(t_app) * 1e3, 4),
@@ -482,8 +485,10 @@ def run_online(args):
            "records": lg.n, "payload_bytes": lg.total_bytes, "n_scale": args.n_scale,
            "batch_ms": round(batch_s * 1e3, 4), "batch_gbs": round(lg.total_bytes / batch_s / 1e9, 2),
            "windows": rows,
-           "note": "host wall clock; appends snapshot device-resident payloads and queue their hashing "
-                   "(FFM_FLAG_ONLINE); each step is synchronous (labels in device memory)"}
+           "note": "host wall clock; appends snapshot device-resident payloads; mode fused: each step runs the "
+                   "fused round 0 on its window (batch record order built on the device); mode append_hash: "
+                   "appends queue the window's hashing (FFM_FLAG_APPEND_HASH), the step verifies two-pass; each step "
+                   "is synchronous (labels in device memory)"}
     print(json.dumps(out), flush=True)
 
 

@@ -69,10 +69,14 @@ enum { FFM_FLAG_TIMING = 1u,     /* record per-stage CUDA events (ffm_last_run_s
        FFM_FLAG_FUSED = 8u,      /* force the fused round 0 (no adaptation) */
        FFM_FLAG_NO_GRAPH = 16u,  /* launch every kernel directly instead of replaying the captured
                                     CUDA graph of a run (default: graph while the log is unchanged) */
-       FFM_FLAG_ONLINE = 32u     /* online mode (S8(f) #2): every append hashes its records right
-                                    away on a hashing stream that follows the staging copies, so the
-                                    next append's staging overlaps it; ffm_online_step then starts
-                                    from the hashes.  Without it a step hashes its window itself. */ };
+       FFM_FLAG_ONLINE = 32u,    /* online mode (S8(f) #2): every append uploads its records' metadata
+                                    right away (staging stream), so ffm_online_step starts from a
+                                    device-resident window; the step runs the fused round 0 on its
+                                    window (each byte read once) */
+       FFM_FLAG_APPEND_HASH = 64u /* with FFM_FLAG_ONLINE: every append also hashes its records on a
+                                    hashing stream that follows the staging copies (the next
+                                    append's staging overlaps it); the step then groups by the full
+                                    digests and re-reads the members to verify them (two-pass) */ };
 
 /* Caller-provided exchange transport of a sharded log (world > 1), used instead of the
    library's own NCCL communicator when NCCL cannot connect the ranks (e.g. several ranks
@@ -246,10 +250,12 @@ int ffm_fold_sites(ffm_log* log, const uint64_t* site_values, const uint32_t* si
  * The stored hashes are a persistent, insert-only device table of every exact class
  * seen so far (key of the full digest, size and channel -> the classes' representatives,
  * whose bytes stay in the HBM arena).  ffm_online_step labels every record appended since
- * the previous step (a window): H2..H4 on the window alone (hashed at append time with
- * FFM_FLAG_ONLINE), then each window class looks its key up in the table and is
- * byte-verified against the stored classes there; classes with no equal stored class
- * are inserted.  A step's work is O(window), never O(prior records) (the table is
+ * the previous step (a window): H1..H4 on the window alone -- by default the batch run's
+ * fused round 0 on the window in its batch record order (built on the device: every byte
+ * read once, leaders hashed, members compared); with FFM_FLAG_APPEND_HASH the appends hash
+ * their records and the step verifies two-pass -- then each window class looks its key up
+ * in the table and is byte-verified against the stored classes there; classes with no
+ * equal stored class are inserted.  A step's work is O(window), never O(prior records) (the table is
  * rehashed only when its capacity doubles).  Labels of earlier records never change, so
  * the concatenated windows equal ffm_dedup_run over the whole log, bit for bit.
  *   duplicate_of [window records] (host or device): gids, or -1

@@ -39,6 +39,7 @@ FFM_FLAG_TWO_PASS = 4
 FFM_FLAG_FUSED = 8
 FFM_FLAG_NO_GRAPH = 16
 FFM_FLAG_ONLINE = 32
+FFM_FLAG_APPEND_HASH = 64
 
 # every symbol include/ffm.h declares (checked by tests/test_abi.py)
 EXPORTS = ["ffm_config_init", "ffm_log_create", "ffm_log_append", "ffm_log_append_batch", "ffm_log_append_batch_ex",
@@ -316,7 +317,8 @@ class FfmLog:
                  digest_bits: int = 64, refine_bits: int = 64, chunk_bytes: int = 0, small_bytes: int = 0,
                  timing: bool = False, stream: int = 0, rank: int = 0, world: int = 1,
                  prefilter: bool = False, two_pass: bool = False, fused: bool = False,
-                 graph: bool = True, online: bool = False, nccl_id: bytes | None = None,
+                 graph: bool = True, online: bool = False, append_hash: bool = False,
+                 nccl_id: bytes | None = None,
                  comm: FfmCommOps | None = None):
         """world > 1 (collective): pass the world's nccl_id (ffm_nccl_unique_id) or a comm
         transport (FfmCommOps, e.g. sharded.HostComm)."""
@@ -328,7 +330,8 @@ class FfmLog:
         cfg.chunk_bytes, cfg.small_bytes = chunk_bytes, small_bytes
         cfg.flags = (FFM_FLAG_TIMING if timing else 0) | (FFM_FLAG_PREFILTER if prefilter else 0) | \
             (FFM_FLAG_TWO_PASS if two_pass else 0) | (FFM_FLAG_FUSED if fused else 0) | \
-            (0 if graph else FFM_FLAG_NO_GRAPH) | (FFM_FLAG_ONLINE if online else 0)
+            (0 if graph else FFM_FLAG_NO_GRAPH) | (FFM_FLAG_ONLINE if online else 0) | \
+            (FFM_FLAG_APPEND_HASH if append_hash else 0)
         cfg.stream = stream or None
         self._keep = (nccl_id, comm)     # alive while the library may use them
         if nccl_id is not None:

@@ -25,6 +25,7 @@ constexpr uint64_t kGatherMax = 1ull << 20;   // device / pinned payloads up to 
 
 struct LocalRun {
     uint64_t n_members, n_res_total, rounds, prefilter_rest;
+    uint64_t n_res0;     // round-0 residuals (kept in keep_res when asked)
     uint64_t n_reread;   // residual members whose bytes were compared again (not settled by difference lists)
     uint64_t n_overflow; // round-0 residuals whose difference list against their head overflowed
     bool two_pass;
@@ -144,7 +145,7 @@ void stage_host(ffm_log* L, const void* src, uint64_t size, uint64_t off) {
 // asynchronously while the next window fills the other half.  The bytes are snapshotted
 // (in the ring, or already in HBM) before the append returns (reading R11).
 // host threads of the pageable staging copies (at most 8: several ranks may share a node)
-int stage_threads() {
+[[maybe_unused]] int stage_threads() {   // (used in an OpenMP pragma)
     static const int t = std::max(1, std::min(8, omp_get_max_threads()));
     return t;
 }
@@ -401,6 +402,7 @@ void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* si
     for (uint64_t i = 0; i < n; ++i) {
         L->payload_bytes += sizes[i];
         L->n_large_chunks += large_chunks(L, sizes[i]);
+        L->n_small_recs += sizes[i] <= L->params.small_bytes;
     }
     L->arena_used = arena_end;
     ++L->epoch;
@@ -565,8 +567,48 @@ DevLog window_view(ffm_log* L, uint64_t a, uint64_t b, bool has_large, cudaStrea
     return D;
 }
 
+// An online window [a, b) in the batch record order (small records by size class, then
+// the large ones), built on the device (stable radix sort of 16-bit size-class keys):
+// the fused round 0 runs on it exactly as on a whole log.  n_small: small records in it.
+DevLog window_view_sorted(ffm_log* L, uint64_t a, uint64_t b, uint64_t n_small, cudaStream_t st,
+                          uint64_t& launches) {
+    DevLog D = window_view(L, a, b, true, st);   // (iota of >= b - a entries)
+    const uint64_t nw = b - a;
+    if (nw > L->word_cap) {
+        if (L->d_word) ck(cudaFree(L->d_word), "cudaFree");
+        if (L->d_wkeys) ck(cudaFree(L->d_wkeys), "cudaFree");
+        if (L->d_wtmp) ck(cudaFree(L->d_wtmp), "cudaFree");
+        L->d_word = nullptr;
+        L->d_wkeys = nullptr;
+        L->d_wtmp = nullptr;
+        const uint64_t c = std::max<uint64_t>(std::max<uint64_t>(nw, 2 * L->word_cap), 4096);
+        ck(cudaMalloc(&L->d_word, 2 * c * sizeof(uint32_t)), "cudaMalloc(window order)");
+        ck(cudaMalloc(&L->d_wkeys, 2 * c * sizeof(uint16_t)), "cudaMalloc(window keys)");
+        size_t tb = 0;
+        if (launch_window_order(nullptr, (uint32_t)c, L->params.small_bytes, nullptr, nullptr, nullptr, nullptr,
+                                nullptr, &tb, st) < 0)
+            throw CudaFail{cudaErrorUnknown, "window order temp size"};
+        L->wtmp_bytes = std::max<size_t>(tb, 256);
+        ck(cudaMalloc(&L->d_wtmp, L->wtmp_bytes), "cudaMalloc(window sort)");
+        L->word_cap = c;
+    }
+    uint32_t* order = L->d_word;
+    uint32_t* inv = L->d_word + L->word_cap;
+    size_t tb = L->wtmp_bytes;
+    const int k = launch_window_order(D.size, (uint32_t)nw, L->params.small_bytes, L->d_wkeys, L->d_iota, order, inv,
+                                      L->d_wtmp, &tb, st);
+    if (k < 0) throw CudaFail{cudaGetLastError(), "window order"};
+    launches += (uint64_t)k;
+    D.small_order = order;
+    D.order_pos = inv;
+    D.n_small = (uint32_t)n_small;
+    D.large_order = order + n_small;
+    D.n_large = (uint32_t)(nw - n_small);
+    return D;
+}
+
 // Online mode (S8(f) #2): the NH sums of records [a, b) into on_A / on_B (global record
-// index), on stream st -- at append time on the hashing stream (FFM_FLAG_ONLINE), else
+// index), on stream st -- at append time on the hashing stream (FFM_FLAG_APPEND_HASH), else
 // at the start of a step.
 void online_hash(ffm_log* L, uint64_t a, uint64_t b, cudaStream_t st, uint64_t& launches) {
     if (a >= b) return;
@@ -628,6 +670,7 @@ void ensure_online(ffm_log* L, uint64_t nw) {
     }
     if (nw > L->on_G_cap) {
         dev_alloc(L->on_G, nw);
+        dev_alloc(L->on_res, nw);
         L->on_G_cap = nw;
     }
 }
@@ -645,7 +688,7 @@ void ensure_online(ffm_log* L, uint64_t nw) {
 // the caller copies again).
 LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& launches, bool label, int64_t* d_dup,
                    bool prefilter = false, const std::function<void()>* pre_sync = nullptr, bool prehashed = false,
-                   int64_t* h_spec = nullptr) {
+                   int64_t* h_spec = nullptr, bool window = false, uint32_t* keep_res = nullptr) {
     const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
     const uint64_t n = D.n;
     Work& W = L->work;
@@ -686,10 +729,14 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         // H2 group-by (round 0): two-pass -- every payload by its full digest; fused -- small
         // payloads by their first 32 bytes, large ones by their first-chunk digest
         uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(2 * std::max<uint64_t>(n, 1)));
-        LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, two_pass ? -1 : 0, W.res[0], s));
+        // fused round 0 with labels: the lookup also writes the speculative labels and the
+        // per-site sums (H5 + H6 need no pass after H3 unless H3 finds residuals)
+        const bool lab0 = label && !two_pass && D.n && label_fused_ok(W, L->params, ns);
+        LCHK(launch_group(D, W, L->params, nullptr, D.n, cap, two_pass ? -1 : 0, W.res[0], s, false, lab0 ? ns : 0,
+                          lab0 ? d_dup : nullptr));
         if (h_spec) {
             // speculative labels, copied to the host on the copy stream during H3
-            LCHK(launch_spec_label(D, W, d_dup, s));
+            if (!lab0) LCHK(launch_spec_label(D, W, d_dup, s));
             ck(cudaEventRecord(L->copy_ev[0], s), "event");
             ck(cudaStreamWaitEvent(L->copy_stream, L->copy_ev[0], 0), "fork copy");
             ck(cudaMemcpyAsync(h_spec, d_dup, (uint64_t)D.n * sizeof(int64_t), cudaMemcpyDeviceToHost,
@@ -714,6 +761,10 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
             LCHK(launch_fused_small(D, W, L->params, W.res[0], side));
             if (timing) ck(cudaEventRecord(L->ev[8], side), "event");
             ck(cudaEventRecord(L->fork_ev[3], side), "event");
+            // per-site sums of the lookup's block rows, off the small pass's critical path
+            if (lab0)
+                LCHK(launch_site_reduce(W.label_part, W.label_cpart, label_hist_rows(L->params.num_sms), ns, W.ben,
+                                        W.cnt, s));
             if (n_large)
                 LCHK(launch_fused(D, W, L->params, n_large, prefilter, W.res[0], s, timing ? L->ev[16] : nullptr,
                                   timing ? L->ev[17] : nullptr));
@@ -721,14 +772,14 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         }
         if (timing) ck(cudaEventRecord(L->ev[3], s), "event");
         // H5 + H6 (speculative: valid unless H3 found residuals)
-        if (label) LCHK(launch_label(D, W, L->params, ns, h_spec ? nullptr : d_dup, s));
+        if (label && !lab0) LCHK(launch_label(D, W, L->params, ns, h_spec ? nullptr : d_dup, s));
         if (h_spec) ck(cudaStreamWaitEvent(s, L->copy_ev[1], 0), "join copy");
         if (timing) ck(cudaEventRecord(L->ev[4], s), "event");
         ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
     };
     // (per-stage timing needs directly recorded events: FFM_FLAG_TIMING runs launch directly)
     // (online windows move their view every step: recapturing would cost more than it saves)
-    const bool graph = !prehashed && !(L->cfg.flags & FFM_FLAG_NO_GRAPH) && !timing;
+    const bool graph = !prehashed && !window && !(L->cfg.flags & FFM_FLAG_NO_GRAPH) && !timing;
     if (graph) {
         // replay a CUDA graph of segment A while the log, its buffers and the run mode are
         // unchanged: one launch instead of ~30 (launch-bound small logs)
@@ -768,6 +819,11 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
     R.prefilter_rest = (uint64_t)L->h_counters[4] | ((uint64_t)L->h_counters[5] << 32);
     uint64_t nres = L->h_counters[0];
     R.n_res_total = nres;
+    R.n_res0 = nres;
+    // (the caller fixes up work it queued on the speculative labels: keep the list, the
+    // resolve rounds reuse the residual buffers)
+    if (nres && keep_res)
+        ck(cudaMemcpyAsync(keep_res, W.res[0], nres * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s), "keep residuals");
     if (nres) {
         // H4 collision resolution: exact classes among the residual members
         if (timing) ck(cudaEventRecord(L->ev[6], s), "event");
@@ -1281,10 +1337,14 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
         push_meta(L, n, sites, sizes, durs, gids, channels, offs, end);
         L->digests_valid = false;
         if (L->cfg.flags & FFM_FLAG_ONLINE) {
-            // online mode: hash the new records now, on the hashing stream after their
-            // staging copies -- the next append's staging overlaps this hashing
+            // online mode: the new records' metadata goes to the device now (the step
+            // starts from a resident window)
             ring_flush(L);
             upload_meta_arrays(L);
+        }
+        if ((L->cfg.flags & FFM_FLAG_ONLINE) && (L->cfg.flags & FFM_FLAG_APPEND_HASH)) {
+            // append-time hashing: hash the new records now, on the hashing stream after
+            // their staging copies -- the next append's staging overlaps this hashing
             ensure_work(L, L->h_size.size());
             ck(cudaEventRecord(L->fork_ev[2], L->stage_stream), "event");
             ck(cudaStreamWaitEvent(L->hash_stream, L->fork_ev[2], 0), "wait staging");
@@ -1464,22 +1524,50 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
         uint64_t launches = 0;
         LocalRun R{};
         if (nw) {
-            // H1 (unless the appends hashed already, FFM_FLAG_ONLINE)
-            const uint64_t h0 = std::max(L->online_hashed, w0);
-            if (h0 < n) online_hash(L, h0, n, s, launches);
-            L->online_hashed = n;
-            uint64_t n_large = 0;
-            for (uint64_t i = w0; i < n; ++i) n_large += large_chunks(L, L->h_size[i]);
-            const DevLog D = window_view(L, w0, n, n_large != 0, s);
-            // H2..H4 on the window: exact window classes (the NH sums are the window's slice
-            // of on_A / on_B)
-            {
+            const uint64_t n_small_w = L->n_small_recs - L->online_small0;
+            const uint64_t n_large = L->n_large_chunks - L->online_chunks0;
+            const bool fused = L->online_hashed <= w0;
+            ensure_online(L, nw);
+            const bool dup_dev = is_device_ptr(dup_out);
+            int64_t* d_dup = dup_dev ? dup_out : W.dup;
+            const uint64_t* wA = fused ? W.accA : L->on_A + w0;
+            const uint64_t* wB = fused ? W.accB : L->on_B + w0;
+            DevLog D;
+            // the window's classes against the stored classes of all earlier windows
+            // ("compared to the stored hashes from prior transfers"), queued on
+            // the round-0 (speculative) labels before run_local's host sync: one sync per
+            // step unless H4 finds residuals (then the fix-up below)
+            const std::function<void()> match = [&]() {
+                LCHK(launch_online_window(D, W, wA, wB, L->otab, L->params, ns, L->on_G, d_dup, L->online_ben,
+                                          L->online_cnt, s));
+                if (!dup_dev)
+                    ck(cudaMemcpyAsync(dup_out, d_dup, nw * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
+                ck(cudaMemcpyAsync(L->h_counters + 2, L->otab.count, sizeof(uint32_t), cudaMemcpyDeviceToHost, s),
+                   "D2H");
+                if (ben_out)
+                    ck(cudaMemcpyAsync(ben_out, L->online_ben, ns * sizeof(uint64_t), cudaMemcpyDefault, s),
+                       "copy ben");
+            };
+            if (fused) {
+                // fused window (default): the batch round 0 on the window in its batch
+                // record order -- each byte read once (leaders hashed, members compared with
+                // their prefix-group leader), full digests for the class representatives
+                D = window_view_sorted(L, w0, n, n_small_w, s, launches);
+                R = run_local(L, D, n_large, launches, false, nullptr, false, &match, false, nullptr, true, L->on_res);
+            } else {
+                // hashed at append time (FFM_FLAG_APPEND_HASH): H2..H4 from the window's NH
+                // sums (the slice of on_A / on_B), two-pass, every member byte-verified
+                const uint64_t h0 = std::max(L->online_hashed, w0);
+                if (h0 < n) online_hash(L, h0, n, s, launches);
+                L->online_hashed = n;
+                D = window_view(L, w0, n, n_large != 0, s);
                 uint64_t* keepA = W.accA;
                 uint64_t* keepB = W.accB;
                 W.accA = L->on_A + w0;
                 W.accB = L->on_B + w0;
                 try {
-                    R = run_local(L, D, n_large, launches, false, nullptr, false, nullptr, true);
+                    R = run_local(L, D, n_large, launches, false, nullptr, false, &match, true, nullptr, true,
+                                  L->on_res);
                 } catch (...) {
                     W.accA = keepA;
                     W.accB = keepB;
@@ -1488,24 +1576,30 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
                 W.accA = keepA;
                 W.accB = keepB;
             }
-            // each window class against the stored classes of all earlier windows ("compared
-            // to the stored hashes from prior transfers"); new classes are stored
-            ensure_online(L, nw);
-            const bool dup_dev = is_device_ptr(dup_out);
-            int64_t* d_dup = dup_dev ? dup_out : W.dup;
-            LCHK(launch_online_window(D, W, L->on_A + w0, L->on_B + w0, L->otab, L->params, ns, L->on_G, d_dup,
-                                      L->online_ben, L->online_cnt, s));
-            if (!dup_dev)
-                ck(cudaMemcpyAsync(dup_out, d_dup, nw * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
-            ck(cudaMemcpyAsync(L->h_counters + 2, L->otab.count, sizeof(uint32_t), cudaMemcpyDeviceToHost, s),
-               "D2H");
+            if (R.n_res0) {
+                // H4 changed the labels of the round-0 residuals: match their classes and
+                // correct their labels and the cumulative sums
+                LCHK(launch_online_fix(D, W, wA, wB, L->otab, L->params, L->on_res, (uint32_t)R.n_res0, L->on_G,
+                                       d_dup, L->online_ben, L->online_cnt, s));
+                if (!dup_dev)
+                    ck(cudaMemcpyAsync(dup_out, d_dup, nw * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
+                ck(cudaMemcpyAsync(L->h_counters + 2, L->otab.count, sizeof(uint32_t), cudaMemcpyDeviceToHost, s),
+                   "D2H");
+                if (ben_out)
+                    ck(cudaMemcpyAsync(ben_out, L->online_ben, ns * sizeof(uint64_t), cudaMemcpyDefault, s),
+                       "copy ben");
+                sync_run(L, "online fix-up sync");
+            }
+        } else {
+            if (ben_out)
+                ck(cudaMemcpyAsync(ben_out, L->online_ben, ns * sizeof(uint64_t), cudaMemcpyDefault, s), "copy ben");
+            sync_run(L, "online sync");
         }
-        if (ben_out)
-            ck(cudaMemcpyAsync(ben_out, L->online_ben, ns * sizeof(uint64_t), cudaMemcpyDefault, s), "copy ben");
-        sync_run(L, "online sync");
         ck(cudaGetLastError(), "online step");
         if (nw) L->online_np = L->h_counters[2];
         L->online_done = n;
+        L->online_small0 = L->n_small_recs;
+        L->online_chunks0 = L->n_large_chunks;
         fill_stats(L, R, launches, false);
         L->stats.n_records = nw;
         L->stats.host_syncs = L->n_syncs;
@@ -1562,6 +1656,7 @@ int ffm_log_reset(ffm_log* L) {
     L->h_gid.clear();
     L->h_chan.clear();
     L->payload_bytes = L->n_large_chunks = L->last_gid = 0;
+    L->n_small_recs = L->online_small0 = L->online_chunks0 = 0;
     L->any_gid = false;
     L->d_meta_n = 0;
     L->d_order_n = 0;

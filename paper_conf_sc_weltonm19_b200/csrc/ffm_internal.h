@@ -147,8 +147,12 @@ int launch_prefix(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_combine(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
 int launch_fused(const DevLog& L, Work& W, const Params& P, uint64_t n_units, bool prefilter, uint32_t* res_out,
                  cudaStream_t st, cudaEvent_t ev_a, cudaEvent_t ev_b);
+// round 0 with label_sites != 0 (label_fused_ok): the leader lookup also writes the
+// speculative labels (label_dup, if non-null) and the per-site sums (W.ben / W.cnt)
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
-                 uint64_t cap, int round, uint32_t* res_out, cudaStream_t st, bool use_diff = false);
+                 uint64_t cap, int round, uint32_t* res_out, cudaStream_t st, bool use_diff = false,
+                 uint32_t label_sites = 0, int64_t* label_dup = nullptr);
+bool label_fused_ok(const Work& W, const Params& P, uint32_t n_sites);
 int launch_verify(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list,
                   uint32_t* res_out, uint64_t vitem_cap, cudaStream_t st, cudaStream_t side, cudaEvent_t ev_fork,
                   cudaEvent_t ev_join);
@@ -168,6 +172,9 @@ int launch_online_rehash(OnlineTable& T, uint32_t np, uint64_t digest_mask, cuda
 int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, const uint64_t* accB,
                          OnlineTable& T, const Params& P, uint32_t n_sites, uint64_t* G, int64_t* dup_out,
                          uint64_t* ben, uint64_t* cnt, cudaStream_t st);
+int launch_online_fix(const DevLog& L, const Work& W, const uint64_t* accA, const uint64_t* accB, OnlineTable& T,
+                      const Params& P, const uint32_t* list, uint32_t n_list, uint64_t* G, int64_t* dup_out,
+                      uint64_t* ben, uint64_t* cnt, cudaStream_t st);
 int launch_merge_label(const DevLog& L, Work& W, ShardWork& S, const Params& P, uint32_t n_sites, int64_t* dup_out,
                        cudaStream_t st);
 int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uint64_t gen, uint64_t n,
@@ -175,6 +182,11 @@ int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uin
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t st);
+// The batch record order of a log view of n records (small ones by 32-byte block count,
+// largest first, stable; then the large ones in index order) and its inverse, on the
+// device: keys [2n] scratch, iota = 0..n-1.  tmp == nullptr: *tmp_bytes = space needed.
+int launch_window_order(const uint64_t* size, uint32_t n, uint32_t small_bytes, uint16_t* keys, const uint32_t* iota,
+                        uint32_t* order, uint32_t* inv, void* tmp, size_t* tmp_bytes, cudaStream_t st);
 int launch_iota(uint32_t* a, uint32_t n, cudaStream_t st);
 int launch_spec_label(const DevLog& L, Work& W, int64_t* dup_out, cudaStream_t st);
 int launch_digest_fill(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
@@ -285,11 +297,22 @@ struct ffm_log {
     uint64_t* on_B = nullptr;
     uint64_t on_cap = 0;
     uint64_t* on_G = nullptr;        // [window] global leader gid of each window class
+    uint32_t* on_res = nullptr;      // [window] the step's round-0 residuals (speculative labels fix-up)
     uint64_t on_G_cap = 0;
     uint64_t* online_ben = nullptr;  // [2 * n_sites] cumulative per-site benefit | duplicate counts
     uint64_t* online_cnt = nullptr;  //   (= online_ben + n_sites)
     uint32_t* d_iota = nullptr;      // identity record order of online windows (0, 1, 2, ...)
     uint64_t iota_cap = 0;
+    // fused online windows: the window's batch record order (small by size class, then
+    // large), built on the device -- [order | inverse] and the sort's key / temp space
+    uint32_t* d_word = nullptr;
+    uint16_t* d_wkeys = nullptr;      // [2 * cap]
+    void* d_wtmp = nullptr;
+    size_t wtmp_bytes = 0;
+    uint64_t word_cap = 0;
+    uint64_t n_small_recs = 0;        // records <= small_bytes appended so far
+    uint64_t online_small0 = 0;       // n_small_recs / n_large_chunks at online_done
+    uint64_t online_chunks0 = 0;
 
     // folded grouping scratch
     void* fold_buf = nullptr;

@@ -441,45 +441,142 @@ __global__ void k_leader(DevLog L, Work W, const uint32_t* __restrict__ list, ui
 // out chunk-major, (chunk c, position p) at lstart[head] + c * (gcount[head] + 1) + p,
 // with the leader itself at p = 0 -- the leader's chunk c is read from HBM once, by
 // its own hashing unit, and re-read from L2 by every member comparing against it.
+// record r's part of the round-0 leader lookup; returns its table leader (the min local
+// index of its group: the candidate of a member, r itself for a leader)
+__device__ __forceinline__ uint32_t leader0_record(const DevLog& L, Work& W, uint32_t r, uint32_t small_bytes,
+                                                   uint32_t* __restrict__ res_out) {
+    const uint32_t i = L.order_pos[r];
+    const uint32_t ld = table_leader(W, W.slot[r]);
+    W.leader[r] = ld;
+    const uint64_t sz = L.size[r];
+    const bool same = L.size[ld] == sz && L.chan[ld] == L.chan[r];
+    if (ld != r) {
+        if (!same) {
+            W.eq[r] = 0;            // key collision across sizes / channels: not equal
+            W.mis[r] = 0;
+            res_out[atomicAdd(&W.counters[0], 1u)] = r;
+        } else {
+            W.eq[r] = 1;
+            W.mis[r] = ~0ull;
+        }
+    }
+    if (sz > small_bytes) {
+        uint32_t head = r, p = 0;
+        if (ld != r && same) {
+            head = ld;
+            p = 1u + atomicAdd(&W.gcount[ld], 1u);
+        }
+        W.fhead[r] = head;
+        W.pos[r] = p;
+    } else {
+        const uint64_t off = L.off[r], loff = (ld != r && same) ? L.off[ld] : ~0ull;
+        W.sdesc[2ull * i] = make_uint4((uint32_t)off, (uint32_t)(off >> 32), (uint32_t)loff, (uint32_t)(loff >> 32));
+        W.sdesc[2ull * i + 1] = make_uint4((uint32_t)sz, r, 0, 0);
+    }
+    return ld;
+}
+
 __global__ void k_leader0(DevLog L, Work W, uint32_t n, uint32_t small_bytes, uint32_t* __restrict__ res_out) {
     // thread r: record r (gid order: its metadata loads and per-record writes coalesce);
     // a small record's compare descriptor lands at its position i in k_fused_small's
     // size-class order
     const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
     bool member = false;
-    if (r < n) {
-        const uint32_t i = L.order_pos[r];
-        const uint32_t ld = table_leader(W, W.slot[r]);
-        W.leader[r] = ld;
-        const uint64_t sz = L.size[r];
-        const bool same = L.size[ld] == sz && L.chan[ld] == L.chan[r];
-        if (ld != r) {
-            member = true;
-            if (!same) {
-                W.eq[r] = 0;            // key collision across sizes / channels: not equal
-                W.mis[r] = 0;
-                res_out[atomicAdd(&W.counters[0], 1u)] = r;
-            } else {
-                W.eq[r] = 1;
-                W.mis[r] = ~0ull;
-            }
-        }
-        if (sz > small_bytes) {
-            uint32_t head = r, p = 0;
-            if (ld != r && same) {
-                head = ld;
-                p = 1u + atomicAdd(&W.gcount[ld], 1u);
-            }
-            W.fhead[r] = head;
-            W.pos[r] = p;
-        } else {
-            const uint64_t off = L.off[r], loff = (ld != r && same) ? L.off[ld] : ~0ull;
-            W.sdesc[2ull * i] = make_uint4((uint32_t)off, (uint32_t)(off >> 32), (uint32_t)loff, (uint32_t)(loff >> 32));
-            W.sdesc[2ull * i + 1] = make_uint4((uint32_t)sz, r, 0, 0);
-        }
-    }
+    if (r < n) member = leader0_record(L, W, r, small_bytes, res_out) != r;
     unsigned b = __ballot_sync(0xFFFFFFFFu, member);
     if ((threadIdx.x & 31) == 0 && b) atomicAdd(&W.counters[1], (uint32_t)__popc(b));
+}
+
+// Round-0 leader lookup with H5 + H6 folded in: each member's table leader is its label
+// unless H3 finds a difference (a residual: the labels and sums are then recomputed after
+// resolution), so the labels (dup_out, if given) and the per-block site histograms of
+// k_label_hist are produced here, from registers the lookup already holds -- no separate
+// pass over the records after H3.  Persistent 1024-thread blocks (one per SM) over the
+// records in gid order; k_site_reduce sums the rows.
+__global__ void __launch_bounds__(1024) k_leader0_label(DevLog L, Work W, uint32_t n, uint32_t small_bytes,
+                                                        uint32_t* __restrict__ res_out, uint32_t n_sites,
+                                                        int64_t* __restrict__ dup_out, uint64_t* __restrict__ part,
+                                                        uint32_t* __restrict__ cpart) {
+    extern __shared__ unsigned long long sben[];
+    uint32_t* scnt = (uint32_t*)(sben + n_sites);
+    for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) {
+        sben[s] = 0;
+        scnt[s] = 0;
+    }
+    __syncthreads();
+    // kL0U records per thread per step, each stage's loads of all of them in flight
+    // together (slot -> table leader -> the leader's metadata are three dependent
+    // latencies per record)
+    constexpr int kL0U = 2;
+    const uint32_t stride = gridDim.x * blockDim.x;
+    uint32_t members = 0;
+    for (uint32_t r0 = blockIdx.x * blockDim.x; r0 < n; r0 += kL0U * stride) {   // block-uniform trip count
+        uint32_t r[kL0U], ld[kL0U];
+#pragma unroll
+        for (int u = 0; u < kL0U; ++u) {
+            r[u] = r0 + threadIdx.x + u * stride;
+            ld[u] = r[u] < n ? W.slot[r[u]] : 0;
+        }
+#pragma unroll
+        for (int u = 0; u < kL0U; ++u) ld[u] = r[u] < n ? table_leader(W, ld[u]) : r[u];
+        uint64_t sz[kL0U], szl[kL0U], ch[kL0U], chl[kL0U];
+#pragma unroll
+        for (int u = 0; u < kL0U; ++u) {
+            const bool ok = r[u] < n;
+            sz[u] = ok ? L.size[r[u]] : 0;
+            ch[u] = ok ? L.chan[r[u]] : 0;
+            szl[u] = ok ? L.size[ld[u]] : 0;
+            chl[u] = ok ? L.chan[ld[u]] : 0;
+        }
+#pragma unroll
+        for (int u = 0; u < kL0U; ++u) {
+            if (r[u] >= n) continue;
+            const uint32_t rr = r[u], l = ld[u];
+            W.leader[rr] = l;
+            const bool member = l != rr;
+            const bool same = szl[u] == sz[u] && chl[u] == ch[u];
+            if (member) {
+                if (!same) {
+                    W.eq[rr] = 0;            // key collision across sizes / channels: not equal
+                    W.mis[rr] = 0;
+                    res_out[atomicAdd(&W.counters[0], 1u)] = rr;
+                } else {
+                    W.eq[rr] = 1;
+                    W.mis[rr] = ~0ull;
+                }
+            }
+            if (sz[u] > small_bytes) {
+                uint32_t head = rr, p = 0;
+                if (member && same) {
+                    head = l;
+                    p = 1u + atomicAdd(&W.gcount[l], 1u);
+                }
+                W.fhead[rr] = head;
+                W.pos[rr] = p;
+            } else {
+                const uint32_t i = L.order_pos[rr];
+                const uint64_t off = L.off[rr], loff = (member && same) ? L.off[l] : ~0ull;
+                W.sdesc[2ull * i] = make_uint4((uint32_t)off, (uint32_t)(off >> 32), (uint32_t)loff, (uint32_t)(loff >> 32));
+                W.sdesc[2ull * i + 1] = make_uint4((uint32_t)sz[u], rr, 0, 0);
+            }
+            if (dup_out) dup_out[rr] = member ? (int64_t)L.gid[l] : -1;
+            if (member) {
+                const uint32_t site = L.site[rr];
+                atomicAdd(&sben[site], (unsigned long long)L.dur[rr]);
+                atomicAdd(&scnt[site], 1u);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kL0U; ++u) members += __popc(__ballot_sync(0xFFFFFFFFu, r[u] < n && ld[u] != r[u]));
+    }
+    if ((threadIdx.x & 31) == 0 && members) atomicAdd(&W.counters[1], members);
+    __syncthreads();
+    uint64_t* row = part + (uint64_t)blockIdx.x * n_sites;
+    uint32_t* crow = cpart + (uint64_t)blockIdx.x * n_sites;
+    for (uint32_t s = threadIdx.x; s < n_sites; s += blockDim.x) {
+        row[s] = sben[s];
+        crow[s] = scnt[s];
+    }
 }
 
 // With FFM_FLAG_PREFILTER a leader whose fused group has no member has a unique
@@ -1763,7 +1860,7 @@ uint64_t fx_entry_cap(uint64_t n_large_chunks, uint32_t chunk_bytes) {
 }
 
 int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list, uint32_t n_list, uint64_t cap,
-                 int round, uint32_t* res_out, cudaStream_t st, bool use_diff) {
+                 int round, uint32_t* res_out, cudaStream_t st, bool use_diff, uint32_t label_sites, int64_t* label_dup) {
     if (n_list == 0) return 0;
     int k = 0;
     if (round > 0) {
@@ -1777,7 +1874,15 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
     k_group_insert<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, cap - 1, P.digest_mask, round,
                                                         P.small_bytes);
     FFM_LAUNCH_CHECK();
-    if (round == 0)
+    if (round == 0 && label_sites) {
+        // H5 + H6 folded into the lookup (speculative; label_fused_ok decided it fits)
+        if (!smem_configured((const void*)k_leader0_label, P.max_smem)) return -1;
+        const uint32_t rows = label_hist_rows(P.num_sms);
+        k_leader0_label<<<rows, 1024, label_smem_bytes(label_sites), st>>>(
+            L, W, n_list, P.small_bytes, res_out, label_sites, label_dup, W.label_part, W.label_cpart);
+        FFM_LAUNCH_CHECK();
+        return k + 2;   // (the caller launches k_site_reduce over the rows: launch_site_reduce)
+    } else if (round == 0)
         k_leader0<<<blocks_for(n_list), 256, 0, st>>>(L, W, n_list, P.small_bytes, res_out);
     else if (round < 0)
         k_leader<<<blocks_for(n_list), 256, 0, st>>>(L, W, nullptr, n_list, P.small_bytes, P.chunk_bytes, res_out, 0);
@@ -1845,6 +1950,10 @@ int launch_site_reduce(const uint64_t* part, const uint32_t* cpart, uint32_t row
 }
 
 size_t label_smem_bytes(uint32_t n_sites) { return (size_t)n_sites * (sizeof(uint64_t) + sizeof(uint32_t)); }
+
+bool label_fused_ok(const Work& W, const Params& P, uint32_t n_sites) {
+    return W.label_part != nullptr && label_smem_bytes(n_sites) <= (size_t)P.max_smem;
+}
 
 int launch_label(const DevLog& L, Work& W, const Params& P, uint32_t n_sites, int64_t* dup_out, cudaStream_t st) {
     if (L.n == 0) {
@@ -1952,6 +2061,35 @@ int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t
     k_invert<<<blocks_for(n), 256, 0, st>>>(order, n, inv);
     FFM_LAUNCH_CHECK();
     return 1;
+}
+
+__global__ void k_window_keys(const uint64_t* __restrict__ size, uint32_t n, uint32_t small_bytes,
+                              uint16_t* __restrict__ keys) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) {
+        const uint64_t sz = size[i];
+        keys[i] = sz <= small_bytes ? (uint16_t)((sz + 31) / 32 + 1) : (uint16_t)0;
+    }
+}
+
+int launch_window_order(const uint64_t* size, uint32_t n, uint32_t small_bytes, uint16_t* keys, const uint32_t* iota,
+                        uint32_t* order, uint32_t* inv, void* tmp, size_t* tmp_bytes, cudaStream_t st) {
+    int bits = 1;
+    while ((1u << bits) <= (small_bytes + 31) / 32 + 1) ++bits;
+    if (!tmp) {
+        return cub::DeviceRadixSort::SortPairsDescending(nullptr, *tmp_bytes, keys, keys + n, iota, order, (int)n, 0,
+                                                         bits) == cudaSuccess ? 0 : -1;
+    }
+    if (n == 0) return 0;
+    k_window_keys<<<blocks_for(n), 256, 0, st>>>(size, n, small_bytes, keys);
+    FFM_LAUNCH_CHECK();
+    // stable: equal block counts keep index order, the large records (key 0) come last
+    if (cub::DeviceRadixSort::SortPairsDescending(tmp, *tmp_bytes, keys, keys + n, iota, order, (int)n, 0, bits, st) !=
+        cudaSuccess)
+        return -1;
+    k_invert<<<blocks_for(n), 256, 0, st>>>(order, n, inv);
+    FFM_LAUNCH_CHECK();
+    return 3;
 }
 
 int launch_zero_counters(Work& W, cudaStream_t st) {

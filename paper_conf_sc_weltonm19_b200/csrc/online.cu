@@ -6,14 +6,16 @@
 // open addressing on the group key of (full digest, size, channel) -> a chain of class
 // representatives in an insert-only pool (gid, arena offset, size, channel, digest).
 // A step labels one window of new records:
-//   1. the window's NH sums were computed at append time on the staging stream
-//      (FFM_FLAG_ONLINE), else at the start of the step;
-//   2. H2-H4 on the window alone -> exact window classes (two-pass round 0 without H1);
-//   3. k_online_match: each window class representative looks its key up in the table
-//      and byte-compares the chained prior representatives of its size / channel /
-//      digest (their bytes stay resident in the HBM arena) -- at most one prior class
-//      can be equal, so the chain order does not matter; a class with no equal stored
-//      class is inserted by the same kernel;
+//   1-2. H1-H4 on the window alone -> exact window classes: by default the batch run's fused
+//      round 0 on the window in its batch record order (built on the device by
+//      launch_window_order); with FFM_FLAG_ONLINE the NH sums were computed at append time
+//      on the hashing stream and the step runs the two-pass round 0 without H1;
+//   3. k_online_probe (thread per record): each window class representative looks its key
+//      up in the table -- absent: the class is new and stored at once; present:
+//      k_online_cmp (8 lanes per listed class) byte-compares the chained prior
+//      representatives of its size / channel / digest (their bytes stay resident in the
+//      HBM arena) -- at most one prior class can be equal, so the chain order does not
+//      matter; a class with no equal stored class is stored by the same kernel;
 //   4. k_online_label: labels (gids) and the cumulative per-site benefit / counts.
 // The table is never rebuilt by a step; it is rehashed only when its capacity doubles.
 #include "digest.cuh"
@@ -44,29 +46,107 @@ __device__ __forceinline__ void online_link(OnlineTable& T, uint64_t key, uint32
     T.pool[idx].next = atomicExch(&T.head[h], idx);
 }
 
-// One 8-lane group per window class representative r (leader[r] == r), grid-stride:
-// look its key up, byte-compare the chained stored classes of its size / channel /
-// digest (32-byte blocks per lane, stopping at the first differing step); with no equal
-// stored class, r's class is stored right away.  Concurrent inserts are safe: a window's
-// classes are pairwise distinct, so a walker that misses (or meets) a class being
-// inserted by another window representative loses nothing, and an entry is complete
-// before the CAS that publishes it.
-__global__ void __launch_bounds__(256) k_online_match(DevLog L, const uint32_t* __restrict__ leader,
+// Store window class r as a new class (its entry is complete before the CAS that
+// publishes it on its key's chain).
+// kFence: chain walkers may run concurrently (k_online_cmp) -- the entry must be visible
+// before the head CAS; k_online_probe has no concurrent walkers (the kernel boundary orders
+// its stores before any walk).
+// ni: the entry's pool index (atomicAdd on T.count, warp-aggregated by the caller)
+template <bool kFence>
+__device__ __forceinline__ void online_store(OnlineTable& T, const DevLog& L, uint32_t r, uint64_t key, uint64_t dig,
+                                             uint32_t ni) {
+    OnlineRep e;
+    e.gid = L.gid[r];
+    e.off = L.off[r];
+    e.size = L.size[r];
+    e.chan = L.chan[r];
+    e.dig = dig;
+    e.pad = 0;
+    uint64_t hh = key & T.mask;
+    while (true) {
+        unsigned long long prev =
+            atomicCAS((unsigned long long*)&T.key[hh], (unsigned long long)kEmptyKey, (unsigned long long)key);
+        if (prev == kEmptyKey || prev == key) break;
+        hh = (hh + 1) & T.mask;
+    }
+    uint32_t old = *reinterpret_cast<volatile uint32_t*>(&T.head[hh]);
+    while (true) {
+        e.next = old;
+        T.pool[ni] = e;
+        if (kFence) __threadfence();
+        const uint32_t seen = atomicCAS(&T.head[hh], old, ni);
+        if (seen == old) break;
+        old = seen;
+    }
+}
+
+// Thread per window record: a window class representative r (leader[r] == r) looks its
+// key up; with the key absent from the table no stored class can equal it and r's class
+// is stored right away (G[r] = its own gid); with the key present r goes to the compare
+// list for k_online_cmp.  Concurrent stores are safe: a window's classes are pairwise
+// distinct, so a class that finds a key stored by another window class of the same
+// step only pays a compare that fails.
+// (list != nullptr: only the listed records -- the residual fix-up of a step)
+__global__ void __launch_bounds__(256) k_online_probe(DevLog L, const uint32_t* __restrict__ leader,
                                                       const uint64_t* __restrict__ accA,
                                                       const uint64_t* __restrict__ accB, OnlineTable T,
-                                                      uint64_t digest_mask, uint64_t refine_mask,
-                                                      uint64_t* __restrict__ G) {
+                                                      uint64_t digest_mask, uint64_t* __restrict__ G,
+                                                      uint32_t* __restrict__ cmp_list, uint32_t* __restrict__ n_cmp,
+                                                      const uint32_t* __restrict__ list, uint32_t n_list) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = threadIdx.x & 31;
+    uint32_t r = 0;
+    bool rep = false;
+    if (i < n_list) {
+        r = list ? list[i] : i;
+        rep = leader[r] == r;
+    }
+    uint64_t key = 0, dig = 0;
+    bool present = false;
+    if (rep) {
+        const uint64_t n = L.size[r];
+        dig = finalize_digest(accA[r], accB[r], n);
+        key = group_key(dig, n, digest_mask, L.chan[r]);
+        present = T.key[online_probe(T, key)] == key;
+    }
+    // one atomic per warp for each of the two appends (list / pool)
+    const unsigned below = (1u << lane) - 1u;
+    const unsigned mp = __ballot_sync(0xFFFFFFFFu, present);
+    const unsigned ms = __ballot_sync(0xFFFFFFFFu, rep && !present);
+    uint32_t bp = 0, bs = 0;
+    if (lane == 0) {
+        if (mp) bp = atomicAdd(n_cmp, (uint32_t)__popc(mp));
+        if (ms) bs = atomicAdd(T.count, (uint32_t)__popc(ms));
+    }
+    bp = __shfl_sync(0xFFFFFFFFu, bp, 0);
+    bs = __shfl_sync(0xFFFFFFFFu, bs, 0);
+    if (present) {
+        cmp_list[bp + __popc(mp & below)] = r;
+    } else if (rep) {
+        G[r] = L.gid[r];
+        online_store<false>(T, L, r, key, dig, bs + __popc(ms & below));
+    }
+}
+
+// One 8-lane group per listed window class r, grid-stride: byte-compare the chained
+// stored classes of its size / channel / digest (32-byte blocks per lane, stopping at the
+// first differing step) -- at most one can be equal; with none, r's class is stored.
+__global__ void __launch_bounds__(256) k_online_cmp(DevLog L, const uint64_t* __restrict__ accA,
+                                                    const uint64_t* __restrict__ accB, OnlineTable T,
+                                                    uint64_t digest_mask, uint64_t refine_mask,
+                                                    uint64_t* __restrict__ G, const uint32_t* __restrict__ cmp_list,
+                                                    const uint32_t* __restrict__ n_cmp) {
     const int g = threadIdx.x & 7;
     const unsigned omask = 0xFFu << (threadIdx.x & 24);
     const uint32_t noct = (gridDim.x * blockDim.x) >> 3;
-    for (uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 3; r < L.n; r += noct) {
-        if (leader[r] != r) continue;   // (uniform per octet)
+    const uint32_t m = *n_cmp;
+    for (uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 3; i < m; i += noct) {
+        const uint32_t r = cmp_list[i];
         const uint64_t n = L.size[r], chan = L.chan[r];
         const uint64_t dig = finalize_digest(accA[r], accB[r], n);
         const uint64_t key = group_key(dig, n, digest_mask, chan);
         const uint64_t h = online_probe(T, key);
-        uint32_t idx = kNoRep;
-        if (T.key[h] == key) idx = *reinterpret_cast<volatile uint32_t*>(&T.head[h]);
+        uint32_t idx = *reinterpret_cast<volatile uint32_t*>(&T.head[h]);
         uint64_t gl = L.gid[r];
         bool found = false;
         const uint8_t* px = L.arena + L.off[r];
@@ -98,33 +178,29 @@ __global__ void __launch_bounds__(256) k_online_match(DevLog L, const uint32_t* 
         }
         if (g == 0) {
             G[r] = gl;
-            if (!found) {   // a new class: stored now
-                const uint32_t ni = atomicAdd(T.count, 1u);
-                OnlineRep e;
-                e.gid = gl;
-                e.off = L.off[r];
-                e.size = n;
-                e.chan = chan;
-                e.dig = dig;
-                e.pad = 0;
-                uint64_t hh = key & T.mask;
-                while (true) {
-                    unsigned long long prev = atomicCAS((unsigned long long*)&T.key[hh], (unsigned long long)kEmptyKey,
-                                                        (unsigned long long)key);
-                    if (prev == kEmptyKey || prev == key) break;
-                    hh = (hh + 1) & T.mask;
-                }
-                uint32_t old = *reinterpret_cast<volatile uint32_t*>(&T.head[hh]);
-                while (true) {
-                    e.next = old;
-                    T.pool[ni] = e;
-                    __threadfence();
-                    const uint32_t seen = atomicCAS(&T.head[hh], old, ni);
-                    if (seen == old) break;
-                    old = seen;
-                }
-            }
+            if (!found) online_store<true>(T, L, r, key, dig, atomicAdd(T.count, 1u));
         }
+    }
+}
+
+// Residual fix-up of a step whose labels went out speculatively (before its H4): a
+// residual r was labelled a duplicate of its round-0 candidate and counted in the
+// cumulative per-site sums; take that back and apply its final label (its class was
+// matched against the table by k_online_probe / k_online_cmp over the residual list).
+__global__ void k_online_fix(DevLog L, const uint32_t* __restrict__ leader, const uint64_t* __restrict__ G,
+                             const uint32_t* __restrict__ list, uint32_t n_list, int64_t* __restrict__ dup_out,
+                             uint64_t* __restrict__ ben, uint64_t* __restrict__ cnt) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n_list) return;
+    const uint32_t r = list[i];
+    const uint32_t s = L.site[r];
+    const uint64_t dur = L.dur[r];
+    const uint64_t g = G[leader[r]];
+    const int64_t d = g == L.gid[r] ? -1 : (int64_t)g;
+    dup_out[r] = d;
+    if (d < 0) {   // (integer sums mod 2^64: subtracting is adding the complement)
+        atomicAdd((unsigned long long*)&ben[s], (unsigned long long)(0 - dur));
+        atomicAdd((unsigned long long*)&cnt[s], ~0ull);
     }
 }
 
@@ -194,8 +270,15 @@ int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, c
                          OnlineTable& T, const Params& P, uint32_t n_sites, uint64_t* G, int64_t* dup_out,
                          uint64_t* ben, uint64_t* cnt, cudaStream_t st) {
     if (L.n == 0) return 0;
-    k_online_match<<<std::min<uint32_t>(blocks_for((uint64_t)L.n * 8), (uint32_t)P.num_sms * 8), 256, 0, st>>>(
-        L, W.leader, accA, accB, T, P.digest_mask, P.refine_mask, G);
+    // the compare list reuses the residual buffer res[1] (free after the window's H4);
+    // its length lives in counters[12]
+    uint32_t* n_cmp = W.counters + 12;
+    if (cudaMemsetAsync(n_cmp, 0, sizeof(uint32_t), st) != cudaSuccess) return -1;
+    k_online_probe<<<blocks_for(L.n), 256, 0, st>>>(L, W.leader, accA, accB, T, P.digest_mask, G, W.res[1], n_cmp,
+                                                    nullptr, L.n);
+    ONLINE_CHECK();
+    k_online_cmp<<<std::min<uint32_t>(blocks_for((uint64_t)L.n * 8), (uint32_t)P.num_sms * 8), 256, 0, st>>>(
+        L, accA, accB, T, P.digest_mask, P.refine_mask, G, W.res[1], n_cmp);
     ONLINE_CHECK();
     const size_t smem = label_smem_bytes(n_sites);
     const uint32_t grid = std::min<uint32_t>(blocks_for(L.n, 1024), (uint32_t)P.num_sms);
@@ -206,7 +289,26 @@ int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, c
         k_online_label<false><<<grid, 1024, 0, st>>>(L, W.leader, G, n_sites, dup_out, ben, cnt);
     }
     ONLINE_CHECK();
-    return 2;
+    return 3;
+}
+
+// After H4 of a step launched with speculative labels: the residual records (list) get
+// their classes matched against the table and their labels / sums corrected.
+int launch_online_fix(const DevLog& L, const Work& W, const uint64_t* accA, const uint64_t* accB, OnlineTable& T,
+                      const Params& P, const uint32_t* list, uint32_t n_list, uint64_t* G, int64_t* dup_out,
+                      uint64_t* ben, uint64_t* cnt, cudaStream_t st) {
+    if (n_list == 0) return 0;
+    uint32_t* n_cmp = W.counters + 12;
+    if (cudaMemsetAsync(n_cmp, 0, sizeof(uint32_t), st) != cudaSuccess) return -1;
+    k_online_probe<<<blocks_for(n_list), 256, 0, st>>>(L, W.leader, accA, accB, T, P.digest_mask, G, W.res[1], n_cmp,
+                                                       list, n_list);
+    ONLINE_CHECK();
+    k_online_cmp<<<std::min<uint32_t>(blocks_for((uint64_t)n_list * 8), (uint32_t)P.num_sms * 8), 256, 0, st>>>(
+        L, accA, accB, T, P.digest_mask, P.refine_mask, G, W.res[1], n_cmp);
+    ONLINE_CHECK();
+    k_online_fix<<<blocks_for(n_list), 256, 0, st>>>(L, W.leader, G, list, n_list, dup_out, ben, cnt);
+    ONLINE_CHECK();
+    return 3;
 }
 
 }  // namespace ffm

@@ -37,17 +37,22 @@ def _online(ffm, lg, cuts, **kw):
     return np.concatenate(dups), bens, batch_d, batch_b
 
 
+MODES = {"step": {}, "online": {"online": True}, "append_hash": {"online": True, "append_hash": True}}
+
+
 @pytest.mark.parametrize("k,ns,ss", [(1, 0.5, 0.25), (2, 0.01, 1.0), (3, 0.03, 1 / 32), (4, 0.1, 1 / 64),
                                      (5, 0.003, 1 / 32)])
 @pytest.mark.parametrize("digest_bits", [64, 0])
-@pytest.mark.parametrize("online", [True, False])
-def test_online_equals_batch_and_oracle(ffm, k, ns, ss, digest_bits, online):
-    """online=True hashes at append time (FFM_FLAG_ONLINE); False hashes in the step."""
+@pytest.mark.parametrize("mode", list(MODES))
+def test_online_equals_batch_and_oracle(ffm, k, ns, ss, digest_bits, mode):
+    """step: the step uploads and processes its window (fused round 0); online: appends
+    upload their metadata (FFM_FLAG_ONLINE), the step runs the fused round 0; append_hash:
+    appends also hash (FFM_FLAG_APPEND_HASH), the step verifies two-pass."""
     lg = loggen.gen_config(k, n_scale=ns, size_scale=ss)
     rng = np.random.default_rng(k)
     cuts = sorted(set(rng.integers(1, lg.n, 6).tolist()))
     want_d, want_b = oracle.dedup(lg)
-    got_d, bens, bd, bb = _online(ffm, lg, cuts, digest_bits=digest_bits, chunk_bytes=4096, online=online)
+    got_d, bens, bd, bb = _online(ffm, lg, cuts, digest_bits=digest_bits, chunk_bytes=4096, **MODES[mode])
     np.testing.assert_array_equal(got_d, want_d)
     np.testing.assert_array_equal(bd, want_d)
     np.testing.assert_array_equal(bb, want_b)
@@ -78,25 +83,27 @@ def test_online_with_channels(ffm):
 
 
 @pytest.mark.parametrize("window", [1, 64, 4096])
-def test_online_fixed_windows_grow_the_table(ffm, window):
+@pytest.mark.parametrize("mode", ["online", "append_hash"])
+def test_online_fixed_windows_grow_the_table(ffm, window, mode):
     """Fixed-size windows over a config-2-shaped log (many small transfers):
     the persistent table grows (rehash on doubling) across steps; the result never changes."""
     lg = loggen.gen_config(2, n_scale=0.004 if window == 1 else 0.02)
     cuts = list(range(window, lg.n, window))
     want_d, want_b = oracle.dedup(lg)
-    got_d, bens, bd, bb = _online(ffm, lg, cuts, online=True)
+    got_d, bens, bd, bb = _online(ffm, lg, cuts, **MODES[mode])
     np.testing.assert_array_equal(got_d, want_d)
     np.testing.assert_array_equal(bens[-1][1], want_b)
     np.testing.assert_array_equal(bd, want_d)
 
 
-def test_online_after_reset_and_forced_collisions_across_windows(ffm):
+@pytest.mark.parametrize("mode", ["online", "append_hash"])
+def test_online_after_reset_and_forced_collisions_across_windows(ffm, mode):
     """ffm_log_reset empties the stored classes too; with digest_bits = refine_bits = 0
     every stored class of a size shares one chain (byte compares decide)."""
     lg = loggen.gen_config(3, n_scale=0.02, size_scale=1 / 64)
     want_d, want_b = oracle.dedup(lg)
     ptrs = lg.payload_ptrs()
-    with ffm.FfmLog(lg.n_sites, digest_bits=0, refine_bits=0, online=True) as log:
+    with ffm.FfmLog(lg.n_sites, digest_bits=0, refine_bits=0, **MODES[mode]) as log:
         for rep in range(2):
             dups = []
             for a in range(0, lg.n, 37):
@@ -109,9 +116,10 @@ def test_online_after_reset_and_forced_collisions_across_windows(ffm):
             log.reset()
 
 
-def test_online_device_payloads_and_outputs(ffm):
-    """Appends of device-resident payloads hashed at append time, labels written to
-    device memory (the streaming shape of bench.py --online)."""
+@pytest.mark.parametrize("mode", ["online", "append_hash"])
+def test_online_device_payloads_and_outputs(ffm, mode):
+    """Appends of device-resident payloads (hashed at append time with append_hash), labels
+    written to device memory (the streaming shape of bench.py --online)."""
     import torch
     lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 32)
     want_d, want_b = oracle.dedup(lg)
@@ -120,7 +128,7 @@ def test_online_device_payloads_and_outputs(ffm):
     dup = torch.empty(lg.n, dtype=torch.int64, device="cuda")
     ben = torch.empty(lg.n_sites, dtype=torch.int64, device="cuda")
     got = []
-    with ffm.FfmLog(lg.n_sites, online=True, chunk_bytes=4096) as log:
+    with ffm.FfmLog(lg.n_sites, chunk_bytes=4096, **MODES[mode]) as log:
         for a in range(0, lg.n, 777):
             e = min(lg.n, a + 777)
             log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e], payload_kind=ffm.FFM_PAYLOAD_DEVICE)

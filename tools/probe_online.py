@@ -11,15 +11,20 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import loggen  # noqa: E402
 import paper_conf_sc_weltonm19_b200 as ffm  # noqa: E402
 
+if os.environ.get("PROBE_LIB"):
+    ffm.set_library_path(os.environ["PROBE_LIB"])
+
 w = int(sys.argv[1]) if len(sys.argv) > 1 else 65536
 nwin = int(sys.argv[2]) if len(sys.argv) > 2 else 8
+append_hash = (sys.argv[3] == "append_hash") if len(sys.argv) > 3 else True
+timing = len(sys.argv) > 4 and sys.argv[4] == "timing"
 lg = loggen.gen_config(2)
 lg.materialize(nthreads=0)
 content = torch.from_numpy(lg.buf).cuda()
 ptrs = (lg.c_off[lg.content] + np.uint64(content.data_ptr())).astype(np.uint64)
 dup = torch.empty(w, dtype=torch.int64, device="cuda")
 ben = torch.empty(lg.n_sites, dtype=torch.int64, device="cuda")
-with ffm.FfmLog(lg.n_sites, online=True, arena_bytes=lg.total_bytes + 128 * lg.n + (1 << 20), max_records=lg.n) as log:
+with ffm.FfmLog(lg.n_sites, online=True, append_hash=append_hash, timing=timing, arena_bytes=lg.total_bytes + 128 * lg.n + (1 << 20), max_records=lg.n) as log:
     for rep in range(2):
         log.reset()
         ta, ts = [], []
@@ -33,5 +38,8 @@ with ffm.FfmLog(lg.n_sites, online=True, arena_bytes=lg.total_bytes + 128 * lg.n
             t2 = time.perf_counter()
             ta.append(t1 - t0)
             ts.append(t2 - t1)
+            if timing and rep == 1:
+                st = log.stats()
+                print({k: round(v, 4) for k, v in st.items() if k.startswith("ms_") or k in ("host_syncs", "kernel_launches", "n_residual", "resolve_rounds")}, flush=True)
         print(f"rep {rep} window {w}: append+hash median {np.median(ta) * 1e3:.3f} ms, step median {np.median(ts) * 1e3:.3f} ms "
               f"stats {log.stats()['host_syncs']} syncs", flush=True)
