@@ -121,6 +121,7 @@ void ensure_arena(ffm_log* L, uint64_t need) {
     L->arena = na;
     L->arena_cap = nc;
     ++L->epoch;
+    ++L->bufgen;
     ++L->arena_gen;   // peers of a sharded log re-map it at their next run
 }
 
@@ -313,6 +314,7 @@ void upload_meta_arrays(ffm_log* L) {
     dev_grow(L->d_gid, cap, n, keep, L->stage_stream);
     cap = c0;
     dev_grow(L->d_chan, cap, n, keep, L->stage_stream);
+    if (cap != L->d_meta_cap) ++L->bufgen;
     L->d_meta_cap = cap;
     uint64_t a = L->d_meta_n, k = n - a;
     cudaStream_t s = L->stage_stream;
@@ -422,6 +424,7 @@ void ensure_work(ffm_log* L, uint64_t n) {
     }
     if (n > W.n_cap || W.accA == nullptr) {
         ++L->epoch;
+        ++L->bufgen;
         uint64_t c = std::max<uint64_t>(n, 1024);
         dev_alloc(W.accA, c);
         dev_alloc(W.accB, c);
@@ -455,11 +458,13 @@ void ensure_work(ffm_log* L, uint64_t n) {
     }
     if (tcap > W.t_cap) {
         ++L->epoch;
+        ++L->bufgen;
         dev_alloc(W.tkey, tcap);
         W.t_cap = tcap;
     }
     if (L->n_large_chunks > W.hitem_cap) {
         ++L->epoch;
+        ++L->bufgen;
         uint64_t c = L->n_large_chunks + L->n_large_chunks / 4 + 64;
         dev_alloc(W.hitems, c);
         dev_alloc(W.hpart, 2 * c);
@@ -468,12 +473,14 @@ void ensure_work(ffm_log* L, uint64_t n) {
     const uint64_t fcap = fx_entry_cap(L->n_large_chunks, L->params.chunk_bytes);
     if (fcap > W.fitem_cap) {
         ++L->epoch;
+        ++L->bufgen;
         const uint64_t c = fcap + fcap / 4;
         dev_alloc(W.fitems, 2 * c);   // 32-byte descriptors
         W.fitem_cap = c;
     }
     if (L->cfg.n_sites > W.site_cap) {
         ++L->epoch;
+        ++L->bufgen;
         dev_alloc(W.ben, 2 * (uint64_t)L->cfg.n_sites);   // [benefit | duplicate counts]: one all-reduce
         W.cnt = W.ben + L->cfg.n_sites;
         if (label_smem_bytes(L->cfg.n_sites) <= (uint64_t)L->params.max_smem) {
@@ -550,6 +557,7 @@ DevLog window_view(ffm_log* L, uint64_t a, uint64_t b, bool has_large, cudaStrea
         ck(cudaMalloc(&L->d_iota, c * sizeof(uint32_t)), "cudaMalloc(iota)");
         if (launch_iota(L->d_iota, (uint32_t)c, st) < 0) throw CudaFail{cudaGetLastError(), "iota"};
         L->iota_cap = c;
+        ++L->bufgen;
     }
     DevLog D = dev_view(L);
     D.off += a;
@@ -568,43 +576,64 @@ DevLog window_view(ffm_log* L, uint64_t a, uint64_t b, bool has_large, cudaStrea
 }
 
 // An online window [a, b) in the batch record order (small records by size class, then
-// the large ones), built on the device (stable radix sort of 16-bit size-class keys):
-// the fused round 0 runs on it exactly as on a whole log.  n_small: small records in it.
-DevLog window_view_sorted(ffm_log* L, uint64_t a, uint64_t b, uint64_t n_small, cudaStream_t st,
-                          uint64_t& launches) {
+// the large ones), its metadata gathered into fixed buffers: window_view_sorted sizes the
+// buffers and returns the view; queue_window_order queues the gather and the order build
+// (a stable device radix sort of 16-bit size-class keys).  n_small: small records in it.
+DevLog window_view_sorted(ffm_log* L, uint64_t a, uint64_t b, uint64_t n_small, cudaStream_t st) {
     DevLog D = window_view(L, a, b, true, st);   // (iota of >= b - a entries)
     const uint64_t nw = b - a;
     if (nw > L->word_cap) {
-        if (L->d_word) ck(cudaFree(L->d_word), "cudaFree");
-        if (L->d_wkeys) ck(cudaFree(L->d_wkeys), "cudaFree");
-        if (L->d_wtmp) ck(cudaFree(L->d_wtmp), "cudaFree");
+        ck(cudaStreamSynchronize(st), "window buffers");
+        for (void* p : {(void*)L->d_word, (void*)L->d_wkeys, L->d_wtmp, (void*)L->wmeta.off, (void*)L->wmeta.size,
+                        (void*)L->wmeta.dur, (void*)L->wmeta.gid, (void*)L->wmeta.chan, (void*)L->wmeta.site})
+            if (p) ck(cudaFree(p), "cudaFree");
         L->d_word = nullptr;
         L->d_wkeys = nullptr;
         L->d_wtmp = nullptr;
+        L->wmeta = WinMeta{};
         const uint64_t c = std::max<uint64_t>(std::max<uint64_t>(nw, 2 * L->word_cap), 4096);
         ck(cudaMalloc(&L->d_word, 2 * c * sizeof(uint32_t)), "cudaMalloc(window order)");
         ck(cudaMalloc(&L->d_wkeys, 2 * c * sizeof(uint16_t)), "cudaMalloc(window keys)");
+        ck(cudaMalloc(&L->wmeta.off, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
+        ck(cudaMalloc(&L->wmeta.size, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
+        ck(cudaMalloc(&L->wmeta.dur, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
+        ck(cudaMalloc(&L->wmeta.gid, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
+        ck(cudaMalloc(&L->wmeta.chan, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
+        ck(cudaMalloc(&L->wmeta.site, c * sizeof(uint32_t)), "cudaMalloc(window meta)");
         size_t tb = 0;
-        if (launch_window_order(nullptr, (uint32_t)c, L->params.small_bytes, nullptr, nullptr, nullptr, nullptr,
-                                nullptr, &tb, st) < 0)
+        if (launch_window_order(D, nullptr, (uint32_t)c, L->wmeta, L->params.small_bytes, nullptr, nullptr, nullptr,
+                                nullptr, nullptr, &tb, st) < 0)
             throw CudaFail{cudaErrorUnknown, "window order temp size"};
         L->wtmp_bytes = std::max<size_t>(tb, 256);
         ck(cudaMalloc(&L->d_wtmp, L->wtmp_bytes), "cudaMalloc(window sort)");
         L->word_cap = c;
+        ++L->bufgen;
     }
-    uint32_t* order = L->d_word;
-    uint32_t* inv = L->d_word + L->word_cap;
-    size_t tb = L->wtmp_bytes;
-    const int k = launch_window_order(D.size, (uint32_t)nw, L->params.small_bytes, L->d_wkeys, L->d_iota, order, inv,
-                                      L->d_wtmp, &tb, st);
-    if (k < 0) throw CudaFail{cudaGetLastError(), "window order"};
-    launches += (uint64_t)k;
-    D.small_order = order;
-    D.order_pos = inv;
+    if (!L->d_wa) {
+        ck(cudaMalloc(&L->d_wa, sizeof(uint64_t)), "cudaMalloc(window start)");
+        ck(cudaMallocHost(&L->h_wa, sizeof(uint64_t)), "cudaMallocHost(window start)");
+    }
+    D.off = L->wmeta.off;
+    D.size = L->wmeta.size;
+    D.site = L->wmeta.site;
+    D.dur = L->wmeta.dur;
+    D.gid = L->wmeta.gid;
+    D.chan = L->wmeta.chan;
+    D.small_order = L->d_word;
+    D.order_pos = L->d_word + L->word_cap;
     D.n_small = (uint32_t)n_small;
-    D.large_order = order + n_small;
+    D.large_order = L->d_word + n_small;
     D.n_large = (uint32_t)(nw - n_small);
     return D;
+}
+
+void queue_window_order(ffm_log* L, const DevLog& D, cudaStream_t st, uint64_t& launches) {
+    size_t tb = L->wtmp_bytes;
+    const int k = launch_window_order(dev_view(L), L->d_wa, D.n, L->wmeta, L->params.small_bytes, L->d_wkeys,
+                                      L->d_iota, const_cast<uint32_t*>(D.small_order),
+                                      const_cast<uint32_t*>(D.order_pos), L->d_wtmp, &tb, st);
+    if (k < 0) throw CudaFail{cudaGetLastError(), "window order"};
+    launches += (uint64_t)k;
 }
 
 // Online mode (S8(f) #2): the NH sums of records [a, b) into on_A / on_B (global record
@@ -654,6 +683,7 @@ void ensure_online(ffm_log* L, uint64_t nw) {
         if (T.pool) ck(cudaFree(T.pool), "cudaFree");
         T.pool = np;
         L->pool_cap = c;
+        ++L->bufgen;
     }
     if (2 * need > T.mask + 1 || !T.key) {
         const uint64_t cap = std::max<uint64_t>(1024, pow2_at_least(4 * need));
@@ -665,6 +695,7 @@ void ensure_online(ffm_log* L, uint64_t nw) {
         ck(cudaMalloc(&T.key, cap * sizeof(uint64_t)), "cudaMalloc(online table)");
         ck(cudaMalloc(&T.head, cap * sizeof(uint32_t)), "cudaMalloc(online table)");
         T.mask = cap - 1;
+        ++L->bufgen;
         if (launch_online_rehash(T, (uint32_t)L->online_np, L->params.digest_mask, s) < 0)
             throw CudaFail{cudaGetLastError(), "online rehash"};
     }
@@ -672,6 +703,7 @@ void ensure_online(ffm_log* L, uint64_t nw) {
         dev_alloc(L->on_G, nw);
         dev_alloc(L->on_res, nw);
         L->on_G_cap = nw;
+        ++L->bufgen;
     }
 }
 
@@ -688,7 +720,9 @@ void ensure_online(ffm_log* L, uint64_t nw) {
 // the caller copies again).
 LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& launches, bool label, int64_t* d_dup,
                    bool prefilter = false, const std::function<void()>* pre_sync = nullptr, bool prehashed = false,
-                   int64_t* h_spec = nullptr, bool window = false, uint32_t* keep_res = nullptr) {
+                   int64_t* h_spec = nullptr, bool window = false, uint32_t* keep_res = nullptr,
+                   GraphSlot* wslot = nullptr, const uint64_t* wextra = nullptr,
+                   const std::function<void()>* pre_a = nullptr) {
     const bool timing = (L->cfg.flags & FFM_FLAG_TIMING) != 0;
     const uint64_t n = D.n;
     Work& W = L->work;
@@ -778,19 +812,29 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         ck(cudaMemcpyAsync(L->h_counters, W.counters, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
     };
     // (per-stage timing needs directly recorded events: FFM_FLAG_TIMING runs launch directly)
-    // (online windows move their view every step: recapturing would cost more than it saves)
-    const bool graph = !prehashed && !window && !(L->cfg.flags & FFM_FLAG_NO_GRAPH) && !timing;
+    // An online window (window) is captured only with a slot of its own (wslot): the
+    // captured step then spans pre_a (the window's metadata gather and order build),
+    // segment A and pre_sync (the match against the stored classes); its key is the
+    // caller's (wextra: buffer generation, window size, outputs), not the log's epoch.
+    const bool graph = !prehashed && (!window || wslot) && !(L->cfg.flags & FFM_FLAG_NO_GRAPH) && !timing;
+    const bool in_graph_sync = graph && window;
+    auto body = [&]() {
+        if (pre_a) (*pre_a)();
+        segment_a();
+        if (in_graph_sync && pre_sync) (*pre_sync)();
+    };
     if (graph) {
         // replay a CUDA graph of segment A while the log, its buffers and the run mode are
         // unchanged: one launch instead of ~30 (launch-bound small logs)
-        const GraphKey key{L->epoch, d_dup, h_spec, two_pass, prefilter, timing};
-        if (!L->graph_exec || !(key == L->graph_key)) {
-            if (L->graph_exec) cudaGraphExecDestroy(L->graph_exec);
-            L->graph_exec = nullptr;
+        GraphSlot& G = window ? *wslot : L->graph;
+        GraphKey key{window ? ~0ull : L->epoch, d_dup, h_spec, two_pass, prefilter, timing};
+        if (wextra)
+            for (int i = 0; i < 4; ++i) key.extra[i] = wextra[i];
+        if (!G.exec || !(key == G.key)) {
             uint64_t before = launches;
             ck(cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed), "begin capture");
             try {
-                segment_a();
+                body();
             } catch (...) {
                 cudaGraph_t g = nullptr;
                 cudaStreamEndCapture(s, &g);
@@ -800,19 +844,31 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
             }
             cudaGraph_t g = nullptr;
             ck(cudaStreamEndCapture(s, &g), "end capture");
-            cudaError_t e = cudaGraphInstantiate(&L->graph_exec, g, 0);
+            // same topology (e.g. the next window of another size): update the executable
+            // graph in place, much cheaper than instantiating it again
+            cudaGraphExecUpdateResultInfo info;
+            cudaError_t e = cudaErrorUnknown;
+            if (G.exec) {
+                e = cudaGraphExecUpdate(G.exec, g, &info);
+                if (e != cudaSuccess) {
+                    cudaGetLastError();
+                    cudaGraphExecDestroy(G.exec);
+                    G.exec = nullptr;
+                }
+            }
+            if (!G.exec) e = cudaGraphInstantiate(&G.exec, g, 0);
             cudaGraphDestroy(g);
             ck(e, "graph instantiate");
-            L->graph_key = key;
-            L->graph_launches = launches - before;
+            G.key = key;
+            G.launches = launches - before;
             launches = before;
         }
-        ck(cudaGraphLaunch(L->graph_exec, s), "graph launch");
-        launches += L->graph_launches;
+        ck(cudaGraphLaunch(G.exec, s), "graph launch");
+        launches += G.launches;
     } else {
-        segment_a();
+        body();
     }
-    if (pre_sync) (*pre_sync)();
+    if (pre_sync && !in_graph_sync) (*pre_sync)();
     sync_run(L, "run sync");
     R.n_members = L->h_counters[1];
     R.two_pass = two_pass;
@@ -1551,9 +1607,21 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
             if (fused) {
                 // fused window (default): the batch round 0 on the window in its batch
                 // record order -- each byte read once (leaders hashed, members compared with
-                // their prefix-group leader), full digests for the class representatives
-                D = window_view_sorted(L, w0, n, n_small_w, s, launches);
-                R = run_local(L, D, n_large, launches, false, nullptr, false, &match, false, nullptr, true, L->on_res);
+                // their prefix-group leader), full digests for the class representatives.
+                // The whole step (gather + order, segment A, match) is one captured CUDA
+                // graph, replayed for the next window of the same size while no buffer
+                // moved; the window's start reaches it through a device word.
+                D = window_view_sorted(L, w0, n, n_small_w, s);
+                *L->h_wa = w0;
+                ck(cudaMemcpyAsync(L->d_wa, L->h_wa, sizeof(uint64_t), cudaMemcpyHostToDevice, s), "window start");
+                const std::function<void()> order = [&]() { queue_window_order(L, D, s, launches); };
+                // (captured copies need device or pinned host outputs)
+                const bool capt = (dup_dev || is_pinned_host(dup_out)) &&
+                                  (!ben_out || is_device_ptr(ben_out) || is_pinned_host(ben_out));
+                const uint64_t extra[4] = {L->bufgen, nw, n_small_w | (n_large << 32),
+                                           (uint64_t)(uintptr_t)dup_out ^ ((uint64_t)(uintptr_t)ben_out << 1)};
+                R = run_local(L, D, n_large, launches, false, nullptr, false, &match, false, nullptr, true, L->on_res,
+                              capt ? &L->wgraph : nullptr, extra, &order);
             } else {
                 // hashed at append time (FFM_FLAG_APPEND_HASH): H2..H4 from the window's NH
                 // sums (the slice of on_A / on_B), two-pass, every member byte-verified
@@ -1678,7 +1746,7 @@ int ffm_log_reset(ffm_log* L) {
     }
     L->digests_valid = false;
     L->prefer_two_pass = false;
-    ++L->epoch;
+    ++L->epoch;   // (no buffer moved: bufgen stays, captured window steps stay valid)
     memset(&L->stats, 0, sizeof(L->stats));
     return FFM_OK;
 }
@@ -1698,7 +1766,8 @@ int ffm_log_destroy(ffm_log* L) {
     free_shard(L->shard);
     if (L->fold_buf) cudaFree(L->fold_buf);
     void* op[] = {L->otab.key, L->otab.head, L->otab.pool, L->otab.count, L->on_A, L->on_B, L->on_G,
-                  L->online_ben, L->d_iota};
+                  L->on_res, L->online_ben, L->d_iota, L->d_word, L->d_wkeys, L->d_wtmp, L->d_wa, L->wmeta.off,
+                  L->wmeta.size, L->wmeta.dur, L->wmeta.gid, L->wmeta.chan, L->wmeta.site};
     for (void* p : op)
         if (p) cudaFree(p);
     for (void* p : L->peer_ptr)
@@ -1715,6 +1784,7 @@ int ffm_log_destroy(ffm_log* L) {
     for (auto e : L->ev)
         if (e) cudaEventDestroy(e);
     if (L->h_counters) cudaFreeHost(L->h_counters);
+    if (L->h_wa) cudaFreeHost(L->h_wa);
     if (L->stage_stream) cudaStreamDestroy(L->stage_stream);
     if (L->side_stream) cudaStreamDestroy(L->side_stream);
     if (L->hash_stream) {
@@ -1727,7 +1797,8 @@ int ffm_log_destroy(ffm_log* L) {
         if (e) cudaEventDestroy(e);
     for (auto e : L->fork_ev)
         if (e) cudaEventDestroy(e);
-    if (L->graph_exec) cudaGraphExecDestroy(L->graph_exec);
+    if (L->graph.exec) cudaGraphExecDestroy(L->graph.exec);
+    if (L->wgraph.exec) cudaGraphExecDestroy(L->wgraph.exec);
     if (L->own_stream && L->stream) cudaStreamDestroy(L->stream);
     cudaGetLastError();
     delete L;

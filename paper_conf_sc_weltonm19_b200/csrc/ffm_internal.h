@@ -127,6 +127,17 @@ struct OnlineTable {
     uint64_t mask = 0;
 };
 
+// The metadata of an online window, gathered into fixed buffers (so that the captured
+// step of a window replays for the next window of the same size).
+struct WinMeta {
+    uint64_t* off = nullptr;
+    uint64_t* size = nullptr;
+    uint64_t* dur = nullptr;
+    uint64_t* gid = nullptr;
+    uint64_t* chan = nullptr;
+    uint32_t* site = nullptr;
+};
+
 struct Params {
     uint64_t digest_mask;
     uint64_t refine_mask;
@@ -185,8 +196,11 @@ int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t
 // The batch record order of a log view of n records (small ones by 32-byte block count,
 // largest first, stable; then the large ones in index order) and its inverse, on the
 // device: keys [2n] scratch, iota = 0..n-1.  tmp == nullptr: *tmp_bytes = space needed.
-int launch_window_order(const uint64_t* size, uint32_t n, uint32_t small_bytes, uint16_t* keys, const uint32_t* iota,
-                        uint32_t* order, uint32_t* inv, void* tmp, size_t* tmp_bytes, cudaStream_t st);
+// The window [*d_a, *d_a + n) of the log L: its metadata gathered into wm, then its
+// batch record order.
+int launch_window_order(const DevLog& L, const uint64_t* d_a, uint32_t n, const WinMeta& wm, uint32_t small_bytes,
+                        uint16_t* keys, const uint32_t* iota, uint32_t* order, uint32_t* inv, void* tmp,
+                        size_t* tmp_bytes, cudaStream_t st);
 int launch_iota(uint32_t* a, uint32_t n, cudaStream_t st);
 int launch_spec_label(const DevLog& L, Work& W, int64_t* dup_out, cudaStream_t st);
 int launch_digest_fill(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
@@ -206,11 +220,21 @@ struct GraphKey {
     const void* dup = nullptr;
     const void* hdup = nullptr;   // pinned host duplicate_of of the speculative D2H (or null)
     bool two_pass = false, prefilter = false, timing = false;
+    uint64_t extra[4] = {0, 0, 0, 0};   // online windows: what else the captured step depends on
     bool operator==(const GraphKey& o) const {
         return epoch == o.epoch && dup == o.dup && hdup == o.hdup && two_pass == o.two_pass &&
-               prefilter == o.prefilter && timing == o.timing;
+               prefilter == o.prefilter && timing == o.timing && extra[0] == o.extra[0] &&
+               extra[1] == o.extra[1] && extra[2] == o.extra[2] && extra[3] == o.extra[3];
     }
 };
+
+// A captured CUDA graph and what it was captured for.
+struct GraphSlot {
+    cudaGraphExec_t exec = nullptr;
+    GraphKey key;
+    uint64_t launches = 0;
+};
+
 
 // The opaque handle.
 struct ffm_log {
@@ -229,9 +253,9 @@ struct ffm_log {
     bool host_ptr_ok = false;      // kernels may dereference registered host pointers
     bool prefer_two_pass = false;  // adaptive round 0 (see run_local)
     uint64_t epoch = 0;            // bumped whenever records or device buffers change
-    cudaGraphExec_t graph_exec = nullptr;   // captured run segment A (see run_local)
-    GraphKey graph_key;
-    uint64_t graph_launches = 0;
+    GraphSlot graph;           // captured run segment A (see run_local)
+    GraphSlot wgraph;          // captured online window step (fused windows)
+    uint64_t bufgen = 0;            // bumped whenever a device buffer a captured graph uses moves
     uint64_t gather_max = 0;       // payloads up to this are gathered by k_gather, above: DMA
     std::string last_error;
 
@@ -306,6 +330,9 @@ struct ffm_log {
     // fused online windows: the window's batch record order (small by size class, then
     // large), built on the device -- [order | inverse] and the sort's key / temp space
     uint32_t* d_word = nullptr;
+    ffm::WinMeta wmeta;               // [cap] the window's metadata (fixed buffers)
+    uint64_t* d_wa = nullptr;         // device: first record of the window
+    uint64_t* h_wa = nullptr;         // pinned mirror
     uint16_t* d_wkeys = nullptr;      // [2 * cap]
     void* d_wtmp = nullptr;
     size_t wtmp_bytes = 0;

@@ -2063,17 +2063,24 @@ int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t
     return 1;
 }
 
-__global__ void k_window_keys(const uint64_t* __restrict__ size, uint32_t n, uint32_t small_bytes,
+__global__ void k_window_meta(DevLog L, const uint64_t* __restrict__ d_a, uint32_t n, WinMeta wm, uint32_t small_bytes,
                               uint16_t* __restrict__ keys) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i < n) {
-        const uint64_t sz = size[i];
-        keys[i] = sz <= small_bytes ? (uint16_t)((sz + 31) / 32 + 1) : (uint16_t)0;
-    }
+    if (i >= n) return;
+    const uint64_t j = *d_a + i;
+    const uint64_t sz = L.size[j];
+    wm.off[i] = L.off[j];
+    wm.size[i] = sz;
+    wm.dur[i] = L.dur[j];
+    wm.gid[i] = L.gid[j];
+    wm.chan[i] = L.chan[j];
+    wm.site[i] = L.site[j];
+    keys[i] = sz <= small_bytes ? (uint16_t)((sz + 31) / 32 + 1) : (uint16_t)0;
 }
 
-int launch_window_order(const uint64_t* size, uint32_t n, uint32_t small_bytes, uint16_t* keys, const uint32_t* iota,
-                        uint32_t* order, uint32_t* inv, void* tmp, size_t* tmp_bytes, cudaStream_t st) {
+int launch_window_order(const DevLog& L, const uint64_t* d_a, uint32_t n, const WinMeta& wm, uint32_t small_bytes,
+                        uint16_t* keys, const uint32_t* iota, uint32_t* order, uint32_t* inv, void* tmp,
+                        size_t* tmp_bytes, cudaStream_t st) {
     int bits = 1;
     while ((1u << bits) <= (small_bytes + 31) / 32 + 1) ++bits;
     if (!tmp) {
@@ -2081,7 +2088,7 @@ int launch_window_order(const uint64_t* size, uint32_t n, uint32_t small_bytes, 
                                                          bits) == cudaSuccess ? 0 : -1;
     }
     if (n == 0) return 0;
-    k_window_keys<<<blocks_for(n), 256, 0, st>>>(size, n, small_bytes, keys);
+    k_window_meta<<<blocks_for(n), 256, 0, st>>>(L, d_a, n, wm, small_bytes, keys);
     FFM_LAUNCH_CHECK();
     // stable: equal block counts keep index order, the large records (key 0) come last
     if (cub::DeviceRadixSort::SortPairsDescending(tmp, *tmp_bytes, keys, keys + n, iota, order, (int)n, 0, bits, st) !=

@@ -117,9 +117,12 @@ def test_online_after_reset_and_forced_collisions_across_windows(ffm, mode):
 
 
 @pytest.mark.parametrize("mode", ["online", "append_hash"])
-def test_online_device_payloads_and_outputs(ffm, mode):
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_online_device_payloads_and_outputs(ffm, mode, digest_bits):
     """Appends of device-resident payloads (hashed at append time with append_hash), labels
-    written to device memory (the streaming shape of bench.py --online)."""
+    written to device memory (the streaming shape of bench.py --online): fused windows of
+    one size replay one captured step; digest_bits = 0 makes every window resolve residuals
+    after its speculative labels (the fix-up path)."""
     import torch
     lg = loggen.gen_config(5, n_scale=0.002, size_scale=1 / 32)
     want_d, want_b = oracle.dedup(lg)
@@ -128,7 +131,7 @@ def test_online_device_payloads_and_outputs(ffm, mode):
     dup = torch.empty(lg.n, dtype=torch.int64, device="cuda")
     ben = torch.empty(lg.n_sites, dtype=torch.int64, device="cuda")
     got = []
-    with ffm.FfmLog(lg.n_sites, chunk_bytes=4096, **MODES[mode]) as log:
+    with ffm.FfmLog(lg.n_sites, chunk_bytes=4096, digest_bits=digest_bits, **MODES[mode]) as log:
         for a in range(0, lg.n, 777):
             e = min(lg.n, a + 777)
             log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e], payload_kind=ffm.FFM_PAYLOAD_DEVICE)
