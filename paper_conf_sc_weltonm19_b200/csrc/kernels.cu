@@ -1321,15 +1321,24 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
     // ahead and gathered by shuffles when the record changes -- the load's destination is
     // read only then, so no step waits on it.
     const uint32_t* sd32 = reinterpret_cast<const uint32_t*>(W.sdesc);
-    uint32_t fi = oct, fw0 = 0;
-    uint64_t foff = 0, floff = 0;
-    uint32_t fn = 0, fr = 0, nd = 0;
+    // producer state of the octet's current record: next word fw0 of fnw, this lane's
+    // next source addresses (own, and the leader's for a compared record), bytes, record
+    uint32_t fi = oct, fw0 = 0, fnw = 0, fn = 0, fr = 0, nd = 0;
+    bool fcmp = false;
+    const uint8_t* fsrc = nullptr;
+    const uint8_t* flsrc = nullptr;
+    auto start_record = [&](uint64_t off, uint64_t loff, uint32_t n, uint32_t rec) {
+        fw0 = 0;
+        fn = n;
+        fr = rec;
+        fnw = (n + 15) >> 4;
+        fcmp = loff != ~0ull;
+        fsrc = L.arena + off + 16 * g;
+        flsrc = L.arena + (fcmp ? loff : off) + 16 * g;
+    };
     if (fi < L.n_small) {
         const uint4 a = W.sdesc[2ull * fi], b = W.sdesc[2ull * fi + 1];
-        foff = (uint64_t)a.y << 32 | a.x;
-        floff = (uint64_t)a.w << 32 | a.z;
-        fn = b.x;
-        fr = b.y;
+        start_record((uint64_t)a.y << 32 | a.x, (uint64_t)a.w << 32 | a.z, b.x, b.y);
         if (fi + noct < L.n_small) nd = sd32[8ull * (fi + noct) + g];
     }
     const int obase = threadIdx.x & 24;
@@ -1340,35 +1349,33 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
         mn = 0;
         mr = 0;
         if (fi < L.n_small) {
-            const uint32_t nw = (fn + 15) >> 4;
-            const bool cmp = floff != ~0ull;
-            // this lane's first word of the step; word j is 128 * j bytes further (immediate
-            // offsets), shared-memory slot j of part p is (2 j + p) * kSaT * 16 further
-            const uint8_t* src = L.arena + foff + 16ull * (fw0 + g);
-            const uint8_t* lsrc = L.arena + (cmp ? floff : foff) + 16ull * (fw0 + g);
+            // word j of the step is 128 * j bytes further (immediate offsets); shared-memory
+            // slot j of part p is (2 j + p) * kSaT * 16 further
             const uint32_t s0 = slot(s, 0, 0);
-            if (fw0 + 8 * kSaJ <= nw) {   // every lane's words exist
+            if (fw0 + 8 * kSaJ <= fnw) {   // every lane's words exist
 #pragma unroll
-                for (int j = 0; j < kSaJ; ++j) cp16(s0 + (uint32_t)(2 * j * kSaT * 16), src + 128 * j, pol_own);
-                if (cmp) {
+                for (int j = 0; j < kSaJ; ++j) cp16(s0 + (uint32_t)(2 * j * kSaT * 16), fsrc + 128 * j, pol_own);
+                if (fcmp) {
 #pragma unroll
                     for (int j = 0; j < kSaJ; ++j)
-                        cp16(s0 + (uint32_t)((2 * j + 1) * kSaT * 16), lsrc + 128 * j, pol_keep);
+                        cp16(s0 + (uint32_t)((2 * j + 1) * kSaT * 16), flsrc + 128 * j, pol_keep);
                 }
             } else {
 #pragma unroll
                 for (int j = 0; j < kSaJ; ++j) {
-                    if (fw0 + 8 * j + g < nw) {
-                        cp16(s0 + (uint32_t)(2 * j * kSaT * 16), src + 128 * j, pol_own);
-                        if (cmp) cp16(s0 + (uint32_t)((2 * j + 1) * kSaT * 16), lsrc + 128 * j, pol_keep);
+                    if (fw0 + 8 * j + g < fnw) {
+                        cp16(s0 + (uint32_t)(2 * j * kSaT * 16), fsrc + 128 * j, pol_own);
+                        if (fcmp) cp16(s0 + (uint32_t)((2 * j + 1) * kSaT * 16), flsrc + 128 * j, pol_keep);
                     }
                 }
             }
-            meta_z = fw0 | (fw0 == 0 ? kSaFirst : 0u) | (cmp ? kSaCmp : 0u);
+            meta_z = fw0 | (fw0 == 0 ? kSaFirst : 0u) | (fcmp ? kSaCmp : 0u);
             mn = fn;
             mr = fr;
             fw0 += 8 * kSaJ;
-            if (fw0 >= nw) meta_z |= kSaLast;
+            fsrc += 128 * kSaJ;
+            flsrc += 128 * kSaJ;
+            if (fw0 >= fnw) meta_z |= kSaLast;
         }
         // last step of the octet's record: move to the next one (shuffles executed by the
         // whole warp; an octet that is not changing ignores them)
@@ -1379,11 +1386,7 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
             const uint32_t d4 = __shfl_sync(0xFFFFFFFFu, nd, obase + 4), d5 = __shfl_sync(0xFFFFFFFFu, nd, obase + 5);
             if (change) {
                 fi += noct;
-                fw0 = 0;
-                foff = (uint64_t)d1 << 32 | d0;
-                floff = (uint64_t)d3 << 32 | d2;
-                fn = d4;
-                fr = d5;
+                start_record((uint64_t)d1 << 32 | d0, (uint64_t)d3 << 32 | d2, d4, d5);
                 if (fi + noct < L.n_small) nd = sd32[8ull * (fi + noct) + g];
             }
         }
@@ -1394,13 +1397,18 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
 
     // ---- consumer state
     LaneKeys K;   // k[0]: stripe position g, k[1]: position g + 8
-    uint32_t ka0[6], ka1[6];   // their stripe-0 keys (fixed per lane: no constant-bank loads per record)
-#pragma unroll
-    for (int jj = 0; jj < 6; ++jj) {
-        ka0[jj] = c_nh.ka[g][jj];
-        ka1[jj] = c_nh.ka[g + 8][jj];
+    // stripe-0 keys of the 16 positions in shared memory (6 keys padded to 8 per position):
+    // a record start reloads a lane's 12 keys with 4 conflict-free 16-byte loads (from the
+    // constant bank the 8 positions of a warp were 8 serialised accesses per key)
+    __shared__ uint4 s_ka[16][2];
+    if (threadIdx.x < 32) {
+        const int q = threadIdx.x >> 1, h = threadIdx.x & 1;
+        s_ka[q][h] = h ? make_uint4(c_nh.ka[q][4], c_nh.ka[q][5], 0u, 0u)
+                       : make_uint4(c_nh.ka[q][0], c_nh.ka[q][1], c_nh.ka[q][2], c_nh.ka[q][3]);
     }
-    uint64_t A = 0, B = 0, A2 = 0, B2 = 0, found = ~0ull;
+    __syncthreads();
+    uint64_t A = 0, B = 0, A2 = 0, B2 = 0;
+    uint32_t found = ~0u;   // first differing 16-byte word of a compared record (lane's own)
     int sc = 0, sf = kSaS - 1;
     // The warp stays converged across the loop (an octet whose records are done idles
     // until all four are), so the octet reductions at record ends use full-mask shuffles
@@ -1417,18 +1425,16 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
         if (!done) {
             if (z & kSaFirst) {
                 A = B = A2 = B2 = 0;
-                found = ~0ull;
-#pragma unroll
-                for (int jj = 0; jj < 6; ++jj) {
-                    K.k[0][jj] = ka0[jj];
-                    K.k[1][jj] = ka1[jj];
-                }
+                found = ~0u;
+                const uint4 a0 = s_ka[g][0], a1 = s_ka[g][1], b0 = s_ka[g + 8][0], b1 = s_ka[g + 8][1];
+                K.k[0][0] = a0.x, K.k[0][1] = a0.y, K.k[0][2] = a0.z, K.k[0][3] = a0.w, K.k[0][4] = a1.x, K.k[0][5] = a1.y;
+                K.k[1][0] = b0.x, K.k[1][1] = b0.y, K.k[1][2] = b0.z, K.k[1][3] = b0.w, K.k[1][4] = b1.x, K.k[1][5] = b1.y;
             }
             const uint32_t w0 = z & 0x0FFFFFFFu, nw = (n + 15) >> 4;
             const bool full = 16 * (w0 + 8 * kSaJ) <= n;   // every word of the step whole
             if (z & kSaCmp) {
                 // member: compare only, until its first differing word
-                if (found == ~0ull) {
+                if (found == ~0u) {
                     uint32_t d = 0;
                     if (full) {
 #pragma unroll
@@ -1446,9 +1452,10 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
                                 uint32_t x[4], y[4];
                                 lds16(slot(sc, j, 0), x);
                                 lds16(slot(sc, j, 1), y);
-                                mask_word(x, n, w);
-                                mask_word(y, n, w);
-                                d |= (x[0] ^ y[0]) | (x[1] ^ y[1]) | (x[2] ^ y[2]) | (x[3] ^ y[3]);
+#pragma unroll
+                                for (int e = 0; e < 4; ++e) x[e] ^= y[e];
+                                if (w + 1 == nw) mask_word(x, n, w);   // only the last word is partial
+                                d |= x[0] | x[1] | x[2] | x[3];
                             }
                         }
                     }
@@ -1487,7 +1494,7 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
                         if (w < nw) {
                             uint32_t x[4];
                             lds16(slot(sc, j, 0), x);
-                            mask_word(x, n, w);
+                            if (w + 1 == nw) mask_word(x, n, w);   // only the last word is partial
                             if (j & 1) nh_word(x[0], x[1], x[2], x[3], K.k[1], A2, B2);
                             else nh_word(x[0], x[1], x[2], x[3], K.k[0], A, B);
                         }
@@ -1496,25 +1503,30 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
                 }
             }
         }
-        // record ends (warp-uniform: any octet finishing one reduces with all four)
+        // record ends (warp-uniform: any octet finishing one reduces with all four); the
+        // NH sums only when a hashed record ends, the first-mismatch minimum only when an
+        // ending compared record has a mismatch (rare)
         const bool last = !done && (z & kSaLast) != 0;
         if (__any_sync(0xFFFFFFFFu, last)) {
-            uint64_t a = A + A2, b = B + B2, f = found;
+            const bool cmp_end = last && (z & kSaCmp) != 0;
+            if (__any_sync(0xFFFFFFFFu, last && !cmp_end)) {
+                uint64_t a = A + A2, b = B + B2;
 #pragma unroll
-            for (int o = 4; o; o >>= 1) {
-                a += __shfl_xor_sync(0xFFFFFFFFu, a, o);
-                b += __shfl_xor_sync(0xFFFFFFFFu, b, o);
-                const uint64_t of = __shfl_xor_sync(0xFFFFFFFFu, f, o);
-                f = of < f ? of : f;
-            }
-            if (last && g == 0) {
-                if (z & kSaCmp) {
-                    if (f != ~0ull) report_mismatch(W, r, f, res_out, false);
-                } else {
+                for (int o = 4; o; o >>= 1) {
+                    a += __shfl_xor_sync(0xFFFFFFFFu, a, o);
+                    b += __shfl_xor_sync(0xFFFFFFFFu, b, o);
+                }
+                if (last && !cmp_end && g == 0) {
                     W.accA[r] = a;
                     W.accB[r] = b;
                     W.digest[r] = finalize_digest(a, b, n);
                 }
+            }
+            if (__any_sync(0xFFFFFFFFu, cmp_end && found != ~0u)) {
+                uint32_t f = found;
+#pragma unroll
+                for (int o = 4; o; o >>= 1) f = min(f, __shfl_xor_sync(0xFFFFFFFFu, f, o));
+                if (cmp_end && g == 0 && f != ~0u) report_mismatch(W, r, f, res_out, false);
             }
         }
         sc = sc + 1 == kSaS ? 0 : sc + 1;
