@@ -48,15 +48,26 @@ for k, ns, ss in [(5, 0.001, 1 / 64), (3, 0.003, 1 / 64), (3, 0.012, 1 / 128), (
                 log.append_log(lg)
             d, b = log.run()
             assert np.array_equal(d, want[0]) and np.array_equal(b, want[1]), (k, db, rb, extra)
-    # online windows (append-time hashing and in-step hashing)
-    for online in (True, False):
-        with ffm.FfmLog(lg.n_sites, digest_bits=8, chunk_bytes=4096, online=online) as log:
-            ptrs = lg.payload_ptrs()
-            got = []
-            for a, e in ((0, lg.n // 3), (lg.n // 3, lg.n)):
-                log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e])
-                got.append(log.online_step()[0].copy())
-            assert np.array_equal(np.concatenate(got), want[0]), ("online", k)
+    # online windows: fused (metadata uploaded by the step / at append time), append-time
+    # hashing (two-pass steps); host outputs (direct launches) and device outputs (the
+    # captured window step, replayed for equal windows, residual fix-up with digest_bits 0)
+    for kw in ({}, {"online": True}, {"online": True, "append_hash": True}):
+        for db, dev_out in ((8, False), (0, True)):
+            with ffm.FfmLog(lg.n_sites, digest_bits=db, chunk_bytes=4096, **kw) as log:
+                ptrs = lg.payload_ptrs()
+                got = []
+                w = max(1, lg.n // 4)
+                dd = torch.empty(w + 1, dtype=torch.int64, device="cuda") if dev_out else None
+                bb = torch.empty(lg.n_sites, dtype=torch.int64, device="cuda") if dev_out else None
+                for a in range(0, lg.n, w):
+                    e = min(lg.n, a + w)
+                    log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e])
+                    if dev_out:
+                        log.online_step(dd, bb)
+                        got.append(dd[:e - a].cpu().numpy().copy())
+                    else:
+                        got.append(log.online_step()[0].copy())
+                assert np.array_equal(np.concatenate(got), want[0]), ("online", k, kw, db)
     # the collective sharded run in one process: a world of 2 whose other rank is empty
     # (header, export, all-gather, merge incl. the same-key segment scan, all-reduce)
     for db in (64, 0):
