@@ -578,34 +578,30 @@ DevLog window_view(ffm_log* L, uint64_t a, uint64_t b, bool has_large, cudaStrea
 // An online window [a, b) in the batch record order (small records by size class, then
 // the large ones), its metadata gathered into fixed buffers: window_view_sorted sizes the
 // buffers and returns the view; queue_window_order queues the gather and the order build
-// (a stable device radix sort of 16-bit size-class keys).  n_small: small records in it.
+// (a counting sort by size class: 2 kernels).  n_small: small records in it.
 DevLog window_view_sorted(ffm_log* L, uint64_t a, uint64_t b, uint64_t n_small, cudaStream_t st) {
     DevLog D = window_view(L, a, b, true, st);   // (iota of >= b - a entries)
     const uint64_t nw = b - a;
     if (nw > L->word_cap) {
         ck(cudaStreamSynchronize(st), "window buffers");
-        for (void* p : {(void*)L->d_word, (void*)L->d_wkeys, L->d_wtmp, (void*)L->wmeta.off, (void*)L->wmeta.size,
-                        (void*)L->wmeta.dur, (void*)L->wmeta.gid, (void*)L->wmeta.chan, (void*)L->wmeta.site})
+        for (void* p : {(void*)L->d_word, (void*)L->wmeta.off, (void*)L->wmeta.size, (void*)L->wmeta.dur,
+                        (void*)L->wmeta.gid, (void*)L->wmeta.chan, (void*)L->wmeta.site})
             if (p) ck(cudaFree(p), "cudaFree");
         L->d_word = nullptr;
-        L->d_wkeys = nullptr;
-        L->d_wtmp = nullptr;
         L->wmeta = WinMeta{};
         const uint64_t c = std::max<uint64_t>(std::max<uint64_t>(nw, 2 * L->word_cap), 4096);
         ck(cudaMalloc(&L->d_word, 2 * c * sizeof(uint32_t)), "cudaMalloc(window order)");
-        ck(cudaMalloc(&L->d_wkeys, 2 * c * sizeof(uint16_t)), "cudaMalloc(window keys)");
         ck(cudaMalloc(&L->wmeta.off, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
         ck(cudaMalloc(&L->wmeta.size, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
         ck(cudaMalloc(&L->wmeta.dur, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
         ck(cudaMalloc(&L->wmeta.gid, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
         ck(cudaMalloc(&L->wmeta.chan, c * sizeof(uint64_t)), "cudaMalloc(window meta)");
         ck(cudaMalloc(&L->wmeta.site, c * sizeof(uint32_t)), "cudaMalloc(window meta)");
-        size_t tb = 0;
-        if (launch_window_order(D, nullptr, (uint32_t)c, L->wmeta, L->params.small_bytes, nullptr, nullptr, nullptr,
-                                nullptr, nullptr, &tb, st) < 0)
-            throw CudaFail{cudaErrorUnknown, "window order temp size"};
-        L->wtmp_bytes = std::max<size_t>(tb, 256);
-        ck(cudaMalloc(&L->d_wtmp, L->wtmp_bytes), "cudaMalloc(window sort)");
+        if (!L->d_wbins) {
+            const uint64_t nb = 3ull * window_bins(L->params.small_bytes);
+            ck(cudaMalloc(&L->d_wbins, nb * sizeof(uint32_t)), "cudaMalloc(window bins)");
+            ck(cudaMemsetAsync(L->d_wbins, 0, nb * sizeof(uint32_t), st), "memset");
+        }
         L->word_cap = c;
         ++L->bufgen;
     }
@@ -628,10 +624,8 @@ DevLog window_view_sorted(ffm_log* L, uint64_t a, uint64_t b, uint64_t n_small, 
 }
 
 void queue_window_order(ffm_log* L, const DevLog& D, cudaStream_t st, uint64_t& launches) {
-    size_t tb = L->wtmp_bytes;
-    const int k = launch_window_order(dev_view(L), L->d_wa, D.n, L->wmeta, L->params.small_bytes, L->d_wkeys,
-                                      L->d_iota, const_cast<uint32_t*>(D.small_order),
-                                      const_cast<uint32_t*>(D.order_pos), L->d_wtmp, &tb, st);
+    const int k = launch_window_order(dev_view(L), L->d_wa, D.n, L->wmeta, L->params.small_bytes, L->d_wbins,
+                                      const_cast<uint32_t*>(D.small_order), const_cast<uint32_t*>(D.order_pos), st);
     if (k < 0) throw CudaFail{cudaGetLastError(), "window order"};
     launches += (uint64_t)k;
 }
@@ -1615,9 +1609,13 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
                 *L->h_wa = w0;
                 ck(cudaMemcpyAsync(L->d_wa, L->h_wa, sizeof(uint64_t), cudaMemcpyHostToDevice, s), "window start");
                 const std::function<void()> order = [&]() { queue_window_order(L, D, s, launches); };
-                // (captured copies need device or pinned host outputs)
+                // (captured copies need device or pinned host outputs; a window size is
+                // captured the second time in a row it occurs -- a one-off size, e.g. the
+                // tail of a stream, launches directly instead of paying a capture)
                 const bool capt = (dup_dev || is_pinned_host(dup_out)) &&
-                                  (!ben_out || is_device_ptr(ben_out) || is_pinned_host(ben_out));
+                                  (!ben_out || is_device_ptr(ben_out) || is_pinned_host(ben_out)) &&
+                                  (nw == L->last_window || (L->wgraph.exec && L->wgraph.key.extra[1] == nw));
+                L->last_window = nw;
                 const uint64_t extra[4] = {L->bufgen, nw, n_small_w | (n_large << 32),
                                            (uint64_t)(uintptr_t)dup_out ^ ((uint64_t)(uintptr_t)ben_out << 1)};
                 R = run_local(L, D, n_large, launches, false, nullptr, false, &match, false, nullptr, true, L->on_res,
@@ -1725,6 +1723,7 @@ int ffm_log_reset(ffm_log* L) {
     L->h_chan.clear();
     L->payload_bytes = L->n_large_chunks = L->last_gid = 0;
     L->n_small_recs = L->online_small0 = L->online_chunks0 = 0;
+    L->last_window = 0;   // (a new stream: its first window of a size launches directly)
     L->any_gid = false;
     L->d_meta_n = 0;
     L->d_order_n = 0;
@@ -1766,7 +1765,7 @@ int ffm_log_destroy(ffm_log* L) {
     free_shard(L->shard);
     if (L->fold_buf) cudaFree(L->fold_buf);
     void* op[] = {L->otab.key, L->otab.head, L->otab.pool, L->otab.count, L->on_A, L->on_B, L->on_G,
-                  L->on_res, L->online_ben, L->d_iota, L->d_word, L->d_wkeys, L->d_wtmp, L->d_wa, L->wmeta.off,
+                  L->on_res, L->online_ben, L->d_iota, L->d_word, L->d_wbins, L->d_wa, L->wmeta.off,
                   L->wmeta.size, L->wmeta.dur, L->wmeta.gid, L->wmeta.chan, L->wmeta.site};
     for (void* p : op)
         if (p) cudaFree(p);

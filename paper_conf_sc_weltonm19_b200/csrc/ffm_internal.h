@@ -193,14 +193,12 @@ int launch_shard_header(const uint32_t* rep_count, const uint32_t* counters, uin
 int launch_gather(const uint64_t* d_desc, uint32_t n, uint8_t* arena, cudaStream_t st);
 int launch_zero_counters(Work& W, cudaStream_t st);
 int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t st);
-// The batch record order of a log view of n records (small ones by 32-byte block count,
-// largest first, stable; then the large ones in index order) and its inverse, on the
-// device: keys [2n] scratch, iota = 0..n-1.  tmp == nullptr: *tmp_bytes = space needed.
-// The window [*d_a, *d_a + n) of the log L: its metadata gathered into wm, then its
-// batch record order.
+// The window [*d_a, *d_a + n) of the log L: its metadata gathered into wm, and its batch
+// record order (small records grouped by 32-byte block count, largest first; then the
+// large ones) and inverse.  bins: [3 * window_bins(small_bytes)] words, zero between calls.
+__host__ __device__ uint32_t window_bins(uint32_t small_bytes);
 int launch_window_order(const DevLog& L, const uint64_t* d_a, uint32_t n, const WinMeta& wm, uint32_t small_bytes,
-                        uint16_t* keys, const uint32_t* iota, uint32_t* order, uint32_t* inv, void* tmp,
-                        size_t* tmp_bytes, cudaStream_t st);
+                        uint32_t* bins, uint32_t* order, uint32_t* inv, cudaStream_t st);
 int launch_iota(uint32_t* a, uint32_t n, cudaStream_t st);
 int launch_spec_label(const DevLog& L, Work& W, int64_t* dup_out, cudaStream_t st);
 int launch_digest_fill(const DevLog& L, Work& W, const Params& P, cudaStream_t st);
@@ -333,10 +331,9 @@ struct ffm_log {
     ffm::WinMeta wmeta;               // [cap] the window's metadata (fixed buffers)
     uint64_t* d_wa = nullptr;         // device: first record of the window
     uint64_t* h_wa = nullptr;         // pinned mirror
-    uint16_t* d_wkeys = nullptr;      // [2 * cap]
-    void* d_wtmp = nullptr;
-    size_t wtmp_bytes = 0;
+    uint32_t* d_wbins = nullptr;      // window order: class counts | cursors | done (zero between steps)
     uint64_t word_cap = 0;
+    uint64_t last_window = 0;         // size of the previous online window
     uint64_t n_small_recs = 0;        // records <= small_bytes appended so far
     uint64_t online_small0 = 0;       // n_small_recs / n_large_chunks at online_done
     uint64_t online_chunks0 = 0;

@@ -1881,8 +1881,11 @@ int launch_group(const DevLog& L, Work& W, const Params& P, const uint32_t* list
         ++k;
     }
     if (cudaMemsetAsync(W.tkey, 0xFF, cap * sizeof(uint64_t), st) != cudaSuccess) return -1;
-    if (cudaMemsetAsync(W.lcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
-    if (cudaMemsetAsync(W.gcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
+    // per-leader large-member counts: only large records use them
+    if (L.n_large) {
+        if (cudaMemsetAsync(W.lcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
+        if (cudaMemsetAsync(W.gcount, 0, ((uint64_t)L.n + 1) * sizeof(uint32_t), st) != cudaSuccess) return -1;
+    }
     k_group_insert<<<blocks_for(n_list), 256, 0, st>>>(L, W, list, n_list, cap - 1, P.digest_mask, round,
                                                         P.small_bytes);
     FFM_LAUNCH_CHECK();
@@ -2075,40 +2078,106 @@ int launch_invert(const uint32_t* order, uint32_t n, uint32_t* inv, cudaStream_t
     return 1;
 }
 
-__global__ void k_window_meta(DevLog L, const uint64_t* __restrict__ d_a, uint32_t n, WinMeta wm, uint32_t small_bytes,
-                              uint16_t* __restrict__ keys) {
+// Online window order (counting sort by size class, 2 kernels): class c of a record =
+// maxb - (its 32-byte block count) for a small one (largest first), maxb + 1 for a large
+// one.  bins = [count | cursor | done], zero between windows.
+__device__ __forceinline__ uint32_t window_class(uint64_t sz, uint32_t small_bytes) {
+    const uint32_t maxb = (small_bytes + 31) / 32;
+    return sz <= small_bytes ? maxb - (uint32_t)((sz + 31) / 32) : maxb + 1;
+}
+
+__host__ __device__ uint32_t window_bins(uint32_t small_bytes) { return (small_bytes + 31) / 32 + 2; }
+
+// gathers the window's metadata into the fixed buffers, counts its classes; the last block
+// turns the counts into the classes' start positions (and zeroes the counts for the next)
+__global__ void __launch_bounds__(1024) k_wclass_count(DevLog L, const uint64_t* __restrict__ d_a, uint32_t n,
+                                                      WinMeta wm, uint32_t small_bytes, uint32_t* __restrict__ bins) {
+    extern __shared__ uint32_t hist[];
+    __shared__ bool last;
+    const uint32_t nb = window_bins(small_bytes);
+    uint32_t* cnt = bins;
+    uint32_t* cur = bins + nb;
+    uint32_t* done = bins + 2 * nb;
+    for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x) hist[b] = 0;
+    __syncthreads();
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= n) return;
-    const uint64_t j = *d_a + i;
-    const uint64_t sz = L.size[j];
-    wm.off[i] = L.off[j];
-    wm.size[i] = sz;
-    wm.dur[i] = L.dur[j];
-    wm.gid[i] = L.gid[j];
-    wm.chan[i] = L.chan[j];
-    wm.site[i] = L.site[j];
-    keys[i] = sz <= small_bytes ? (uint16_t)((sz + 31) / 32 + 1) : (uint16_t)0;
+    if (i < n) {
+        const uint64_t j = *d_a + i;
+        const uint64_t sz = L.size[j];
+        wm.off[i] = L.off[j];
+        wm.size[i] = sz;
+        wm.dur[i] = L.dur[j];
+        wm.gid[i] = L.gid[j];
+        wm.chan[i] = L.chan[j];
+        wm.site[i] = L.site[j];
+        atomicAdd(&hist[window_class(sz, small_bytes)], 1u);
+    }
+    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x)
+        if (hist[b]) atomicAdd(&cnt[b], hist[b]);
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) last = atomicAdd(done, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (!last) return;
+    // the last block: exclusive scan of the counts (read and zeroed atomically)
+    for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x) hist[b] = atomicExch(&cnt[b], 0u);
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        uint32_t base = 0;
+        for (uint32_t b0 = 0; b0 < nb; b0 += 32) {
+            const uint32_t b = b0 + threadIdx.x;
+            const uint32_t v = b < nb ? hist[b] : 0u;
+            uint32_t x = v;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+                if ((int)threadIdx.x >= o) x += y;
+            }
+            if (b < nb) cur[b] = base + x - v;
+            base += __shfl_sync(0xFFFFFFFFu, x, 31);
+        }
+        if (threadIdx.x == 0) *done = 0;
+    }
+}
+
+// each record takes the next position of its class: ranks within the block from shared
+// memory atomics, then one global atomic per (block, class present) reserves the range
+__global__ void __launch_bounds__(1024) k_wclass_scatter(const WinMeta wm, uint32_t n, uint32_t small_bytes,
+                                                         uint32_t* __restrict__ bins, uint32_t* __restrict__ order,
+                                                         uint32_t* __restrict__ inv) {
+    extern __shared__ uint32_t hist[];   // [nb] counts, then [nb] bases
+    const uint32_t nb = window_bins(small_bytes);
+    uint32_t* base = hist + nb;
+    for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x) hist[b] = 0;
+    __syncthreads();
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    uint32_t c = 0, rank = 0;
+    if (i < n) {
+        c = window_class(wm.size[i], small_bytes);
+        rank = atomicAdd(&hist[c], 1u);
+    }
+    __syncthreads();
+    for (uint32_t b = threadIdx.x; b < nb; b += blockDim.x)
+        if (hist[b]) base[b] = atomicAdd(&bins[nb + b], hist[b]);
+    __syncthreads();
+    if (i < n) {
+        const uint32_t pos = base[c] + rank;
+        order[pos] = i;
+        inv[i] = pos;
+    }
 }
 
 int launch_window_order(const DevLog& L, const uint64_t* d_a, uint32_t n, const WinMeta& wm, uint32_t small_bytes,
-                        uint16_t* keys, const uint32_t* iota, uint32_t* order, uint32_t* inv, void* tmp,
-                        size_t* tmp_bytes, cudaStream_t st) {
-    int bits = 1;
-    while ((1u << bits) <= (small_bytes + 31) / 32 + 1) ++bits;
-    if (!tmp) {
-        return cub::DeviceRadixSort::SortPairsDescending(nullptr, *tmp_bytes, keys, keys + n, iota, order, (int)n, 0,
-                                                         bits) == cudaSuccess ? 0 : -1;
-    }
+                        uint32_t* bins, uint32_t* order, uint32_t* inv, cudaStream_t st) {
     if (n == 0) return 0;
-    k_window_meta<<<blocks_for(n), 256, 0, st>>>(L, d_a, n, wm, small_bytes, keys);
+    const uint32_t nb = window_bins(small_bytes);
+    k_wclass_count<<<blocks_for(n, 1024), 1024, nb * sizeof(uint32_t), st>>>(L, d_a, n, wm, small_bytes, bins);
     FFM_LAUNCH_CHECK();
-    // stable: equal block counts keep index order, the large records (key 0) come last
-    if (cub::DeviceRadixSort::SortPairsDescending(tmp, *tmp_bytes, keys, keys + n, iota, order, (int)n, 0, bits, st) !=
-        cudaSuccess)
-        return -1;
-    k_invert<<<blocks_for(n), 256, 0, st>>>(order, n, inv);
+    k_wclass_scatter<<<blocks_for(n, 1024), 1024, 2 * nb * sizeof(uint32_t), st>>>(wm, n, small_bytes, bins, order,
+                                                                                  inv);
     FFM_LAUNCH_CHECK();
-    return 3;
+    return 2;
 }
 
 int launch_zero_counters(Work& W, cudaStream_t st) {

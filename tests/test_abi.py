@@ -82,3 +82,13 @@ def test_product_never_imports_the_oracle():
                     assert bad not in txt, (f, bad)
     out = subprocess.run(["nm", "-D", ffm._LIB_PATH], capture_output=True, text=True).stdout
     assert "oracle" not in out
+
+
+def test_binding_constants_match_the_header():
+    """Every FFM_* enum value include/ffm.h defines has the same value in the binding."""
+    src = re.sub(r"/\*.*?\*/", "", open(os.path.join(ROOT, "include", "ffm.h")).read(), flags=re.S)
+    consts = {m.group(1): int(m.group(2)) for m in re.finditer(r"\b(FFM_[A-Z_0-9]+)\s*=\s*(-?\d+)u?\b", src)}
+    assert {"FFM_OK", "FFM_E_NODEV", "FFM_PAYLOAD_DEVICE", "FFM_FLAG_ONLINE", "FFM_FLAG_APPEND_HASH",
+            "FFM_SHARD_CONTIGUOUS"} <= set(consts)
+    for name, value in consts.items():
+        assert getattr(ffm, name) == value, name
