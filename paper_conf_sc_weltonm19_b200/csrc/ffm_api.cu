@@ -823,7 +823,7 @@ LocalRun run_local(ffm_log* L, const DevLog& D, uint64_t n_large, uint64_t& laun
         GraphSlot& G = window ? *wslot : L->graph;
         GraphKey key{window ? ~0ull : L->epoch, d_dup, h_spec, two_pass, prefilter, timing};
         if (wextra)
-            for (int i = 0; i < 4; ++i) key.extra[i] = wextra[i];
+            for (int i = 0; i < GraphKey::kExtra; ++i) key.extra[i] = wextra[i];
         if (!G.exec || !(key == G.key)) {
             uint64_t before = launches;
             ck(cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed), "begin capture");
@@ -1616,8 +1616,8 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
                                   (!ben_out || is_device_ptr(ben_out) || is_pinned_host(ben_out)) &&
                                   (nw == L->last_window || (L->wgraph.exec && L->wgraph.key.extra[1] == nw));
                 L->last_window = nw;
-                const uint64_t extra[4] = {L->bufgen, nw, n_small_w | (n_large << 32),
-                                           (uint64_t)(uintptr_t)dup_out ^ ((uint64_t)(uintptr_t)ben_out << 1)};
+                const uint64_t extra[GraphKey::kExtra] = {L->bufgen, nw, n_small_w, n_large,
+                                                          (uint64_t)(uintptr_t)dup_out, (uint64_t)(uintptr_t)ben_out};
                 R = run_local(L, D, n_large, launches, false, nullptr, false, &match, false, nullptr, true, L->on_res,
                               capt ? &L->wgraph : nullptr, extra, &order);
             } else {

@@ -218,11 +218,13 @@ struct GraphKey {
     const void* dup = nullptr;
     const void* hdup = nullptr;   // pinned host duplicate_of of the speculative D2H (or null)
     bool two_pass = false, prefilter = false, timing = false;
-    uint64_t extra[4] = {0, 0, 0, 0};   // online windows: what else the captured step depends on
+    static constexpr int kExtra = 6;
+    uint64_t extra[kExtra] = {0, 0, 0, 0, 0, 0};   // online windows: what else the captured step depends on
     bool operator==(const GraphKey& o) const {
-        return epoch == o.epoch && dup == o.dup && hdup == o.hdup && two_pass == o.two_pass &&
-               prefilter == o.prefilter && timing == o.timing && extra[0] == o.extra[0] &&
-               extra[1] == o.extra[1] && extra[2] == o.extra[2] && extra[3] == o.extra[3];
+        bool same = epoch == o.epoch && dup == o.dup && hdup == o.hdup && two_pass == o.two_pass &&
+                    prefilter == o.prefilter && timing == o.timing;
+        for (int i = 0; i < kExtra; ++i) same = same && extra[i] == o.extra[i];
+        return same;
     }
 };
 

@@ -1409,19 +1409,19 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
     __syncthreads();
     uint64_t A = 0, B = 0, A2 = 0, B2 = 0;
     uint32_t found = ~0u;   // first differing 16-byte word of a compared record (lane's own)
-    int sc = 0, sf = kSaS - 1;
     // The warp stays converged across the loop (an octet whose records are done idles
     // until all four are), so the octet reductions at record ends use full-mask shuffles
     // (xor 4 / 2 / 1 stay inside an octet) executed warp-uniformly -- no per-octet masks.
-#pragma unroll 1
-    while (true) {
+    // one iteration consuming stage sc and refilling stage sf; unrolled over the two
+    // stages so every shared-memory slot address is a compile-time offset
+    auto iteration = [&](const int sc, const int sf) -> bool {
         // refill the stage consumed last iteration (its values were used, so read), then
         // wait for the oldest: S-1 steps stay in flight while this one is hashed
         const uint32_t n = mn, r = mr, z = meta_z;   // the step fetched last iteration
         fetch(sf);
         asm volatile("cp.async.wait_group %0;" ::"n"(kSaS - 1) : "memory");
         const bool done = (z & kSaEnd) != 0;
-        if (__all_sync(0xFFFFFFFFu, done)) break;
+        if (__all_sync(0xFFFFFFFFu, done)) return false;
         if (!done) {
             if (z & kSaFirst) {
                 A = B = A2 = B2 = 0;
@@ -1529,8 +1529,10 @@ __global__ void __launch_bounds__(kSaT) k_fused_small(DevLog L, Work W, uint32_t
                 if (cmp_end && g == 0 && f != ~0u) report_mismatch(W, r, f, res_out, false);
             }
         }
-        sc = sc + 1 == kSaS ? 0 : sc + 1;
-        sf = sf + 1 == kSaS ? 0 : sf + 1;
+        return true;
+    };
+#pragma unroll 1
+    while (iteration(0, 1) && iteration(1, 0)) {
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
 }
