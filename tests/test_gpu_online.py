@@ -139,3 +139,29 @@ def test_online_device_payloads_and_outputs(ffm, mode, digest_bits):
             got.append(dup[:e - a].cpu().numpy().copy())
     np.testing.assert_array_equal(np.concatenate(got), want_d)
     np.testing.assert_array_equal(ben.cpu().numpy().view(np.uint64), want_b)
+
+
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_online_pinned_host_outputs_and_table_growth(ffm, digest_bits):
+    """Labels into pinned host memory (the captured window step copies into it), windows of
+    one size long enough to replay the captured step several times while the stored-class
+    table grows (rehash: the captured step must be re-made), a reset mid-stream, and a
+    tail window of another size."""
+    import torch
+    lg = loggen.gen_config(2, n_scale=0.03)
+    want_d, want_b = oracle.dedup(lg)
+    ptrs = lg.payload_ptrs()
+    dup = torch.empty(lg.n, dtype=torch.int64).pin_memory()
+    ben = torch.empty(lg.n_sites, dtype=torch.int64).pin_memory()
+    w = 997
+    with ffm.FfmLog(lg.n_sites, digest_bits=digest_bits, online=True) as log:
+        for rep in range(2):
+            got = []
+            for a in range(0, lg.n, w):
+                e = min(lg.n, a + w)
+                log.append_batch(lg.site[a:e], lg.size[a:e], ptrs[a:e], lg.dur[a:e])
+                log.online_step(dup, ben)
+                got.append(dup[:e - a].numpy().copy())
+            np.testing.assert_array_equal(np.concatenate(got), want_d)
+            np.testing.assert_array_equal(ben.numpy().view(np.uint64), want_b)
+            log.reset()
