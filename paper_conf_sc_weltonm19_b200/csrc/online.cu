@@ -8,7 +8,7 @@
 // A step labels one window of new records:
 //   1-2. H1-H4 on the window alone -> exact window classes: by default the batch run's fused
 //      round 0 on the window in its batch record order (built on the device by
-//      launch_window_order); with FFM_FLAG_ONLINE the NH sums were computed at append time
+//      launch_window_order); with FFM_FLAG_APPEND_HASH the NH sums were computed at append time
 //      on the hashing stream and the step runs the two-pass round 0 without H1;
 //   3. k_online_probe (thread per record): each window class representative looks its key
 //      up in the table -- absent: the class is new and stored at once; present:
