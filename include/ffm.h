@@ -255,7 +255,8 @@ int ffm_fold_sites(ffm_log* log, const uint64_t* site_values, const uint32_t* si
  * read once, leaders hashed, members compared); with FFM_FLAG_APPEND_HASH the appends hash
  * their records and the step verifies two-pass -- then each window class looks its key up
  * in the table and is byte-verified against the stored classes there; classes with no
- * equal stored class are inserted.  A step's work is O(window), never O(prior records) (the table is
+ * equal stored class are inserted.  A window of <= 8 small records is labelled by one warp,
+ * record by record in gid order, directly against the table (one launch per step).  A step's work is O(window), never O(prior records) (the table is
  * rehashed only when its capacity doubles).  Labels of earlier records never change, so
  * the concatenated windows equal ffm_dedup_run over the whole log, bit for bit.
  *   duplicate_of [window records] (host or device): gids, or -1

@@ -1573,9 +1573,23 @@ int ffm_online_step(ffm_log* L, int64_t* dup_out, uint64_t* ben_out, uint64_t* n
         }
         uint64_t launches = 0;
         LocalRun R{};
-        if (nw) {
+        const uint64_t n_large_w = L->n_large_chunks - L->online_chunks0;
+        if (nw && nw <= kTinyWindow && !n_large_w && L->online_hashed <= w0) {
+            // a tiny window (a few small records, e.g. one intercepted call): one warp labels
+            // them in order against the table -- one launch, one sync
+            ensure_online(L, nw);
+            const bool dup_dev = is_device_ptr(dup_out);
+            int64_t* d_dup = dup_dev ? dup_out : W.dup;
+            const DevLog D = window_view(L, w0, n, false, s);
+            LCHK(launch_online_tiny(D, L->otab, L->params, d_dup, L->online_ben, L->online_cnt, s));
+            if (!dup_dev) ck(cudaMemcpyAsync(dup_out, d_dup, nw * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "D2H dup");
+            ck(cudaMemcpyAsync(L->h_counters + 2, L->otab.count, sizeof(uint32_t), cudaMemcpyDeviceToHost, s), "D2H");
+            if (ben_out)
+                ck(cudaMemcpyAsync(ben_out, L->online_ben, ns * sizeof(uint64_t), cudaMemcpyDefault, s), "copy ben");
+            sync_run(L, "online sync");
+        } else if (nw) {
             const uint64_t n_small_w = L->n_small_recs - L->online_small0;
-            const uint64_t n_large = L->n_large_chunks - L->online_chunks0;
+            const uint64_t n_large = n_large_w;
             const bool fused = L->online_hashed <= w0;
             ensure_online(L, nw);
             const bool dup_dev = is_device_ptr(dup_out);

@@ -183,6 +183,10 @@ int launch_online_rehash(OnlineTable& T, uint32_t np, uint64_t digest_mask, cuda
 int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, const uint64_t* accB,
                          OnlineTable& T, const Params& P, uint32_t n_sites, uint64_t* G, int64_t* dup_out,
                          uint64_t* ben, uint64_t* cnt, cudaStream_t st);
+// tiny windows: one warp labels the records in order against the table (ffm_online_step)
+constexpr uint32_t kTinyWindow = 8;
+int launch_online_tiny(const DevLog& L, OnlineTable& T, const Params& P, int64_t* dup_out, uint64_t* ben,
+                       uint64_t* cnt, cudaStream_t st);
 int launch_online_fix(const DevLog& L, const Work& W, const uint64_t* accA, const uint64_t* accB, OnlineTable& T,
                       const Params& P, const uint32_t* list, uint32_t n_list, uint64_t* G, int64_t* dup_out,
                       uint64_t* ben, uint64_t* cnt, cudaStream_t st);

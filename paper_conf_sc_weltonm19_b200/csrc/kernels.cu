@@ -30,31 +30,6 @@ namespace ffm {
 // The per-stripe key steps DA are compile-time constants (immediate operands), so a
 // lane keeps only its 12 current keys in registers.
 // ----------------------------------------------------------------------------
-struct NHKeys {
-    uint32_t ka[16][6];
-};
-
-constexpr uint64_t sm64(uint64_t x) {
-    x += 0x9E3779B97F4A7C15ull;
-    x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
-    x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
-    return x ^ (x >> 31);
-}
-
-constexpr NHKeys make_nh_keys() {
-    NHKeys k{};
-    uint64_t s = 0xD10E5E5FF1ull;
-    for (int g = 0; g < 16; ++g)
-        for (int j = 0; j < 6; ++j) k.ka[g][j] = (uint32_t)(sm64(s++) >> 16);
-    return k;
-}
-
-// per-stripe key increments (odd => full period mod 2^32)
-__host__ __device__ constexpr uint32_t kDA(int j) {
-    return j == 0 ? 0x9E3779B9u : j == 1 ? 0x7F4A7C15u : j == 2 ? 0xF39CC061u
-         : j == 3 ? 0x5CEDC835u : j == 4 ? 0x1B873593u : 0xCC9E2D51u;
-}
-
 __constant__ NHKeys c_nh = make_nh_keys();
 
 struct LaneKeys {

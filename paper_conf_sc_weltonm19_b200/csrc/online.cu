@@ -204,6 +204,94 @@ __global__ void k_online_fix(DevLog L, const uint32_t* __restrict__ leader, cons
     }
 }
 
+// Tiny windows (<= kTinyWindow small records; ffm_online_step): one warp labels the
+// window's records one after another, in gid order, directly against the table -- the
+// record's NH digest (lane l takes 16-byte words l, l + 32, ...), its
+// key's chain byte-compared, a new class stored at once -- so a duplicate inside the window
+// finds its class in the table like any earlier one.  No group-by, no record order, one
+// launch: the per-call latency of the paper's per-transfer check.
+__global__ void __launch_bounds__(32) k_online_tiny(DevLog L, OnlineTable T, NHKeys nk, uint64_t digest_mask,
+                                                    uint64_t refine_mask, int64_t* __restrict__ dup_out,
+                                                    uint64_t* __restrict__ ben, uint64_t* __restrict__ cnt) {
+    __shared__ uint32_t ska[16][6];
+    const int lane = threadIdx.x;
+    for (int i = lane; i < 96; i += 32) ska[i / 6][i % 6] = nk.ka[i / 6][i % 6];
+    __syncwarp();
+    for (uint32_t r = 0; r < L.n; ++r) {
+        const uint64_t n = L.size[r], chan = L.chan[r];
+        const uint8_t* px = L.arena + L.off[r];
+        const uint64_t nw = (n + 15) >> 4;
+        uint64_t A = 0, B = 0;
+        for (uint64_t q = lane; q < nw; q += 32) {
+            uint4 v = *reinterpret_cast<const uint4*>(px + 16 * q);
+            uint32_t w[4] = {v.x, v.y, v.z, v.w};
+            const int32_t valid = (int32_t)(n - 16 * q);
+            if (valid < 16) {
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const int32_t vb = valid - 4 * i;
+                    w[i] &= vb >= 4 ? 0xFFFFFFFFu : (vb <= 0 ? 0u : ((1u << (8 * vb)) - 1u));
+                }
+            }
+            uint32_t k[6];
+            const uint32_t s = (uint32_t)(q >> 4);
+#pragma unroll
+            for (int j = 0; j < 6; ++j) k[j] = ska[q & 15][j] + s * kDA(j);
+            A += (uint64_t)(w[0] + k[0]) * (uint64_t)(w[1] + k[1]);
+            A += (uint64_t)(w[2] + k[2]) * (uint64_t)(w[3] + k[3]);
+            B += (uint64_t)(w[0] + k[2]) * (uint64_t)(w[1] + k[3]);
+            B += (uint64_t)(w[2] + k[4]) * (uint64_t)(w[3] + k[5]);
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            A += __shfl_xor_sync(0xFFFFFFFFu, A, o);
+            B += __shfl_xor_sync(0xFFFFFFFFu, B, o);
+        }
+        const uint64_t dig = finalize_digest(A, B, n);
+        const uint64_t key = group_key(dig, n, digest_mask, chan);
+        const uint64_t h = online_probe(T, key);
+        uint32_t idx = 0xFFFFFFFFu;   // (kNoRep)
+        if (T.key[h] == key) idx = *reinterpret_cast<volatile uint32_t*>(&T.head[h]);
+        uint64_t gl = L.gid[r];
+        bool found = false;
+        const uint64_t nblk = (n + 31) >> 5;
+        while (idx != kNoRep && !found) {
+            const OnlineRep e = T.pool[idx];
+            if (e.size == n && e.chan == chan && ((e.dig ^ dig) & refine_mask) == 0) {
+                const uint8_t* py = L.arena + e.off;
+                bool diff = false;
+                for (uint64_t b0 = 0; b0 < nblk && !diff; b0 += 32) {
+                    const uint64_t b = b0 + lane;
+                    bool d = false;
+                    if (b < nblk) {
+                        Blk x = ld_stream(px + 32 * b);
+                        Blk y = ld_keep(py + 32 * b);
+                        mask_tail(x, n, b);
+                        mask_tail(y, n, b);
+                        d = !blk_equal(x, y);
+                    }
+                    diff = __any_sync(0xFFFFFFFFu, d);
+                }
+                if (!diff) {
+                    gl = e.gid;
+                    found = true;
+                }
+            }
+            idx = e.next;
+        }
+        if (lane == 0) {
+            if (!found) online_store<false>(T, L, r, key, dig, atomicAdd(T.count, 1u));
+            const int64_t d = found ? (int64_t)gl : -1;
+            dup_out[r] = d;
+            if (d >= 0) {
+                ben[L.site[r]] += L.dur[r];
+                cnt[L.site[r]] += 1;
+            }
+        }
+        __syncwarp();   // (the next record's probe may meet this one's new entry)
+    }
+}
+
 // Capacity growth: re-link every stored representative into a fresh (larger) table.
 __global__ void k_online_rehash(OnlineTable T, uint32_t np, uint64_t digest_mask) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -290,6 +378,14 @@ int launch_online_window(const DevLog& L, const Work& W, const uint64_t* accA, c
     }
     ONLINE_CHECK();
     return 3;
+}
+
+int launch_online_tiny(const DevLog& L, OnlineTable& T, const Params& P, int64_t* dup_out, uint64_t* ben,
+                       uint64_t* cnt, cudaStream_t st) {
+    if (L.n == 0) return 0;
+    k_online_tiny<<<1, 32, 0, st>>>(L, T, make_nh_keys(), P.digest_mask, P.refine_mask, dup_out, ben, cnt);
+    ONLINE_CHECK();
+    return 1;
 }
 
 // After H4 of a step launched with speculative labels: the residual records (list) get

@@ -165,3 +165,24 @@ def test_online_pinned_host_outputs_and_table_growth(ffm, digest_bits):
             np.testing.assert_array_equal(np.concatenate(got), want_d)
             np.testing.assert_array_equal(ben.numpy().view(np.uint64), want_b)
             log.reset()
+
+
+@pytest.mark.parametrize("digest_bits", [64, 0])
+def test_online_tiny_and_regular_windows_interleaved(ffm, digest_bits):
+    """Windows of 1..12 records: the tiny ones (<= 8 small records) are labelled by one warp
+    in order against the table, the others by the fused window step; both store classes the
+    other finds (same digest, same table).  digest_bits = 0: every class of a size shares one
+    chain; channels split equal bytes."""
+    lg = loggen.gen_config(2, n_scale=0.004)
+    lg.channel = (lg.site.astype(np.uint64) % np.uint64(2))
+    want_d, want_b = oracle.dedup(lg)
+    rng = np.random.default_rng(7)
+    cuts, c = [], 0
+    while c < lg.n:
+        c += int(rng.integers(1, 13))
+        cuts.append(min(c, lg.n))
+    got_d, bens, bd, bb = _online(ffm, lg, cuts[:-1], digest_bits=digest_bits, online=True)
+    np.testing.assert_array_equal(got_d, want_d)
+    np.testing.assert_array_equal(bens[-1][1], want_b)
+    for end, b in bens[::50]:
+        np.testing.assert_array_equal(b, oracle.dedup(lg.subset(np.arange(end)))[1])
