@@ -99,7 +99,8 @@ typedef struct ffm_config {
     int32_t  rank, world;  /* shard id / count; 0, 1 for one GPU.  world > 1 makes ffm_log_create
                               and ffm_dedup_run collective (see "Sharded logs" below) */
     uint64_t arena_bytes;  /* initial HBM payload arena capacity (bytes); grows x2 on demand */
-    uint64_t max_records;  /* initial record capacity hint; grows on demand */
+    uint64_t max_records;  /* initial record capacity hint; grows on demand (within it the host
+                              copy of the metadata is page-locked: its uploads are async DMA) */
     uint32_t digest_bits;  /* 64 normally.  < 64 truncates the group-by digest to FORCE
                               collisions (test / verify-stress knob, BASELINE config 3);
                               results never change.  0 => group by size alone. */

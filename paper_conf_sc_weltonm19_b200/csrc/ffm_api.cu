@@ -380,10 +380,35 @@ int plan_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* si
     return FFM_OK;
 }
 
+// The host metadata vectors are page-locked while they stay within the capacity reserved
+// at create (cfg.max_records): their uploads are then plain asynchronous DMA.  Growing past
+// it reallocates them -- unregistered first, pageable from then on.
+void pin_meta(ffm_log* L, bool on) {
+    void* ptrs[] = {L->h_site.data(), L->h_size.data(), L->h_off.data(), L->h_dur.data(), L->h_gid.data(),
+                    L->h_chan.data()};
+    const size_t bytes[] = {L->h_site.capacity() * 4, L->h_size.capacity() * 8, L->h_off.capacity() * 8,
+                            L->h_dur.capacity() * 8, L->h_gid.capacity() * 8, L->h_chan.capacity() * 8};
+    if (on && !L->meta_pinned) {
+        bool ok = true;
+        for (int i = 0; i < 6; ++i) ok = ok && bytes[i] && cudaHostRegister(ptrs[i], bytes[i], cudaHostRegisterDefault) == cudaSuccess;
+        cudaGetLastError();
+        L->meta_pinned = ok;
+        if (!ok)
+            for (int i = 0; i < 6; ++i) cudaHostUnregister(ptrs[i]);   // (the ones that did register)
+        cudaGetLastError();
+    } else if (!on && L->meta_pinned) {
+        ck(cudaStreamSynchronize(L->stage_stream), "unpin sync");   // no upload still reads them
+        for (int i = 0; i < 6; ++i) cudaHostUnregister(ptrs[i]);
+        cudaGetLastError();
+        L->meta_pinned = false;
+    }
+}
+
 void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes, const uint64_t* durs,
                const uint64_t* gids, const uint64_t* chans, const std::vector<uint64_t>& offs, uint64_t arena_end) {
     const uint64_t base = L->h_size.size();
     bool any = base > 0;
+    if (L->meta_pinned && base + n > L->h_size.capacity()) pin_meta(L, false);   // about to reallocate
     L->h_site.insert(L->h_site.end(), sites, sites + n);
     L->h_size.insert(L->h_size.end(), sizes, sizes + n);
     L->h_off.insert(L->h_off.end(), offs.begin(), offs.begin() + n);
@@ -1284,6 +1309,7 @@ int ffm_log_create(const ffm_config* cfg, ffm_log** out) {
             L->h_dur.reserve(cfg->max_records);
             L->h_gid.reserve(cfg->max_records);
             L->h_chan.reserve(cfg->max_records);
+            pin_meta(L, true);
         }
     } catch (const CudaFail& f) {
         int code = (f.e == cudaErrorMemoryAllocation) ? FFM_E_NOMEM : FFM_E_CUDA;
@@ -1318,8 +1344,16 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
     try {
         ck(cudaSetDevice(L->device), "cudaSetDevice");
         ensure_arena(L, end);
-        std::vector<uint64_t> desc;
-        if (kind == FFM_PAYLOAD_DEVICE || kind == FFM_PAYLOAD_HOST_PINNED) desc.reserve(3 * n);
+        // k_gather descriptors (source, arena offset, bytes), written into page-locked
+        // staging (the previous append's copy of it completed: appends sync before return)
+        if (3 * n > L->h_desc_cap) {
+            if (L->h_desc) ck(cudaFreeHost(L->h_desc), "cudaFreeHost");
+            L->h_desc = nullptr;
+            const uint64_t c = std::max<uint64_t>(3 * n, 2 * L->h_desc_cap);
+            ck(cudaMallocHost(&L->h_desc, c * sizeof(uint64_t)), "cudaMallocHost(desc)");
+            L->h_desc_cap = c;
+        }
+        uint64_t nde = 0;   // descriptor words written
         bool need_sync = false, ordered = false;
         PtrCache pc;
         std::vector<PageablePiece> pageable;   // consecutive pageable records, staged together
@@ -1362,36 +1396,37 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
                    "copy");
             } else {
                 need_sync = true;     // k_gather reads caller memory (HBM, or pinned host over PCIe)
-                desc.push_back((uint64_t)(uintptr_t)payloads[i]);
-                desc.push_back(offs[i]);
-                desc.push_back(sizes[i]);
+                L->h_desc[nde++] = (uint64_t)(uintptr_t)payloads[i];
+                L->h_desc[nde++] = offs[i];
+                L->h_desc[nde++] = sizes[i];
             }
         }
         stage_pageable(L, pageable);
-        if (!desc.empty()) {
-            uint64_t nd = desc.size() / 3;
+        if (nde) {
+            uint64_t nd = nde / 3;
             uint64_t cap = L->desc_cap;
-            if (desc.size() > cap) {
+            if (nde > cap) {
+                ck(cudaStreamSynchronize(L->stage_stream), "desc grow");
                 if (L->d_desc) ck(cudaFree(L->d_desc), "cudaFree");
                 L->d_desc = nullptr;
-                cap = std::max<uint64_t>(desc.size(), 2 * cap);
+                cap = std::max<uint64_t>(nde, 2 * cap);
                 ck(cudaMalloc(&L->d_desc, cap * sizeof(uint64_t)), "cudaMalloc(desc)");
                 L->desc_cap = cap;
             }
-            ck(cudaMemcpyAsync(L->d_desc, desc.data(), desc.size() * 8, cudaMemcpyHostToDevice, L->stage_stream),
-               "desc H2D");
+            ck(cudaMemcpyAsync(L->d_desc, L->h_desc, nde * 8, cudaMemcpyHostToDevice, L->stage_stream), "desc H2D");
             if (launch_gather(L->d_desc, (uint32_t)nd, L->arena, L->stage_stream) < 0)
                 throw CudaFail{cudaGetLastError(), "k_gather"};
         }
-        if (need_sync) ck(cudaStreamSynchronize(L->stage_stream), "append sync");   // snapshot before return
         push_meta(L, n, sites, sizes, durs, gids, channels, offs, end);
         L->digests_valid = false;
         if (L->cfg.flags & FFM_FLAG_ONLINE) {
-            // online mode: the new records' metadata goes to the device now (the step
-            // starts from a resident window)
+            // online mode: the new records' metadata goes to the device now, overlapping
+            // the payload gather (the step starts from a resident window)
             ring_flush(L);
             upload_meta_arrays(L);
+            need_sync = true;
         }
+        if (need_sync) ck(cudaStreamSynchronize(L->stage_stream), "append sync");   // snapshot before return
         if ((L->cfg.flags & FFM_FLAG_ONLINE) && (L->cfg.flags & FFM_FLAG_APPEND_HASH)) {
             // append-time hashing: hash the new records now, on the hashing stream after
             // their staging copies -- the next append's staging overlaps this hashing
@@ -1798,6 +1833,12 @@ int ffm_log_destroy(ffm_log* L) {
         if (e) cudaEventDestroy(e);
     if (L->h_counters) cudaFreeHost(L->h_counters);
     if (L->h_wa) cudaFreeHost(L->h_wa);
+    if (L->h_desc) cudaFreeHost(L->h_desc);
+    if (L->meta_pinned) {
+        void* mp[] = {L->h_site.data(), L->h_size.data(), L->h_off.data(), L->h_dur.data(), L->h_gid.data(),
+                      L->h_chan.data()};
+        for (void* p : mp) cudaHostUnregister(p);
+    }
     if (L->stage_stream) cudaStreamDestroy(L->stage_stream);
     if (L->side_stream) cudaStreamDestroy(L->side_stream);
     if (L->hash_stream) {

@@ -351,6 +351,9 @@ struct ffm_log {
     // gather descriptors for device payloads
     uint64_t* d_desc = nullptr;
     uint64_t desc_cap = 0;
+    uint64_t* h_desc = nullptr;     // page-locked staging of the descriptors
+    uint64_t h_desc_cap = 0;
+    bool meta_pinned = false;       // h_site .. h_chan page-locked (within the reserved capacity)
 
     // run state
     ffm::Work work;
