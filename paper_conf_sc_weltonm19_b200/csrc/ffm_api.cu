@@ -4,6 +4,8 @@
 #include <cuda_runtime.h>
 #include <omp.h>
 #include <stdio.h>
+
+#include <chrono>
 #include <stdlib.h>
 #include <string.h>
 
@@ -11,6 +13,7 @@
 #include <functional>
 #include <new>
 #include <string>
+#include <iterator>
 #include <vector>
 
 #include "ffm_internal.h"
@@ -404,33 +407,81 @@ void pin_meta(ffm_log* L, bool on) {
     }
 }
 
+// gids g, g + 1, ... as an iterator range (no temporary, no zero-fill pass)
+struct CountIt {
+    using iterator_category = std::random_access_iterator_tag;
+    using value_type = uint64_t;
+    using difference_type = std::ptrdiff_t;
+    using pointer = const uint64_t*;
+    using reference = uint64_t;
+    uint64_t v;
+    uint64_t operator*() const { return v; }
+    CountIt& operator++() { ++v; return *this; }
+    CountIt operator++(int) { CountIt t = *this; ++v; return t; }
+    CountIt& operator--() { --v; return *this; }
+    CountIt operator--(int) { CountIt t = *this; --v; return t; }
+    CountIt operator-(difference_type d) const { return CountIt{v - (uint64_t)d}; }
+    CountIt& operator-=(difference_type d) { v -= (uint64_t)d; return *this; }
+    bool operator>(const CountIt& o) const { return v > o.v; }
+    bool operator<=(const CountIt& o) const { return v <= o.v; }
+    bool operator>=(const CountIt& o) const { return v >= o.v; }
+    difference_type operator-(const CountIt& o) const { return (difference_type)(v - o.v); }
+    CountIt operator+(difference_type d) const { return CountIt{v + (uint64_t)d}; }
+    CountIt& operator+=(difference_type d) { v += (uint64_t)d; return *this; }
+    uint64_t operator[](difference_type d) const { return v + (uint64_t)d; }
+    bool operator==(const CountIt& o) const { return v == o.v; }
+    bool operator!=(const CountIt& o) const { return v != o.v; }
+    bool operator<(const CountIt& o) const { return v < o.v; }
+};
+
+// Appends the batch's metadata to the host copies: the six arrays copied concurrently and
+// the running sums reduced in parallel for large batches (the append's host cost).
 void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes, const uint64_t* durs,
                const uint64_t* gids, const uint64_t* chans, const std::vector<uint64_t>& offs, uint64_t arena_end) {
     const uint64_t base = L->h_size.size();
-    bool any = base > 0;
+    const bool any = base > 0;
     if (L->meta_pinned && base + n > L->h_size.capacity()) pin_meta(L, false);   // about to reallocate
-    L->h_site.insert(L->h_site.end(), sites, sites + n);
-    L->h_size.insert(L->h_size.end(), sizes, sizes + n);
-    L->h_off.insert(L->h_off.end(), offs.begin(), offs.begin() + n);
-    L->h_dur.insert(L->h_dur.end(), durs, durs + n);
-    if (chans)
-        L->h_chan.insert(L->h_chan.end(), chans, chans + n);
-    else
-        L->h_chan.resize(base + n, 0);
-    if (gids) {
-        L->h_gid.insert(L->h_gid.end(), gids, gids + n);
-        L->any_gid = true;
-    } else {
-        L->h_gid.resize(base + n);
-        uint64_t g = any ? L->last_gid + 1 : 0;
-        for (uint64_t i = 0; i < n; ++i) L->h_gid[base + i] = g + i;
+    const uint64_t g0 = gids ? 0 : (any ? L->last_gid + 1 : 0);
+    const bool par = n >= 65536;
+#pragma omp parallel sections num_threads(6) if (par)
+    {
+#pragma omp section
+        L->h_site.insert(L->h_site.end(), sites, sites + n);
+#pragma omp section
+        L->h_size.insert(L->h_size.end(), sizes, sizes + n);
+#pragma omp section
+        L->h_off.insert(L->h_off.end(), offs.begin(), offs.begin() + n);
+#pragma omp section
+        L->h_dur.insert(L->h_dur.end(), durs, durs + n);
+#pragma omp section
+        {
+            if (chans)
+                L->h_chan.insert(L->h_chan.end(), chans, chans + n);
+            else
+                L->h_chan.resize(base + n, 0);
+        }
+#pragma omp section
+        {
+            if (gids)
+                L->h_gid.insert(L->h_gid.end(), gids, gids + n);
+            else
+                L->h_gid.insert(L->h_gid.end(), CountIt{g0}, CountIt{g0 + n});
+        }
     }
+    if (gids) L->any_gid = true;
     if (n) L->last_gid = L->h_gid.back();
+    uint64_t pb = 0, nlc = 0, nsr = 0;
+    const uint64_t cb = L->params.chunk_bytes, sb = L->params.small_bytes;
+#pragma omp parallel for reduction(+ : pb, nlc, nsr) num_threads(8) if (par)
     for (uint64_t i = 0; i < n; ++i) {
-        L->payload_bytes += sizes[i];
-        L->n_large_chunks += large_chunks(L, sizes[i]);
-        L->n_small_recs += sizes[i] <= L->params.small_bytes;
+        const uint64_t z = sizes[i];
+        pb += z;
+        nlc += z > sb ? (z + cb - 1) / cb : 0;
+        nsr += z <= sb;
     }
+    L->payload_bytes += pb;
+    L->n_large_chunks += nlc;
+    L->n_small_recs += nsr;
     L->arena_used = arena_end;
     ++L->epoch;
 }
@@ -1329,9 +1380,17 @@ int ffm_log_append_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const ui
     return ffm_log_append_batch_ex(L, n, sites, sizes, payloads, durs, gids, nullptr, kind);
 }
 
+#ifdef FFM_APPEND_TIMES
+#define FFM_AT(tag) fprintf(stderr, "[append] %s %.3f ms\n", tag, std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - at0).count())
+#else
+#define FFM_AT(tag)
+#endif
 int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes,
                             const void* const* payloads, const uint64_t* durs, const uint64_t* gids,
                             const uint64_t* channels, int kind) {
+#ifdef FFM_APPEND_TIMES
+    const auto at0 = std::chrono::steady_clock::now();
+#endif
     int st = check_state(L);
     if (st) return st;
     if (n == 0) return FFM_OK;
@@ -1341,6 +1400,7 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
     uint64_t end = 0;
     int rc = plan_batch(L, n, sites, sizes, payloads, gids, offs, end);
     if (rc) return rc;
+    FFM_AT("plan");
     try {
         ck(cudaSetDevice(L->device), "cudaSetDevice");
         ensure_arena(L, end);
@@ -1357,7 +1417,74 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
         bool need_sync = false, ordered = false;
         PtrCache pc;
         std::vector<PageablePiece> pageable;   // consecutive pageable records, staged together
-        for (uint64_t i = 0; i < n; ++i) {
+        // a large batch of device or page-locked payloads: classified and its descriptors
+        // written by the host threads in parallel (no ring staging can occur)
+        const bool par = (kind == FFM_PAYLOAD_DEVICE || kind == FFM_PAYLOAD_HOST_PINNED) && n >= 65536;
+        if (par) {
+            if (kind == FFM_PAYLOAD_DEVICE) {
+                // device payloads may still be being produced (see below)
+                ordered = true;
+                ck(cudaEventRecord(L->fork_ev[0], cudaStreamLegacy), "event");
+                ck(cudaStreamWaitEvent(L->stage_stream, L->fork_ev[0], 0), "wait producer");
+                if (L->stream != cudaStreamLegacy) {
+                    ck(cudaEventRecord(L->fork_ev[1], L->stream), "event");
+                    ck(cudaStreamWaitEvent(L->stage_stream, L->fork_ev[1], 0), "wait producer");
+                }
+            }
+            if (L->ring_fill) ring_flush(L);
+            std::vector<uint8_t> act(n);   // 0: nothing (empty), 1: k_gather, 2: copy engine
+            const int T = stage_threads();
+            std::vector<uint64_t> cnt(T + 1, 0);
+            int used = 1;
+            const uint64_t gmax = L->gather_max;
+            const bool hp_ok = L->host_ptr_ok;
+            const int mydev = L->device;
+#pragma omp parallel num_threads(T)
+            {
+                const int t = omp_get_thread_num(), nt = omp_get_num_threads();
+                const uint64_t lo = n * t / nt, hi = n * (t + 1) / nt;
+                PtrCache pct;
+                uint64_t c = 0;
+                for (uint64_t i = lo; i < hi; ++i) {
+                    if (sizes[i] == 0) {
+                        act[i] = 0;
+                        continue;
+                    }
+                    int pdev = mydev;
+                    if (kind == FFM_PAYLOAD_DEVICE) {
+                        int d = -1;   // (a peer GPU's memory is never dereferenced by k_gather)
+                        if (pct.classify(payloads[i], &d) == FFM_PAYLOAD_DEVICE) pdev = d;
+                    }
+                    const bool dma = sizes[i] > gmax || (kind == FFM_PAYLOAD_HOST_PINNED && !hp_ok) ||
+                                     (kind == FFM_PAYLOAD_DEVICE && pdev != mydev);
+                    act[i] = dma ? 2 : 1;
+                    c += !dma;
+                }
+                cnt[t + 1] = c;
+#pragma omp barrier
+#pragma omp single
+                {
+                    used = nt;
+                    for (int k = 0; k < nt; ++k) cnt[k + 1] += cnt[k];
+                }
+                uint64_t k = 3 * cnt[t];
+                for (uint64_t i = lo; i < hi; ++i) {
+                    if (act[i] != 1) continue;
+                    L->h_desc[k++] = (uint64_t)(uintptr_t)payloads[i];
+                    L->h_desc[k++] = offs[i];
+                    L->h_desc[k++] = sizes[i];
+                }
+            }
+            nde = 3 * cnt[used];
+            need_sync = nde != 0;
+            for (uint64_t i = 0; i < n; ++i) {
+                if (act[i] != 2) continue;
+                need_sync = true;   // async copy engine from caller memory: sync before return
+                ck(cudaMemcpyAsync(L->arena + offs[i], payloads[i], sizes[i], cudaMemcpyDefault, L->stage_stream),
+                   "copy");
+            }
+        }
+        for (uint64_t i = 0; i < (par ? 0 : n); ++i) {
             if (sizes[i] == 0) continue;
             int src = kind, pdev = L->device;
             if (kind == FFM_PAYLOAD_AUTO) {
@@ -1402,6 +1529,7 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
             }
         }
         stage_pageable(L, pageable);
+        FFM_AT("staging loop");
         if (nde) {
             uint64_t nd = nde / 3;
             uint64_t cap = L->desc_cap;
@@ -1417,7 +1545,9 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
             if (launch_gather(L->d_desc, (uint32_t)nd, L->arena, L->stage_stream) < 0)
                 throw CudaFail{cudaGetLastError(), "k_gather"};
         }
+        FFM_AT("desc + gather queued");
         push_meta(L, n, sites, sizes, durs, gids, channels, offs, end);
+        FFM_AT("push_meta");
         L->digests_valid = false;
         if (L->cfg.flags & FFM_FLAG_ONLINE) {
             // online mode: the new records' metadata goes to the device now, overlapping
@@ -1426,7 +1556,9 @@ int ffm_log_append_batch_ex(ffm_log* L, uint64_t n, const uint32_t* sites, const
             upload_meta_arrays(L);
             need_sync = true;
         }
+        FFM_AT("meta upload queued");
         if (need_sync) ck(cudaStreamSynchronize(L->stage_stream), "append sync");   // snapshot before return
+        FFM_AT("synced");
         if ((L->cfg.flags & FFM_FLAG_ONLINE) && (L->cfg.flags & FFM_FLAG_APPEND_HASH)) {
             // append-time hashing: hash the new records now, on the hashing stream after
             // their staging copies -- the next append's staging overlaps this hashing

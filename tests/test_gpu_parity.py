@@ -619,3 +619,34 @@ def test_empty_log_and_all_empty_payloads(ffm):
     for i in range(1, n):
         want[sites[i]] += durs[i]
     assert ben.tolist() == want
+
+
+@pytest.mark.parametrize("kind", ["device", "pinned"])
+def test_large_batch_parallel_staging(ffm, kind):
+    """A batch of >= 65,536 device or page-locked payloads is classified and its gather
+    descriptors written by the host threads in parallel; empty payloads and payloads
+    above the gather limit (copy engines) mixed in; bytes snapshotted before return."""
+    import torch
+    lg = loggen.gen_config(2, n_scale=0.12)
+    host = lg.materialize()
+    buf = torch.from_numpy(host.copy()).cuda() if kind == "device" else torch.from_numpy(host.copy()).pin_memory()
+    ptrs = (lg.c_off[lg.content] + np.uint64(buf.data_ptr())).astype(np.uint64)
+    sizes = lg.size.copy()
+    sizes[::997] = 0                                  # empty payloads (all equal, R7)
+    big = np.zeros(3 << 20, np.uint8)                 # > the 1 MiB gather limit: copy engines
+    big[::4099] = 7
+    bt = torch.from_numpy(big).cuda() if kind == "device" else torch.from_numpy(big).pin_memory()
+    sizes[5::20011] = big.size
+    ptrs[5::20011] = bt.data_ptr()
+    lg2 = loggen.from_payloads([host[lg.c_off[lg.content[i]]:lg.c_off[lg.content[i]] + sizes[i]].tobytes()
+                                if ptrs[i] != bt.data_ptr() else big.tobytes() for i in range(lg.n)],
+                               lg.site, lg.dur, lg.n_sites)
+    pk = ffm.FFM_PAYLOAD_DEVICE if kind == "device" else ffm.FFM_PAYLOAD_HOST_PINNED
+    with ffm.FfmLog(lg.n_sites) as log:
+        log.append_batch(lg.site, sizes, ptrs, lg.dur, payload_kind=pk)
+        buf.zero_()                                   # snapshot taken: later writes are invisible
+        bt.zero_()
+        dup, ben = log.run()
+    want_d, want_b = oracle.dedup(lg2)
+    np.testing.assert_array_equal(dup, want_d)
+    np.testing.assert_array_equal(ben, want_b)

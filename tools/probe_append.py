@@ -11,6 +11,9 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import loggen  # noqa: E402
 import paper_conf_sc_weltonm19_b200 as ffm  # noqa: E402
 
+if os.environ.get("PROBE_LIB"):
+    ffm.set_library_path(os.environ["PROBE_LIB"])
+
 lg = loggen.gen_config(2)
 lg.materialize(nthreads=0)
 content = torch.from_numpy(lg.buf).cuda()
