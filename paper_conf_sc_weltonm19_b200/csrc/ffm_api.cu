@@ -356,30 +356,65 @@ int check_state(ffm_log* L) {
 }
 
 // Validate + assign arena offsets for a batch; returns FFM_OK or an error without
-// touching the log.
+// touching the log.  Slots are 32-byte aligned, so offs[i] = base + sum over earlier
+// records of align_up(size, 32): a prefix sum, split over the host threads for a large
+// batch (each thread's chunk checked and summed, then offset by the chunks before it); an
+// error is reported for the first offending record, as the serial check would.
 int plan_batch(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* sizes, const void* const* payloads,
                const uint64_t* gids, std::vector<uint64_t>& offs, uint64_t& arena_end) {
-    uint64_t cur = L->arena_used;
-    uint64_t last = L->last_gid;
-    bool any = L->any_gid || !L->h_gid.empty();
+    const bool any0 = L->any_gid || !L->h_gid.empty();
+    const uint64_t last0 = L->last_gid;
     uint64_t base_n = L->h_size.size();
     if (base_n + n >= 0xFFFFFFFFull) return set_err(L, FFM_E_RANGE, "too many records for one log (2^32-1)");
     if (L->cfg.world > 1 && !gids)
         return set_err(L, FFM_E_INVAL, "a sharded log needs the records' global gids (gids == NULL)");
     offs.resize(n);
-    for (uint64_t i = 0; i < n; ++i) {
-        if (sites[i] >= L->cfg.n_sites) return set_err(L, FFM_E_RANGE, "call_site >= n_sites");
-        if (sizes[i] > 0 && payloads[i] == nullptr) return set_err(L, FFM_E_INVAL, "NULL payload with size > 0");
-        uint64_t g = gids ? gids[i] : (any ? last + 1 : 0);
-        if (gids && any && g <= last) return set_err(L, FFM_E_RANGE, "gids must be strictly increasing");
-        if (g >> 63) return set_err(L, FFM_E_RANGE, "gid >= 2^63 (duplicate_of is int64)");
-        last = g;
-        any = true;
-        cur = align_up(cur, kArenaAlign);
-        offs[i] = cur;
-        cur += sizes[i];
+    // record i's problem (0: none), independent of the others but for the gid order
+    auto check = [&](uint64_t i) -> int {
+        if (sites[i] >= L->cfg.n_sites) return 1;
+        if (sizes[i] > 0 && payloads[i] == nullptr) return 2;
+        if (gids) {
+            if ((i > 0 || any0) && gids[i] <= (i > 0 ? gids[i - 1] : last0)) return 3;
+            if (gids[i] >> 63) return 4;
+        } else if (((any0 ? last0 + 1 : 0) + i) >> 63) {
+            return 4;
+        }
+        return 0;
+    };
+    const uint64_t base = align_up(L->arena_used, kArenaAlign);
+    const int T = n >= 65536 ? stage_threads() : 1;
+    std::vector<uint64_t> part(T + 1, 0), bad(T, ~0ull);
+    int used = 1;
+#pragma omp parallel num_threads(T) if (T > 1)
+    {
+        const int t = omp_get_thread_num(), nt = omp_get_num_threads();
+        const uint64_t lo = n * t / nt, hi = n * (t + 1) / nt;
+        uint64_t sum = 0;
+        for (uint64_t i = lo; i < hi; ++i) {
+            if (bad[t] == ~0ull && check(i)) bad[t] = i;
+            offs[i] = sum;
+            sum += align_up(sizes[i], kArenaAlign);
+        }
+        part[t + 1] = sum;
+#pragma omp barrier
+#pragma omp single
+        {
+            used = nt;
+            for (int k = 0; k < nt; ++k) part[k + 1] += part[k];
+        }
+        for (uint64_t i = lo; i < hi; ++i) offs[i] += base + part[t];
     }
-    arena_end = cur;
+    uint64_t first = ~0ull;
+    for (int t = 0; t < used; ++t) first = std::min(first, bad[t]);
+    if (first != ~0ull) {
+        switch (check(first)) {
+            case 1: return set_err(L, FFM_E_RANGE, "call_site >= n_sites");
+            case 2: return set_err(L, FFM_E_INVAL, "NULL payload with size > 0");
+            case 3: return set_err(L, FFM_E_RANGE, "gids must be strictly increasing");
+            default: return set_err(L, FFM_E_RANGE, "gid >= 2^63 (duplicate_of is int64)");
+        }
+    }
+    arena_end = n ? offs[n - 1] + sizes[n - 1] : L->arena_used;
     return FFM_OK;
 }
 
@@ -409,29 +444,18 @@ void pin_meta(ffm_log* L, bool on) {
 
 // gids g, g + 1, ... as an iterator range (no temporary, no zero-fill pass)
 struct CountIt {
-    using iterator_category = std::random_access_iterator_tag;
+    using iterator_category = std::forward_iterator_tag;
     using value_type = uint64_t;
     using difference_type = std::ptrdiff_t;
     using pointer = const uint64_t*;
     using reference = uint64_t;
     uint64_t v;
     uint64_t operator*() const { return v; }
-    CountIt& operator++() { ++v; return *this; }
-    CountIt operator++(int) { CountIt t = *this; ++v; return t; }
-    CountIt& operator--() { --v; return *this; }
-    CountIt operator--(int) { CountIt t = *this; --v; return t; }
-    CountIt operator-(difference_type d) const { return CountIt{v - (uint64_t)d}; }
-    CountIt& operator-=(difference_type d) { v -= (uint64_t)d; return *this; }
-    bool operator>(const CountIt& o) const { return v > o.v; }
-    bool operator<=(const CountIt& o) const { return v <= o.v; }
-    bool operator>=(const CountIt& o) const { return v >= o.v; }
-    difference_type operator-(const CountIt& o) const { return (difference_type)(v - o.v); }
-    CountIt operator+(difference_type d) const { return CountIt{v + (uint64_t)d}; }
-    CountIt& operator+=(difference_type d) { v += (uint64_t)d; return *this; }
-    uint64_t operator[](difference_type d) const { return v + (uint64_t)d; }
-    bool operator==(const CountIt& o) const { return v == o.v; }
+    CountIt& operator++() {
+        ++v;
+        return *this;
+    }
     bool operator!=(const CountIt& o) const { return v != o.v; }
-    bool operator<(const CountIt& o) const { return v < o.v; }
 };
 
 // Appends the batch's metadata to the host copies: the six arrays copied concurrently and
@@ -442,7 +466,7 @@ void push_meta(ffm_log* L, uint64_t n, const uint32_t* sites, const uint64_t* si
     const bool any = base > 0;
     if (L->meta_pinned && base + n > L->h_size.capacity()) pin_meta(L, false);   // about to reallocate
     const uint64_t g0 = gids ? 0 : (any ? L->last_gid + 1 : 0);
-    const bool par = n >= 65536;
+    [[maybe_unused]] const bool par = n >= 65536;   // (used in the OpenMP clauses)
 #pragma omp parallel sections num_threads(6) if (par)
     {
 #pragma omp section

@@ -650,3 +650,34 @@ def test_large_batch_parallel_staging(ffm, kind):
     want_d, want_b = oracle.dedup(lg2)
     np.testing.assert_array_equal(dup, want_d)
     np.testing.assert_array_equal(ben, want_b)
+
+
+def test_large_batch_errors_leave_log_unchanged(ffm):
+    """A batch of >= 65,536 records is planned by the host threads in parallel: the first
+    offending record decides the error (as record-by-record checking would) and the log is
+    left unchanged."""
+    n = 100_000
+    x = np.zeros(64, np.uint8)
+    sites = np.zeros(n, np.uint32)
+    sizes = np.full(n, 64, np.uint64)
+    ptrs = np.full(n, x.ctypes.data, np.uint64)
+    durs = np.ones(n, np.uint64)
+    gids = np.arange(n, dtype=np.uint64) * 2
+    with ffm.FfmLog(4) as log:
+        s2 = sites.copy()
+        s2[90_000] = 4                        # call_site out of range, later than ...
+        g2 = gids.copy()
+        g2[70_001] = g2[70_000]               # ... a gid that is not increasing: reported first
+        with pytest.raises(ffm.FfmError) as e:
+            log.append_batch(s2, sizes, ptrs, durs, gids=g2)
+        assert e.value.code == ffm.FFM_E_RANGE and "increasing" in str(e.value)
+        p2 = ptrs.copy()
+        p2[66_000] = 0                        # NULL payload before the out-of-range site
+        with pytest.raises(ffm.FfmError) as e:
+            log.append_batch(s2, sizes, p2, durs, gids=gids)
+        assert e.value.code == ffm.FFM_E_INVAL
+        assert log.count == 0
+        log.append_batch(sites, sizes, ptrs, durs, gids=gids)
+        assert log.count == n
+        dup, ben = log.run()
+        assert dup[0] == -1 and (dup[1:] == 0).all() and int(ben[0]) == n - 1
